@@ -1,0 +1,364 @@
+/*
+ * oracle.c -- plain, slow, single-threaded fp64 CPU oracle for the PASTA MTTKRP hot path.
+ *
+ * TEST INFRASTRUCTURE ONLY.  Only tests/, __graft_entry__.smoke() and bench.py's
+ * cpu_baseline / --impl reference legs may load or call this library.  The product
+ * path (libpasta.so, paper_conf_iiswc_lilwlob20_b200/) never does, and it shares no
+ * source, header, table or helper with this file.
+ *
+ * Citations: "P:N" = line N of the paper text (/root/reference/PAPER.md,
+ * Li et al., "A Sparse Tensor Benchmark Suite for CPUs and GPUs", IISWC'20).
+ * "R#k" = reading k in DESIGN.md section "Readings of the paper".
+ *
+ * Every routine below follows the definition or algorithm it cites in the order the
+ * paper states it; the only library primitive used is qsort.  Compile with
+ * -ffp-contract=off so that no multiply-add is fused (the generator's fp64 cell
+ * decision must be reproducible bit for bit, R#20).
+ *
+ * Pins (tests/test_oracle_*.py): brute force X_(n)(KRP) on dense tiny tensors,
+ * rank-1 closed form, all-ones slice sums, N=2 SpMM (scipy), R=1 chained TTV,
+ * linearity/order/mode-permutation invariants, an independent Python Morton
+ * conversion, HiCOO storage formula, binomial popcount marginal of the
+ * generator.  No routine here is "parity unpinned".
+ */
+#include <math.h>
+#include <stdint.h>
+#include <stdlib.h>
+#include <string.h>
+
+#define ORACLE_MAX_ORDER 8
+
+/* ------------------------------------------------------------------------- */
+/* O-MTTKRP: Eq. 3 with the Khatri-Rao product of Eq. 4 folded  */
+/* into the nonzero loop, as the paper describes (Alg. 3). */
+/*   Mref(i_n(x), r) += val(x) * prod_{k != n} U^(k)(i_k(x), r)               */
+/*   Aref(i_n(x), r) += |val(x) * prod_{k != n} U^(k)(i_k(x), r)|             */
+/* Factors are row-major [I_k][R] (footnote 2; R#4).                   */
+/* Returns 0, or -1 on invalid arguments.                                     */
+/* ------------------------------------------------------------------------- */
+int oracle_mttkrp(uint32_t order, const uint32_t *dims, uint64_t nnz,
+                  const uint32_t *const *inds, const float *vals, uint32_t mode,
+                  const float *const *factors, uint32_t R, double *Mref, double *Aref)
+{
+    if (order < 1 || order > ORACLE_MAX_ORDER || mode >= order || R < 1) return -1;
+    uint64_t rows = dims[mode];
+    for (uint64_t e = 0; e < rows * R; ++e) { Mref[e] = 0.0; Aref[e] = 0.0; }
+    for (uint64_t x = 0; x < nnz; ++x) {
+        uint64_t i = inds[mode][x];
+        for (uint32_t r = 0; r < R; ++r) {
+            double t = (double)vals[x];
+            for (uint32_t k = 0; k < order; ++k) {
+                if (k == mode) continue;
+                t *= (double)factors[k][(uint64_t)inds[k][x] * R + r];
+            }
+            Mref[i * R + r] += t;
+            Aref[i * R + r] += fabs(t);
+        }
+    }
+    return 0;
+}
+
+/* Same definition restricted to a set of output rows (for full-size sampled
+ * parity).  rows[] must be strictly increasing; Mref/Aref are [nsel][R]. */
+int oracle_mttkrp_rows(uint32_t order, const uint32_t *dims, uint64_t nnz,
+                       const uint32_t *const *inds, const float *vals, uint32_t mode,
+                       const float *const *factors, uint32_t R, uint32_t nsel,
+                       const uint32_t *rows, double *Mref, double *Aref)
+{
+    if (order < 1 || order > ORACLE_MAX_ORDER || mode >= order || R < 1) return -1;
+    (void)dims;
+    for (uint64_t e = 0; e < (uint64_t)nsel * R; ++e) { Mref[e] = 0.0; Aref[e] = 0.0; }
+    for (uint64_t x = 0; x < nnz; ++x) {
+        uint32_t i = inds[mode][x];
+        /* binary search i in rows[0..nsel) */
+        uint32_t lo = 0, hi = nsel;
+        while (lo < hi) {
+            uint32_t mid = lo + (hi - lo) / 2;
+            if (rows[mid] < i) lo = mid + 1; else hi = mid;
+        }
+        if (lo == nsel || rows[lo] != i) continue;
+        for (uint32_t r = 0; r < R; ++r) {
+            double t = (double)vals[x];
+            for (uint32_t k = 0; k < order; ++k) {
+                if (k == mode) continue;
+                t *= (double)factors[k][(uint64_t)inds[k][x] * R + r];
+            }
+            Mref[(uint64_t)lo * R + r] += t;
+            Aref[(uint64_t)lo * R + r] += fabs(t);
+        }
+    }
+    return 0;
+}
+
+/* ------------------------------------------------------------------------- */
+/* O-HiCOO-MTTKRP (Alg. 3): for block b, the pointers are rebased   */
+/* by binds(b)*B*R, i.e. i_k = binds_k(b)*B + einds_k(x) (R#5: A_b means the  */
+/* output).  Then the same accumulation as O-MTTKRP.                          */
+/* ------------------------------------------------------------------------- */
+int oracle_mttkrp_hicoo(uint32_t order, const uint32_t *dims, uint32_t block_bits,
+                        uint64_t nblocks, const uint64_t *bptr,
+                        const uint32_t *const *binds, const uint8_t *const *einds,
+                        const float *vals, uint32_t mode, const float *const *factors,
+                        uint32_t R, double *Mref, double *Aref)
+{
+    if (order < 1 || order > ORACLE_MAX_ORDER || mode >= order || R < 1) return -1;
+    uint64_t B = 1ull << block_bits;
+    uint64_t rows = dims[mode];
+    for (uint64_t e = 0; e < rows * R; ++e) { Mref[e] = 0.0; Aref[e] = 0.0; }
+    for (uint64_t b = 0; b < nblocks; ++b) {
+        for (uint64_t x = bptr[b]; x < bptr[b + 1]; ++x) {
+            uint64_t i = (uint64_t)binds[mode][b] * B + einds[mode][x];
+            for (uint32_t r = 0; r < R; ++r) {
+                double t = (double)vals[x];
+                for (uint32_t k = 0; k < order; ++k) {
+                    if (k == mode) continue;
+                    uint64_t ik = (uint64_t)binds[k][b] * B + einds[k][x];
+                    t *= (double)factors[k][ik * R + r];
+                }
+                Mref[i * R + r] += t;
+                Aref[i * R + r] += fabs(t);
+            }
+        }
+    }
+    return 0;
+}
+
+/* ------------------------------------------------------------------------- */
+/* Sorting helpers (qsort over an index permutation; ties broken by original  */
+/* position so that the result is a stable sort, R#15).                       */
+/* ------------------------------------------------------------------------- */
+static uint32_t g_order;
+static const uint32_t *const *g_inds;
+static uint32_t g_first_mode;
+
+/* O-mode-sort comparator: lexicographic on (i_n, i_{n+1 mod N}, ..., i_{n-1}),
+ * which makes equal output rows contiguous (a2; "pre-processing to trade
+ * for less kernel computation time", "naturally sorted in a mode order"). */
+static int cmp_mode_lex(const void *pa, const void *pb)
+{
+    uint64_t a = *(const uint64_t *)pa, b = *(const uint64_t *)pb;
+    for (uint32_t j = 0; j < g_order; ++j) {
+        uint32_t k = (g_first_mode + j) % g_order;
+        uint32_t va = g_inds[k][a], vb = g_inds[k][b];
+        if (va != vb) return va < vb ? -1 : 1;
+    }
+    return a < b ? -1 : (a > b ? 1 : 0);
+}
+
+/* Morton (Z) order comparator for HiCOO ("Morton order sorting implied by
+ * the HiCOO format"; R#13): the first differing bit of the level-major
+ * interleave (MSB level first, mode 0 first within a level) decides.  That bit
+ * lives in mode k* = argmax_k msb(a_k XOR b_k), ties to the smallest k. */
+static int msb_less(uint32_t x, uint32_t y) { return x < y && x < (x ^ y); }
+static int cmp_morton(const void *pa, const void *pb)
+{
+    uint64_t a = *(const uint64_t *)pa, b = *(const uint64_t *)pb;
+    int best = -1;
+    uint32_t best_x = 0;
+    for (uint32_t k = 0; k < g_order; ++k) {
+        uint32_t x = g_inds[k][a] ^ g_inds[k][b];
+        if (msb_less(best_x, x)) { best = (int)k; best_x = x; }
+    }
+    if (best >= 0) {
+        uint32_t va = g_inds[best][a], vb = g_inds[best][b];
+        return va < vb ? -1 : 1;
+    }
+    return a < b ? -1 : (a > b ? 1 : 0);
+}
+
+/* Mode-n sort of a COO tensor.  Writes the permuted copy into out_inds/out_vals. */
+int oracle_mode_sort(uint32_t order, uint64_t nnz, const uint32_t *const *inds,
+                     const float *vals, uint32_t mode, uint32_t *const *out_inds,
+                     float *out_vals)
+{
+    if (order < 1 || order > ORACLE_MAX_ORDER || mode >= order) return -1;
+    uint64_t *perm = (uint64_t *)malloc((nnz ? nnz : 1) * sizeof(uint64_t));
+    if (!perm) return -2;
+    for (uint64_t x = 0; x < nnz; ++x) perm[x] = x;
+    g_order = order; g_inds = inds; g_first_mode = mode;
+    qsort(perm, nnz, sizeof(uint64_t), cmp_mode_lex);
+    for (uint64_t x = 0; x < nnz; ++x) {
+        for (uint32_t k = 0; k < order; ++k) out_inds[k][x] = inds[k][perm[x]];
+        out_vals[x] = vals[perm[x]];
+    }
+    free(perm);
+    return 0;
+}
+
+/* ------------------------------------------------------------------------- */
+/* O-HiCOO conversion (R#10, R#12-R#14):             */
+/*  1. sort nonzeros into Morton order of their full coordinates;             */
+/*  2. scan: a new block starts where (i_k >> b) differs for any k;           */
+/*  3. emit bptr (u64, bptr[n_b] = M), binds_k(blk) = i_k >> b (u32),          */
+/*     einds_k(x) = i_k & (B-1) (u8), val (bitwise copy).                     */
+/* Output arrays are caller-allocated with capacity M (bptr: M+1).            */
+/* Returns n_b (>= 0) or -1 on invalid arguments.                             */
+/* ------------------------------------------------------------------------- */
+int64_t oracle_coo_to_hicoo(uint32_t order, uint64_t nnz, const uint32_t *const *inds,
+                            const float *vals, uint32_t block_bits, uint64_t *bptr,
+                            uint32_t *const *binds, uint8_t *const *einds, float *out_vals)
+{
+    if (order < 1 || order > ORACLE_MAX_ORDER || block_bits < 1 || block_bits > 8) return -1;
+    uint64_t *perm = (uint64_t *)malloc((nnz ? nnz : 1) * sizeof(uint64_t));
+    if (!perm) return -2;
+    for (uint64_t x = 0; x < nnz; ++x) perm[x] = x;
+    g_order = order; g_inds = inds;
+    qsort(perm, nnz, sizeof(uint64_t), cmp_morton);
+    uint32_t emask = (1u << block_bits) - 1u;
+    int64_t nb = 0;
+    for (uint64_t x = 0; x < nnz; ++x) {
+        uint64_t p = perm[x];
+        int new_block = (x == 0);
+        if (!new_block) {
+            uint64_t q = perm[x - 1];
+            for (uint32_t k = 0; k < order; ++k)
+                if ((inds[k][p] >> block_bits) != (inds[k][q] >> block_bits)) new_block = 1;
+        }
+        if (new_block) {
+            bptr[nb] = x;
+            for (uint32_t k = 0; k < order; ++k) binds[k][nb] = inds[k][p] >> block_bits;
+            ++nb;
+        }
+        for (uint32_t k = 0; k < order; ++k) einds[k][x] = (uint8_t)(inds[k][p] & emask);
+        out_vals[x] = vals[p];
+    }
+    bptr[nb] = nnz;
+    free(perm);
+    return nb;
+}
+
+/* ------------------------------------------------------------------------- */
+/* Stochastic Kronecker ("ball-dropping") tensor generator, P:223-227 (R#19-  */
+/* R#23).  Counter-based randomness so the product generator can implement    */
+/* the very same draw sequence independently:                                 */
+/*   mix64 = SplitMix64 finaliser;  K = mix64(seed ^ 0x5851F42D4C957F2D);     */
+/*   h(d, s) = mix64(K ^ mix64((s << 40) | d));  u = (h >> 11) * 2^-53.       */
+/* Draw d, level l (s = l): choose initiator cell c = first c with            */
+/*   u * cum[last] < cum[c]   (cum = running fp64 sum of the 2^N table);      */
+/* mode k takes bit ((c >> k) & 1) at bit position l while l < L_k =          */
+/* ceil(log2 I_k).  A draw with any i_k >= I_k is stripped.           */
+/* Value of draw d: (float)(lo + (hi - lo) * u(d, 0xFFFF)).                   */
+/* Result: the first M distinct coordinates in draw order (each keeps the     */
+/* value of its first draw), emitted in lexicographic (i_0, ..., i_{N-1})     */
+/* order.  Returns 0, -1 invalid, -2 no memory, -3 could not reach M.         */
+/* ------------------------------------------------------------------------- */
+static uint64_t mix64(uint64_t z)
+{
+    z ^= z >> 30; z *= 0xbf58476d1ce4e5b9ull;
+    z ^= z >> 27; z *= 0x94d049bb133111ebull;
+    z ^= z >> 31;
+    return z;
+}
+static double gen_uniform(uint64_t key, uint64_t d, uint64_t s)
+{
+    uint64_t h = mix64(key ^ mix64((s << 40) | d));
+    return (double)(h >> 11) * (1.0 / 9007199254740992.0);
+}
+
+typedef struct { uint32_t c[ORACLE_MAX_ORDER]; uint64_t d; } draw_rec;
+static uint32_t g_gen_order;
+static int cmp_draw_coords_then_d(const void *pa, const void *pb)
+{
+    const draw_rec *a = (const draw_rec *)pa, *b = (const draw_rec *)pb;
+    for (uint32_t k = 0; k < g_gen_order; ++k)
+        if (a->c[k] != b->c[k]) return a->c[k] < b->c[k] ? -1 : 1;
+    return a->d < b->d ? -1 : (a->d > b->d ? 1 : 0);
+}
+static int cmp_draw_d(const void *pa, const void *pb)
+{
+    const draw_rec *a = (const draw_rec *)pa, *b = (const draw_rec *)pb;
+    return a->d < b->d ? -1 : (a->d > b->d ? 1 : 0);
+}
+
+int oracle_gen_powerlaw(uint32_t order, const uint32_t *dims, uint64_t nnz, uint64_t seed,
+                        const double *initiator, double q, float val_lo, float val_hi,
+                        uint32_t *const *out_inds, float *out_vals)
+{
+    if (order < 1 || order > ORACLE_MAX_ORDER) return -1;
+    uint32_t ncell = 1u << order;
+    double table[1u << ORACLE_MAX_ORDER], cum[1u << ORACLE_MAX_ORDER];
+    if (initiator) {
+        for (uint32_t c = 0; c < ncell; ++c) table[c] = initiator[c];
+    } else {
+        if (!(q > 0.0 && q < 1.0)) q = 0.75;
+        for (uint32_t c = 0; c < ncell; ++c) {
+            double p = 1.0;
+            for (uint32_t k = 0; k < order; ++k) p = p * (((c >> k) & 1u) ? (1.0 - q) : q);
+            table[c] = p;
+        }
+    }
+    double run = 0.0;
+    uint32_t last_pos = 0;
+    for (uint32_t c = 0; c < ncell; ++c) {
+        if (table[c] < 0.0) return -1;
+        run = run + table[c];
+        cum[c] = run;
+        if (table[c] > 0.0) last_pos = c;
+    }
+    if (!(run > 0.0)) return -1;
+    uint32_t L[ORACLE_MAX_ORDER], Lmax = 0;
+    double cells = 1.0;
+    for (uint32_t k = 0; k < order; ++k) {
+        if (dims[k] < 1) return -1;
+        uint32_t l = 0;
+        while (l < 32 && ((uint64_t)1 << l) < dims[k]) ++l;
+        L[k] = l;
+        if (l > Lmax) Lmax = l;
+        cells *= (double)dims[k];
+    }
+    if ((double)nnz > cells) return -1;
+    uint64_t key = mix64(seed ^ 0x5851F42D4C957F2Dull);
+
+    uint64_t D = nnz + nnz / 16 + 4096;
+    uint64_t cap = 64 * nnz + (1ull << 22);
+    for (;;) {
+        draw_rec *rec = (draw_rec *)malloc(D * sizeof(draw_rec));
+        if (!rec) return -2;
+        uint64_t nvalid = 0;
+        for (uint64_t d = 0; d < D; ++d) {
+            draw_rec r;
+            memset(&r, 0, sizeof(r));
+            r.d = d;
+            for (uint32_t l = 0; l < Lmax; ++l) {
+                double u = gen_uniform(key, d, l) * run;
+                uint32_t cell = last_pos;
+                for (uint32_t c = 0; c < ncell; ++c)
+                    if (u < cum[c]) { cell = c; break; }
+                for (uint32_t k = 0; k < order; ++k)
+                    if (l < L[k]) r.c[k] |= ((cell >> k) & 1u) << l;
+            }
+            int ok = 1;
+            for (uint32_t k = 0; k < order; ++k) if (r.c[k] >= dims[k]) ok = 0;
+            if (ok) rec[nvalid++] = r;
+        }
+        g_gen_order = order;
+        qsort(rec, nvalid, sizeof(draw_rec), cmp_draw_coords_then_d);
+        uint64_t nuniq = 0;
+        for (uint64_t x = 0; x < nvalid; ++x) {
+            int dup = 0;
+            if (nuniq > 0) {
+                dup = 1;
+                for (uint32_t k = 0; k < order; ++k)
+                    if (rec[x].c[k] != rec[nuniq - 1].c[k]) dup = 0;
+            }
+            if (!dup) rec[nuniq++] = rec[x];
+        }
+        if (nuniq >= nnz) {
+            qsort(rec, nuniq, sizeof(draw_rec), cmp_draw_d);           /* first-drawn order */
+            qsort(rec, nnz, sizeof(draw_rec), cmp_draw_coords_then_d); /* keep M, lex order */
+            double lo = (double)val_lo, diff = (double)val_hi - (double)val_lo;
+            for (uint64_t x = 0; x < nnz; ++x) {
+                for (uint32_t k = 0; k < order; ++k) out_inds[k][x] = rec[x].c[k];
+                double u = gen_uniform(key, rec[x].d, 0xFFFF);
+                double v = lo + diff * u;
+                out_vals[x] = (float)v;
+            }
+            free(rec);
+            return 0;
+        }
+        free(rec);
+        if (D >= cap) return -3;
+        D = D + D / 2 + 2 * (nnz - nuniq) + 4096; /* geometric growth */
+        if (D > cap) D = cap;
+    }
+}
