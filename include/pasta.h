@@ -1,0 +1,204 @@
+/*
+ * pasta.h -- C ABI of libpasta, a B200-native (sm_100a) sparse MTTKRP library on COO and
+ * HiCOO tensors, after Li et al., "A Sparse Tensor Benchmark Suite for CPUs and GPUs"
+ * (IISWC'20).  "P:N" cites line N of that paper's text; "R#k" cites reading k
+ * of DESIGN.md ("Readings of the paper").
+ *
+ * Conventions for every entry point
+ *   - Returns pasta_status; nothing throws or aborts across the ABI.  On a non-OK status
+ *     pasta_last_error() returns a thread-local, human-readable message.
+ *   - Arguments are validated before any side effect (EINVAL / ERANGE).  A CUDA launch or
+ *     runtime failure maps to PASTA_ECUDA.  Faults of asynchronous kernels surface at the
+ *     next synchronising call.
+ *   - Tensor handles (pasta_coo, pasta_hicoo) are opaque and library-owned; free them with
+ *     pasta_*_free (NULL-safe).  Their arrays live in device memory of the device that was
+ *     current at creation.  Handles are immutable after creation except for lazily built,
+ *     cached per-mode copies (pasta_*_prepare); calls on one handle must be serialised by
+ *     the caller until every mode it uses is prepared, after which they are thread-safe.
+ *   - Factor and output matrices are caller-owned DEVICE memory (e.g. torch tensors),
+ *     row-major [I_k][R] with leading dimension R (footnote 2; Alg. 3's bi*B*R
+ *     rebasing; R#4).  The library never frees them.
+ *   - Indices are 0-based uint32 ("32 bits"), values fp32.  Modes are
+ *     0-based (R#6).  Maximum order PASTA_MAX_ORDER.
+ *   - `stream` is a cudaStream_t (NULL = legacy default stream).  MTTKRP calls are
+ *     asynchronous on it; creation / conversion / export calls synchronise.
+ */
+#ifndef PASTA_H
+#define PASTA_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define PASTA_MAX_ORDER 8
+
+typedef enum {
+    PASTA_OK = 0,
+    PASTA_EINVAL = -1,       /* invalid argument (NULL pointer, mode >= order, R == 0, ...) */
+    PASTA_EIO = -2,          /* file could not be opened / read / written                  */
+    PASTA_EFORMAT = -3,      /* malformed input file                                        */
+    PASTA_ERANGE = -4,       /* an index >= its dimension, a size beyond 32-bit limits      */
+    PASTA_ENOMEM = -5,       /* host or device allocation failed                             */
+    PASTA_ECUDA = -6,        /* CUDA runtime / launch error                                  */
+    PASTA_EUNSUPPORTED = -7  /* valid request this build does not implement                  */
+} pasta_status;
+
+typedef struct pasta_coo pasta_coo;     /* COO tensor, device-resident          */
+typedef struct pasta_hicoo pasta_hicoo; /* HiCOO tensor, device-resident        */
+
+/* Optional device allocator hook (e.g. torch's caching allocator).  alloc returns device
+ * memory of `bytes` usable on `stream` or NULL; free releases it.  NULL hook -> cudaMalloc. */
+typedef struct {
+    void *(*alloc)(size_t bytes, void *stream, void *ctx);
+    void (*free)(void *ptr, void *stream, void *ctx);
+    void *ctx;
+} pasta_allocator;
+
+/* Thread-local text describing the last non-OK status of this thread ("" if none). */
+const char *pasta_last_error(void);
+/* Library version string, e.g. "pasta-b200 0.1 sm_100a". */
+const char *pasta_version(void);
+/* Install (or with NULL, remove) the device allocator hook.  Affects later allocations. */
+pasta_status pasta_set_allocator(const pasta_allocator *alloc);
+
+/* ---------------------------------------------------------------- ingest (a1) --------- */
+
+/* Load a COO tensor from a FROSTT-style text file (R#17): one nonzero per line,
+ * whitespace-separated 1-based indices followed by the value; '#' lines are comments.
+ * The order is the token count of the first data line minus one; dims are the per-mode
+ * maximum index.  Repeated coordinates are kept as separate nonzeros (MTTKRP is linear in
+ * them, R#15).  Errors: EIO (open/read), EFORMAT (ragged line, index 0, bad number),
+ * ERANGE (index > 2^32-1 or > 2^32-1 nonzeros). */
+pasta_status pasta_load_coo(const char *path, pasta_coo **out);
+
+/* Write `x` (canonical order) as a 1-based text file readable by pasta_load_coo.
+ * Values are printed with 9 significant digits (exact fp32 round trip).  EIO on failure. */
+pasta_status pasta_save_coo(const pasta_coo *x, const char *path);
+
+/* Create a COO tensor from HOST arrays (copied; the caller keeps ownership).
+ * inds: `order` pointers to nnz uint32 each; vals: nnz floats.  Every index must be
+ * < dims[k] (ERANGE otherwise).  The input order is kept as the canonical order. */
+pasta_status pasta_coo_from_arrays(uint32_t order, const uint32_t *dims, uint64_t nnz,
+                                   const uint32_t *const *inds, const float *vals,
+                                   pasta_coo **out);
+
+/* Synthetic tensor generator parameters (R#19-R#23). */
+typedef struct {
+    uint32_t kind;            /* 0 uniform (q = 0.5), 1 Stochastic Kronecker (default),
+                                 2 FireHose slice power law (not implemented: EUNSUPPORTED) */
+    const double *initiator;  /* 2^order non-negative cell weights, cell c sets bit k of mode
+                                 k's index to (c >> k) & 1; NULL -> product form from q     */
+    double q;                 /* product-form P(bit = 0) per mode per level; 0 -> 0.75      */
+    uint32_t permute;         /* must be 0 (random relabelling: EUNSUPPORTED)                */
+    float val_lo, val_hi;     /* values uniform in [val_lo, val_hi); both 0 -> [-1, 1)       */
+} pasta_gen_params;
+
+/* Stochastic Kronecker tensor by ball dropping (R#20-R#21): draw d chooses, at each
+ * level l < L_k = ceil(log2 I_k), an initiator cell with the counter-based uniform
+ * u(d, l) = (mix64(K ^ mix64((l << 40) | d)) >> 11) * 2^-53,  K = mix64(seed ^
+ * 0x5851F42D4C957F2D), mix64 = SplitMix64 finaliser; mode k takes the cell's bit k as bit l
+ * of i_k; draws with any i_k >= I_k are stripped.  The tensor is the first `nnz` distinct
+ * coordinates in draw order, each with value lo + (hi - lo) * u(d_first, 0xFFFF) (fp64,
+ * rounded to fp32), stored in lexicographic (i_0, ..., i_{N-1}) order.  Runs on the GPU.
+ * Errors: EINVAL (order, dims, nnz > prod dims, bad initiator), ERANGE (more than 2^32-2
+ * draws would be needed), EUNSUPPORTED (kind 2, permute). */
+pasta_status pasta_gen_powerlaw(uint32_t order, const uint32_t *dims, uint64_t nnz,
+                                uint64_t seed, const pasta_gen_params *params,
+                                pasta_coo **out);
+
+/* ------------------------------------------------------------- formats (a2, a3) ------ */
+
+/* HiCOO conversion (R#10-R#14): Morton (Z) order of the full
+ * coordinates (level-major interleave, MSB level first, mode 0 first within a level; ties
+ * by canonical position), blocks of B = 2^block_bits per mode (block_bits 1..8; 7 -> the
+ * paper's B = 128), bptr u64, binds u32 = i >> b, einds u8 = i & (B-1).  Bit-exact
+ * with the oracle's conversion.  Runs on the GPU. */
+pasta_status pasta_coo_to_hicoo(const pasta_coo *x, uint32_t block_bits, pasta_hicoo **out);
+
+/* Build (once; cached in the handle) the mode-`mode` working copy: for COO the nonzeros
+ * stably sorted lexicographically by (i_mode, i_mode+1, ..., i_mode-1) (a2);
+ * for HiCOO the blocks stably sorted by binds_mode and, inside each block, the entries
+ * stably sorted by einds_mode (R#27).  Optional: MTTKRP prepares on first use. */
+pasta_status pasta_coo_prepare(pasta_coo *x, uint32_t mode, void *stream);
+pasta_status pasta_hicoo_prepare(pasta_hicoo *h, uint32_t mode, void *stream);
+
+/* --------------------------------------------------------------- MTTKRP (a5-a8) ------ */
+
+/* out = X_(mode) (U^(N-1) (.) ... (.) U^(mode+1) (.) U^(mode-1) (.) ... (.) U^(0))
+ * (Eq. 3; Eq. 4) computed directly over the nonzeros:
+ *   out(i_mode(x), r) += val(x) * prod_{k != mode} U^(k)(i_k(x), r).
+ * factors: `order` DEVICE pointers, U^(k) row-major [dims[k]][R]; factors[mode] is not
+ * read and may be NULL.  out: DEVICE [dims[mode]][R] row-major, OVERWRITTEN (zeroed, then
+ * accumulated, R#1) on the rows this handle owns: all rows, or [row_lo, row_hi) of a shard
+ * made for this mode.  fp32 arithmetic; partial sums combined with fp32 atomics at segment
+ * boundaries (R#24).  Asynchronous on `stream`.  Prepares the mode on first use
+ * (synchronising once).  R >= 1 (any value; R % 4 == 0 and 16-byte aligned pointers take
+ * the 128-bit vector path). */
+pasta_status pasta_mttkrp_coo(pasta_coo *x, uint32_t mode, const float *const *factors,
+                              uint32_t R, float *out, void *stream);
+pasta_status pasta_mttkrp_hicoo(pasta_hicoo *h, uint32_t mode, const float *const *factors,
+                                uint32_t R, float *out, void *stream);
+
+/* End-to-end variant over ALL modes with HOST buffers (the e2e path): copies the `order`
+ * factor matrices host->device (pinned host memory gives full PCIe/C2C bandwidth), computes
+ * MTTKRP for every mode into library-owned device buffers, copies the `order` results back
+ * to host_out[k] ([dims[k]][R] row-major) and synchronises `stream`.  Device staging
+ * buffers are cached in the handle. */
+pasta_status pasta_mttkrp_coo_allmodes_host(pasta_coo *x, const float *const *host_factors,
+                                            uint32_t R, float *const *host_out, void *stream);
+
+/* --------------------------------------------------------------- multi-GPU (a9) ------ */
+
+/* counts[r] = number of nonzeros with i_mode == r, r < dims[mode] (HOST uint64 buffer). */
+pasta_status pasta_coo_row_counts(const pasta_coo *x, uint32_t mode, uint64_t *counts);
+/* Host-only: nnz-balanced contiguous row ranges.  bounds[p] = min{ r : S(r) >= p*T/nparts }
+ * with S(r) = sum_{i<r} counts[i], T = S(nrows); bounds[0] = 0, bounds[nparts] = nrows.
+ * bounds has nparts + 1 entries.  Needs no GPU. */
+pasta_status pasta_row_partition(uint32_t nrows, const uint64_t *counts, uint32_t nparts,
+                                 uint32_t *bounds);
+/* pasta_coo_row_counts + pasta_row_partition. */
+pasta_status pasta_coo_partition(const pasta_coo *x, uint32_t mode, uint32_t nparts,
+                                 uint32_t *bounds);
+/* New handle holding the nonzeros with row_lo <= i_mode < row_hi (global indices and dims
+ * kept; the mode-`mode` copy comes prepared).  MTTKRP of that mode on the shard writes only
+ * rows [row_lo, row_hi) of `out`. */
+pasta_status pasta_coo_shard(pasta_coo *x, uint32_t mode, uint32_t row_lo, uint32_t row_hi,
+                             pasta_coo **out);
+
+/* ------------------------------------------------------------ introspection ---------- */
+
+pasta_status pasta_coo_info(const pasta_coo *x, uint32_t *order, uint32_t *dims,
+                            uint64_t *nnz);
+/* Copy the canonical arrays to HOST buffers (inds: `order` pointers to nnz uint32). */
+pasta_status pasta_coo_export(const pasta_coo *x, uint32_t *const *inds, float *vals);
+/* Copy the mode-`mode` sorted copy to HOST buffers (prepares it if needed). */
+pasta_status pasta_coo_export_mode(pasta_coo *x, uint32_t mode, uint32_t *const *inds,
+                                   float *vals);
+pasta_status pasta_hicoo_info(const pasta_hicoo *h, uint32_t *order, uint32_t *dims,
+                              uint32_t *block_bits, uint64_t *nblocks, uint64_t *nnz);
+/* Copy the canonical (Morton-ordered) HiCOO arrays to HOST buffers: bptr[nblocks+1],
+ * binds: `order` pointers to nblocks uint32, einds: `order` pointers to nnz uint8, vals. */
+pasta_status pasta_hicoo_export(const pasta_hicoo *h, uint64_t *bptr, uint32_t *const *binds,
+                                uint8_t *const *einds, float *vals);
+void pasta_coo_free(pasta_coo *x);
+void pasta_hicoo_free(pasta_hicoo *h);
+
+/* -------------------------------------------------------------- measurement ---------- */
+
+/* Number of kernels this library has launched in this process (all kinds). */
+uint64_t pasta_launch_count(void);
+/* When enabled, every MTTKRP main-kernel launch is bracketed by CUDA events recorded on
+ * its own stream.  pasta_profile_read synchronises those events and returns the summed
+ * device time (ms) and the launch count of kernel family `which` (0 = COO MTTKRP,
+ * 1 = HiCOO MTTKRP, 2 = output zero-fill), then clears the record if `reset`. */
+pasta_status pasta_profile_enable(int on);
+pasta_status pasta_profile_read(uint32_t which, double *total_ms, uint64_t *launches,
+                                int reset);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* PASTA_H */

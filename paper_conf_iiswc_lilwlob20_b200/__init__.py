@@ -1,0 +1,372 @@
+"""pasta-b200: B200-native sparse MTTKRP on COO and HiCOO (Li et al., IISWC'20).
+
+Thin Python binding over the C ABI of ``lib/libpasta.so`` (``include/pasta.h``): the
+functions carry the C names and only marshal arguments.  Every compute step (generation,
+sorting, HiCOO conversion, MTTKRP) runs in the library's CUDA kernels; PyTorch supplies
+device memory, streams and process groups.  There is no CPU fallback: importing works
+without a GPU, but compute calls raise ``PastaError`` (PASTA_ECUDA) when no device exists.
+"""
+from __future__ import annotations
+
+import ctypes as C
+from typing import Optional, Sequence
+
+import numpy as np
+
+from ._native import MAX_ORDER, Allocator, ALLOC_FN, FREE_FN, GenParams, PastaError, check, lib
+
+__all__ = [
+    "PastaError", "Coo", "Hicoo", "pasta_version", "pasta_set_allocator", "use_torch_allocator",
+    "pasta_load_coo", "pasta_save_coo", "pasta_coo_from_arrays", "pasta_gen_powerlaw",
+    "pasta_coo_to_hicoo", "pasta_coo_prepare", "pasta_hicoo_prepare", "pasta_mttkrp_coo",
+    "pasta_mttkrp_hicoo", "pasta_mttkrp_coo_allmodes_host", "pasta_coo_row_counts",
+    "pasta_row_partition", "pasta_coo_partition", "pasta_coo_shard", "pasta_coo_info",
+    "pasta_coo_export", "pasta_coo_export_mode", "pasta_hicoo_info", "pasta_hicoo_export",
+    "pasta_launch_count", "pasta_profile_enable", "pasta_profile_read",
+]
+
+_u32p = C.POINTER(C.c_uint32)
+_u64p = C.POINTER(C.c_uint64)
+_f32p = C.POINTER(C.c_float)
+_u8p = C.POINTER(C.c_uint8)
+
+
+class Coo:
+    """Owning wrapper of a ``pasta_coo*`` (device-resident COO tensor)."""
+
+    def __init__(self, ptr: int):
+        self._p = C.c_void_p(ptr)
+        order, dims, nnz = pasta_coo_info(self)
+        self.order, self.dims, self.nnz = order, dims, nnz
+
+    @property
+    def ptr(self):
+        return self._p
+
+    def free(self):
+        if self._p and self._p.value:
+            lib().pasta_coo_free(self._p)
+            self._p = C.c_void_p(None)
+
+    def __del__(self):
+        try:
+            self.free()
+        except Exception:
+            pass
+
+
+class Hicoo:
+    """Owning wrapper of a ``pasta_hicoo*`` (device-resident HiCOO tensor)."""
+
+    def __init__(self, ptr: int):
+        self._p = C.c_void_p(ptr)
+        info = pasta_hicoo_info(self)
+        self.order, self.dims, self.block_bits, self.nblocks, self.nnz = info
+
+    @property
+    def ptr(self):
+        return self._p
+
+    def free(self):
+        if self._p and self._p.value:
+            lib().pasta_hicoo_free(self._p)
+            self._p = C.c_void_p(None)
+
+    def __del__(self):
+        try:
+            self.free()
+        except Exception:
+            pass
+
+
+def _np_ptr(a: np.ndarray, t):
+    return a.ctypes.data_as(t)
+
+
+def _stream_ptr(stream):
+    import torch
+    if stream is None:
+        stream = torch.cuda.current_stream()
+    return C.c_void_p(stream.cuda_stream)
+
+
+# ----------------------------------------------------------------------------- library
+def pasta_version() -> str:
+    return lib().pasta_version().decode()
+
+
+_alloc_keepalive = []
+
+
+def pasta_set_allocator(alloc_fn=None, free_fn=None) -> None:
+    """Install python callables ``alloc_fn(nbytes, stream_ptr) -> int`` / ``free_fn(ptr, stream_ptr)``
+    as the device allocator hook, or remove the hook when both are None."""
+    if alloc_fn is None and free_fn is None:
+        check(lib().pasta_set_allocator(None))
+        _alloc_keepalive.clear()
+        return
+
+    def _a(nbytes, stream, ctx):
+        try:
+            return alloc_fn(int(nbytes), stream)
+        except Exception:
+            return None
+
+    def _f(ptr, stream, ctx):
+        try:
+            free_fn(ptr, stream)
+        except Exception:
+            pass
+
+    a, f = ALLOC_FN(_a), FREE_FN(_f)
+    s = Allocator(a, f, None)
+    _alloc_keepalive[:] = [a, f, s]
+    check(lib().pasta_set_allocator(C.byref(s)))
+
+
+def use_torch_allocator() -> None:
+    """Route libpasta device allocations through torch's caching allocator."""
+    import torch
+
+    def alloc(nbytes, stream):
+        return torch.cuda.caching_allocator_alloc(max(nbytes, 1), torch.cuda.current_device(),
+                                                  stream or 0)
+
+    def free(ptr, stream):
+        torch.cuda.caching_allocator_delete(ptr)
+
+    pasta_set_allocator(alloc, free)
+
+
+# ----------------------------------------------------------------------------- ingest
+def pasta_load_coo(path: str) -> Coo:
+    out = C.c_void_p()
+    check(lib().pasta_load_coo(path.encode(), C.byref(out)))
+    return Coo(out.value)
+
+
+def pasta_save_coo(x: Coo, path: str) -> None:
+    check(lib().pasta_save_coo(x.ptr, path.encode()))
+
+
+def pasta_coo_from_arrays(dims: Sequence[int], inds: np.ndarray, vals: np.ndarray) -> Coo:
+    """Create a device COO tensor from host arrays ``inds`` (u32 [N, M]) and ``vals`` (f32 [M])."""
+    dims_a = np.ascontiguousarray(dims, dtype=np.uint32)
+    order = dims_a.shape[0]
+    vals = np.ascontiguousarray(vals, dtype=np.float32)
+    inds = np.ascontiguousarray(inds, dtype=np.uint32).reshape(order, vals.shape[0])
+    rows = [np.ascontiguousarray(inds[k]) for k in range(order)]
+    arr = (_u32p * max(order, 1))(*[_np_ptr(r, _u32p) for r in rows])
+    out = C.c_void_p()
+    check(lib().pasta_coo_from_arrays(order, _np_ptr(dims_a, _u32p), vals.shape[0], arr,
+                                      _np_ptr(vals, _f32p), C.byref(out)))
+    return Coo(out.value)
+
+
+def pasta_gen_powerlaw(dims: Sequence[int], nnz: int, seed: int, kind: int = 1,
+                       initiator: Optional[Sequence[float]] = None, q: float = 0.0,
+                       val_lo: float = -1.0, val_hi: float = 1.0, permute: int = 0) -> Coo:
+    """Stochastic Kronecker tensor on the GPU; see include/pasta.h."""
+    dims_a = np.ascontiguousarray(dims, dtype=np.uint32)
+    p = GenParams()
+    p.kind, p.q, p.permute, p.val_lo, p.val_hi = kind, q, permute, val_lo, val_hi
+    keep = None
+    if initiator is not None:
+        keep = np.ascontiguousarray(initiator, dtype=np.float64)
+        p.initiator = keep.ctypes.data_as(C.POINTER(C.c_double))
+    out = C.c_void_p()
+    check(lib().pasta_gen_powerlaw(dims_a.shape[0], _np_ptr(dims_a, _u32p), nnz, seed, C.byref(p),
+                                   C.byref(out)))
+    del keep
+    return Coo(out.value)
+
+
+# ----------------------------------------------------------------------------- formats
+def pasta_coo_to_hicoo(x: Coo, block_bits: int = 7) -> Hicoo:
+    out = C.c_void_p()
+    check(lib().pasta_coo_to_hicoo(x.ptr, block_bits, C.byref(out)))
+    return Hicoo(out.value)
+
+
+def pasta_coo_prepare(x: Coo, mode: int, stream=None) -> None:
+    check(lib().pasta_coo_prepare(x.ptr, mode, _stream_ptr(stream)))
+
+
+def pasta_hicoo_prepare(h: Hicoo, mode: int, stream=None) -> None:
+    check(lib().pasta_hicoo_prepare(h.ptr, mode, _stream_ptr(stream)))
+
+
+# ----------------------------------------------------------------------------- MTTKRP
+def _factor_ptrs(order, mode, factors, R):
+    import torch
+    ptrs = (C.c_void_p * order)()
+    for k in range(order):
+        f = factors[k] if k < len(factors) else None
+        if k == mode:
+            ptrs[k] = None
+            continue
+        if f is None or not isinstance(f, torch.Tensor) or not f.is_cuda:
+            raise PastaError(-1, f"factors[{k}] must be a CUDA tensor")
+        if f.dtype != torch.float32 or not f.is_contiguous() or f.dim() != 2 or f.shape[1] != R:
+            raise PastaError(-1, f"factors[{k}] must be a contiguous float32 [I_k, R] tensor")
+        ptrs[k] = f.data_ptr()
+    return ptrs
+
+
+def _check_out(out, rows, R):
+    import torch
+    if not (isinstance(out, torch.Tensor) and out.is_cuda and out.dtype == torch.float32
+            and out.is_contiguous() and tuple(out.shape) == (rows, R)):
+        raise PastaError(-1, f"out must be a contiguous float32 CUDA tensor of shape ({rows}, {R})")
+
+
+def _rank(factors, mode, R=None):
+    if R is not None:
+        return int(R)
+    for k, f in enumerate(factors):
+        if k != mode and f is not None:
+            return int(f.shape[1])
+    raise PastaError(-1, "no factor matrix given")
+
+
+def pasta_mttkrp_coo(x: Coo, mode: int, factors, out=None, stream=None, R=None):
+    """Mode-`mode` MTTKRP (Eq. 3) on COO; returns ``out`` (float32 [I_mode, R] CUDA tensor)."""
+    import torch
+    R = _rank(factors, mode, R)
+    if not 0 <= mode < x.order:
+        raise PastaError(-1, f"mode {mode} >= order {x.order}")
+    if out is None:
+        dev = next((f.device for k, f in enumerate(factors) if k != mode and f is not None),
+                   torch.device("cuda", torch.cuda.current_device()))
+        out = torch.empty((x.dims[mode], R), dtype=torch.float32, device=dev)
+    _check_out(out, x.dims[mode], R)
+    ptrs = _factor_ptrs(x.order, mode, factors, R)
+    check(lib().pasta_mttkrp_coo(x.ptr, mode, ptrs, R, C.c_void_p(out.data_ptr()),
+                                 _stream_ptr(stream)))
+    return out
+
+
+def pasta_mttkrp_hicoo(h: Hicoo, mode: int, factors, out=None, stream=None, R=None):
+    """Mode-`mode` MTTKRP on HiCOO (Alg. 3 semantics); returns ``out``."""
+    import torch
+    R = _rank(factors, mode, R)
+    if not 0 <= mode < h.order:
+        raise PastaError(-1, f"mode {mode} >= order {h.order}")
+    if out is None:
+        dev = next((f.device for k, f in enumerate(factors) if k != mode and f is not None),
+                   torch.device("cuda", torch.cuda.current_device()))
+        out = torch.empty((h.dims[mode], R), dtype=torch.float32, device=dev)
+    _check_out(out, h.dims[mode], R)
+    ptrs = _factor_ptrs(h.order, mode, factors, R)
+    check(lib().pasta_mttkrp_hicoo(h.ptr, mode, ptrs, R, C.c_void_p(out.data_ptr()),
+                                   _stream_ptr(stream)))
+    return out
+
+
+def pasta_mttkrp_coo_allmodes_host(x: Coo, host_factors, host_out, stream=None) -> None:
+    """All-modes MTTKRP from/to HOST tensors or arrays (float32, contiguous, ideally pinned)."""
+    R = int(host_factors[0].shape[1])
+    fp = (C.c_void_p * x.order)()
+    op = (C.c_void_p * x.order)()
+    for k in range(x.order):
+        f, o = host_factors[k], host_out[k]
+        fp[k] = f.data_ptr() if hasattr(f, "data_ptr") else f.ctypes.data
+        op[k] = o.data_ptr() if hasattr(o, "data_ptr") else o.ctypes.data
+    check(lib().pasta_mttkrp_coo_allmodes_host(x.ptr, fp, R, op, _stream_ptr(stream)))
+
+
+# ----------------------------------------------------------------------------- multi-GPU
+def pasta_coo_row_counts(x: Coo, mode: int) -> np.ndarray:
+    counts = np.zeros(x.dims[mode], np.uint64)
+    check(lib().pasta_coo_row_counts(x.ptr, mode, _np_ptr(counts, _u64p)))
+    return counts
+
+
+def pasta_row_partition(counts: np.ndarray, nparts: int) -> np.ndarray:
+    """Host-only nnz-balanced contiguous row ranges (needs no GPU)."""
+    counts = np.ascontiguousarray(counts, dtype=np.uint64)
+    bounds = np.zeros(nparts + 1, np.uint32)
+    check(lib().pasta_row_partition(counts.shape[0], _np_ptr(counts, _u64p), nparts,
+                                    _np_ptr(bounds, _u32p)))
+    return bounds
+
+
+def pasta_coo_partition(x: Coo, mode: int, nparts: int) -> np.ndarray:
+    bounds = np.zeros(nparts + 1, np.uint32)
+    check(lib().pasta_coo_partition(x.ptr, mode, nparts, _np_ptr(bounds, _u32p)))
+    return bounds
+
+
+def pasta_coo_shard(x: Coo, mode: int, row_lo: int, row_hi: int) -> Coo:
+    out = C.c_void_p()
+    check(lib().pasta_coo_shard(x.ptr, mode, row_lo, row_hi, C.byref(out)))
+    return Coo(out.value)
+
+
+# ----------------------------------------------------------------------------- introspection
+def pasta_coo_info(x: Coo):
+    order = C.c_uint32()
+    dims = (C.c_uint32 * MAX_ORDER)()
+    nnz = C.c_uint64()
+    check(lib().pasta_coo_info(x.ptr, C.byref(order), dims, C.byref(nnz)))
+    return order.value, tuple(dims[: order.value]), nnz.value
+
+
+def _export(fn, x, *extra):
+    inds = [np.zeros(max(x.nnz, 1), np.uint32) for _ in range(x.order)]
+    vals = np.zeros(max(x.nnz, 1), np.float32)
+    arr = (_u32p * x.order)(*[_np_ptr(i, _u32p) for i in inds])
+    check(fn(x.ptr, *extra, arr, _np_ptr(vals, _f32p)))
+    return np.stack([i[: x.nnz] for i in inds]), vals[: x.nnz].copy()
+
+
+def pasta_coo_export(x: Coo):
+    """Canonical arrays -> (inds u32 [N, M], vals f32 [M]) on the host."""
+    return _export(lib().pasta_coo_export, x)
+
+
+def pasta_coo_export_mode(x: Coo, mode: int):
+    """Mode-`mode` sorted copy -> (inds, vals) on the host."""
+    return _export(lib().pasta_coo_export_mode, x, mode)
+
+
+def pasta_hicoo_info(h: Hicoo):
+    order = C.c_uint32()
+    dims = (C.c_uint32 * MAX_ORDER)()
+    bb = C.c_uint32()
+    nb = C.c_uint64()
+    nnz = C.c_uint64()
+    check(lib().pasta_hicoo_info(h.ptr, C.byref(order), dims, C.byref(bb), C.byref(nb),
+                                 C.byref(nnz)))
+    return order.value, tuple(dims[: order.value]), bb.value, nb.value, nnz.value
+
+
+def pasta_hicoo_export(h: Hicoo) -> dict:
+    nb, M, N = h.nblocks, h.nnz, h.order
+    bptr = np.zeros(nb + 1, np.uint64)
+    binds = [np.zeros(max(nb, 1), np.uint32) for _ in range(N)]
+    einds = [np.zeros(max(M, 1), np.uint8) for _ in range(N)]
+    vals = np.zeros(max(M, 1), np.float32)
+    bp = (_u32p * N)(*[_np_ptr(b, _u32p) for b in binds])
+    ep = (_u8p * N)(*[_np_ptr(e, _u8p) for e in einds])
+    check(lib().pasta_hicoo_export(h.ptr, _np_ptr(bptr, _u64p), bp, ep, _np_ptr(vals, _f32p)))
+    return {"order": N, "block_bits": h.block_bits, "nblocks": nb, "nnz": M, "bptr": bptr,
+            "binds": np.stack([b[:nb] for b in binds]), "einds": np.stack([e[:M] for e in einds]),
+            "vals": vals[:M].copy()}
+
+
+# ----------------------------------------------------------------------------- measurement
+def pasta_launch_count() -> int:
+    return int(lib().pasta_launch_count())
+
+
+def pasta_profile_enable(on: bool = True) -> None:
+    check(lib().pasta_profile_enable(1 if on else 0))
+
+
+def pasta_profile_read(which: int, reset: bool = True):
+    """Summed device ms and launch count of kernel family `which` (0 COO, 1 HiCOO, 2 zero)."""
+    ms = C.c_double()
+    n = C.c_uint64()
+    check(lib().pasta_profile_read(which, C.byref(ms), C.byref(n), 1 if reset else 0))
+    return ms.value, n.value

@@ -1,0 +1,699 @@
+// capi.cu -- the extern "C" boundary of libpasta (include/pasta.h): validation, handles,
+// errors, host-side IO / partitioning and measurement hooks.  Every compute step runs in
+// the kernels of gen.cu, sort.cu, hicoo.cu and mttkrp.cu.
+#include <cerrno>
+#include <cinttypes>
+#include <cmath>
+#include <cstdio>
+#include <cstdlib>
+#include <memory>
+#include <new>
+
+#include "internal.cuh"
+
+namespace pasta {
+
+// ----------------------------------------------------------------------------- errors
+static thread_local std::string t_last_error;
+
+void set_last_error(pasta_status code, const std::string &msg) {
+  (void)code;
+  t_last_error = msg;
+}
+
+static std::atomic<uint64_t> g_launches{0};
+void count_launch() { g_launches.fetch_add(1, std::memory_order_relaxed); }
+
+// ----------------------------------------------------------------------------- memory
+static std::mutex g_alloc_mu;
+static pasta_allocator g_alloc{nullptr, nullptr, nullptr};
+static bool g_alloc_set = false;
+
+void *dev_alloc(size_t bytes, cudaStream_t s) {
+  pasta_allocator a;
+  bool set;
+  {
+    std::lock_guard<std::mutex> lk(g_alloc_mu);
+    a = g_alloc;
+    set = g_alloc_set;
+  }
+  void *p = nullptr;
+  if (set) {
+    p = a.alloc(bytes, reinterpret_cast<void *>(s), a.ctx);
+    if (!p) fail(PASTA_ENOMEM, "device allocation of " + std::to_string(bytes) + " bytes failed (hook)");
+    return p;
+  }
+  cudaError_t e = cudaMalloc(&p, bytes);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    fail(e == cudaErrorMemoryAllocation ? PASTA_ENOMEM : PASTA_ECUDA,
+         "cudaMalloc(" + std::to_string(bytes) + "): " + cudaGetErrorString(e));
+  }
+  return p;
+}
+
+void dev_free(void *p, cudaStream_t s) {
+  if (!p) return;
+  pasta_allocator a;
+  bool set;
+  {
+    std::lock_guard<std::mutex> lk(g_alloc_mu);
+    a = g_alloc;
+    set = g_alloc_set;
+  }
+  if (set) {
+    a.free(p, reinterpret_cast<void *>(s), a.ctx);
+  } else {
+    cudaFree(p);
+  }
+}
+
+// ----------------------------------------------------------------------------- profiling
+static std::mutex g_prof_mu;
+static std::atomic<bool> g_prof_on{false};
+struct ProfRec {
+  cudaEvent_t a, b;
+};
+static std::vector<ProfRec> g_prof[kProfKinds];
+
+ProfScope::ProfScope(int k, cudaStream_t st) : kind(k), s(st) {
+  if (!g_prof_on.load(std::memory_order_relaxed)) return;
+  if (cudaEventCreate(&a) != cudaSuccess || cudaEventCreate(&b) != cudaSuccess) {
+    cudaGetLastError();
+    a = b = nullptr;
+    return;
+  }
+  cudaEventRecord(a, s);
+}
+ProfScope::~ProfScope() {
+  if (!a) return;
+  cudaEventRecord(b, s);
+  std::lock_guard<std::mutex> lk(g_prof_mu);
+  g_prof[kind].push_back({a, b});
+}
+
+}  // namespace pasta
+
+using namespace pasta;
+
+#define API_BEGIN try {
+#define API_END                                                            \
+  return PASTA_OK;                                                         \
+  }                                                                        \
+  catch (const pasta::Error &e) {                                          \
+    set_last_error(e.code, e.msg);                                         \
+    return e.code;                                                         \
+  }                                                                        \
+  catch (const std::bad_alloc &) {                                         \
+    set_last_error(PASTA_ENOMEM, "host allocation failed");                \
+    return PASTA_ENOMEM;                                                   \
+  }                                                                        \
+  catch (...) {                                                            \
+    set_last_error(PASTA_EINVAL, "unexpected internal exception");         \
+    return PASTA_EINVAL;                                                   \
+  }
+
+static void require(bool cond, const char *msg) {
+  if (!cond) fail(PASTA_EINVAL, msg);
+}
+
+static cudaStream_t as_stream(void *s) { return reinterpret_cast<cudaStream_t>(s); }
+
+static void check_device(int dev) {
+  int cur = -1;
+  PASTA_CUDA(cudaGetDevice(&cur));
+  if (cur != dev)
+    fail(PASTA_EINVAL, "handle lives on device " + std::to_string(dev) + " but device " +
+                           std::to_string(cur) + " is current");
+}
+
+static int current_device() {
+  int d = 0;
+  PASTA_CUDA(cudaGetDevice(&d));
+  return d;
+}
+
+static void validate_dims(uint32_t order, const uint32_t *dims) {
+  require(order >= 1 && order <= kMaxOrder, "order must be in 1..PASTA_MAX_ORDER");
+  require(dims != nullptr, "dims is NULL");
+  for (uint32_t k = 0; k < order; ++k) require(dims[k] >= 1, "every dimension must be >= 1");
+}
+
+// Upload host arrays into a fresh handle (indices already validated).
+static std::unique_ptr<pasta_coo> coo_upload(uint32_t order, const uint32_t *dims, uint64_t nnz,
+                                             const uint32_t *const *inds, const float *vals,
+                                             cudaStream_t s) {
+  auto x = std::make_unique<pasta_coo>();
+  x->order = order;
+  for (uint32_t k = 0; k < order; ++k) x->dims[k] = dims[k];
+  x->nnz = nnz;
+  x->device = current_device();
+  for (uint32_t k = 0; k < order; ++k) {
+    x->inds[k].alloc(nnz, s);
+    if (nnz)
+      PASTA_CUDA(cudaMemcpyAsync(x->inds[k].p, inds[k], nnz * sizeof(uint32_t), cudaMemcpyHostToDevice, s));
+  }
+  x->val.alloc(nnz, s);
+  if (nnz) PASTA_CUDA(cudaMemcpyAsync(x->val.p, vals, nnz * sizeof(float), cudaMemcpyHostToDevice, s));
+  PASTA_CUDA(cudaStreamSynchronize(s));
+  const uint32_t *ip[kMaxOrder];
+  for (uint32_t k = 0; k < order; ++k) ip[k] = x->inds[k].p;
+  x->lex_sorted = is_lex_sorted_device(ip, order, nnz, s);
+  return x;
+}
+
+namespace pasta {
+
+void coo_prepare_mode(pasta_coo *x, uint32_t mode, cudaStream_t s) {
+  CooModeCopy &mc = x->mc[mode];
+  if (mc.ready) return;
+  const uint32_t N = x->order;
+  const uint64_t M = x->nnz;
+  if (mode == 0 && x->lex_sorted) {  // canonical order already is the mode-0 order
+    for (uint32_t k = 0; k < N; ++k) mc.inds[k] = x->inds[k].p;
+    mc.val = x->val.p;
+    mc.ready = true;
+    return;
+  }
+  DevArray<uint32_t> perm(M, s);
+  iota_u32(perm.p, M, s);
+  const uint32_t *comps[kMaxOrder];
+  uint32_t bits[kMaxOrder];
+  for (uint32_t j = 0; j < N; ++j) {
+    uint32_t k = (mode + j) % N;
+    comps[j] = x->inds[k].p;
+    bits[j] = ceil_log2(x->dims[k]);
+  }
+  lexsort(comps, bits, int(N), perm, M, s);
+  for (uint32_t k = 0; k < N; ++k) {
+    mc.own_inds[k].alloc(M, s);
+    gather_u32(x->inds[k].p, perm.p, mc.own_inds[k].p, M, s);
+    mc.inds[k] = mc.own_inds[k].p;
+  }
+  mc.own_val.alloc(M, s);
+  gather_f32(x->val.p, perm.p, mc.own_val.p, M, s);
+  mc.val = mc.own_val.p;
+  PASTA_CUDA(cudaStreamSynchronize(s));
+  mc.ready = true;
+}
+
+}  // namespace pasta
+
+// ================================================================== extern "C" ABI ======
+extern "C" {
+
+const char *pasta_last_error(void) { return t_last_error.c_str(); }
+
+const char *pasta_version(void) { return "pasta-b200 0.1 sm_100a"; }
+
+pasta_status pasta_set_allocator(const pasta_allocator *alloc) {
+  API_BEGIN
+  std::lock_guard<std::mutex> lk(g_alloc_mu);
+  if (alloc) {
+    require(alloc->alloc && alloc->free, "allocator hook needs both alloc and free");
+    g_alloc = *alloc;
+    g_alloc_set = true;
+  } else {
+    g_alloc = pasta_allocator{nullptr, nullptr, nullptr};
+    g_alloc_set = false;
+  }
+  API_END
+}
+
+// ---------------------------------------------------------------------------- ingest
+pasta_status pasta_load_coo(const char *path, pasta_coo **out) {
+  API_BEGIN
+  require(path && out, "path/out is NULL");
+  *out = nullptr;
+  FILE *f = std::fopen(path, "rb");
+  if (!f) fail(PASTA_EIO, std::string("cannot open ") + path);
+  std::string text;
+  {
+    char buf[1 << 16];
+    size_t got;
+    while ((got = std::fread(buf, 1, sizeof(buf), f)) > 0) text.append(buf, got);
+    bool err = std::ferror(f);
+    std::fclose(f);
+    if (err) fail(PASTA_EIO, std::string("read error on ") + path);
+  }
+  std::vector<std::vector<uint32_t>> inds;
+  std::vector<float> vals;
+  uint32_t order = 0;
+  std::vector<uint32_t> dims;
+  size_t pos = 0, line_no = 0;
+  std::vector<std::string> tok;
+  while (pos < text.size()) {
+    size_t eol = text.find('\n', pos);
+    if (eol == std::string::npos) eol = text.size();
+    ++line_no;
+    const char *p = text.c_str() + pos, *end = text.c_str() + eol;
+    pos = eol + 1;
+    while (p < end && (*p == ' ' || *p == '\t' || *p == '\r')) ++p;
+    if (p == end || *p == '#') continue;
+    tok.clear();
+    while (p < end) {
+      const char *q = p;
+      while (q < end && *q != ' ' && *q != '\t' && *q != '\r') ++q;
+      tok.emplace_back(p, q);
+      p = q;
+      while (p < end && (*p == ' ' || *p == '\t' || *p == '\r')) ++p;
+    }
+    if (order == 0) {
+      if (tok.size() < 2 || tok.size() - 1 > kMaxOrder)
+        fail(PASTA_EFORMAT, "line " + std::to_string(line_no) + ": expected 2..9 tokens");
+      order = uint32_t(tok.size() - 1);
+      inds.resize(order);
+      dims.assign(order, 0);
+    }
+    if (tok.size() != order + 1)
+      fail(PASTA_EFORMAT, "line " + std::to_string(line_no) + ": ragged line");
+    for (uint32_t k = 0; k < order; ++k) {
+      errno = 0;
+      char *e = nullptr;
+      unsigned long long v = std::strtoull(tok[k].c_str(), &e, 10);
+      if (errno || !e || *e != '\0' || tok[k][0] == '-')
+        fail(PASTA_EFORMAT, "line " + std::to_string(line_no) + ": bad index '" + tok[k] + "'");
+      if (v == 0) fail(PASTA_EFORMAT, "line " + std::to_string(line_no) + ": indices are 1-based");
+      if (v > 0xFFFFFFFFull) fail(PASTA_ERANGE, "line " + std::to_string(line_no) + ": index too large");
+      inds[k].push_back(uint32_t(v - 1));
+      if (uint32_t(v) > dims[k]) dims[k] = uint32_t(v);
+    }
+    errno = 0;
+    char *e = nullptr;
+    float fv = std::strtof(tok[order].c_str(), &e);
+    if (!e || *e != '\0') fail(PASTA_EFORMAT, "line " + std::to_string(line_no) + ": bad value");
+    vals.push_back(fv);
+    if (vals.size() > 0xFFFFFFFEull) fail(PASTA_ERANGE, "more than 2^32-2 nonzeros");
+  }
+  if (order == 0) fail(PASTA_EFORMAT, std::string("no nonzeros in ") + path);
+  const uint32_t *ip[kMaxOrder];
+  for (uint32_t k = 0; k < order; ++k) ip[k] = inds[k].data();
+  auto x = coo_upload(order, dims.data(), vals.size(), ip, vals.data(), nullptr);
+  *out = x.release();
+  API_END
+}
+
+pasta_status pasta_save_coo(const pasta_coo *x, const char *path) {
+  API_BEGIN
+  require(x && path, "x/path is NULL");
+  check_device(x->device);
+  std::vector<std::vector<uint32_t>> h(x->order, std::vector<uint32_t>(x->nnz));
+  std::vector<float> v(x->nnz);
+  for (uint32_t k = 0; k < x->order; ++k)
+    if (x->nnz) PASTA_CUDA(cudaMemcpy(h[k].data(), x->inds[k].p, x->nnz * 4, cudaMemcpyDeviceToHost));
+  if (x->nnz) PASTA_CUDA(cudaMemcpy(v.data(), x->val.p, x->nnz * 4, cudaMemcpyDeviceToHost));
+  FILE *f = std::fopen(path, "wb");
+  if (!f) fail(PASTA_EIO, std::string("cannot create ") + path);
+  bool ok = true;
+  for (uint64_t i = 0; i < x->nnz && ok; ++i) {
+    for (uint32_t k = 0; k < x->order; ++k) ok &= std::fprintf(f, "%u ", h[k][i] + 1) > 0;
+    ok &= std::fprintf(f, "%.9g\n", double(v[i])) > 0;
+  }
+  ok &= std::fclose(f) == 0;
+  if (!ok) fail(PASTA_EIO, std::string("write error on ") + path);
+  API_END
+}
+
+pasta_status pasta_coo_from_arrays(uint32_t order, const uint32_t *dims, uint64_t nnz,
+                                   const uint32_t *const *inds, const float *vals, pasta_coo **out) {
+  API_BEGIN
+  require(out != nullptr, "out is NULL");
+  *out = nullptr;
+  validate_dims(order, dims);
+  require(nnz == 0 || (inds && vals), "inds/vals is NULL");
+  if (nnz > 0xFFFFFFFEull) fail(PASTA_ERANGE, "more than 2^32-2 nonzeros");
+  for (uint32_t k = 0; k < order && nnz; ++k) {
+    require(inds[k] != nullptr, "inds[k] is NULL");
+    for (uint64_t i = 0; i < nnz; ++i)
+      if (inds[k][i] >= dims[k])
+        fail(PASTA_ERANGE, "index " + std::to_string(inds[k][i]) + " >= dims[" + std::to_string(k) + "]");
+  }
+  auto x = coo_upload(order, dims, nnz, inds, vals, nullptr);
+  *out = x.release();
+  API_END
+}
+
+pasta_status pasta_gen_powerlaw(uint32_t order, const uint32_t *dims, uint64_t nnz, uint64_t seed,
+                                const pasta_gen_params *params, pasta_coo **out) {
+  API_BEGIN
+  require(out != nullptr, "out is NULL");
+  *out = nullptr;
+  validate_dims(order, dims);
+  pasta_gen_params p{1, nullptr, 0.0, 0, 0.f, 0.f};
+  if (params) p = *params;
+  if (p.kind == 2) fail(PASTA_EUNSUPPORTED, "FireHose slice power-law generator (kind 2) is not implemented");
+  require(p.kind <= 1, "unknown generator kind");
+  if (p.permute) fail(PASTA_EUNSUPPORTED, "label permutation is not implemented");
+  double cells = 1.0;
+  for (uint32_t k = 0; k < order; ++k) cells *= double(dims[k]);
+  require(double(nnz) <= cells, "nnz exceeds the number of cells");
+  if (nnz > 0xFFFFFFFEull) fail(PASTA_ERANGE, "more than 2^32-2 nonzeros");
+  const uint32_t ncell = 1u << order;
+  double table[1 << kMaxOrder];
+  if (p.kind == 0) {
+    for (uint32_t c = 0; c < ncell; ++c) {
+      double v = 1.0;
+      for (uint32_t k = 0; k < order; ++k) v = v * 0.5;
+      table[c] = v;
+    }
+  } else if (p.initiator) {
+    double sum = 0.0;
+    for (uint32_t c = 0; c < ncell; ++c) {
+      require(p.initiator[c] >= 0.0 && std::isfinite(p.initiator[c]), "initiator weights must be >= 0");
+      table[c] = p.initiator[c];
+      sum += table[c];
+    }
+    require(sum > 0.0, "initiator weights sum to zero");
+  } else {
+    double q = (p.q > 0.0 && p.q < 1.0) ? p.q : 0.75;
+    require(p.q == 0.0 || (p.q > 0.0 && p.q < 1.0), "q must be in (0, 1)");
+    for (uint32_t c = 0; c < ncell; ++c) {
+      double v = 1.0;
+      for (uint32_t k = 0; k < order; ++k) v = v * (((c >> k) & 1u) ? (1.0 - q) : q);
+      table[c] = v;
+    }
+  }
+  float lo = p.val_lo, hi = p.val_hi;
+  if (lo == 0.f && hi == 0.f) { lo = -1.f; hi = 1.f; }
+  require(lo < hi, "val_lo must be < val_hi");
+  auto x = std::make_unique<pasta_coo>();
+  x->order = order;
+  for (uint32_t k = 0; k < order; ++k) x->dims[k] = dims[k];
+  x->nnz = nnz;
+  x->device = current_device();
+  gen_powerlaw_device(x.get(), seed, table, ncell, lo, hi, nullptr);
+  x->lex_sorted = true;
+  *out = x.release();
+  API_END
+}
+
+// ---------------------------------------------------------------------------- formats
+pasta_status pasta_coo_to_hicoo(const pasta_coo *x, uint32_t block_bits, pasta_hicoo **out) {
+  API_BEGIN
+  require(x && out, "x/out is NULL");
+  *out = nullptr;
+  require(block_bits >= 1 && block_bits <= 8, "block_bits must be in 1..8 (8-bit element indices, P:181)");
+  check_device(x->device);
+  auto h = std::make_unique<pasta_hicoo>();
+  h->order = x->order;
+  for (uint32_t k = 0; k < x->order; ++k) h->dims[k] = x->dims[k];
+  h->block_bits = block_bits;
+  h->device = x->device;
+  coo_to_hicoo_device(x, h.get(), nullptr);
+  *out = h.release();
+  API_END
+}
+
+pasta_status pasta_coo_prepare(pasta_coo *x, uint32_t mode, void *stream) {
+  API_BEGIN
+  require(x != nullptr, "x is NULL");
+  require(mode < x->order, "mode >= order");
+  check_device(x->device);
+  std::lock_guard<std::mutex> lk(x->mu);
+  coo_prepare_mode(x, mode, as_stream(stream));
+  API_END
+}
+
+pasta_status pasta_hicoo_prepare(pasta_hicoo *h, uint32_t mode, void *stream) {
+  API_BEGIN
+  require(h != nullptr, "h is NULL");
+  require(mode < h->order, "mode >= order");
+  check_device(h->device);
+  std::lock_guard<std::mutex> lk(h->mu);
+  hicoo_prepare_mode(h, mode, as_stream(stream));
+  API_END
+}
+
+// ---------------------------------------------------------------------------- MTTKRP
+static void validate_mttkrp(uint32_t order, uint32_t mode, const float *const *factors, uint32_t R,
+                            const float *out) {
+  require(mode < order, "mode >= order");
+  require(R >= 1, "R must be >= 1");
+  require(factors != nullptr, "factors is NULL");
+  require(out != nullptr, "out is NULL");
+  for (uint32_t k = 0; k < order; ++k)
+    if (k != mode) require(factors[k] != nullptr, "factors[k] is NULL for a mode k != mode");
+}
+
+pasta_status pasta_mttkrp_coo(pasta_coo *x, uint32_t mode, const float *const *factors, uint32_t R,
+                              float *out, void *stream) {
+  API_BEGIN
+  require(x != nullptr, "x is NULL");
+  validate_mttkrp(x->order, mode, factors, R, out);
+  check_device(x->device);
+  cudaStream_t s = as_stream(stream);
+  if (!x->mc[mode].ready) {
+    std::lock_guard<std::mutex> lk(x->mu);
+    coo_prepare_mode(x, mode, s);
+  }
+  uint64_t lo = 0, hi = x->dims[mode];
+  if (x->shard_mode == int(mode)) { lo = x->row_lo; hi = x->row_hi; }
+  launch_zero_rows(out, lo, hi, R, s);
+  launch_coo_mttkrp(x, mode, factors, R, out, s);
+  API_END
+}
+
+pasta_status pasta_mttkrp_hicoo(pasta_hicoo *h, uint32_t mode, const float *const *factors, uint32_t R,
+                                float *out, void *stream) {
+  API_BEGIN
+  require(h != nullptr, "h is NULL");
+  validate_mttkrp(h->order, mode, factors, R, out);
+  check_device(h->device);
+  cudaStream_t s = as_stream(stream);
+  if (!h->mc[mode].ready) {
+    std::lock_guard<std::mutex> lk(h->mu);
+    hicoo_prepare_mode(h, mode, s);
+  }
+  launch_zero_rows(out, 0, h->dims[mode], R, s);
+  launch_hicoo_mttkrp(h, mode, factors, R, out, s);
+  API_END
+}
+
+pasta_status pasta_mttkrp_coo_allmodes_host(pasta_coo *x, const float *const *host_factors, uint32_t R,
+                                            float *const *host_out, void *stream) {
+  API_BEGIN
+  require(x && host_factors && host_out, "x/host_factors/host_out is NULL");
+  require(R >= 1, "R must be >= 1");
+  for (uint32_t k = 0; k < x->order; ++k)
+    require(host_factors[k] && host_out[k], "host_factors[k]/host_out[k] is NULL");
+  check_device(x->device);
+  cudaStream_t s = as_stream(stream);
+  std::lock_guard<std::mutex> lk(x->mu);
+  for (uint32_t k = 0; k < x->order; ++k) coo_prepare_mode(x, k, s);
+  if (x->stage_R != R) {
+    for (uint32_t k = 0; k < x->order; ++k) {
+      x->stage_f[k].alloc(uint64_t(x->dims[k]) * R, s);
+      x->stage_o[k].alloc(uint64_t(x->dims[k]) * R, s);
+    }
+    x->stage_R = R;
+  }
+  const float *dfac[kMaxOrder];
+  for (uint32_t k = 0; k < x->order; ++k) {
+    PASTA_CUDA(cudaMemcpyAsync(x->stage_f[k].p, host_factors[k], uint64_t(x->dims[k]) * R * sizeof(float),
+                               cudaMemcpyHostToDevice, s));
+    dfac[k] = x->stage_f[k].p;
+  }
+  for (uint32_t m = 0; m < x->order; ++m) {
+    uint64_t lo = 0, hi = x->dims[m];
+    if (x->shard_mode == int(m)) { lo = x->row_lo; hi = x->row_hi; }
+    launch_zero_rows(x->stage_o[m].p, lo, hi, R, s);
+    launch_coo_mttkrp(x, m, dfac, R, x->stage_o[m].p, s);
+    PASTA_CUDA(cudaMemcpyAsync(host_out[m], x->stage_o[m].p, uint64_t(x->dims[m]) * R * sizeof(float),
+                               cudaMemcpyDeviceToHost, s));
+  }
+  PASTA_CUDA(cudaStreamSynchronize(s));
+  API_END
+}
+
+// ---------------------------------------------------------------------------- multi-GPU
+pasta_status pasta_coo_row_counts(const pasta_coo *x, uint32_t mode, uint64_t *counts) {
+  API_BEGIN
+  require(x && counts, "x/counts is NULL");
+  require(mode < x->order, "mode >= order");
+  check_device(x->device);
+  row_counts_device(x->inds[mode].p, x->nnz, x->dims[mode], counts, nullptr);
+  API_END
+}
+
+pasta_status pasta_row_partition(uint32_t nrows, const uint64_t *counts, uint32_t nparts,
+                                 uint32_t *bounds) {
+  API_BEGIN
+  require(nparts >= 1, "nparts must be >= 1");
+  require(bounds != nullptr && (nrows == 0 || counts != nullptr), "counts/bounds is NULL");
+  // S(r) = sum_{i<r} counts[i];  bounds[p] = min{r : S(r) * nparts >= p * T}
+  unsigned __int128 T = 0;
+  for (uint32_t r = 0; r < nrows; ++r) T += counts[r];
+  bounds[0] = 0;
+  uint32_t p = 1;
+  unsigned __int128 S = 0;
+  for (uint32_t r = 0; r <= nrows && p < nparts; ++r) {
+    while (p < nparts && S * nparts >= T * p) bounds[p++] = r;
+    if (r < nrows) S += counts[r];
+  }
+  while (p < nparts) bounds[p++] = nrows;
+  bounds[nparts] = nrows;
+  API_END
+}
+
+pasta_status pasta_coo_partition(const pasta_coo *x, uint32_t mode, uint32_t nparts, uint32_t *bounds) {
+  API_BEGIN
+  require(x && bounds, "x/bounds is NULL");
+  require(mode < x->order, "mode >= order");
+  std::vector<uint64_t> counts(x->dims[mode]);
+  pasta_status st = pasta_coo_row_counts(x, mode, counts.data());
+  if (st != PASTA_OK) fail(st, t_last_error);
+  st = pasta_row_partition(x->dims[mode], counts.data(), nparts, bounds);
+  if (st != PASTA_OK) fail(st, t_last_error);
+  API_END
+}
+
+pasta_status pasta_coo_shard(pasta_coo *x, uint32_t mode, uint32_t row_lo, uint32_t row_hi,
+                             pasta_coo **out) {
+  API_BEGIN
+  require(x && out, "x/out is NULL");
+  *out = nullptr;
+  require(mode < x->order, "mode >= order");
+  require(row_lo <= row_hi && row_hi <= x->dims[mode], "need row_lo <= row_hi <= dims[mode]");
+  check_device(x->device);
+  cudaStream_t s = nullptr;
+  {
+    std::lock_guard<std::mutex> lk(x->mu);
+    coo_prepare_mode(x, mode, s);
+  }
+  const CooModeCopy &mc = x->mc[mode];
+  uint64_t a = lower_bound_device(mc.inds[mode], x->nnz, row_lo, s);
+  uint64_t b = row_hi >= x->dims[mode] ? x->nnz : lower_bound_device(mc.inds[mode], x->nnz, row_hi, s);
+  auto y = std::make_unique<pasta_coo>();
+  y->order = x->order;
+  for (uint32_t k = 0; k < x->order; ++k) y->dims[k] = x->dims[k];
+  y->nnz = b - a;
+  y->device = x->device;
+  for (uint32_t k = 0; k < x->order; ++k) {
+    y->inds[k].alloc(y->nnz, s);
+    if (y->nnz)
+      PASTA_CUDA(cudaMemcpyAsync(y->inds[k].p, mc.inds[k] + a, y->nnz * 4, cudaMemcpyDeviceToDevice, s));
+  }
+  y->val.alloc(y->nnz, s);
+  if (y->nnz) PASTA_CUDA(cudaMemcpyAsync(y->val.p, mc.val + a, y->nnz * 4, cudaMemcpyDeviceToDevice, s));
+  PASTA_CUDA(cudaStreamSynchronize(s));
+  y->lex_sorted = (mode == 0) ? true : false;
+  CooModeCopy &ym = y->mc[mode];
+  for (uint32_t k = 0; k < y->order; ++k) ym.inds[k] = y->inds[k].p;
+  ym.val = y->val.p;
+  ym.ready = true;
+  y->shard_mode = int(mode);
+  y->row_lo = row_lo;
+  y->row_hi = row_hi;
+  *out = y.release();
+  API_END
+}
+
+// ---------------------------------------------------------------------------- introspection
+pasta_status pasta_coo_info(const pasta_coo *x, uint32_t *order, uint32_t *dims, uint64_t *nnz) {
+  API_BEGIN
+  require(x != nullptr, "x is NULL");
+  if (order) *order = x->order;
+  if (dims)
+    for (uint32_t k = 0; k < x->order; ++k) dims[k] = x->dims[k];
+  if (nnz) *nnz = x->nnz;
+  API_END
+}
+
+static void export_arrays(uint32_t order, uint64_t nnz, const uint32_t *const *dinds, const float *dval,
+                          uint32_t *const *inds, float *vals) {
+  for (uint32_t k = 0; k < order; ++k) {
+    require(!inds || inds[k] || !nnz, "inds[k] is NULL");
+    if (inds && inds[k] && nnz)
+      PASTA_CUDA(cudaMemcpy(inds[k], dinds[k], nnz * sizeof(uint32_t), cudaMemcpyDeviceToHost));
+  }
+  if (vals && nnz) PASTA_CUDA(cudaMemcpy(vals, dval, nnz * sizeof(float), cudaMemcpyDeviceToHost));
+}
+
+pasta_status pasta_coo_export(const pasta_coo *x, uint32_t *const *inds, float *vals) {
+  API_BEGIN
+  require(x != nullptr, "x is NULL");
+  check_device(x->device);
+  const uint32_t *di[kMaxOrder];
+  for (uint32_t k = 0; k < x->order; ++k) di[k] = x->inds[k].p;
+  export_arrays(x->order, x->nnz, di, x->val.p, inds, vals);
+  API_END
+}
+
+pasta_status pasta_coo_export_mode(pasta_coo *x, uint32_t mode, uint32_t *const *inds, float *vals) {
+  API_BEGIN
+  require(x != nullptr, "x is NULL");
+  require(mode < x->order, "mode >= order");
+  check_device(x->device);
+  {
+    std::lock_guard<std::mutex> lk(x->mu);
+    coo_prepare_mode(x, mode, nullptr);
+  }
+  export_arrays(x->order, x->nnz, x->mc[mode].inds, x->mc[mode].val, inds, vals);
+  API_END
+}
+
+pasta_status pasta_hicoo_info(const pasta_hicoo *h, uint32_t *order, uint32_t *dims, uint32_t *block_bits,
+                              uint64_t *nblocks, uint64_t *nnz) {
+  API_BEGIN
+  require(h != nullptr, "h is NULL");
+  if (order) *order = h->order;
+  if (dims)
+    for (uint32_t k = 0; k < h->order; ++k) dims[k] = h->dims[k];
+  if (block_bits) *block_bits = h->block_bits;
+  if (nblocks) *nblocks = h->nblocks;
+  if (nnz) *nnz = h->nnz;
+  API_END
+}
+
+pasta_status pasta_hicoo_export(const pasta_hicoo *h, uint64_t *bptr, uint32_t *const *binds,
+                                uint8_t *const *einds, float *vals) {
+  API_BEGIN
+  require(h != nullptr, "h is NULL");
+  check_device(h->device);
+  if (bptr) PASTA_CUDA(cudaMemcpy(bptr, h->bptr.p, (h->nblocks + 1) * 8, cudaMemcpyDeviceToHost));
+  for (uint32_t k = 0; k < h->order; ++k) {
+    if (binds && binds[k] && h->nblocks)
+      PASTA_CUDA(cudaMemcpy(binds[k], h->binds[k].p, h->nblocks * 4, cudaMemcpyDeviceToHost));
+    if (einds && einds[k] && h->nnz)
+      PASTA_CUDA(cudaMemcpy(einds[k], h->einds[k].p, h->nnz, cudaMemcpyDeviceToHost));
+  }
+  if (vals && h->nnz) PASTA_CUDA(cudaMemcpy(vals, h->val.p, h->nnz * 4, cudaMemcpyDeviceToHost));
+  API_END
+}
+
+void pasta_coo_free(pasta_coo *x) { delete x; }
+void pasta_hicoo_free(pasta_hicoo *h) { delete h; }
+
+// ---------------------------------------------------------------------------- measurement
+uint64_t pasta_launch_count(void) { return g_launches.load(); }
+
+pasta_status pasta_profile_enable(int on) {
+  API_BEGIN
+  g_prof_on.store(on != 0);
+  API_END
+}
+
+pasta_status pasta_profile_read(uint32_t which, double *total_ms, uint64_t *launches, int reset) {
+  API_BEGIN
+  require(which < kProfKinds, "which must be 0 (COO), 1 (HiCOO) or 2 (zero-fill)");
+  std::lock_guard<std::mutex> lk(g_prof_mu);
+  double sum = 0.0;
+  for (auto &r : g_prof[which]) {
+    PASTA_CUDA(cudaEventSynchronize(r.b));
+    float ms = 0.f;
+    PASTA_CUDA(cudaEventElapsedTime(&ms, r.a, r.b));
+    sum += ms;
+  }
+  if (total_ms) *total_ms = sum;
+  if (launches) *launches = g_prof[which].size();
+  if (reset) {
+    for (auto &r : g_prof[which]) {
+      cudaEventDestroy(r.a);
+      cudaEventDestroy(r.b);
+    }
+    g_prof[which].clear();
+  }
+  API_END
+}
+
+}  // extern "C"

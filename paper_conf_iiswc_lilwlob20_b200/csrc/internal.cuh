@@ -1,0 +1,186 @@
+// internal.cuh -- shared internals of libpasta (never installed; not part of the ABI).
+// Citations: P:N = line N of the paper text; R#k = DESIGN.md reading k.
+#pragma once
+
+#include <cuda_runtime.h>
+
+#include <atomic>
+#include <cstdint>
+#include <cstring>
+#include <mutex>
+#include <string>
+#include <utility>
+#include <vector>
+
+#include "../../include/pasta.h"
+
+namespace pasta {
+
+constexpr int kMaxOrder = PASTA_MAX_ORDER;
+
+// ----------------------------------------------------------------------------- errors
+struct Error {
+  pasta_status code;
+  std::string msg;
+};
+[[noreturn]] inline void fail(pasta_status code, const std::string &msg) { throw Error{code, msg}; }
+void set_last_error(pasta_status code, const std::string &msg);
+
+#define PASTA_CUDA(expr)                                                                  \
+  do {                                                                                    \
+    cudaError_t _e = (expr);                                                              \
+    if (_e != cudaSuccess)                                                                \
+      ::pasta::fail(PASTA_ECUDA, std::string(#expr) + ": " + cudaGetErrorString(_e));     \
+  } while (0)
+
+#define PASTA_LAUNCHED()                                                                  \
+  do {                                                                                    \
+    ::pasta::count_launch();                                                              \
+    cudaError_t _e = cudaGetLastError();                                                  \
+    if (_e != cudaSuccess)                                                                \
+      ::pasta::fail(PASTA_ECUDA, std::string("kernel launch: ") + cudaGetErrorString(_e)); \
+  } while (0)
+
+void count_launch();
+
+// ----------------------------------------------------------------------------- memory
+void *dev_alloc(size_t bytes, cudaStream_t s);
+void dev_free(void *p, cudaStream_t s);
+
+// Owning device array (allocated through the allocator hook, else cudaMalloc).
+template <class T>
+struct DevArray {
+  T *p = nullptr;
+  size_t n = 0;
+  DevArray() = default;
+  explicit DevArray(size_t count, cudaStream_t s = nullptr) { alloc(count, s); }
+  DevArray(const DevArray &) = delete;
+  DevArray &operator=(const DevArray &) = delete;
+  DevArray(DevArray &&o) noexcept : p(o.p), n(o.n) { o.p = nullptr; o.n = 0; }
+  DevArray &operator=(DevArray &&o) noexcept {
+    if (this != &o) { reset(); p = o.p; n = o.n; o.p = nullptr; o.n = 0; }
+    return *this;
+  }
+  ~DevArray() { reset(); }
+  void alloc(size_t count, cudaStream_t s = nullptr) {
+    reset();
+    n = count;
+    p = static_cast<T *>(dev_alloc((count ? count : 1) * sizeof(T), s));
+  }
+  void reset() {
+    if (p) dev_free(p, nullptr);
+    p = nullptr;
+    n = 0;
+  }
+  T *get() const { return p; }
+  size_t bytes() const { return n * sizeof(T); }
+};
+
+// ----------------------------------------------------------------------------- handles
+struct CooModeCopy {
+  bool ready = false;
+  const uint32_t *inds[kMaxOrder] = {};  // sorted by (i_mode, i_mode+1, ...), may alias canon
+  const float *val = nullptr;
+  DevArray<uint32_t> own_inds[kMaxOrder];
+  DevArray<float> own_val;
+};
+
+struct HicooModeCopy {
+  bool ready = false;
+  DevArray<uint64_t> bptr;               // nblocks + 1
+  DevArray<uint32_t> binds[kMaxOrder];   // nblocks each
+  DevArray<uint8_t> einds[kMaxOrder];    // nnz each
+  DevArray<float> val;                   // nnz
+};
+
+}  // namespace pasta
+
+struct pasta_coo {
+  uint32_t order = 0;
+  uint32_t dims[pasta::kMaxOrder] = {};
+  uint64_t nnz = 0;
+  int device = 0;
+  bool lex_sorted = false;  // canonical order == mode-0 lexicographic order
+  pasta::DevArray<uint32_t> inds[pasta::kMaxOrder];
+  pasta::DevArray<float> val;
+  pasta::CooModeCopy mc[pasta::kMaxOrder];
+  int shard_mode = -1;  // >= 0: this handle is the [row_lo, row_hi) shard of that mode
+  uint32_t row_lo = 0, row_hi = 0;
+  // e2e staging (pasta_mttkrp_coo_allmodes_host)
+  uint32_t stage_R = 0;
+  pasta::DevArray<float> stage_f[pasta::kMaxOrder];
+  pasta::DevArray<float> stage_o[pasta::kMaxOrder];
+  std::mutex mu;
+};
+
+struct pasta_hicoo {
+  uint32_t order = 0;
+  uint32_t dims[pasta::kMaxOrder] = {};
+  uint32_t block_bits = 7;
+  uint64_t nblocks = 0;
+  uint64_t nnz = 0;
+  int device = 0;
+  pasta::DevArray<uint64_t> bptr;
+  pasta::DevArray<uint32_t> binds[pasta::kMaxOrder];
+  pasta::DevArray<uint8_t> einds[pasta::kMaxOrder];
+  pasta::DevArray<float> val;
+  pasta::HicooModeCopy mc[pasta::kMaxOrder];
+  std::mutex mu;
+};
+
+namespace pasta {
+
+inline uint32_t ceil_log2(uint64_t v) {
+  uint32_t l = 0;
+  while (l < 64 && (uint64_t(1) << l) < v) ++l;
+  return l;
+}
+
+// ------------------------------------------------------------------------- sort helpers
+// Stable lexicographic sort of the permutation `perm` (length M, initialised by the
+// caller) by device u32 component arrays comps[0] (most significant) .. comps[nc-1],
+// where comps[c] has bits[c] significant bits.  Indexing: key of position x is
+// comps[c][perm[x]].  Implemented as LSD passes of CUB radix sort over 64-bit packed keys.
+void lexsort(const uint32_t *const *comps, const uint32_t *bits, int nc, DevArray<uint32_t> &perm,
+             uint64_t M, cudaStream_t s);
+// Morton-order sort (R#13) of the coordinate arrays `inds` (order N): stable, by the
+// level-major interleave of Lm-bit coordinates.  perm initialised by the caller.
+void morton_sort(const uint32_t *const *inds, uint32_t order, uint32_t Lm, DevArray<uint32_t> &perm,
+                 uint64_t M, cudaStream_t s);
+// out[x] = in[perm[x]]
+void gather_u32(const uint32_t *in, const uint32_t *perm, uint32_t *out, uint64_t M, cudaStream_t s);
+void gather_f32(const float *in, const uint32_t *perm, float *out, uint64_t M, cudaStream_t s);
+void gather_u8(const uint8_t *in, const uint32_t *perm, uint8_t *out, uint64_t M, cudaStream_t s);
+void iota_u32(uint32_t *p, uint64_t M, cudaStream_t s);
+// idx_out[0..count) = positions x < M with flags[x] != 0, ascending.  Returns count.
+uint64_t select_flagged(const uint8_t *flags, uint64_t M, DevArray<uint32_t> &idx_out, cudaStream_t s);
+
+// ------------------------------------------------------------------------- operations
+void coo_prepare_mode(pasta_coo *x, uint32_t mode, cudaStream_t s);
+void hicoo_prepare_mode(pasta_hicoo *h, uint32_t mode, cudaStream_t s);
+void gen_powerlaw_device(pasta_coo *x, uint64_t seed, const double *table, uint32_t ncell,
+                         float val_lo, float val_hi, cudaStream_t s);
+void coo_to_hicoo_device(const pasta_coo *x, pasta_hicoo *h, cudaStream_t s);
+
+void launch_zero_rows(float *out, uint64_t row_lo, uint64_t row_hi, uint32_t R, cudaStream_t s);
+void launch_coo_mttkrp(const pasta_coo *x, uint32_t mode, const float *const *factors, uint32_t R,
+                       float *out, cudaStream_t s);
+void launch_hicoo_mttkrp(const pasta_hicoo *h, uint32_t mode, const float *const *factors,
+                         uint32_t R, float *out, cudaStream_t s);
+void row_counts_device(const uint32_t *rows, uint64_t nnz, uint32_t nrows, uint64_t *counts_host,
+                       cudaStream_t s);
+// first position x in the sorted array a[0..M) with a[x] >= v (device binary search).
+uint64_t lower_bound_device(const uint32_t *a, uint64_t M, uint32_t v, cudaStream_t s);
+bool is_lex_sorted_device(const uint32_t *const *inds, uint32_t order, uint64_t M, cudaStream_t s);
+
+// ------------------------------------------------------------------------- profiling
+enum ProfKind { kProfCoo = 0, kProfHicoo = 1, kProfZero = 2, kProfKinds = 3 };
+struct ProfScope {
+  cudaEvent_t a = nullptr, b = nullptr;
+  int kind;
+  cudaStream_t s;
+  ProfScope(int kind, cudaStream_t s);
+  ~ProfScope();
+};
+
+}  // namespace pasta

@@ -1,0 +1,417 @@
+// mttkrp.cu -- sm_100a MTTKRP kernels on COO (a6) and HiCOO (a7), and the output zero-fill (a5).
+//
+// What is computed (Eq. 3; Eq. 4; folded into the nonzero loop):
+//     out(i_n(x), r) += val(x) * prod_{k != n} U^(k)(i_k(x), r)
+//
+// Design (B200-first, not the paper's P100/V100 kernels):
+//   * Input is the mode-n working copy: nonzeros sorted so equal output rows are contiguous
+//     (COO: lexicographic from mode n; HiCOO: blocks by binds_n, entries by einds_n, R#27).
+//   * A warp owns a contiguous chunk of nonzeros; its 32 lanes form G = 32/LPN groups of LPN
+//     lanes.  Group g walks a contiguous run of S = chunk/G nonzeros; within the group each
+//     lane owns VW (=4 -> one 128-bit LDG) consecutive columns r of every factor row, so one
+//     group-load fetches a whole 4R-byte row (64 B at R = 16) -- the coalescing direction the
+//     paper's 2-D blocks use (x = R).
+//   * Index/value streams: 128-bit vector loads (4 nonzeros per load per array, COO) or
+//     32-bit loads of 4 packed 8-bit element indices (HiCOO).
+//   * All U gathers of an unrolled step are issued before any is consumed (memory-level
+//     parallelism is the whole game for this gather-bound kernel).
+//   * Rank-R partial sums stay in registers while the output row does not change
+//     (segmented reduction over runs of equal i_n).  A finished segment that began and
+//     ended inside the run is owned by this group alone -> plain 128-bit store; the first
+//     and last segment of a run may be shared with neighbours -> red.global.add.v4.f32
+//     (one vector atomic per boundary, not per nonzero, cf. P:157/P:282 atomics).
+//   * No tensor cores: the path is a gather/scatter, not a dense contraction.
+#include "internal.cuh"
+
+namespace pasta {
+
+namespace {
+
+constexpr int kWarpsPerCta = 8;
+constexpr int kThreads = kWarpsPerCta * 32;
+
+struct KArgs {
+  uint64_t nnz;
+  uint64_t chunk;  // nonzeros per warp; chunk % (4 * G) == 0
+  uint32_t order, R;
+  // COO streams (mode-n copy)
+  const uint32_t *irow;                 // i_n
+  const uint32_t *io[kMaxOrder - 1];    // i_k, k != n, ascending k
+  const float *val;
+  // HiCOO streams (mode-n copy)
+  const uint64_t *bptr;
+  uint64_t nblocks;
+  const uint32_t *brow;
+  const uint32_t *bo[kMaxOrder - 1];
+  const uint8_t *erow;
+  const uint8_t *eo[kMaxOrder - 1];
+  uint32_t bbits;
+  // factors of the other modes (ascending k), output
+  const float *Uo[kMaxOrder - 1];
+  float *out;
+};
+
+template <int VW>
+struct Vec {
+  float v[VW];
+};
+
+template <int VW>
+__device__ __forceinline__ Vec<VW> ldg_vec(const float *p) {
+  Vec<VW> r;
+  if constexpr (VW == 4) {
+    float4 t = __ldg(reinterpret_cast<const float4 *>(p));
+    r.v[0] = t.x; r.v[1] = t.y; r.v[2] = t.z; r.v[3] = t.w;
+  } else {
+#pragma unroll
+    for (int i = 0; i < VW; ++i) r.v[i] = __ldg(p + i);
+  }
+  return r;
+}
+
+template <int VW>
+__device__ __forceinline__ void red_vec(float *p, const Vec<VW> &a) {
+  if constexpr (VW == 4) {
+    asm volatile("red.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(p), "f"(a.v[0]), "f"(a.v[1]),
+                 "f"(a.v[2]), "f"(a.v[3])
+                 : "memory");
+  } else {
+#pragma unroll
+    for (int i = 0; i < VW; ++i) atomicAdd(p + i, a.v[i]);
+  }
+}
+
+template <int VW>
+__device__ __forceinline__ void st_vec(float *p, const Vec<VW> &a) {
+  if constexpr (VW == 4) {
+    *reinterpret_cast<float4 *>(p) = make_float4(a.v[0], a.v[1], a.v[2], a.v[3]);
+  } else {
+#pragma unroll
+    for (int i = 0; i < VW; ++i) p[i] = a.v[i];
+  }
+}
+
+// Index source policies --------------------------------------------------------------------
+// load(x, cnt, row[], idx[][], v[]) fills U entries starting at x (cnt valid, x % 4 == 0).
+
+template <int NO, int U>
+struct CooSrc {
+  // rows are globally sorted: a segment strictly inside a run is owned by that run
+  static constexpr bool kSortedRows = true;
+  __device__ __forceinline__ void init(const KArgs &, uint64_t) {}
+  __device__ __forceinline__ void load(const KArgs &a, uint64_t x, int cnt, uint32_t (&row)[U],
+                                       uint32_t (&idx)[NO > 0 ? NO : kMaxOrder - 1][U], float (&v)[U], int no) {
+    if (cnt == U) {
+#pragma unroll
+      for (int q = 0; q < U; q += 4) {
+        uint4 r4 = __ldg(reinterpret_cast<const uint4 *>(a.irow + x + q));
+        row[q] = r4.x; row[q + 1] = r4.y; row[q + 2] = r4.z; row[q + 3] = r4.w;
+        float4 v4 = __ldg(reinterpret_cast<const float4 *>(a.val + x + q));
+        v[q] = v4.x; v[q + 1] = v4.y; v[q + 2] = v4.z; v[q + 3] = v4.w;
+#pragma unroll
+        for (int j = 0; j < (NO > 0 ? NO : kMaxOrder - 1); ++j) {
+          if (j < no) {
+            uint4 i4 = __ldg(reinterpret_cast<const uint4 *>(a.io[j] + x + q));
+            idx[j][q] = i4.x; idx[j][q + 1] = i4.y; idx[j][q + 2] = i4.z; idx[j][q + 3] = i4.w;
+          }
+        }
+      }
+    } else {
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        if (u < cnt) {
+          row[u] = __ldg(a.irow + x + u);
+          v[u] = __ldg(a.val + x + u);
+#pragma unroll
+          for (int j = 0; j < (NO > 0 ? NO : kMaxOrder - 1); ++j)
+            if (j < no) idx[j][u] = __ldg(a.io[j] + x + u);
+        }
+      }
+    }
+  }
+};
+
+template <int NO, int U>
+struct HicooSrc {
+  // rows repeat across blocks of one block row (R#27): every flush is an atomic
+  static constexpr bool kSortedRows = false;
+  uint64_t b, bend;
+  uint32_t base_row;
+  uint32_t base[NO > 0 ? NO : kMaxOrder - 1];
+  int no;
+  __device__ __forceinline__ void set_block(const KArgs &a) {
+    bend = __ldg(a.bptr + b + 1);
+    base_row = __ldg(a.brow + b) << a.bbits;
+#pragma unroll
+    for (int j = 0; j < (NO > 0 ? NO : kMaxOrder - 1); ++j)
+      if (j < no) base[j] = __ldg(a.bo[j] + b) << a.bbits;
+  }
+  __device__ __forceinline__ void init(const KArgs &a, uint64_t x0) {
+    no = int(a.order) - 1;
+    uint64_t lo = 0, hi = a.nblocks;  // last block with bptr[b] <= x0
+    while (hi - lo > 1) {
+      uint64_t mid = (lo + hi) / 2;
+      if (__ldg(a.bptr + mid) <= x0) lo = mid; else hi = mid;
+    }
+    b = lo;
+    set_block(a);
+  }
+  __device__ __forceinline__ void load(const KArgs &a, uint64_t x, int cnt, uint32_t (&row)[U],
+                                       uint32_t (&idx)[NO > 0 ? NO : kMaxOrder - 1][U], float (&v)[U], int) {
+    uint32_t er[U], ej[NO > 0 ? NO : kMaxOrder - 1][U];
+    if (cnt == U) {
+#pragma unroll
+      for (int q = 0; q < U; q += 4) {
+        uint32_t w = __ldg(reinterpret_cast<const uint32_t *>(a.erow + x + q));
+        er[q] = w & 0xff; er[q + 1] = (w >> 8) & 0xff; er[q + 2] = (w >> 16) & 0xff; er[q + 3] = w >> 24;
+        float4 v4 = __ldg(reinterpret_cast<const float4 *>(a.val + x + q));
+        v[q] = v4.x; v[q + 1] = v4.y; v[q + 2] = v4.z; v[q + 3] = v4.w;
+#pragma unroll
+        for (int j = 0; j < (NO > 0 ? NO : kMaxOrder - 1); ++j) {
+          if (j < no) {
+            uint32_t e = __ldg(reinterpret_cast<const uint32_t *>(a.eo[j] + x + q));
+            ej[j][q] = e & 0xff; ej[j][q + 1] = (e >> 8) & 0xff; ej[j][q + 2] = (e >> 16) & 0xff;
+            ej[j][q + 3] = e >> 24;
+          }
+        }
+      }
+    } else {
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        if (u < cnt) {
+          er[u] = __ldg(a.erow + x + u);
+          v[u] = __ldg(a.val + x + u);
+#pragma unroll
+          for (int j = 0; j < (NO > 0 ? NO : kMaxOrder - 1); ++j)
+            if (j < no) ej[j][u] = __ldg(a.eo[j] + x + u);
+        }
+      }
+    }
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      if (u < cnt) {
+        while (x + u >= bend) { ++b; set_block(a); }  // walk to the entry's block
+        row[u] = base_row + er[u];
+#pragma unroll
+        for (int j = 0; j < (NO > 0 ? NO : kMaxOrder - 1); ++j)
+          if (j < no) idx[j][u] = base[j] + ej[j][u];
+      }
+    }
+  }
+};
+
+// NO = number of other modes (order - 1) when specialised, 0 = generic (<= kMaxOrder - 1).
+template <class Src, int NO, int LPN, int VW, int U>
+__global__ void __launch_bounds__(kThreads) mttkrp_kernel(const KArgs a) {
+  constexpr int G = 32 / LPN;
+  constexpr int NOA = NO > 0 ? NO : kMaxOrder - 1;  // register array extent
+  const int lane = threadIdx.x & 31;
+  const int g = lane / LPN, lig = lane % LPN;
+  const uint64_t w = uint64_t(blockIdx.x) * kWarpsPerCta + (threadIdx.x >> 5);
+  const uint64_t c0 = w * a.chunk;
+  if (c0 >= a.nnz) return;
+  const uint64_t S = a.chunk / G;
+  const uint64_t x0 = c0 + uint64_t(g) * S;
+  uint64_t x1 = x0 + S;
+  if (x1 > a.nnz) x1 = a.nnz;
+  if (x0 >= x1) return;
+  const int no = NO > 0 ? NO : int(a.order) - 1;
+  const uint32_t R = a.R;
+
+  for (uint32_t col = uint32_t(lig) * VW; col < R; col += LPN * VW) {
+    Src src;
+    src.init(a, x0);
+    Vec<VW> acc;
+#pragma unroll
+    for (int i = 0; i < VW; ++i) acc.v[i] = 0.f;
+    uint32_t cur = 0xFFFFFFFFu;
+    bool first = true;
+    for (uint64_t x = x0; x < x1; x += U) {
+      const int cnt = (x1 - x) >= uint64_t(U) ? U : int(x1 - x);
+      uint32_t row[U];
+      uint32_t idx[NOA][U];
+      float v[U];
+      src.load(a, x, cnt, row, idx, v, no);
+      // issue every gather of this step before consuming any
+      Vec<VW> f[NOA][U];
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+#pragma unroll
+        for (int j = 0; j < NOA; ++j) {
+          if (j < no && u < cnt) f[j][u] = ldg_vec<VW>(a.Uo[j] + uint64_t(idx[j][u]) * R + col);
+        }
+      }
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        if (u < cnt) {
+          Vec<VW> t;
+#pragma unroll
+          for (int i = 0; i < VW; ++i) t.v[i] = v[u];
+#pragma unroll
+          for (int j = 0; j < NOA; ++j) {
+            if (j < no) {
+#pragma unroll
+              for (int i = 0; i < VW; ++i) t.v[i] *= f[j][u].v[i];
+            }
+          }
+          if (row[u] == cur) {
+#pragma unroll
+            for (int i = 0; i < VW; ++i) acc.v[i] += t.v[i];
+          } else {
+            if (cur != 0xFFFFFFFFu) {
+              float *dst = a.out + uint64_t(cur) * R + col;
+              if (first || !Src::kSortedRows) red_vec<VW>(dst, acc); else st_vec<VW>(dst, acc);
+              first = false;
+            }
+            cur = row[u];
+            acc = t;
+          }
+        }
+      }
+    }
+    if (cur != 0xFFFFFFFFu) red_vec<VW>(a.out + uint64_t(cur) * R + col, acc);
+  }
+}
+
+template <int VW>
+__global__ void zero_rows_kernel(float *__restrict__ out, uint64_t n) {
+  for (uint64_t e = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; e < n;
+       e += uint64_t(gridDim.x) * blockDim.x) {
+    if constexpr (VW == 4) reinterpret_cast<float4 *>(out)[e] = make_float4(0.f, 0.f, 0.f, 0.f);
+    else out[e] = 0.f;
+  }
+}
+
+int sm_count() {
+  static int n = 0;
+  if (!n) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
+    if (n <= 0) n = 148;
+  }
+  return n;
+}
+
+template <class Src, int NO, int LPN, int VW>
+void launch_t(const KArgs &a, cudaStream_t s) {
+  uint64_t nwarps = (a.nnz + a.chunk - 1) / a.chunk;
+  uint64_t nblk = (nwarps + kWarpsPerCta - 1) / kWarpsPerCta;
+  if (nblk == 0) return;
+  if (nblk > 0x7FFFFFFFull) fail(PASTA_ERANGE, "mttkrp: grid too large");
+  constexpr int U = 4;
+  mttkrp_kernel<Src, NO, LPN, VW, U><<<unsigned(nblk), kThreads, 0, s>>>(a);
+  PASTA_LAUNCHED();
+}
+
+template <template <int, int> class SrcT, int NO, int VW>
+void launch_lpn(const KArgs &a, int lpn, cudaStream_t s) {
+  switch (lpn) {
+    case 1: launch_t<SrcT<NO, 4>, NO, 1, VW>(a, s); break;
+    case 2: launch_t<SrcT<NO, 4>, NO, 2, VW>(a, s); break;
+    case 4: launch_t<SrcT<NO, 4>, NO, 4, VW>(a, s); break;
+    case 8: launch_t<SrcT<NO, 4>, NO, 8, VW>(a, s); break;
+    case 16: launch_t<SrcT<NO, 4>, NO, 16, VW>(a, s); break;
+    default: launch_t<SrcT<NO, 4>, NO, 32, VW>(a, s); break;
+  }
+}
+
+template <template <int, int> class SrcT>
+void dispatch(KArgs &a, bool vec4, cudaStream_t s) {
+  // lanes per nonzero: smallest power of two covering R / VW columns, at most 32
+  const uint32_t VWv = vec4 ? 4 : 1;
+  uint32_t need = (a.R + VWv - 1) / VWv;
+  int lpn = 1;
+  while (lpn < 32 && uint32_t(lpn) < need) lpn <<= 1;
+  const int G = 32 / lpn;
+  // run length per group: 128 nonzeros (multiple of 4), chunk = G * run
+  const uint64_t run = 128;
+  a.chunk = uint64_t(G) * run;
+  const int no = int(a.order) - 1;
+  if (vec4) {
+    if (no == 2) launch_lpn<SrcT, 2, 4>(a, lpn, s);
+    else if (no == 3) launch_lpn<SrcT, 3, 4>(a, lpn, s);
+    else launch_lpn<SrcT, 0, 4>(a, lpn, s);
+  } else {
+    if (no == 2) launch_lpn<SrcT, 2, 1>(a, lpn, s);
+    else if (no == 3) launch_lpn<SrcT, 3, 1>(a, lpn, s);
+    else launch_lpn<SrcT, 0, 1>(a, lpn, s);
+  }
+}
+
+bool aligned16(const void *p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
+
+}  // namespace
+
+void launch_zero_rows(float *out, uint64_t row_lo, uint64_t row_hi, uint32_t R, cudaStream_t s) {
+  if (row_hi <= row_lo) return;
+  ProfScope prof(kProfZero, s);
+  float *p = out + row_lo * R;
+  uint64_t n = (row_hi - row_lo) * uint64_t(R);
+  uint64_t grid = uint64_t(sm_count()) * 8;
+  if (aligned16(p) && n % 4 == 0) {
+    zero_rows_kernel<4><<<unsigned(grid), 256, 0, s>>>(p, n / 4);
+  } else {
+    zero_rows_kernel<1><<<unsigned(grid), 256, 0, s>>>(p, n);
+  }
+  PASTA_LAUNCHED();
+}
+
+static bool vec4_ok(uint32_t order, uint32_t mode, const float *const *factors, uint32_t R,
+                    const float *out) {
+  if (R % 4 != 0 || !aligned16(out)) return false;
+  for (uint32_t k = 0; k < order; ++k)
+    if (k != mode && !aligned16(factors[k])) return false;
+  return true;
+}
+
+void launch_coo_mttkrp(const pasta_coo *x, uint32_t mode, const float *const *factors, uint32_t R,
+                       float *out, cudaStream_t s) {
+  const CooModeCopy &mc = x->mc[mode];
+  KArgs a{};
+  a.nnz = x->nnz;
+  a.order = x->order;
+  a.R = R;
+  a.irow = mc.inds[mode];
+  a.val = mc.val;
+  int j = 0;
+  for (uint32_t k = 0; k < x->order; ++k) {
+    if (k == mode) continue;
+    a.io[j] = mc.inds[k];
+    a.Uo[j] = factors[k];
+    ++j;
+  }
+  a.out = out;
+  if (a.nnz == 0) return;
+  ProfScope prof(kProfCoo, s);
+  dispatch<CooSrc>(a, vec4_ok(x->order, mode, factors, R, out), s);
+}
+
+void launch_hicoo_mttkrp(const pasta_hicoo *h, uint32_t mode, const float *const *factors,
+                         uint32_t R, float *out, cudaStream_t s) {
+  const HicooModeCopy &mc = h->mc[mode];
+  KArgs a{};
+  a.nnz = h->nnz;
+  a.order = h->order;
+  a.R = R;
+  a.bptr = mc.bptr.p;
+  a.nblocks = h->nblocks;
+  a.brow = mc.binds[mode].p;
+  a.erow = mc.einds[mode].p;
+  a.val = mc.val.p;
+  a.bbits = h->block_bits;
+  int j = 0;
+  for (uint32_t k = 0; k < h->order; ++k) {
+    if (k == mode) continue;
+    a.bo[j] = mc.binds[k].p;
+    a.eo[j] = mc.einds[k].p;
+    a.Uo[j] = factors[k];
+    ++j;
+  }
+  a.out = out;
+  if (a.nnz == 0) return;
+  ProfScope prof(kProfHicoo, s);
+  dispatch<HicooSrc>(a, vec4_ok(h->order, mode, factors, R, out), s);
+}
+
+}  // namespace pasta

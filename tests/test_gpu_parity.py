@@ -1,0 +1,297 @@
+"""GPU parity: the CUDA path (through the C ABI) against the fp64 oracle.
+
+Tolerance (BASELINE.json north_star): |gpu - ref| <= 1e-4 * sum|terms| + 1e-6
+per output element.  Integer / byte work (generator, mode sort, HiCOO conversion) is
+compared bit for bit.  Inputs come from synth_inputs or from the oracle's own generator,
+never from the CUDA path.
+"""
+import numpy as np
+import pytest
+
+import synth_inputs as si
+
+pytestmark = pytest.mark.gpu
+
+TOL_REL, TOL_ABS = 1e-4, 1e-6
+
+
+@pytest.fixture(scope="module")
+def env(oracle_mod):
+    import torch
+
+    import paper_conf_iiswc_lilwlob20_b200 as pasta
+    assert torch.cuda.is_available(), "GPU tests need a CUDA device"
+    torch.cuda.set_device(0)
+    return pasta, oracle_mod, torch
+
+
+def _check(got, ref, ab, what=""):
+    g = got.detach().cpu().numpy().astype(np.float64) if hasattr(got, "detach") else got
+    excess = np.abs(g - ref) - (TOL_REL * ab + TOL_ABS)
+    i = np.unravel_index(np.argmax(excess), excess.shape) if excess.size else None
+    assert excess.size == 0 or excess.max() <= 0, (
+        f"{what}: tolerance exceeded at {i}: gpu={g[i]!r} ref={ref[i]!r} sumabs={ab[i]!r}")
+
+
+def _dev(torch, U):
+    return [torch.from_numpy(np.ascontiguousarray(u)).cuda() for u in U]
+
+
+def test_config1_all_modes_coo_and_hicoo(env):
+    pasta, oracle, torch = env
+    cfg = si.CONFIGS["c1"]
+    dims, R = cfg["dims"], cfg["R"]
+    inds, vals = si.uniform_coo(dims, cfg["nnz"], seed=cfg["seed"])
+    U = si.factors(dims, R, seed=cfg["seed"])
+    Ud = _dev(torch, U)
+    x = pasta.pasta_coo_from_arrays(dims, inds, vals)
+    h = pasta.pasta_coo_to_hicoo(x, 7)
+    for n in range(3):
+        ref, ab = oracle.mttkrp(dims, inds, vals, n, U)
+        _check(pasta.pasta_mttkrp_coo(x, n, Ud), ref, ab, f"coo mode {n}")
+        _check(pasta.pasta_mttkrp_hicoo(h, n, Ud), ref, ab, f"hicoo mode {n}")
+
+
+CASES = [
+    # dims, nnz, R, generator, block_bits
+    ((300, 200, 500), 50_013, 16, "powerlaw", 7),
+    ((300, 200, 500), 50_013, 32, "uniform", 7),
+    ((1000, 900), 30_001, 16, "powerlaw", 5),          # N = 2 (SpMM)
+    ((60, 70, 80, 90), 40_007, 16, "powerlaw", 4),     # N = 4
+    ((20, 30, 25, 12, 9), 20_003, 8, "uniform", 3),    # N = 5, generic order path
+    ((400, 300, 200), 25_000, 1, "powerlaw", 7),       # R = 1, scalar path
+    ((400, 300, 200), 25_000, 3, "uniform", 6),        # R % 4 != 0
+    ((400, 300, 200), 25_000, 40, "powerlaw", 7),      # R = 40: 16 lanes, ragged lanes
+    ((400, 300, 200), 12_345, 160, "powerlaw", 8),     # R > 128: column loop
+    ((1, 500, 300), 20_000, 16, "uniform", 7),         # a dimension of 1
+    ((4096, 4096, 4096), 200_000, 16, "powerlaw", 7),  # several tiles, hypersparse blocks
+]
+
+
+@pytest.mark.parametrize("dims,nnz,R,gen,bb", CASES)
+def test_random_tensors_all_modes(env, dims, nnz, R, gen, bb):
+    pasta, oracle, torch = env
+    seed = nnz + R
+    mk = si.powerlaw_coo if gen == "powerlaw" else si.uniform_coo
+    inds, vals = mk(dims, nnz, seed=seed)  # shuffled (unsorted) input order
+    U = si.factors(dims, R, seed=seed)
+    Ud = _dev(torch, U)
+    x = pasta.pasta_coo_from_arrays(dims, inds, vals)
+    h = pasta.pasta_coo_to_hicoo(x, bb)
+    for n in range(len(dims)):
+        ref, ab = oracle.mttkrp(dims, inds, vals, n, U)
+        _check(pasta.pasta_mttkrp_coo(x, n, Ud), ref, ab, f"coo {dims} R={R} mode {n}")
+        _check(pasta.pasta_mttkrp_hicoo(h, n, Ud), ref, ab, f"hicoo {dims} R={R} mode {n}")
+
+
+def test_hot_row_spanning_many_warps(env):
+    """2M nonzeros in one output row: the segmented reduction must carry across groups,
+    warps and CTAs, and hierarchical summation must stay inside the tolerance."""
+    pasta, oracle, torch = env
+    dims = (5000, 3000, 2000)
+    inds, vals = si.hot_row_coo(dims, 2_000_000, 100_000, seed=3, mode=0, hot_row=1234)
+    U = si.factors(dims, 16, seed=5)
+    Ud = _dev(torch, U)
+    x = pasta.pasta_coo_from_arrays(dims, inds, vals)
+    h = pasta.pasta_coo_to_hicoo(x, 7)
+    for n in range(3):
+        ref, ab = oracle.mttkrp(dims, inds, vals, n, U)
+        _check(pasta.pasta_mttkrp_coo(x, n, Ud), ref, ab, f"coo hot mode {n}")
+        _check(pasta.pasta_mttkrp_hicoo(h, n, Ud), ref, ab, f"hicoo hot mode {n}")
+
+
+def test_output_is_overwritten_and_empty_rows_zero(env):
+    pasta, oracle, torch = env
+    dims = (1000, 50, 60)
+    inds, vals = si.uniform_coo((1000, 50, 60), 3000, seed=1)
+    keep = inds[0] % 3 != 0  # every third row empty
+    inds, vals = np.ascontiguousarray(inds[:, keep]), vals[keep]
+    U = si.factors(dims, 16, seed=2)
+    Ud = _dev(torch, U)
+    x = pasta.pasta_coo_from_arrays(dims, inds, vals)
+    h = pasta.pasta_coo_to_hicoo(x, 7)
+    ref, ab = oracle.mttkrp(dims, inds, vals, 0, U)
+    for fn, t in ((pasta.pasta_mttkrp_coo, x), (pasta.pasta_mttkrp_hicoo, h)):
+        out = torch.full((dims[0], 16), 7.0, device="cuda")
+        fn(t, 0, Ud, out=out)
+        _check(out, ref, ab, fn.__name__)
+        assert torch.all(out[0::3] == 0)
+
+
+def test_empty_tensor_and_order_one(env):
+    pasta, oracle, torch = env
+    dims = (10, 20, 30)
+    x = pasta.pasta_coo_from_arrays(dims, np.zeros((3, 0), np.uint32), np.zeros(0, np.float32))
+    Ud = _dev(torch, si.factors(dims, 16, seed=0))
+    out = torch.full((20, 16), 3.0, device="cuda")
+    pasta.pasta_mttkrp_coo(x, 1, Ud, out=out)
+    assert torch.all(out == 0)
+    h = pasta.pasta_coo_to_hicoo(x, 7)
+    assert h.nblocks == 0
+    out.fill_(3.0)
+    pasta.pasta_mttkrp_hicoo(h, 1, Ud, out=out)
+    assert torch.all(out == 0)
+    # order 1: the empty Khatri-Rao product; MTTKRP = slice sums in every column
+    i1 = np.array([[5, 1, 5, 9]], np.uint32)
+    v1 = np.array([1.0, 2.0, -0.5, 4.0], np.float32)
+    x1 = pasta.pasta_coo_from_arrays((10,), i1, v1)
+    got = pasta.pasta_mttkrp_coo(x1, 0, [None], R=4).cpu().numpy()
+    ref, ab = oracle.mttkrp((10,), i1, v1, 0, [None], R=4)
+    _check(got, ref, ab, "order 1")
+
+
+def test_generator_bit_exact_with_oracle(env):
+    pasta, oracle, torch = env
+    cases = [
+        dict(dims=(12092, 9184, 28818), nnz=200_000, seed=1002),
+        dict(dims=(6066, 5699, 244268, 1176), nnz=100_000, seed=1004),
+        dict(dims=(64, 64, 64), nnz=20_000, seed=7),  # many repeated draws
+        dict(dims=(1 << 16, 1 << 16), nnz=5000, seed=3, initiator=[0.57, 0.19, 0.19, 0.05]),
+        dict(dims=(100, 100, 100), nnz=10_000, seed=1001, kind=0),
+    ]
+    for c in cases:
+        kind = c.get("kind", 1)
+        x = pasta.pasta_gen_powerlaw(c["dims"], c["nnz"], c["seed"], kind=kind,
+                                     initiator=c.get("initiator"))
+        gi, gv = pasta.pasta_coo_export(x)
+        oi, ov = oracle.gen_powerlaw(c["dims"], c["nnz"], c["seed"], initiator=c.get("initiator"),
+                                     q=0.5 if kind == 0 else 0.75)
+        np.testing.assert_array_equal(gi, oi)
+        np.testing.assert_array_equal(gv.view(np.uint32), ov.view(np.uint32))
+
+
+def test_mode_sort_bit_exact_with_oracle(env):
+    pasta, oracle, torch = env
+    dims = (3000, 200, 4000, 50)
+    inds, vals = si.powerlaw_coo(dims, 100_000, seed=4)
+    x = pasta.pasta_coo_from_arrays(dims, inds, vals)
+    for n in range(4):
+        gi, gv = pasta.pasta_coo_export_mode(x, n)
+        oi, ov = oracle.mode_sort(inds, vals, n)
+        np.testing.assert_array_equal(gi, oi)
+        np.testing.assert_array_equal(gv.view(np.uint32), ov.view(np.uint32))
+
+
+@pytest.mark.parametrize("dims,nnz,bb", [((300, 200, 500), 50_013, 7), ((60, 70, 80, 90), 40_007, 4),
+                                         ((4096, 4096, 4096), 200_000, 7), ((1000, 900), 30_001, 1),
+                                         ((1 << 20, 3, 1 << 12), 30_000, 8)])
+def test_hicoo_conversion_bit_exact(env, dims, nnz, bb):
+    pasta, oracle, torch = env
+    inds, vals = si.powerlaw_coo(dims, nnz, seed=nnz)
+    x = pasta.pasta_coo_from_arrays(dims, inds, vals)
+    h = pasta.pasta_hicoo_export(pasta.pasta_coo_to_hicoo(x, bb))
+    o = oracle.coo_to_hicoo(inds, vals, bb)
+    assert h["nblocks"] == o["nblocks"]
+    np.testing.assert_array_equal(h["bptr"], o["bptr"])
+    np.testing.assert_array_equal(h["binds"], o["binds"])
+    np.testing.assert_array_equal(h["einds"], o["einds"])
+    np.testing.assert_array_equal(h["vals"].view(np.uint32), o["vals"].view(np.uint32))
+
+
+def test_shards_cover_the_output(env):
+    pasta, oracle, torch = env
+    dims = (2000, 300, 400)
+    inds, vals = si.hot_row_coo(dims, 20_000, 60_000, seed=9, mode=1, hot_row=17)
+    U = si.factors(dims, 16, seed=4)
+    Ud = _dev(torch, U)
+    x = pasta.pasta_coo_from_arrays(dims, inds, vals)
+    for n in range(3):
+        ref, ab = oracle.mttkrp(dims, inds, vals, n, U)
+        counts = pasta.pasta_coo_row_counts(x, n)
+        np.testing.assert_array_equal(counts, np.bincount(inds[n], minlength=dims[n]))
+        for P in (1, 3, 8):
+            bounds = pasta.pasta_coo_partition(x, n, P)
+            np.testing.assert_array_equal(bounds, pasta.pasta_row_partition(counts, P))
+            out = torch.full((dims[n], 16), float("nan"), device="cuda")
+            total = 0
+            for p in range(P):
+                s = pasta.pasta_coo_shard(x, n, int(bounds[p]), int(bounds[p + 1]))
+                total += s.nnz
+                pasta.pasta_mttkrp_coo(s, n, Ud, out=out)  # writes only its rows
+            assert total == vals.shape[0]
+            _check(out, ref, ab, f"shards mode {n} P={P}")
+
+
+def test_allmodes_host_e2e_matches_device(env):
+    pasta, oracle, torch = env
+    dims = (500, 400, 300)
+    inds, vals = si.powerlaw_coo(dims, 60_000, seed=11)
+    U = si.factors(dims, 16, seed=12)
+    x = pasta.pasta_coo_from_arrays(dims, inds, vals)
+    hf = [torch.from_numpy(u).pin_memory() for u in U]
+    ho = [torch.empty((d, 16), dtype=torch.float32).pin_memory() for d in dims]
+    pasta.pasta_mttkrp_coo_allmodes_host(x, hf, ho)
+    for n in range(3):
+        ref, ab = oracle.mttkrp(dims, inds, vals, n, U)
+        _check(ho[n].numpy().astype(np.float64), ref, ab, f"e2e mode {n}")
+
+
+def test_tns_roundtrip(env, tmp_path):
+    pasta, oracle, torch = env
+    dims = (50, 60, 70)
+    inds, vals = si.uniform_coo(dims, 2000, seed=2)
+    p = tmp_path / "t.tns"
+    with open(p, "w") as f:
+        f.write("# FROSTT-style, 1-based\n")
+        for x in range(vals.shape[0]):
+            f.write(" ".join(str(int(inds[k, x]) + 1) for k in range(3)) + f" {float(vals[x]):.9g}\n")
+    t = pasta.pasta_load_coo(str(p))
+    assert t.order == 3 and t.nnz == 2000
+    assert t.dims == tuple(int(inds[k].max()) + 1 for k in range(3))
+    gi, gv = pasta.pasta_coo_export(t)
+    np.testing.assert_array_equal(gi, inds)
+    np.testing.assert_array_equal(gv, vals)
+    q = tmp_path / "u.tns"
+    pasta.pasta_save_coo(t, str(q))
+    t2 = pasta.pasta_load_coo(str(q))
+    gi2, gv2 = pasta.pasta_coo_export(t2)
+    np.testing.assert_array_equal(gi2, inds)
+    np.testing.assert_array_equal(gv2, vals)
+
+
+def test_misaligned_factor_takes_scalar_path(env):
+    pasta, oracle, torch = env
+    dims = (300, 200, 100)
+    inds, vals = si.uniform_coo(dims, 20_000, seed=8)
+    U = si.factors(dims, 16, seed=8)
+    x = pasta.pasta_coo_from_arrays(dims, inds, vals)
+    Ud = []
+    for u in U:  # a view starting 4 bytes into a buffer: not 16-byte aligned
+        buf = torch.empty(u.size + 1, dtype=torch.float32, device="cuda")
+        v = buf[1:].view(u.shape)
+        v.copy_(torch.from_numpy(u))
+        Ud.append(v)
+    for n in range(3):
+        ref, ab = oracle.mttkrp(dims, inds, vals, n, U)
+        _check(pasta.pasta_mttkrp_coo(x, n, Ud), ref, ab, f"misaligned mode {n}")
+
+
+def test_profile_and_launch_counters(env):
+    pasta, oracle, torch = env
+    dims = (300, 200, 100)
+    inds, vals = si.uniform_coo(dims, 20_000, seed=8)
+    Ud = _dev(torch, si.factors(dims, 16, seed=8))
+    x = pasta.pasta_coo_from_arrays(dims, inds, vals)
+    pasta.pasta_mttkrp_coo(x, 0, Ud)
+    pasta.pasta_profile_read(0, reset=True)
+    pasta.pasta_profile_enable(True)
+    n0 = pasta.pasta_launch_count()
+    for _ in range(3):
+        pasta.pasta_mttkrp_coo(x, 0, Ud)
+    ms, n = pasta.pasta_profile_read(0, reset=True)
+    pasta.pasta_profile_enable(False)
+    assert n == 3 and ms > 0
+    assert pasta.pasta_launch_count() - n0 == 6  # zero-fill + MTTKRP per call
+
+
+def test_errors_on_device(env):
+    pasta, oracle, torch = env
+    dims = (10, 10, 10)
+    x = pasta.pasta_coo_from_arrays(dims, np.zeros((3, 1), np.uint32), np.ones(1, np.float32))
+    Ud = _dev(torch, si.factors(dims, 4, seed=0))
+    with pytest.raises(pasta.PastaError):
+        pasta.pasta_mttkrp_coo(x, 3, Ud)
+    with pytest.raises(pasta.PastaError):
+        pasta.pasta_coo_to_hicoo(x, 9)
+    with pytest.raises(pasta.PastaError):
+        pasta.pasta_coo_shard(x, 0, 5, 3)
