@@ -1,0 +1,354 @@
+#!/usr/bin/env python
+"""bench.py -- MTTKRP GFLOP/s and HBM GB/s against the measured B200 roofline.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config h|c2|c3|c4|c1] [--impl reference]
+
+One STEP = COO MTTKRP of every mode (output zero-fill + kernel, the paper times all modes and
+averages) over the synthetic tensor resident in HBM; at N > 1 each rank runs its
+nnz-balanced row shard of every mode and the owned output rows are all-gathered (NCCL).
+Rank 0 prints one JSON line.  GFLOP/s uses the nominal N*M*R flops per mode (Table I
+generalised; R#7).
+
+The default workload is the north_star target: a 100M-nonzero 3rd-order power-law tensor,
+regL-shaped (2^23)^3 (Table II s3), R = 16.
+
+--impl reference times the fp64 CPU oracle (oracle/, the slow correctness reference) on a
+bounded sample of the same workload on the host cores; under torchrun only rank 0 works.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+import synth_inputs as si  # noqa: E402
+
+METRIC = "MTTKRP GFLOP/s and HBM GB/s vs ~8 TB/s roofline at 1/2/4/8 B200"
+FALLBACK_HBM_GBS = 6650.0
+
+
+def model_flops(order, nnz, R):
+    """N*M*R per mode (N-1 multiplies + 1 add per r per nonzero; Table I's 3MR at N = 3)."""
+    return order * nnz * R
+
+
+def model_bytes_coo(order, nnz, R):
+    """Table I COO upper bound generalised (R#8): 4(N+1)M stream + 4NRM factor/output rows."""
+    return 4 * (order + 1) * nnz + 4 * order * R * nnz
+
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        with open(p) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, torch copy)"
+    except Exception:
+        return FALLBACK_HBM_GBS, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+class ClockSampler:
+    """nvidia-smi clocks and throttle reasons sampled DURING the timed region."""
+
+    FIELDS = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index = index
+        self.proc = None
+        self.path = None
+
+    def start(self):
+        fd, self.path = tempfile.mkstemp(prefix="clocks_", suffix=".csv")
+        os.close(fd)
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}",
+                 "--format=csv,noheader,nounits", "-lms", "100"],
+                stdout=open(self.path, "w"), stderr=subprocess.DEVNULL)
+        except Exception:
+            self.proc = None
+        time.sleep(0.3)
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        time.sleep(0.15)
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        rows = []
+        with open(self.path) as f:
+            for line in f:
+                parts = [p.strip() for p in line.split(",")]
+                if len(parts) >= 8:
+                    rows.append(parts)
+        os.unlink(self.path)
+        if not rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["no samples"]}
+        sm = [float(r[0]) for r in rows if r[0].replace(".", "").isdigit()]
+        smax = max(float(r[1]) for r in rows if r[1].replace(".", "").isdigit())
+        loaded = [s for s in sm if s > 0.5 * smax] or sm
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in rows for i in range(4) if r[4 + i].lower() == "active"})
+        return {"sm_mhz": statistics.median(loaded), "sm_max_mhz": smax, "reasons": reasons,
+                "samples": len(rows), "power_w_max": max(float(r[2]) for r in rows
+                                                           if r[2].replace(".", "").isdigit())}
+
+
+def dist_env():
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return world, rank, local
+
+
+def cpu_baseline(cfg, R, sample_nnz, steps=1, warmup=0):
+    """The fp64 oracle (as it stands, single thread) on a bounded sample of the workload:
+    the first `sample_nnz` distinct coordinates of the SAME counter-based draw sequence
+    (the oracle's own generator), all modes.  Returns (GFLOP/s, seconds per step)."""
+    import oracle
+    dims = cfg["dims"]
+    inds, vals = oracle.gen_powerlaw(dims, sample_nnz, cfg["seed"], q=0.5 if cfg["kind"] ==
+                                     "uniform" else 0.75)
+    U = si.factors(dims, R, seed=cfg["seed"])
+    times = []
+    for it in range(warmup + steps):
+        t0 = time.perf_counter()
+        for n in range(len(dims)):
+            oracle.mttkrp(dims, inds, vals, n, U)
+        if it >= warmup:
+            times.append(time.perf_counter() - t0)
+    t = sum(times) / len(times)
+    flops = len(dims) * model_flops(len(dims), sample_nnz, R)
+    return flops / t / 1e9, t
+
+
+def ncu_traffic(config_key):
+    """DRAM bytes per COO-MTTKRP launch from the committed ncu --set full summary, if any."""
+    p = os.path.join(ROOT, "profiles", "ncu_summary.json")
+    try:
+        with open(p) as f:
+            d = json.load(f)
+        e = d.get(config_key, {}).get("coo_mttkrp")
+        return float(e["dram_bytes_per_launch"]) if e else None
+    except Exception:
+        return None
+
+
+def run_reference(args, cfg, world, rank):
+    if rank != 0:
+        return
+    R = cfg["R"]
+    sample = args.ref_sample
+    gflops, t = cpu_baseline(cfg, R, sample, steps=args.steps, warmup=args.warmup)
+    cores = 1
+    line = {
+        "impl": "reference", "metric": METRIC, "value": round(gflops, 4), "unit": "GFLOP/s",
+        "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": round(t * 1e3, 3), "higher_is_better": True, "scaling": "strong",
+        "vs_baseline": None, "dtype": "f64", "data": "synthetic (oracle generator, same draws)",
+        "config": {"workload": f"{args.config}: {cfg['name']}", "dims": list(cfg["dims"]),
+                   "nnz": cfg["nnz"], "R": R, "format": "COO", "modes": "all"},
+        "cpu_baseline": {"value": round(gflops, 4), "unit": "GFLOP/s", "cores": cores,
+                         "kind": "oracle",
+                         "sample": f"first {sample} distinct nonzeros of the workload's draw "
+                                   f"sequence, all {len(cfg['dims'])} modes per step"},
+        "e2e": {"value": round(gflops, 4), "unit": "GFLOP/s", "h2d_bytes_per_step": 0,
+                "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=100)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--config", default="h", choices=sorted(si.CONFIGS))
+    ap.add_argument("--impl", default="pasta", choices=["pasta", "reference"])
+    ap.add_argument("--ref-sample", type=int, default=1_000_000)
+    ap.add_argument("--cpu-sample", type=int, default=4_000_000)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--e2e-steps", type=int, default=10)
+    args = ap.parse_args()
+    if args.warmup < 3:
+        args.warmup = 3  # timing rule: >= 3 warm-up steps
+    cfg = si.CONFIGS[args.config]
+    world, rank, local = dist_env()
+
+    if args.impl == "reference":
+        run_reference(args, cfg, world, rank)
+        return
+
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_iiswc_lilwlob20_b200 as pasta
+    from paper_conf_iiswc_lilwlob20_b200.parallel import RowPartitionedMTTKRP
+
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    stream = torch.cuda.current_stream()
+
+    dims, R, M = cfg["dims"], cfg["R"], cfg["nnz"]
+    N = len(dims)
+    t0 = time.perf_counter()
+    x = pasta.pasta_gen_powerlaw(dims, M, cfg["seed"], kind=0 if cfg["kind"] == "uniform" else 1)
+    torch.cuda.synchronize()
+    t_gen = time.perf_counter() - t0
+    t0 = time.perf_counter()
+    for n in range(N):
+        pasta.pasta_coo_prepare(x, n)
+    torch.cuda.synchronize()
+    t_prep = time.perf_counter() - t0
+    g = torch.Generator(device=dev)
+    g.manual_seed(cfg["seed"])
+    U = [torch.rand((d, R), generator=g, device=dev, dtype=torch.float32) for d in dims]
+
+    if world > 1:
+        part = RowPartitionedMTTKRP(x, rank, world, R, dev)
+        shard_nnz = part.shard_nnz()
+        x_local = None
+        del x
+        torch.cuda.synchronize()
+
+        def step():
+            part.step(U, gather=True)
+    else:
+        outs = [torch.empty((d, R), dtype=torch.float32, device=dev) for d in dims]
+        shard_nnz = [M] * N
+
+        def step():
+            for n in range(N):
+                pasta.pasta_mttkrp_coo(x, n, U, out=outs[n])
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+
+    clocks = ClockSampler(local)
+    if rank == 0:
+        clocks.start()
+    pasta.pasta_profile_read(0, reset=True)
+    pasta.pasta_profile_read(2, reset=True)
+    pasta.pasta_profile_enable(True)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    launches0 = pasta.pasta_launch_count()
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    ev0.record(stream)
+    for _ in range(args.steps):
+        step()
+    ev1.record(stream)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    launches = pasta.pasta_launch_count() - launches0
+    pasta.pasta_profile_enable(False)
+    elapsed_ms = ev0.elapsed_time(ev1)
+    kern_ms, kern_n = pasta.pasta_profile_read(0, reset=True)
+    zero_ms, zero_n = pasta.pasta_profile_read(2, reset=True)
+    clk = clocks.stop() if rank == 0 else None
+    if world > 1:
+        t = torch.tensor([elapsed_ms], device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        elapsed_ms = float(t.item())
+
+    ms_per_step = elapsed_ms / args.steps
+    total_flops = N * model_flops(N, M, R)  # all ranks together, every mode
+    value = total_flops / (ms_per_step * 1e-3) / 1e9
+
+    # e2e: the same metric through the public C ABI with HOST buffers (pinned)
+    e2e = None
+    if world == 1 and args.e2e_steps > 0:
+        hf = [u.cpu().pin_memory() for u in U]
+        ho = [torch.empty((d, R), dtype=torch.float32).pin_memory() for d in dims]
+        pasta.pasta_mttkrp_coo_allmodes_host(x, hf, ho)  # warm-up (allocates staging)
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(args.e2e_steps):
+            pasta.pasta_mttkrp_coo_allmodes_host(x, hf, ho)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        e_ms = e0.elapsed_time(e1) / args.e2e_steps
+        nbytes = sum(d * R * 4 for d in dims)
+        e2e = {"value": round(total_flops / (e_ms * 1e-3) / 1e9, 3), "unit": "GFLOP/s",
+               "h2d_bytes_per_step": nbytes, "d2h_bytes_per_step": nbytes,
+               "ms_per_step": round(e_ms, 3),
+               "path": "pasta_mttkrp_coo_allmodes_host (pinned host factors in, results out)"}
+        del hf, ho
+
+    if rank != 0:
+        if world > 1:
+            dist.destroy_process_group()
+        return
+
+    peak, peak_src = load_peaks()
+    per_launch_nnz = max(shard_nnz)  # rank 0's launches cover its shard
+    my_launch_nnz = [shard_nnz[n] for n in range(N)]
+    avg_launch_ms = kern_ms / max(kern_n, 1)
+    launch_bytes = sum(model_bytes_coo(N, m, R) for m in my_launch_nnz) / N
+    achieved = launch_bytes / (avg_launch_ms * 1e-3) / 1e9
+    traffic = ncu_traffic(args.config) if world == 1 else None
+
+    cpu = None
+    if not args.no_cpu_baseline and world == 1:
+        sample = min(args.cpu_sample, M)
+        gf, t = cpu_baseline(cfg, R, sample)
+        cpu = {"value": round(gf, 4), "unit": "GFLOP/s", "cores": 1, "kind": "oracle",
+               "sample": f"first {sample} distinct nonzeros of the same draw sequence (oracle "
+                         f"generator), all {N} modes, 1 run, 1 host thread"}
+
+    line = {
+        "metric": METRIC, "value": round(value, 3), "unit": "GFLOP/s", "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms_per_step, 4),
+        "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f32",
+        "data": f"synthetic: GPU Stochastic Kronecker generator (q=0.75), seed {cfg['seed']}",
+        "config": {"workload": f"{args.config}: {cfg['name']}", "dims": list(dims), "nnz": M,
+                   "R": R, "format": "COO", "modes": f"all {N} per step",
+                   "parallelism": f"row-partitioned x{world}" + (" + NCCL all-gather" if world > 1
+                                                                  else ""),
+                   "l2": "no flush: per-step working set (COO copies + factors + outputs) "
+                         "> 126 MB L2"},
+        "model_gbs": round(model_bytes_coo(N, M, R) * N / (ms_per_step * 1e-3) / 1e9, 1),
+        "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
+                     "frac": round(achieved / peak, 4), "traffic": traffic,
+                     "kernel": "mttkrp_kernel<CooSrc> (a6)",
+                     "bytes_model": "4(N+1)M + 4NRM per launch (Table I, P:117)",
+                     "avg_launch_ms": round(avg_launch_ms, 4), "launches": kern_n,
+                     "peak_source": peak_src},
+        "zero_fill_ms_per_step": round(zero_ms / args.steps, 4),
+        "preprocess_s": {"generate": round(t_gen, 3), "mode_sort_all": round(t_prep, 3)},
+        "clocks": clk,
+        "e2e": e2e,
+        "gpu_launches": launches,
+        "cpu_baseline": cpu,
+        "max_shard_nnz": per_launch_nnz,
+    }
+    print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()
