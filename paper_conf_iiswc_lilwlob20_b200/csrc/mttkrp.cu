@@ -21,6 +21,8 @@
 //     and last segment of a run may be shared with neighbours -> red.global.add.v4.f32
 //     (one vector atomic per boundary, not per nonzero, cf. P:157/P:282 atomics).
 //   * No tensor cores: the path is a gather/scatter, not a dense contraction.
+#include <cstdlib>
+
 #include "internal.cuh"
 
 namespace pasta {
@@ -201,8 +203,20 @@ struct HicooSrc {
 };
 
 // NO = number of other modes (order - 1) when specialised, 0 = generic (<= kMaxOrder - 1).
-template <class Src, int NO, int LPN, int VW, int U>
-__global__ void __launch_bounds__(kThreads) mttkrp_kernel(const KArgs a) {
+// Kernel variant knobs: U nonzeros per unrolled step, PF = software-pipelined prefetch of
+// the next step's index/value stream (so the stream latency hides behind the gathers),
+// MINB = minimum resident CTAs per SM requested from ptxas (register cap).
+template <int U_, bool PF_, int MINB_>
+struct Tune {
+  static constexpr int U = U_;
+  static constexpr bool PF = PF_;
+  static constexpr int MINB = MINB_;
+};
+
+// NO = number of other modes (order - 1) when specialised, 0 = generic (<= kMaxOrder - 1).
+template <class Src, int NO, int LPN, int VW, class T>
+__global__ void __launch_bounds__(kThreads, T::MINB) mttkrp_kernel(const KArgs a) {
+  constexpr int U = T::U;
   constexpr int G = 32 / LPN;
   constexpr int NOA = NO > 0 ? NO : kMaxOrder - 1;  // register array extent
   const int lane = threadIdx.x & 31;
@@ -226,12 +240,22 @@ __global__ void __launch_bounds__(kThreads) mttkrp_kernel(const KArgs a) {
     for (int i = 0; i < VW; ++i) acc.v[i] = 0.f;
     uint32_t cur = 0xFFFFFFFFu;
     bool first = true;
+    uint32_t row[U];
+    uint32_t idx[NOA][U];
+    float v[U];
+    int cnt = (x1 - x0) >= uint64_t(U) ? U : int(x1 - x0);
+    if (T::PF) src.load(a, x0, cnt, row, idx, v, no);
     for (uint64_t x = x0; x < x1; x += U) {
-      const int cnt = (x1 - x) >= uint64_t(U) ? U : int(x1 - x);
-      uint32_t row[U];
-      uint32_t idx[NOA][U];
-      float v[U];
-      src.load(a, x, cnt, row, idx, v, no);
+      uint32_t rown[U];
+      uint32_t idxn[NOA][U];
+      float vn[U];
+      const uint64_t xn = x + U;
+      const int cntn = xn >= x1 ? 0 : ((x1 - xn) >= uint64_t(U) ? U : int(x1 - xn));
+      if (T::PF) {
+        if (cntn > 0) src.load(a, xn, cntn, rown, idxn, vn, no);  // next step's stream
+      } else {
+        src.load(a, x, cnt, row, idx, v, no);
+      }
       // issue every gather of this step before consuming any
       Vec<VW> f[NOA][U];
 #pragma unroll
@@ -268,6 +292,16 @@ __global__ void __launch_bounds__(kThreads) mttkrp_kernel(const KArgs a) {
           }
         }
       }
+      if (T::PF) {
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+          row[u] = rown[u];
+          v[u] = vn[u];
+#pragma unroll
+          for (int j = 0; j < NOA; ++j) idx[j][u] = idxn[j][u];
+        }
+      }
+      cnt = cntn;
     }
     if (cur != 0xFFFFFFFFu) red_vec<VW>(a.out + uint64_t(cur) * R + col, acc);
   }
@@ -293,27 +327,53 @@ int sm_count() {
   return n;
 }
 
-template <class Src, int NO, int LPN, int VW>
+template <class Src, int NO, int LPN, int VW, class T>
 void launch_t(const KArgs &a, cudaStream_t s) {
   uint64_t nwarps = (a.nnz + a.chunk - 1) / a.chunk;
   uint64_t nblk = (nwarps + kWarpsPerCta - 1) / kWarpsPerCta;
   if (nblk == 0) return;
   if (nblk > 0x7FFFFFFFull) fail(PASTA_ERANGE, "mttkrp: grid too large");
-  constexpr int U = 4;
-  mttkrp_kernel<Src, NO, LPN, VW, U><<<unsigned(nblk), kThreads, 0, s>>>(a);
+  mttkrp_kernel<Src, NO, LPN, VW, T><<<unsigned(nblk), kThreads, 0, s>>>(a);
   PASTA_LAUNCHED();
 }
 
-template <template <int, int> class SrcT, int NO, int VW>
-void launch_lpn(const KArgs &a, int lpn, cudaStream_t s) {
-  switch (lpn) {
-    case 1: launch_t<SrcT<NO, 4>, NO, 1, VW>(a, s); break;
-    case 2: launch_t<SrcT<NO, 4>, NO, 2, VW>(a, s); break;
-    case 4: launch_t<SrcT<NO, 4>, NO, 4, VW>(a, s); break;
-    case 8: launch_t<SrcT<NO, 4>, NO, 8, VW>(a, s); break;
-    case 16: launch_t<SrcT<NO, 4>, NO, 16, VW>(a, s); break;
-    default: launch_t<SrcT<NO, 4>, NO, 32, VW>(a, s); break;
+using TuneDefault = Tune<4, false, 1>;
+
+// Variants selectable with PASTA_MTTKRP_VARIANT for tuning sweeps (vector path, N = 3, 4,
+// R = 16 / 32).
+template <template <int, int> class SrcT, int NO, int LPN>
+void launch_variant(const KArgs &a, int variant, cudaStream_t s) {
+  switch (variant) {
+    case 1: launch_t<SrcT<NO, 4>, NO, LPN, 4, Tune<4, true, 1>>(a, s); break;
+    case 2: launch_t<SrcT<NO, 8>, NO, LPN, 4, Tune<8, false, 1>>(a, s); break;
+    case 3: launch_t<SrcT<NO, 4>, NO, LPN, 4, Tune<4, true, 3>>(a, s); break;
+    case 4: launch_t<SrcT<NO, 8>, NO, LPN, 4, Tune<8, true, 2>>(a, s); break;
+    case 5: launch_t<SrcT<NO, 4>, NO, LPN, 4, Tune<4, false, 4>>(a, s); break;
+    case 6: launch_t<SrcT<NO, 4>, NO, LPN, 4, Tune<4, false, 3>>(a, s); break;
+    case 7: launch_t<SrcT<NO, 8>, NO, LPN, 4, Tune<8, false, 2>>(a, s); break;
+    default: launch_t<SrcT<NO, 4>, NO, LPN, 4, TuneDefault>(a, s); break;
   }
+}
+
+template <template <int, int> class SrcT, int NO, int VW>
+void launch_lpn(const KArgs &a, int lpn, int variant, cudaStream_t s) {
+  if constexpr (VW == 4 && (NO == 2 || NO == 3)) {
+    if (lpn == 4) return launch_variant<SrcT, NO, 4>(a, variant, s);
+    if (lpn == 8) return launch_variant<SrcT, NO, 8>(a, variant, s);
+  }
+  switch (lpn) {
+    case 1: launch_t<SrcT<NO, 4>, NO, 1, VW, TuneDefault>(a, s); break;
+    case 2: launch_t<SrcT<NO, 4>, NO, 2, VW, TuneDefault>(a, s); break;
+    case 4: launch_t<SrcT<NO, 4>, NO, 4, VW, TuneDefault>(a, s); break;
+    case 8: launch_t<SrcT<NO, 4>, NO, 8, VW, TuneDefault>(a, s); break;
+    case 16: launch_t<SrcT<NO, 4>, NO, 16, VW, TuneDefault>(a, s); break;
+    default: launch_t<SrcT<NO, 4>, NO, 32, VW, TuneDefault>(a, s); break;
+  }
+}
+
+int env_int(const char *name, int dflt) {
+  const char *v = getenv(name);
+  return (v && *v) ? atoi(v) : dflt;
 }
 
 template <template <int, int> class SrcT>
@@ -324,18 +384,20 @@ void dispatch(KArgs &a, bool vec4, cudaStream_t s) {
   int lpn = 1;
   while (lpn < 32 && uint32_t(lpn) < need) lpn <<= 1;
   const int G = 32 / lpn;
-  // run length per group: 128 nonzeros (multiple of 4), chunk = G * run
-  const uint64_t run = 128;
+  // run length per group (multiple of 8), chunk = G * run
+  uint64_t run = uint64_t(env_int("PASTA_MTTKRP_RUN", 128));
+  run = run < 8 ? 8 : (run / 8) * 8;
   a.chunk = uint64_t(G) * run;
+  const int variant = env_int("PASTA_MTTKRP_VARIANT", 0);
   const int no = int(a.order) - 1;
   if (vec4) {
-    if (no == 2) launch_lpn<SrcT, 2, 4>(a, lpn, s);
-    else if (no == 3) launch_lpn<SrcT, 3, 4>(a, lpn, s);
-    else launch_lpn<SrcT, 0, 4>(a, lpn, s);
+    if (no == 2) launch_lpn<SrcT, 2, 4>(a, lpn, variant, s);
+    else if (no == 3) launch_lpn<SrcT, 3, 4>(a, lpn, variant, s);
+    else launch_lpn<SrcT, 0, 4>(a, lpn, variant, s);
   } else {
-    if (no == 2) launch_lpn<SrcT, 2, 1>(a, lpn, s);
-    else if (no == 3) launch_lpn<SrcT, 3, 1>(a, lpn, s);
-    else launch_lpn<SrcT, 0, 1>(a, lpn, s);
+    if (no == 2) launch_lpn<SrcT, 2, 1>(a, lpn, variant, s);
+    else if (no == 3) launch_lpn<SrcT, 3, 1>(a, lpn, variant, s);
+    else launch_lpn<SrcT, 0, 1>(a, lpn, variant, s);
   }
 }
 
