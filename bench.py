@@ -47,6 +47,11 @@ def model_bytes_coo(order, nnz, R):
     return 4 * (order + 1) * nnz + 4 * order * R * nnz
 
 
+def model_bytes_hicoo(order, nnz, nblocks, R, B=128):
+    """Table I HiCOO bound generalised (R#8): (N+4)M + (8+4N)n_b + 4NR min(n_b B, M)."""
+    return (order + 4) * nnz + (8 + 4 * order) * nblocks + 4 * order * R * min(nblocks * B, nnz)
+
+
 def load_peaks():
     p = os.path.join(ROOT, "MEASURED_PEAKS.json")
     try:
@@ -137,13 +142,13 @@ def cpu_baseline(cfg, R, sample_nnz, steps=1, warmup=0):
     return flops / t / 1e9, t
 
 
-def ncu_traffic(config_key):
-    """DRAM bytes per COO-MTTKRP launch from the committed ncu --set full summary, if any."""
+def ncu_traffic(config_key, family="coo_mttkrp"):
+    """DRAM bytes per MTTKRP launch from the committed ncu --set full summary, if any."""
     p = os.path.join(ROOT, "profiles", "ncu_summary.json")
     try:
         with open(p) as f:
             d = json.load(f)
-        e = d.get(config_key, {}).get("coo_mttkrp")
+        e = d.get(config_key, {}).get(family)
         return float(e["dram_bytes_per_launch"]) if e else None
     except Exception:
         return None
@@ -184,6 +189,7 @@ def main():
     ap.add_argument("--cpu-sample", type=int, default=4_000_000)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=10)
+    ap.add_argument("--hicoo-steps", type=int, default=20)
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3  # timing rule: >= 3 warm-up steps
@@ -298,6 +304,51 @@ def main():
                "path": "pasta_mttkrp_coo_allmodes_host (pinned host factors in, results out)"}
         del hf, ho
 
+    # a7: HiCOO MTTKRP (B = 128) on the same tensor, every mode per step
+    hicoo = None
+    if world == 1 and args.hicoo_steps > 0:
+        t0 = time.perf_counter()
+        h = pasta.pasta_coo_to_hicoo(x, 7)
+        torch.cuda.synchronize()
+        t_conv = time.perf_counter() - t0
+        t0 = time.perf_counter()
+        for n in range(N):
+            pasta.pasta_hicoo_prepare(h, n)
+        torch.cuda.synchronize()
+        t_hprep = time.perf_counter() - t0
+        houts = [torch.empty((d, R), dtype=torch.float32, device=dev) for d in dims]
+        for _ in range(3):
+            for n in range(N):
+                pasta.pasta_mttkrp_hicoo(h, n, U, out=houts[n])
+        torch.cuda.synchronize()
+        pasta.pasta_profile_read(1, reset=True)
+        pasta.pasta_profile_enable(True)
+        h0, h1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        h0.record(stream)
+        for _ in range(args.hicoo_steps):
+            for n in range(N):
+                pasta.pasta_mttkrp_hicoo(h, n, U, out=houts[n])
+        h1.record(stream)
+        torch.cuda.synchronize()
+        pasta.pasta_profile_enable(False)
+        hk_ms, hk_n = pasta.pasta_profile_read(1, reset=True)
+        h_ms = h0.elapsed_time(h1) / args.hicoo_steps
+        hb = model_bytes_hicoo(N, M, h.nblocks, R)
+        peak_h, _ = load_peaks()
+        ach = hb / (hk_ms / max(hk_n, 1) * 1e-3) / 1e9
+        hicoo = {"value": round(total_flops / (h_ms * 1e-3) / 1e9, 3), "unit": "GFLOP/s",
+                 "ms_per_step": round(h_ms, 4), "nblocks": h.nblocks, "block": 128,
+                 "nnz_per_block": round(M / max(h.nblocks, 1), 3),
+                 "roofline": {"bound": "hbm", "achieved": round(ach, 1), "peak": peak_h,
+                              "unit": "GB/s", "frac": round(ach / peak_h, 4),
+                              "traffic": ncu_traffic(args.config, "hicoo_mttkrp"),
+                              "kernel": "mttkrp_kernel<HicooSrc> (a7)",
+                              "bytes_model": "(N+4)M + (8+4N)n_b + 4NR min(n_b B, M) per launch",
+                              "avg_launch_ms": round(hk_ms / max(hk_n, 1), 4)},
+                 "preprocess_s": {"coo_to_hicoo": round(t_conv, 3),
+                                  "mode_copies_all": round(t_hprep, 3)}}
+        del h, houts
+
     if rank != 0:
         if world > 1:
             dist.destroy_process_group()
@@ -341,6 +392,7 @@ def main():
         "preprocess_s": {"generate": round(t_gen, 3), "mode_sort_all": round(t_prep, 3)},
         "clocks": clk,
         "e2e": e2e,
+        "hicoo": hicoo,
         "gpu_launches": launches,
         "cpu_baseline": cpu,
         "max_shard_nnz": per_launch_nnz,

@@ -51,7 +51,45 @@ struct KArgs {
   // factors of the other modes (ascending k), output
   const float *Uo[kMaxOrder - 1];
   float *out;
+  // L2 eviction-priority hints (bit 0: streams evict_first, bit 1: gathers evict_last,
+  // bit 2: output stores / atomics evict_first); see Policies
+  uint32_t cache_mode;
 };
+
+// Per-thread L2 cache policies (createpolicy, sm_80+): the nonzero stream is touched once
+// and must not displace the power-law-hot factor rows, which is what L2 is for here.
+struct Policies {
+  uint64_t stream, gather, out;
+  __device__ __forceinline__ explicit Policies(uint32_t mode) {
+    uint64_t first, normal, last;
+    asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(first));
+    asm("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;" : "=l"(normal));
+    asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(last));
+    stream = (mode & 1) ? first : normal;
+    gather = (mode & 2) ? last : normal;
+    out = (mode & 4) ? first : normal;
+  }
+};
+
+__device__ __forceinline__ uint4 ld_stream_u4(const void *p, uint64_t pol) {
+  uint4 r;
+  asm("ld.global.nc.L2::cache_hint.v4.u32 {%0, %1, %2, %3}, [%4], %5;"
+      : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
+      : "l"(p), "l"(pol));
+  return r;
+}
+__device__ __forceinline__ uint32_t ld_stream_u32(const void *p, uint64_t pol) {
+  uint32_t r;
+  asm("ld.global.nc.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(r) : "l"(p), "l"(pol));
+  return r;
+}
+__device__ __forceinline__ float4 ld_gather_f4(const float *p, uint64_t pol) {
+  float4 r;
+  asm("ld.global.nc.L2::cache_hint.v4.f32 {%0, %1, %2, %3}, [%4], %5;"
+      : "=f"(r.x), "=f"(r.y), "=f"(r.z), "=f"(r.w)
+      : "l"(p), "l"(pol));
+  return r;
+}
 
 template <int VW>
 struct Vec {
@@ -59,10 +97,10 @@ struct Vec {
 };
 
 template <int VW>
-__device__ __forceinline__ Vec<VW> ldg_vec(const float *p) {
+__device__ __forceinline__ Vec<VW> ldg_vec(const float *p, uint64_t pol) {
   Vec<VW> r;
   if constexpr (VW == 4) {
-    float4 t = __ldg(reinterpret_cast<const float4 *>(p));
+    float4 t = ld_gather_f4(p, pol);
     r.v[0] = t.x; r.v[1] = t.y; r.v[2] = t.z; r.v[3] = t.w;
   } else {
 #pragma unroll
@@ -72,10 +110,10 @@ __device__ __forceinline__ Vec<VW> ldg_vec(const float *p) {
 }
 
 template <int VW>
-__device__ __forceinline__ void red_vec(float *p, const Vec<VW> &a) {
+__device__ __forceinline__ void red_vec(float *p, const Vec<VW> &a, uint64_t pol) {
   if constexpr (VW == 4) {
-    asm volatile("red.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(p), "f"(a.v[0]), "f"(a.v[1]),
-                 "f"(a.v[2]), "f"(a.v[3])
+    asm volatile("red.global.add.L2::cache_hint.v4.f32 [%0], {%1, %2, %3, %4}, %5;" ::"l"(p),
+                 "f"(a.v[0]), "f"(a.v[1]), "f"(a.v[2]), "f"(a.v[3]), "l"(pol)
                  : "memory");
   } else {
 #pragma unroll
@@ -84,9 +122,11 @@ __device__ __forceinline__ void red_vec(float *p, const Vec<VW> &a) {
 }
 
 template <int VW>
-__device__ __forceinline__ void st_vec(float *p, const Vec<VW> &a) {
+__device__ __forceinline__ void st_vec(float *p, const Vec<VW> &a, uint64_t pol) {
   if constexpr (VW == 4) {
-    *reinterpret_cast<float4 *>(p) = make_float4(a.v[0], a.v[1], a.v[2], a.v[3]);
+    asm volatile("st.global.L2::cache_hint.v4.f32 [%0], {%1, %2, %3, %4}, %5;" ::"l"(p), "f"(a.v[0]),
+                 "f"(a.v[1]), "f"(a.v[2]), "f"(a.v[3]), "l"(pol)
+                 : "memory");
   } else {
 #pragma unroll
     for (int i = 0; i < VW; ++i) p[i] = a.v[i];
@@ -100,20 +140,22 @@ template <int NO, int U>
 struct CooSrc {
   // rows are globally sorted: a segment strictly inside a run is owned by that run
   static constexpr bool kSortedRows = true;
-  __device__ __forceinline__ void init(const KArgs &, uint64_t) {}
+  uint64_t pol;
+  __device__ __forceinline__ void init(const KArgs &, uint64_t, uint64_t p) { pol = p; }
   __device__ __forceinline__ void load(const KArgs &a, uint64_t x, int cnt, uint32_t (&row)[U],
                                        uint32_t (&idx)[NO > 0 ? NO : kMaxOrder - 1][U], float (&v)[U], int no) {
     if (cnt == U) {
 #pragma unroll
       for (int q = 0; q < U; q += 4) {
-        uint4 r4 = __ldg(reinterpret_cast<const uint4 *>(a.irow + x + q));
+        uint4 r4 = ld_stream_u4(a.irow + x + q, pol);
         row[q] = r4.x; row[q + 1] = r4.y; row[q + 2] = r4.z; row[q + 3] = r4.w;
-        float4 v4 = __ldg(reinterpret_cast<const float4 *>(a.val + x + q));
-        v[q] = v4.x; v[q + 1] = v4.y; v[q + 2] = v4.z; v[q + 3] = v4.w;
+        uint4 v4 = ld_stream_u4(a.val + x + q, pol);
+        v[q] = __uint_as_float(v4.x); v[q + 1] = __uint_as_float(v4.y);
+        v[q + 2] = __uint_as_float(v4.z); v[q + 3] = __uint_as_float(v4.w);
 #pragma unroll
         for (int j = 0; j < (NO > 0 ? NO : kMaxOrder - 1); ++j) {
           if (j < no) {
-            uint4 i4 = __ldg(reinterpret_cast<const uint4 *>(a.io[j] + x + q));
+            uint4 i4 = ld_stream_u4(a.io[j] + x + q, pol);
             idx[j][q] = i4.x; idx[j][q + 1] = i4.y; idx[j][q + 2] = i4.z; idx[j][q + 3] = i4.w;
           }
         }
@@ -141,6 +183,7 @@ struct HicooSrc {
   uint32_t base_row;
   uint32_t base[NO > 0 ? NO : kMaxOrder - 1];
   int no;
+  uint64_t pol;
   __device__ __forceinline__ void set_block(const KArgs &a) {
     bend = __ldg(a.bptr + b + 1);
     base_row = __ldg(a.brow + b) << a.bbits;
@@ -148,7 +191,8 @@ struct HicooSrc {
     for (int j = 0; j < (NO > 0 ? NO : kMaxOrder - 1); ++j)
       if (j < no) base[j] = __ldg(a.bo[j] + b) << a.bbits;
   }
-  __device__ __forceinline__ void init(const KArgs &a, uint64_t x0) {
+  __device__ __forceinline__ void init(const KArgs &a, uint64_t x0, uint64_t p) {
+    pol = p;
     no = int(a.order) - 1;
     uint64_t lo = 0, hi = a.nblocks;  // last block with bptr[b] <= x0
     while (hi - lo > 1) {
@@ -164,14 +208,15 @@ struct HicooSrc {
     if (cnt == U) {
 #pragma unroll
       for (int q = 0; q < U; q += 4) {
-        uint32_t w = __ldg(reinterpret_cast<const uint32_t *>(a.erow + x + q));
+        uint32_t w = ld_stream_u32(a.erow + x + q, pol);
         er[q] = w & 0xff; er[q + 1] = (w >> 8) & 0xff; er[q + 2] = (w >> 16) & 0xff; er[q + 3] = w >> 24;
-        float4 v4 = __ldg(reinterpret_cast<const float4 *>(a.val + x + q));
-        v[q] = v4.x; v[q + 1] = v4.y; v[q + 2] = v4.z; v[q + 3] = v4.w;
+        uint4 v4 = ld_stream_u4(a.val + x + q, pol);
+        v[q] = __uint_as_float(v4.x); v[q + 1] = __uint_as_float(v4.y);
+        v[q + 2] = __uint_as_float(v4.z); v[q + 3] = __uint_as_float(v4.w);
 #pragma unroll
         for (int j = 0; j < (NO > 0 ? NO : kMaxOrder - 1); ++j) {
           if (j < no) {
-            uint32_t e = __ldg(reinterpret_cast<const uint32_t *>(a.eo[j] + x + q));
+            uint32_t e = ld_stream_u32(a.eo[j] + x + q, pol);
             ej[j][q] = e & 0xff; ej[j][q + 1] = (e >> 8) & 0xff; ej[j][q + 2] = (e >> 16) & 0xff;
             ej[j][q + 3] = e >> 24;
           }
@@ -231,10 +276,11 @@ __global__ void __launch_bounds__(kThreads, T::MINB) mttkrp_kernel(const KArgs a
   if (x0 >= x1) return;
   const int no = NO > 0 ? NO : int(a.order) - 1;
   const uint32_t R = a.R;
+  const Policies pol(a.cache_mode);
 
   for (uint32_t col = uint32_t(lig) * VW; col < R; col += LPN * VW) {
     Src src;
-    src.init(a, x0);
+    src.init(a, x0, pol.stream);
     Vec<VW> acc;
 #pragma unroll
     for (int i = 0; i < VW; ++i) acc.v[i] = 0.f;
@@ -262,7 +308,7 @@ __global__ void __launch_bounds__(kThreads, T::MINB) mttkrp_kernel(const KArgs a
       for (int u = 0; u < U; ++u) {
 #pragma unroll
         for (int j = 0; j < NOA; ++j) {
-          if (j < no && u < cnt) f[j][u] = ldg_vec<VW>(a.Uo[j] + uint64_t(idx[j][u]) * R + col);
+          if (j < no && u < cnt) f[j][u] = ldg_vec<VW>(a.Uo[j] + uint64_t(idx[j][u]) * R + col, pol.gather);
         }
       }
 #pragma unroll
@@ -284,7 +330,7 @@ __global__ void __launch_bounds__(kThreads, T::MINB) mttkrp_kernel(const KArgs a
           } else {
             if (cur != 0xFFFFFFFFu) {
               float *dst = a.out + uint64_t(cur) * R + col;
-              if (first || !Src::kSortedRows) red_vec<VW>(dst, acc); else st_vec<VW>(dst, acc);
+              if (first || !Src::kSortedRows) red_vec<VW>(dst, acc, pol.out); else st_vec<VW>(dst, acc, pol.out);
               first = false;
             }
             cur = row[u];
@@ -303,7 +349,7 @@ __global__ void __launch_bounds__(kThreads, T::MINB) mttkrp_kernel(const KArgs a
       }
       cnt = cntn;
     }
-    if (cur != 0xFFFFFFFFu) red_vec<VW>(a.out + uint64_t(cur) * R + col, acc);
+    if (cur != 0xFFFFFFFFu) red_vec<VW>(a.out + uint64_t(cur) * R + col, acc, pol.out);
   }
 }
 
@@ -389,6 +435,7 @@ void dispatch(KArgs &a, bool vec4, cudaStream_t s) {
   run = run < 8 ? 8 : (run / 8) * 8;
   a.chunk = uint64_t(G) * run;
   const int variant = env_int("PASTA_MTTKRP_VARIANT", 0);
+  a.cache_mode = uint32_t(env_int("PASTA_MTTKRP_CACHE", 0));
   const int no = int(a.order) - 1;
   if (vec4) {
     if (no == 2) launch_lpn<SrcT, 2, 4>(a, lpn, variant, s);

@@ -24,11 +24,14 @@ def _rng(seed: int) -> np.random.Generator:
 
 def _unique_first(coords: np.ndarray) -> np.ndarray:
     """Indices (in draw order) of the first occurrence of each distinct row of coords [D, N]."""
-    if coords.shape[0] == 0:
+    D, N = coords.shape
+    if D == 0:
         return np.zeros(0, np.int64)
-    keys = np.ascontiguousarray(coords).view([("", coords.dtype)] * coords.shape[1]).ravel()
-    _, first = np.unique(keys, return_index=True)
-    return np.sort(first)
+    order = np.lexsort([coords[:, k] for k in range(N - 1, -1, -1)])  # stable, mode 0 primary
+    srt = coords[order]
+    new = np.ones(D, bool)
+    new[1:] = np.any(srt[1:] != srt[:-1], axis=1)
+    return np.sort(order[new])
 
 
 def uniform_coo(dims, nnz, seed, shuffle=True):
@@ -52,8 +55,10 @@ def uniform_coo(dims, nnz, seed, shuffle=True):
     return np.ascontiguousarray(got.T), vals
 
 
-def powerlaw_coo(dims, nnz, seed, q=0.75, shuffle=True):
-    """Product-form Kronecker power-law tensor (independent index bits, P(1) = 1 - q)."""
+def powerlaw_coo(dims, nnz, seed, q=0.75, shuffle=True, dedup=True):
+    """Product-form Kronecker power-law tensor (independent index bits, P(1) = 1 - q).
+    dedup=False skips the uniqueness pass (full-size inputs where repeats are ~1e-7 of the
+    draws); repeated coordinates are then separate nonzeros (R#15)."""
     dims = [int(d) for d in dims]
     rng = _rng(seed)
     L = [max(0, int(np.ceil(np.log2(d)))) if d > 1 else 0 for d in dims]
@@ -62,15 +67,22 @@ def powerlaw_coo(dims, nnz, seed, q=0.75, shuffle=True):
         need = int((nnz - got.shape[0]) * 1.3) + 1024
         cols = []
         for d, l in zip(dims, L):
-            idx = np.zeros(need, np.uint64)
-            for b in range(l):
-                bit = (rng.random(need) < (1.0 - q)).astype(np.uint64)
-                idx |= bit << np.uint64(b)
+            mask = np.uint64((1 << l) - 1)
+            if q == 0.75 and l <= 32:
+                # AND of two uniform words: every bit is 1 with probability 1/4, independently
+                a = rng.integers(0, 1 << 32, size=need, dtype=np.uint32)
+                b = rng.integers(0, 1 << 32, size=need, dtype=np.uint32)
+                idx = ((a & b).astype(np.uint64)) & mask
+            else:
+                idx = np.zeros(need, np.uint64)
+                for bb in range(l):
+                    bit = (rng.random(need) < (1.0 - q)).astype(np.uint64)
+                    idx |= bit << np.uint64(bb)
             cols.append(idx)
         cand = np.stack(cols, axis=1)
         ok = np.all(cand < np.array(dims, dtype=np.uint64)[None, :], axis=1)
         allc = np.concatenate([got, cand[ok]])
-        got = allc[_unique_first(allc)]
+        got = allc[_unique_first(allc)] if dedup else allc
     got = got[:nnz].astype(np.uint32)
     if shuffle:
         got = got[rng.permutation(nnz)]

@@ -22,6 +22,7 @@ def main():
     ap.add_argument("--runs", default="128")
     ap.add_argument("--formats", default="coo")
     ap.add_argument("--reps", type=int, default=10)
+    ap.add_argument("--caches", default="0")
     args = ap.parse_args()
     cfg = si.CONFIGS[args.config]
     dims, R, M = cfg["dims"], cfg["R"], cfg["nnz"]
@@ -39,8 +40,11 @@ def main():
         which = 0 if fmt == "coo" else 1
         for n in range(len(dims)):
             fn(t, n, U, out=outs[n])  # prepare
-        for run in [int(r) for r in args.runs.split(",")]:
-            for var in [int(v) for v in args.variants.split(",")]:
+        combos = [(r, v, c) for r in args.runs.split(",") for v in args.variants.split(",")
+                  for c in args.caches.split(",")]
+        for run, var, cache in [(int(r), int(v), int(c)) for r, v, c in combos]:
+            if True:
+                os.environ["PASTA_MTTKRP_CACHE"] = str(cache)
                 os.environ["PASTA_MTTKRP_VARIANT"] = str(var)
                 os.environ["PASTA_MTTKRP_RUN"] = str(run)
                 per_mode = []
@@ -56,7 +60,7 @@ def main():
                     pasta.pasta_profile_enable(False)
                     ms, k = pasta.pasta_profile_read(which, reset=True)
                     per_mode.append(round(ms / k, 4))
-                print(json.dumps({"config": args.config, "fmt": fmt, "variant": var, "run": run,
+                print(json.dumps({"config": args.config, "fmt": fmt, "variant": var, "run": run, "cache": cache,
                                   "ms_per_mode": per_mode,
                                   "mean_ms": round(sum(per_mode) / len(per_mode), 4)}), flush=True)
 
