@@ -2,6 +2,9 @@
 // HiCOO working copy used by the GPU MTTKRP (R#27).
 #include <cub/cub.cuh>
 
+#include <cstdlib>
+#include <vector>
+
 #include "internal.cuh"
 
 namespace pasta {
@@ -83,6 +86,68 @@ __global__ void u8_to_u32_kernel(const uint8_t *__restrict__ in, uint64_t M, uin
     out[x] = in[x];
 }
 
+// light[x] = 1 iff the block of entry x holds fewer than heavy_min entries
+__global__ void light_entry_kernel(const uint64_t *__restrict__ bptr, const uint32_t *__restrict__ blk,
+                                   uint64_t M, uint32_t heavy_min, uint32_t *__restrict__ light) {
+  for (uint64_t x = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; x < M;
+       x += uint64_t(gridDim.x) * blockDim.x) {
+    uint32_t b = blk[x];
+    light[x] = (bptr[b + 1] - bptr[b]) < heavy_min ? 1u : 0u;
+  }
+}
+
+__global__ void light_block_kernel(const uint64_t *__restrict__ bptr, uint64_t nb, uint32_t heavy_min,
+                                   uint32_t *__restrict__ light) {
+  for (uint64_t b = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; b < nb;
+       b += uint64_t(gridDim.x) * blockDim.x)
+    light[b] = (bptr[b + 1] - bptr[b]) < heavy_min ? 1u : 0u;
+}
+
+__global__ void piece_count_kernel(const uint64_t *__restrict__ bptr, uint64_t nh, uint32_t piece,
+                                   uint64_t *__restrict__ cnt) {
+  for (uint64_t s = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; s <= nh;
+       s += uint64_t(gridDim.x) * blockDim.x)
+    cnt[s] = s == nh ? 0 : (bptr[s + 1] - bptr[s] + piece - 1) / piece;
+}
+
+__global__ void piece_emit_kernel(const uint64_t *__restrict__ off, uint64_t nh, uint32_t *__restrict__ out) {
+  for (uint64_t s = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; s < nh;
+       s += uint64_t(gridDim.x) * blockDim.x)
+    for (uint64_t j = off[s]; j < off[s + 1]; ++j) {
+      out[2 * j] = uint32_t(s);
+      out[2 * j + 1] = uint32_t(j - off[s]);
+    }
+}
+
+// rowslice: flag[x] = 1 iff position x starts a new (block, einds_mode) slice
+__global__ void slice_flag_kernel(const uint32_t *__restrict__ blkp, const uint32_t *__restrict__ enp,
+                                  uint64_t M, uint8_t *__restrict__ flag) {
+  for (uint64_t x = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; x < M;
+       x += uint64_t(gridDim.x) * blockDim.x)
+    flag[x] = (x == 0) || blkp[x] != blkp[x - 1] || enp[x] != enp[x - 1];
+}
+
+struct SliceOut {
+  const uint32_t *binds[kMaxOrder];
+  uint32_t *base[kMaxOrder];
+  uint32_t order, mode, bbits;
+};
+
+__global__ void slice_emit_kernel(SliceOut o, const uint32_t *__restrict__ starts, uint64_t nsb, uint64_t M,
+                                  const uint32_t *__restrict__ blkp, const uint32_t *__restrict__ enp,
+                                  uint64_t *__restrict__ sbptr, uint32_t *__restrict__ sbrow) {
+  for (uint64_t j = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; j <= nsb;
+       j += uint64_t(gridDim.x) * blockDim.x) {
+    if (j == nsb) { sbptr[nsb] = M; continue; }
+    uint32_t x = starts[j];
+    uint32_t b = blkp[x];
+    sbptr[j] = x;
+    sbrow[j] = (o.binds[o.mode][b] << o.bbits) + enp[x];
+    for (uint32_t k = 0; k < o.order; ++k)
+      if (k != o.mode) o.base[k][j] = o.binds[k][b] << o.bbits;
+  }
+}
+
 __global__ void sched_counts_kernel(const uint64_t *__restrict__ bptr, const uint32_t *__restrict__ sched,
                                     uint64_t nb, uint64_t *__restrict__ cnt) {
   for (uint64_t s = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; s <= nb;
@@ -146,11 +211,80 @@ void coo_to_hicoo_device(const pasta_coo *x, pasta_hicoo *h, cudaStream_t s) {
   PASTA_CUDA(cudaStreamSynchronize(s));
 }
 
-// Per-mode copy (R#27): blocks stably sorted by binds_mode, entries inside a block stably
-// sorted by einds_mode, so equal output rows are contiguous runs (segmented reduction).
+// Per-mode copy (R#27): blocks stably sorted by (light, binds_mode), entries inside a block
+// stably sorted by einds_mode, so equal output rows are contiguous runs (segmented
+// reduction); heavy blocks come first and get CTA work items (pieces) for the tile-staged
+// kernel.
+static void hicoo_prepare_rowslice(pasta_hicoo *h, uint32_t mode, cudaStream_t s) {
+  HicooModeCopy &mc = h->mc[mode];
+  const uint32_t N = h->order;
+  const uint64_t M = h->nnz, nb = h->nblocks;
+  const uint32_t bb = h->block_bits;
+  mc.layout = 0;
+  for (uint32_t k = 0; k < N; ++k)
+    if (k != mode) mc.einds[k].alloc(M, s);
+  mc.val.alloc(M, s);
+  if (M == 0) {
+    mc.nsb = 0;
+    mc.sbptr.alloc(1, s);
+    uint64_t zero = 0;
+    PASTA_CUDA(cudaMemcpyAsync(mc.sbptr.p, &zero, sizeof(zero), cudaMemcpyHostToDevice, s));
+    PASTA_CUDA(cudaStreamSynchronize(s));
+    mc.ready = true;
+    return;
+  }
+  // entry order: (binds_mode[blk], einds_mode, blk); ties keep Morton order (stable)
+  DevArray<uint32_t> blk(M, s), c0(M, s), en(M, s);
+  entry_block_kernel<<<grid_for(M), kThreads, 0, s>>>(h->bptr.p, nb, M, blk.p);
+  PASTA_LAUNCHED();
+  gather_binds_kernel<<<grid_for(M), kThreads, 0, s>>>(h->binds[mode].p, blk.p, M, c0.p);
+  PASTA_LAUNCHED();
+  u8_to_u32_kernel<<<grid_for(M), kThreads, 0, s>>>(h->einds[mode].p, M, en.p);
+  PASTA_LAUNCHED();
+  uint64_t nbr = (uint64_t(h->dims[mode]) + (1ull << bb) - 1) >> bb;
+  const uint32_t *comps[3] = {c0.p, en.p, blk.p};
+  uint32_t bits[3] = {ceil_log2(nbr), bb, ceil_log2(nb)};
+  DevArray<uint32_t> perm(M, s);
+  iota_u32(perm.p, M, s);
+  lexsort(comps, bits, 3, perm, M, s);
+  c0.reset();
+  DevArray<uint32_t> blkp(M, s), enp(M, s);
+  gather_u32(blk.p, perm.p, blkp.p, M, s);
+  gather_u32(en.p, perm.p, enp.p, M, s);
+  for (uint32_t k = 0; k < N; ++k)
+    if (k != mode) gather_u8(h->einds[k].p, perm.p, mc.einds[k].p, M, s);
+  gather_f32(h->val.p, perm.p, mc.val.p, M, s);
+  DevArray<uint8_t> flag(M, s);
+  slice_flag_kernel<<<grid_for(M), kThreads, 0, s>>>(blkp.p, enp.p, M, flag.p);
+  PASTA_LAUNCHED();
+  DevArray<uint32_t> starts;
+  mc.nsb = select_flagged(flag.p, M, starts, s);
+  mc.sbptr.alloc(mc.nsb + 1, s);
+  mc.sbrow.alloc(mc.nsb, s);
+  SliceOut o{};
+  o.order = N;
+  o.mode = mode;
+  o.bbits = bb;
+  for (uint32_t k = 0; k < N; ++k) {
+    o.binds[k] = h->binds[k].p;
+    if (k != mode) {
+      mc.sbbase[k].alloc(mc.nsb, s);
+      o.base[k] = mc.sbbase[k].p;
+    }
+  }
+  slice_emit_kernel<<<grid_for(mc.nsb + 1), kThreads, 0, s>>>(o, starts.p, mc.nsb, M, blkp.p, enp.p,
+                                                              mc.sbptr.p, mc.sbrow.p);
+  PASTA_LAUNCHED();
+  PASTA_CUDA(cudaStreamSynchronize(s));
+  mc.ready = true;
+}
+
 void hicoo_prepare_mode(pasta_hicoo *h, uint32_t mode, cudaStream_t s) {
   HicooModeCopy &mc = h->mc[mode];
   if (mc.ready) return;
+  const char *lay = getenv("PASTA_HICOO_LAYOUT");
+  if (!(lay && std::string(lay) == "block")) return hicoo_prepare_rowslice(h, mode, s);
+  mc.layout = 1;
   const uint32_t N = h->order;
   const uint64_t M = h->nnz, nb = h->nblocks;
   const uint32_t bb = h->block_bits;
@@ -167,28 +301,37 @@ void hicoo_prepare_mode(pasta_hicoo *h, uint32_t mode, cudaStream_t s) {
     mc.ready = true;
     return;
   }
-  // entry permutation: (binds_mode[blk], blk, einds_mode)
-  DevArray<uint32_t> blk(M, s), c0(M, s), c2(M, s);
+  // Heavy blocks (>= heavy_min entries: staging their factor tiles pays, Table I's
+  // min{n_b B, M} term) go first, light ones after; each part by binds_mode.
+  const char *env = getenv("PASTA_HICOO_HEAVY");
+  mc.heavy_min = (env && *env) ? uint32_t(atoi(env)) : 256u;
+  if (mc.heavy_min == 0) mc.heavy_min = 0xFFFFFFFFu;  // 0 disables the heavy path
+  // entry permutation: (light[blk], binds_mode[blk], blk, einds_mode)
+  DevArray<uint32_t> blk(M, s), c0(M, s), c2(M, s), lt(M, s);
   entry_block_kernel<<<grid_for(M), kThreads, 0, s>>>(h->bptr.p, nb, M, blk.p);
   PASTA_LAUNCHED();
   gather_binds_kernel<<<grid_for(M), kThreads, 0, s>>>(h->binds[mode].p, blk.p, M, c0.p);
   PASTA_LAUNCHED();
   u8_to_u32_kernel<<<grid_for(M), kThreads, 0, s>>>(h->einds[mode].p, M, c2.p);
   PASTA_LAUNCHED();
+  light_entry_kernel<<<grid_for(M), kThreads, 0, s>>>(h->bptr.p, blk.p, M, mc.heavy_min, lt.p);
+  PASTA_LAUNCHED();
   uint64_t nbr = (uint64_t(h->dims[mode]) + (1ull << bb) - 1) >> bb;  // block rows of this mode
-  const uint32_t *comps[3] = {c0.p, blk.p, c2.p};
-  uint32_t bits[3] = {ceil_log2(nbr), ceil_log2(nb), bb};
+  const uint32_t *comps[4] = {lt.p, c0.p, blk.p, c2.p};
+  uint32_t bits[4] = {1, ceil_log2(nbr), ceil_log2(nb), bb};
   DevArray<uint32_t> perm(M, s);
   iota_u32(perm.p, M, s);
-  lexsort(comps, bits, 3, perm, M, s);
+  lexsort(comps, bits, 4, perm, M, s);
   for (uint32_t k = 0; k < N; ++k) gather_u8(h->einds[k].p, perm.p, mc.einds[k].p, M, s);
   gather_f32(h->val.p, perm.p, mc.val.p, M, s);
-  // block schedule: blocks stably sorted by binds_mode (same order the entries now follow)
-  DevArray<uint32_t> sched(nb, s);
+  // block schedule: blocks stably sorted by (light, binds_mode), the order entries now follow
+  DevArray<uint32_t> sched(nb, s), blt(nb, s);
   iota_u32(sched.p, nb, s);
-  const uint32_t *bc[1] = {h->binds[mode].p};
-  uint32_t bbit[1] = {ceil_log2(nbr)};
-  lexsort(bc, bbit, 1, sched, nb, s);
+  light_block_kernel<<<grid_for(nb), kThreads, 0, s>>>(h->bptr.p, nb, mc.heavy_min, blt.p);
+  PASTA_LAUNCHED();
+  const uint32_t *bc[2] = {blt.p, h->binds[mode].p};
+  uint32_t bbit[2] = {1, ceil_log2(nbr)};
+  lexsort(bc, bbit, 2, sched, nb, s);
   DevArray<uint64_t> cnt(nb + 1, s);
   sched_counts_kernel<<<grid_for(nb + 1), kThreads, 0, s>>>(h->bptr.p, sched.p, nb, cnt.p);
   PASTA_LAUNCHED();
@@ -197,6 +340,34 @@ void hicoo_prepare_mode(pasta_hicoo *h, uint32_t mode, cudaStream_t s) {
   DevArray<uint8_t> tmp(tmp_bytes, s);
   PASTA_CUDA(cub::DeviceScan::ExclusiveSum(tmp.p, tmp_bytes, cnt.p, mc.bptr.p, nb + 1, s));
   count_launch();
+  // number of heavy blocks = blocks whose light flag is 0
+  {
+    std::vector<uint32_t> hl(nb);
+    PASTA_CUDA(cudaMemcpyAsync(hl.data(), blt.p, nb * sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
+    PASTA_CUDA(cudaStreamSynchronize(s));
+    uint64_t nh = 0;
+    for (uint64_t b = 0; b < nb; ++b) nh += hl[b] == 0;
+    mc.n_heavy = nh;
+  }
+  PASTA_CUDA(cudaMemcpyAsync(&mc.heavy_nnz, mc.bptr.p + mc.n_heavy, sizeof(uint64_t),
+                             cudaMemcpyDeviceToHost, s));
+  PASTA_CUDA(cudaStreamSynchronize(s));
+  // CTA work items of the heavy part: (block, piece) with at most `piece` entries each
+  if (mc.n_heavy) {
+    DevArray<uint64_t> pc(mc.n_heavy + 1, s), off(mc.n_heavy + 1, s);
+    piece_count_kernel<<<grid_for(mc.n_heavy + 1), kThreads, 0, s>>>(mc.bptr.p, mc.n_heavy, mc.piece, pc.p);
+    PASTA_LAUNCHED();
+    size_t tb = 0;
+    PASTA_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, tb, pc.p, off.p, mc.n_heavy + 1, s));
+    DevArray<uint8_t> t2(tb, s);
+    PASTA_CUDA(cub::DeviceScan::ExclusiveSum(t2.p, tb, pc.p, off.p, mc.n_heavy + 1, s));
+    count_launch();
+    PASTA_CUDA(cudaMemcpyAsync(&mc.n_pieces, off.p + mc.n_heavy, sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
+    PASTA_CUDA(cudaStreamSynchronize(s));
+    mc.pieces.alloc(2 * mc.n_pieces, s);
+    piece_emit_kernel<<<grid_for(mc.n_heavy), kThreads, 0, s>>>(off.p, mc.n_heavy, mc.pieces.p);
+    PASTA_LAUNCHED();
+  }
   for (uint32_t k = 0; k < N; ++k) gather_u32(h->binds[k].p, sched.p, mc.binds[k].p, nb, s);
   PASTA_CUDA(cudaStreamSynchronize(s));
   mc.ready = true;

@@ -87,10 +87,27 @@ struct CooModeCopy {
 
 struct HicooModeCopy {
   bool ready = false;
+  // blocks ordered (heavy first, then light; each part by binds_mode), entries inside a block
+  // by einds_mode (R#27)
   DevArray<uint64_t> bptr;               // nblocks + 1
   DevArray<uint32_t> binds[kMaxOrder];   // nblocks each
   DevArray<uint8_t> einds[kMaxOrder];    // nnz each
   DevArray<float> val;                   // nnz
+  uint64_t n_heavy = 0;                  // blocks [0, n_heavy) hold >= heavy_min entries
+  uint64_t heavy_nnz = 0;                // = bptr[n_heavy]
+  uint32_t heavy_min = 0;
+  uint32_t piece = 4096;                 // max entries per CTA work item
+  DevArray<uint32_t> pieces;             // 2 per item: (block, piece index within block)
+  uint64_t n_pieces = 0;
+  // layout 0 ("row slices", default): entries sorted by output row across the blocks of a
+  // block row; a slice = the entries of one block sharing einds_mode, with its own row and
+  // other-mode block bases.  Uses einds[k] (k != mode) and val; not bptr/binds/pieces.
+  // layout 1 ("blocks"): the block-major copy above (heavy blocks TMA-staged).
+  int layout = 0;
+  uint64_t nsb = 0;
+  DevArray<uint64_t> sbptr;              // nsb + 1
+  DevArray<uint32_t> sbrow;              // nsb: output row of the slice
+  DevArray<uint32_t> sbbase[kMaxOrder];  // nsb each (k != mode): binds_k << block_bits
 };
 
 }  // namespace pasta

@@ -33,7 +33,10 @@ constexpr int kWarpsPerCta = 8;
 constexpr int kThreads = kWarpsPerCta * 32;
 
 struct KArgs {
-  uint64_t nnz;
+  uint64_t nnz;      // absolute end of the processed range
+  uint64_t x_begin;  // absolute start (multiple of 4)
+  uint64_t x_skip;   // entries below this absolute position are not processed
+  uint64_t b_begin;  // HiCOO: first block of the range
   uint64_t chunk;  // nonzeros per warp; chunk % (4 * G) == 0
   uint32_t order, R;
   // COO streams (mode-n copy)
@@ -48,6 +51,11 @@ struct KArgs {
   const uint8_t *erow;
   const uint8_t *eo[kMaxOrder - 1];
   uint32_t bbits;
+  // HiCOO row-slice copy (layout 0)
+  const uint64_t *sbptr;
+  uint64_t nsb;
+  const uint32_t *sbrow;
+  const uint32_t *sbbase[kMaxOrder - 1];
   // factors of the other modes (ascending k), output
   const float *Uo[kMaxOrder - 1];
   float *out;
@@ -144,7 +152,7 @@ struct CooSrc {
   __device__ __forceinline__ void init(const KArgs &, uint64_t, uint64_t p) { pol = p; }
   __device__ __forceinline__ void load(const KArgs &a, uint64_t x, int cnt, uint32_t (&row)[U],
                                        uint32_t (&idx)[NO > 0 ? NO : kMaxOrder - 1][U], float (&v)[U], int no) {
-    if (cnt == U) {
+    if (cnt == U && (x & 3) == 0) {
 #pragma unroll
       for (int q = 0; q < U; q += 4) {
         uint4 r4 = ld_stream_u4(a.irow + x + q, pol);
@@ -194,7 +202,7 @@ struct HicooSrc {
   __device__ __forceinline__ void init(const KArgs &a, uint64_t x0, uint64_t p) {
     pol = p;
     no = int(a.order) - 1;
-    uint64_t lo = 0, hi = a.nblocks;  // last block with bptr[b] <= x0
+    uint64_t lo = a.b_begin, hi = a.nblocks;  // last block with bptr[b] <= x0
     while (hi - lo > 1) {
       uint64_t mid = (lo + hi) / 2;
       if (__ldg(a.bptr + mid) <= x0) lo = mid; else hi = mid;
@@ -205,7 +213,7 @@ struct HicooSrc {
   __device__ __forceinline__ void load(const KArgs &a, uint64_t x, int cnt, uint32_t (&row)[U],
                                        uint32_t (&idx)[NO > 0 ? NO : kMaxOrder - 1][U], float (&v)[U], int) {
     uint32_t er[U], ej[NO > 0 ? NO : kMaxOrder - 1][U];
-    if (cnt == U) {
+    if (cnt == U && (x & 3) == 0) {
 #pragma unroll
       for (int q = 0; q < U; q += 4) {
         uint32_t w = ld_stream_u32(a.erow + x + q, pol);
@@ -247,6 +255,95 @@ struct HicooSrc {
   }
 };
 
+// HiCOO row-slice policy (layout 0, R#27): a slice = the entries of one block that share
+// einds_n; slices are ordered by output row, so rows are globally sorted as in COO.  Per
+// entry only the 8-bit element indices of the other modes and the value are streamed; the
+// row and the other-mode block bases (Alg. 3's rebased pointers) come per slice.
+template <int NO, int U>
+struct HicooRowSrc {
+  static constexpr bool kSortedRows = true;
+  static constexpr int NOA = NO > 0 ? NO : kMaxOrder - 1;
+  // current slice and the next one, loaded one slice ahead so that advancing through
+  // short slices does not wait on a dependent load
+  uint64_t sb, sbend, nend;
+  uint32_t srow, nrow;
+  uint32_t base[NOA], nbase[NOA];
+  int no;
+  uint64_t pol;
+  __device__ __forceinline__ void load_next(const KArgs &a) {
+    const uint64_t n1 = sb + 1 < a.nsb ? sb + 1 : sb;  // clamp: never read past the end
+    nend = __ldg(a.sbptr + n1 + 1);
+    nrow = __ldg(a.sbrow + n1);
+#pragma unroll
+    for (int j = 0; j < NOA; ++j)
+      if (j < no) nbase[j] = __ldg(a.sbbase[j] + n1);
+  }
+  __device__ __forceinline__ void advance(const KArgs &a) {
+    ++sb;
+    sbend = nend;
+    srow = nrow;
+#pragma unroll
+    for (int j = 0; j < NOA; ++j) base[j] = nbase[j];
+    load_next(a);
+  }
+  __device__ __forceinline__ void init(const KArgs &a, uint64_t x0, uint64_t p) {
+    pol = p;
+    no = int(a.order) - 1;
+    uint64_t lo = 0, hi = a.nsb;  // last slice with sbptr[sb] <= x0
+    while (hi - lo > 1) {
+      uint64_t mid = (lo + hi) / 2;
+      if (__ldg(a.sbptr + mid) <= x0) lo = mid; else hi = mid;
+    }
+    sb = lo;
+    sbend = __ldg(a.sbptr + sb + 1);
+    srow = __ldg(a.sbrow + sb);
+#pragma unroll
+    for (int j = 0; j < NOA; ++j)
+      if (j < no) base[j] = __ldg(a.sbbase[j] + sb);
+    load_next(a);
+  }
+  __device__ __forceinline__ void load(const KArgs &a, uint64_t x, int cnt, uint32_t (&row)[U],
+                                       uint32_t (&idx)[NOA][U], float (&v)[U], int) {
+    uint32_t ej[NOA][U];
+    if (cnt == U && (x & 3) == 0) {
+#pragma unroll
+      for (int q = 0; q < U; q += 4) {
+        uint4 v4 = ld_stream_u4(a.val + x + q, pol);
+        v[q] = __uint_as_float(v4.x); v[q + 1] = __uint_as_float(v4.y);
+        v[q + 2] = __uint_as_float(v4.z); v[q + 3] = __uint_as_float(v4.w);
+#pragma unroll
+        for (int j = 0; j < NOA; ++j) {
+          if (j < no) {
+            uint32_t e = ld_stream_u32(a.eo[j] + x + q, pol);
+            ej[j][q] = e & 0xff; ej[j][q + 1] = (e >> 8) & 0xff; ej[j][q + 2] = (e >> 16) & 0xff;
+            ej[j][q + 3] = e >> 24;
+          }
+        }
+      }
+    } else {
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        if (u < cnt) {
+          v[u] = __ldg(a.val + x + u);
+#pragma unroll
+          for (int j = 0; j < NOA; ++j)
+            if (j < no) ej[j][u] = __ldg(a.eo[j] + x + u);
+        }
+      }
+    }
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      if (u < cnt) {
+        while (x + u >= sbend) advance(a);  // walk to the entry's slice
+        row[u] = srow;
+#pragma unroll
+        for (int j = 0; j < NOA; ++j)
+          if (j < no) idx[j][u] = base[j] + ej[j][u];
+      }
+    }
+  }
+};
+
 // NO = number of other modes (order - 1) when specialised, 0 = generic (<= kMaxOrder - 1).
 // Kernel variant knobs: U nonzeros per unrolled step, PF = software-pipelined prefetch of
 // the next step's index/value stream (so the stream latency hides behind the gathers),
@@ -267,12 +364,13 @@ __global__ void __launch_bounds__(kThreads, T::MINB) mttkrp_kernel(const KArgs a
   const int lane = threadIdx.x & 31;
   const int g = lane / LPN, lig = lane % LPN;
   const uint64_t w = uint64_t(blockIdx.x) * kWarpsPerCta + (threadIdx.x >> 5);
-  const uint64_t c0 = w * a.chunk;
+  const uint64_t c0 = a.x_begin + w * a.chunk;
   if (c0 >= a.nnz) return;
   const uint64_t S = a.chunk / G;
-  const uint64_t x0 = c0 + uint64_t(g) * S;
+  uint64_t x0 = c0 + uint64_t(g) * S;
   uint64_t x1 = x0 + S;
   if (x1 > a.nnz) x1 = a.nnz;
+  if (x0 < a.x_skip) x0 = a.x_skip;
   if (x0 >= x1) return;
   const int no = NO > 0 ? NO : int(a.order) - 1;
   const uint32_t R = a.R;
@@ -353,6 +451,154 @@ __global__ void __launch_bounds__(kThreads, T::MINB) mttkrp_kernel(const KArgs a
   }
 }
 
+// ---------------------------------------------------------------------------------------
+// HiCOO heavy-block kernel (a7, dense part).  One CTA per work item = one tensor block (or a
+// <= `piece`-entry slice of a huge one), the paper's HiCOO-GPU mapping, made B200-
+// native: thread 0 stages the block's (N-1) factor-row tiles U_k[bk*B .. bk*B+B) -- contiguous
+// B*R*4-byte ranges, Alg. 3's rebased pointers C_b, B_b -- into shared memory with
+// 1-D TMA bulk copies (cp.async.bulk, completion on an mbarrier); the CTA's 64 lane groups
+// then walk contiguous runs of the block's entries (sorted by einds_n), gather rows from the
+// staged tiles (LDS.128), keep rank-R partial sums in registers while einds_n repeats, and
+// flush each finished segment with one red.global.add.v4.f32.
+struct HArgs {
+  const uint32_t *pieces;
+  uint32_t piece;
+  const uint64_t *bptr;
+  const uint32_t *brow;
+  const uint32_t *bo[kMaxOrder - 1];
+  const uint8_t *erow;
+  const uint8_t *eo[kMaxOrder - 1];
+  const float *val;
+  const float *Uo[kMaxOrder - 1];
+  uint32_t dims_o[kMaxOrder - 1];
+  float *out;
+  uint32_t order, R, bbits;
+  uint32_t cache_mode;
+};
+
+__device__ __forceinline__ uint32_t smem_addr(const void *p) {
+  return uint32_t(__cvta_generic_to_shared(p));
+}
+
+__device__ __forceinline__ void mbar_wait(uint32_t addr, uint32_t parity) {
+  uint32_t done = 0;
+  do {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+        "selp.u32 %0, 1, 0, p;\n\t}"
+        : "=r"(done)
+        : "r"(addr), "r"(parity)
+        : "memory");
+  } while (!done);
+}
+
+template <int NO, int LPN>
+__global__ void __launch_bounds__(kThreads) hicoo_heavy_kernel(const HArgs a) {
+  extern __shared__ __align__(128) float tiles[];  // [no][B][R]
+  __shared__ __align__(8) uint64_t mbar;
+  constexpr int G = 32 / LPN;
+  constexpr int NOA = NO > 0 ? NO : kMaxOrder - 1;
+  constexpr int U = 4;
+  const int no = NO > 0 ? NO : int(a.order) - 1;
+  const uint32_t R = a.R;
+  const uint32_t B = 1u << a.bbits;
+  const uint32_t s = __ldg(a.pieces + 2 * blockIdx.x);
+  const uint32_t pj = __ldg(a.pieces + 2 * blockIdx.x + 1);
+  const uint64_t eb = __ldg(a.bptr + s), ee = __ldg(a.bptr + s + 1);
+  const uint64_t lo = eb + uint64_t(pj) * a.piece;
+  const uint64_t hi = (lo + a.piece < ee) ? lo + a.piece : ee;
+  const uint32_t mb = smem_addr(&mbar);
+  if (threadIdx.x == 0) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(mb) : "memory");
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    uint32_t total = 0;
+    uint32_t bytes[NOA];
+    uint64_t base[NOA];
+#pragma unroll
+    for (int j = 0; j < NOA; ++j) {
+      if (j < no) {
+        base[j] = uint64_t(__ldg(a.bo[j] + s)) << a.bbits;
+        uint64_t rows = a.dims_o[j] - base[j];
+        if (rows > B) rows = B;
+        bytes[j] = uint32_t(rows * R * 4u);
+        total += bytes[j];
+      }
+    }
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(mb), "r"(total) : "memory");
+#pragma unroll
+    for (int j = 0; j < NOA; ++j) {
+      if (j < no)
+        asm volatile(
+            "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                smem_addr(tiles + size_t(j) * B * R)),
+            "l"(a.Uo[j] + base[j] * R), "r"(bytes[j]), "r"(mb)
+            : "memory");
+    }
+  }
+  const uint32_t base_row = __ldg(a.brow + s) << a.bbits;
+  const int lane = threadIdx.x & 31, g = lane / LPN, lig = lane % LPN;
+  const int gid = int(threadIdx.x >> 5) * G + g;
+  const uint64_t ngroups = uint64_t(kWarpsPerCta) * G;
+  const uint64_t run = (hi - lo + ngroups - 1) / ngroups;
+  const uint64_t x0 = lo + uint64_t(gid) * run;
+  const uint64_t x1 = (x0 + run < hi) ? x0 + run : hi;
+  const Policies pol(a.cache_mode);
+  mbar_wait(mb, 0);  // every thread waits: the tiles have landed
+  if (x0 >= x1) return;
+
+  for (uint32_t col = uint32_t(lig) * 4; col < R; col += LPN * 4) {
+    Vec<4> acc;
+#pragma unroll
+    for (int i = 0; i < 4; ++i) acc.v[i] = 0.f;
+    uint32_t cur = 0xFFFFFFFFu;
+    for (uint64_t x = x0; x < x1; x += U) {
+      const int cnt = (x1 - x) >= uint64_t(U) ? U : int(x1 - x);
+      uint32_t er[U], ej[NOA][U];
+      float v[U];
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        if (u < cnt) {
+          er[u] = __ldg(a.erow + x + u);
+          v[u] = __ldg(a.val + x + u);
+#pragma unroll
+          for (int j = 0; j < NOA; ++j)
+            if (j < no) ej[j][u] = __ldg(a.eo[j] + x + u);
+        }
+      }
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        if (u < cnt) {
+          Vec<4> t;
+#pragma unroll
+          for (int i = 0; i < 4; ++i) t.v[i] = v[u];
+#pragma unroll
+          for (int j = 0; j < NOA; ++j) {
+            if (j < no) {
+              const float4 f =
+                  *reinterpret_cast<const float4 *>(tiles + (size_t(j) * B + ej[j][u]) * R + col);
+              t.v[0] *= f.x; t.v[1] *= f.y; t.v[2] *= f.z; t.v[3] *= f.w;
+            }
+          }
+          if (er[u] == cur) {
+#pragma unroll
+            for (int i = 0; i < 4; ++i) acc.v[i] += t.v[i];
+          } else {
+            if (cur != 0xFFFFFFFFu) red_vec<4>(a.out + uint64_t(base_row + cur) * R + col, acc, pol.out);
+            cur = er[u];
+            acc = t;
+          }
+        }
+      }
+    }
+    if (cur != 0xFFFFFFFFu) red_vec<4>(a.out + uint64_t(base_row + cur) * R + col, acc, pol.out);
+  }
+}
+
 template <int VW>
 __global__ void zero_rows_kernel(float *__restrict__ out, uint64_t n) {
   for (uint64_t e = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; e < n;
@@ -375,7 +621,7 @@ int sm_count() {
 
 template <class Src, int NO, int LPN, int VW, class T>
 void launch_t(const KArgs &a, cudaStream_t s) {
-  uint64_t nwarps = (a.nnz + a.chunk - 1) / a.chunk;
+  uint64_t nwarps = (a.nnz - a.x_begin + a.chunk - 1) / a.chunk;
   uint64_t nblk = (nwarps + kWarpsPerCta - 1) / kWarpsPerCta;
   if (nblk == 0) return;
   if (nblk > 0x7FFFFFFFull) fail(PASTA_ERANGE, "mttkrp: grid too large");
@@ -496,9 +742,50 @@ void launch_coo_mttkrp(const pasta_coo *x, uint32_t mode, const float *const *fa
   dispatch<CooSrc>(a, vec4_ok(x->order, mode, factors, R, out), s);
 }
 
+template <int NO>
+void launch_heavy_lpn(const HArgs &h, int lpn, uint64_t n_pieces, size_t smem, cudaStream_t s) {
+  auto go = [&](auto kern) {
+    if (smem > 48 * 1024)
+      PASTA_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem)));
+    kern<<<unsigned(n_pieces), kThreads, smem, s>>>(h);
+    PASTA_LAUNCHED();
+  };
+  switch (lpn) {
+    case 1: go(hicoo_heavy_kernel<NO, 1>); break;
+    case 2: go(hicoo_heavy_kernel<NO, 2>); break;
+    case 4: go(hicoo_heavy_kernel<NO, 4>); break;
+    case 8: go(hicoo_heavy_kernel<NO, 8>); break;
+    case 16: go(hicoo_heavy_kernel<NO, 16>); break;
+    default: go(hicoo_heavy_kernel<NO, 32>); break;
+  }
+}
+
 void launch_hicoo_mttkrp(const pasta_hicoo *h, uint32_t mode, const float *const *factors,
                          uint32_t R, float *out, cudaStream_t s) {
   const HicooModeCopy &mc = h->mc[mode];
+  if (mc.layout == 0) {
+    KArgs a{};
+    a.nnz = h->nnz;
+    a.order = h->order;
+    a.R = R;
+    a.sbptr = mc.sbptr.p;
+    a.nsb = mc.nsb;
+    a.sbrow = mc.sbrow.p;
+    a.val = mc.val.p;
+    int j = 0;
+    for (uint32_t k = 0; k < h->order; ++k) {
+      if (k == mode) continue;
+      a.sbbase[j] = mc.sbbase[k].p;
+      a.eo[j] = mc.einds[k].p;
+      a.Uo[j] = factors[k];
+      ++j;
+    }
+    a.out = out;
+    if (a.nnz == 0) return;
+    ProfScope prof(kProfHicoo, s);
+    dispatch<HicooRowSrc>(a, vec4_ok(h->order, mode, factors, R, out), s);
+    return;
+  }
   KArgs a{};
   a.nnz = h->nnz;
   a.order = h->order;
@@ -509,18 +796,52 @@ void launch_hicoo_mttkrp(const pasta_hicoo *h, uint32_t mode, const float *const
   a.erow = mc.einds[mode].p;
   a.val = mc.val.p;
   a.bbits = h->block_bits;
+  HArgs ha{};
   int j = 0;
   for (uint32_t k = 0; k < h->order; ++k) {
     if (k == mode) continue;
     a.bo[j] = mc.binds[k].p;
     a.eo[j] = mc.einds[k].p;
     a.Uo[j] = factors[k];
+    ha.bo[j] = mc.binds[k].p;
+    ha.eo[j] = mc.einds[k].p;
+    ha.Uo[j] = factors[k];
+    ha.dims_o[j] = h->dims[k];
     ++j;
   }
   a.out = out;
   if (a.nnz == 0) return;
   ProfScope prof(kProfHicoo, s);
-  dispatch<HicooSrc>(a, vec4_ok(h->order, mode, factors, R, out), s);
+  const bool vec4 = vec4_ok(h->order, mode, factors, R, out);
+  const size_t smem = size_t(h->order - 1) * (size_t(1) << h->block_bits) * R * sizeof(float);
+  const bool heavy = vec4 && mc.n_pieces > 0 && smem <= 160 * 1024;
+  if (heavy) {
+    ha.pieces = mc.pieces.p;
+    ha.piece = mc.piece;
+    ha.bptr = mc.bptr.p;
+    ha.brow = mc.binds[mode].p;
+    ha.erow = mc.einds[mode].p;
+    ha.val = mc.val.p;
+    ha.out = out;
+    ha.order = h->order;
+    ha.R = R;
+    ha.bbits = h->block_bits;
+    ha.cache_mode = uint32_t(env_int("PASTA_MTTKRP_CACHE", 0));
+    uint32_t need = (R + 3) / 4;
+    int lpn = 1;
+    while (lpn < 32 && uint32_t(lpn) < need) lpn <<= 1;
+    const int no = int(h->order) - 1;
+    if (no == 2) launch_heavy_lpn<2>(ha, lpn, mc.n_pieces, smem, s);
+    else if (no == 3) launch_heavy_lpn<3>(ha, lpn, mc.n_pieces, smem, s);
+    else launch_heavy_lpn<0>(ha, lpn, mc.n_pieces, smem, s);
+    // the light blocks: warp runs over the rest of the per-mode copy (the run grid starts
+    // 16-byte aligned; entries before heavy_nnz are skipped)
+    a.x_begin = mc.heavy_nnz & ~uint64_t(3);
+    a.x_skip = mc.heavy_nnz;
+    a.b_begin = mc.n_heavy;
+    if (mc.heavy_nnz == h->nnz) return;
+  }
+  dispatch<HicooSrc>(a, vec4, s);
 }
 
 }  // namespace pasta

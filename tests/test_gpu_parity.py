@@ -295,3 +295,23 @@ def test_errors_on_device(env):
         pasta.pasta_coo_to_hicoo(x, 9)
     with pytest.raises(pasta.PastaError):
         pasta.pasta_coo_shard(x, 0, 5, 3)
+
+
+@pytest.mark.parametrize("heavy", ["128", "16"])
+def test_hicoo_block_layout_with_tma_staged_heavy_blocks(env, heavy, monkeypatch):
+    """The block-major HiCOO copy (PASTA_HICOO_LAYOUT=block): heavy blocks are processed one
+    per CTA from factor tiles staged in shared memory by TMA bulk copies, light blocks by the
+    warp-run kernel.  Same tolerance as every other path."""
+    pasta, oracle, torch = env
+    monkeypatch.setenv("PASTA_HICOO_LAYOUT", "block")
+    monkeypatch.setenv("PASTA_HICOO_HEAVY", heavy)
+    for dims, nnz, R, bb in [((300, 200, 500), 50_013, 16, 7), ((60, 70, 80, 90), 40_007, 32, 4),
+                             ((5000, 3000, 2000), 200_000, 16, 7)]:
+        inds, vals = si.powerlaw_coo(dims, nnz, seed=nnz)
+        U = si.factors(dims, R, seed=3)
+        Ud = _dev(torch, U)
+        x = pasta.pasta_coo_from_arrays(dims, inds, vals)
+        h = pasta.pasta_coo_to_hicoo(x, bb)
+        for n in range(len(dims)):
+            ref, ab = oracle.mttkrp(dims, inds, vals, n, U)
+            _check(pasta.pasta_mttkrp_hicoo(h, n, Ud), ref, ab, f"block layout {dims} mode {n}")
