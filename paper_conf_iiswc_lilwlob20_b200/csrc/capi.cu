@@ -487,20 +487,36 @@ pasta_status pasta_mttkrp_coo_allmodes_host(pasta_coo *x, const float *const *ho
     }
     x->stage_R = R;
   }
+  // Pipelined: factors go up on a copy stream in the order the modes need them
+  // (U1..U_{N-1}, then U0), mode m's kernel starts as soon as its factors have landed,
+  // and its result goes down on a second copy stream while later modes compute
+  // (PCIe/C2C is full duplex).
+  E2EStreams &e = x->e2e;
+  e.init();
+  const uint32_t N = x->order;
   const float *dfac[kMaxOrder];
-  for (uint32_t k = 0; k < x->order; ++k) {
+  PASTA_CUDA(cudaEventRecord(e.start, s));
+  PASTA_CUDA(cudaStreamWaitEvent(e.h2d, e.start, 0));
+  for (uint32_t j = 0; j < N; ++j) {
+    uint32_t k = (j + 1) % N;  // 1, 2, ..., N-1, 0
     PASTA_CUDA(cudaMemcpyAsync(x->stage_f[k].p, host_factors[k], uint64_t(x->dims[k]) * R * sizeof(float),
-                               cudaMemcpyHostToDevice, s));
+                               cudaMemcpyHostToDevice, e.h2d));
+    PASTA_CUDA(cudaEventRecord(e.f[k], e.h2d));
     dfac[k] = x->stage_f[k].p;
   }
-  for (uint32_t m = 0; m < x->order; ++m) {
+  for (uint32_t m = 0; m < N; ++m) {
+    for (uint32_t k = 0; k < N; ++k)
+      if (k != m) PASTA_CUDA(cudaStreamWaitEvent(s, e.f[k], 0));
     uint64_t lo = 0, hi = x->dims[m];
     if (x->shard_mode == int(m)) { lo = x->row_lo; hi = x->row_hi; }
     launch_zero_rows(x->stage_o[m].p, lo, hi, R, s);
     launch_coo_mttkrp(x, m, dfac, R, x->stage_o[m].p, s);
+    PASTA_CUDA(cudaEventRecord(e.o[m], s));
+    PASTA_CUDA(cudaStreamWaitEvent(e.d2h, e.o[m], 0));
     PASTA_CUDA(cudaMemcpyAsync(host_out[m], x->stage_o[m].p, uint64_t(x->dims[m]) * R * sizeof(float),
-                               cudaMemcpyDeviceToHost, s));
+                               cudaMemcpyDeviceToHost, e.d2h));
   }
+  PASTA_CUDA(cudaStreamSynchronize(e.d2h));
   PASTA_CUDA(cudaStreamSynchronize(s));
   API_END
 }

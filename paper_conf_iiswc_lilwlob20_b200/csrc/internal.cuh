@@ -76,6 +76,34 @@ struct DevArray {
   size_t bytes() const { return n * sizeof(T); }
 };
 
+// Copy streams and events of the end-to-end host path (created on first use).
+struct E2EStreams {
+  cudaStream_t h2d = nullptr, d2h = nullptr;
+  cudaEvent_t f[kMaxOrder] = {}, o[kMaxOrder] = {}, start = nullptr;
+  bool ready = false;
+  void init() {
+    if (ready) return;
+    cudaStreamCreateWithFlags(&h2d, cudaStreamNonBlocking);
+    cudaStreamCreateWithFlags(&d2h, cudaStreamNonBlocking);
+    for (int k = 0; k < kMaxOrder; ++k) {
+      cudaEventCreateWithFlags(&f[k], cudaEventDisableTiming);
+      cudaEventCreateWithFlags(&o[k], cudaEventDisableTiming);
+    }
+    cudaEventCreateWithFlags(&start, cudaEventDisableTiming);
+    ready = true;
+  }
+  ~E2EStreams() {
+    if (!ready) return;
+    for (int k = 0; k < kMaxOrder; ++k) {
+      cudaEventDestroy(f[k]);
+      cudaEventDestroy(o[k]);
+    }
+    cudaEventDestroy(start);
+    cudaStreamDestroy(h2d);
+    cudaStreamDestroy(d2h);
+  }
+};
+
 // ----------------------------------------------------------------------------- handles
 struct CooModeCopy {
   bool ready = false;
@@ -127,6 +155,7 @@ struct pasta_coo {
   uint32_t stage_R = 0;
   pasta::DevArray<float> stage_f[pasta::kMaxOrder];
   pasta::DevArray<float> stage_o[pasta::kMaxOrder];
+  pasta::E2EStreams e2e;
   std::mutex mu;
 };
 

@@ -148,6 +148,7 @@ template <int NO, int U>
 struct CooSrc {
   // rows are globally sorted: a segment strictly inside a run is owned by that run
   static constexpr bool kSortedRows = true;
+  static constexpr int kMinBlocks = 1;
   uint64_t pol;
   __device__ __forceinline__ void init(const KArgs &, uint64_t, uint64_t p) { pol = p; }
   __device__ __forceinline__ void load(const KArgs &a, uint64_t x, int cnt, uint32_t (&row)[U],
@@ -187,6 +188,7 @@ template <int NO, int U>
 struct HicooSrc {
   // rows repeat across blocks of one block row (R#27): every flush is an atomic
   static constexpr bool kSortedRows = false;
+  static constexpr int kMinBlocks = 2;
   uint64_t b, bend;
   uint32_t base_row;
   uint32_t base[NO > 0 ? NO : kMaxOrder - 1];
@@ -262,6 +264,7 @@ struct HicooSrc {
 template <int NO, int U>
 struct HicooRowSrc {
   static constexpr bool kSortedRows = true;
+  static constexpr int kMinBlocks = 2;  // cap registers at 128: >= 16 resident warps per SM
   static constexpr int NOA = NO > 0 ? NO : kMaxOrder - 1;
   // current slice and the next one, loaded one slice ahead so that advancing through
   // short slices does not wait on a dependent load
@@ -629,7 +632,8 @@ void launch_t(const KArgs &a, cudaStream_t s) {
   PASTA_LAUNCHED();
 }
 
-using TuneDefault = Tune<4, false, 1>;
+template <class Src>
+using TuneDefault = Tune<4, false, Src::kMinBlocks>;
 
 // Variants selectable with PASTA_MTTKRP_VARIANT for tuning sweeps (vector path, N = 3, 4,
 // R = 16 / 32).
@@ -643,7 +647,7 @@ void launch_variant(const KArgs &a, int variant, cudaStream_t s) {
     case 5: launch_t<SrcT<NO, 4>, NO, LPN, 4, Tune<4, false, 4>>(a, s); break;
     case 6: launch_t<SrcT<NO, 4>, NO, LPN, 4, Tune<4, false, 3>>(a, s); break;
     case 7: launch_t<SrcT<NO, 8>, NO, LPN, 4, Tune<8, false, 2>>(a, s); break;
-    default: launch_t<SrcT<NO, 4>, NO, LPN, 4, TuneDefault>(a, s); break;
+    default: launch_t<SrcT<NO, 4>, NO, LPN, 4, TuneDefault<SrcT<NO, 4>>>(a, s); break;
   }
 }
 
@@ -654,12 +658,12 @@ void launch_lpn(const KArgs &a, int lpn, int variant, cudaStream_t s) {
     if (lpn == 8) return launch_variant<SrcT, NO, 8>(a, variant, s);
   }
   switch (lpn) {
-    case 1: launch_t<SrcT<NO, 4>, NO, 1, VW, TuneDefault>(a, s); break;
-    case 2: launch_t<SrcT<NO, 4>, NO, 2, VW, TuneDefault>(a, s); break;
-    case 4: launch_t<SrcT<NO, 4>, NO, 4, VW, TuneDefault>(a, s); break;
-    case 8: launch_t<SrcT<NO, 4>, NO, 8, VW, TuneDefault>(a, s); break;
-    case 16: launch_t<SrcT<NO, 4>, NO, 16, VW, TuneDefault>(a, s); break;
-    default: launch_t<SrcT<NO, 4>, NO, 32, VW, TuneDefault>(a, s); break;
+    case 1: launch_t<SrcT<NO, 4>, NO, 1, VW, TuneDefault<SrcT<NO, 4>>>(a, s); break;
+    case 2: launch_t<SrcT<NO, 4>, NO, 2, VW, TuneDefault<SrcT<NO, 4>>>(a, s); break;
+    case 4: launch_t<SrcT<NO, 4>, NO, 4, VW, TuneDefault<SrcT<NO, 4>>>(a, s); break;
+    case 8: launch_t<SrcT<NO, 4>, NO, 8, VW, TuneDefault<SrcT<NO, 4>>>(a, s); break;
+    case 16: launch_t<SrcT<NO, 4>, NO, 16, VW, TuneDefault<SrcT<NO, 4>>>(a, s); break;
+    default: launch_t<SrcT<NO, 4>, NO, 32, VW, TuneDefault<SrcT<NO, 4>>>(a, s); break;
   }
 }
 

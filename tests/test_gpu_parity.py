@@ -315,3 +315,25 @@ def test_hicoo_block_layout_with_tma_staged_heavy_blocks(env, heavy, monkeypatch
         for n in range(len(dims)):
             ref, ab = oracle.mttkrp(dims, inds, vals, n, U)
             _check(pasta.pasta_mttkrp_hicoo(h, n, Ud), ref, ab, f"block layout {dims} mode {n}")
+
+
+def test_row_partitioned_runner_two_ranks_on_one_gpu(env):
+    """parallel.RowPartitionedMTTKRP for world = 2, both ranks simulated on this GPU without a
+    process group (gather=False): the union of each rank's owned rows equals the oracle."""
+    pasta, oracle, torch = env
+    from paper_conf_iiswc_lilwlob20_b200.parallel import RowPartitionedMTTKRP
+    dims = (3000, 800, 1200)
+    inds, vals = si.hot_row_coo(dims, 50_000, 150_000, seed=21, mode=2, hot_row=5)
+    U = si.factors(dims, 16, seed=6)
+    Ud = _dev(torch, U)
+    x = pasta.pasta_coo_from_arrays(dims, inds, vals)
+    parts = [RowPartitionedMTTKRP(x, r, 2, 16, torch.device("cuda")) for r in range(2)]
+    assert sum(sum(p.shard_nnz()) for p in parts) == 3 * vals.shape[0]
+    outs = [p.step(Ud, gather=False) for p in parts]
+    for n in range(3):
+        ref, ab = oracle.mttkrp(dims, inds, vals, n, U)
+        full = torch.empty((dims[n], 16), device="cuda")
+        for r in range(2):
+            lo, hi = int(parts[r].bounds[n][r]), int(parts[r].bounds[n][r + 1])
+            full[lo:hi] = outs[r][n][lo:hi]
+        _check(full, ref, ab, f"rank-partitioned mode {n}")
