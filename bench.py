@@ -206,10 +206,17 @@ def main():
     import paper_conf_iiswc_lilwlob20_b200 as pasta
     from paper_conf_iiswc_lilwlob20_b200.parallel import RowPartitionedMTTKRP
 
-    torch.cuda.set_device(local)
-    dev = torch.device("cuda", local)
+    # PASTA_BENCH_SHARED_GPU=1 (tests only): every rank on cuda:0 with the gloo backend, to
+    # exercise the N > 1 code path on a single-GPU box; real runs use one GPU per rank + NCCL
+    shared = os.environ.get("PASTA_BENCH_SHARED_GPU") == "1"
+    local_dev = 0 if shared else local
+    torch.cuda.set_device(local_dev)
+    dev = torch.device("cuda", local_dev)
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        if shared:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=dev)
     stream = torch.cuda.current_stream()
 
     dims, R, M = cfg["dims"], cfg["R"], cfg["nnz"]
@@ -250,7 +257,7 @@ def main():
     if world > 1:
         dist.barrier()
 
-    clocks = ClockSampler(local)
+    clocks = ClockSampler(local_dev)
     if rank == 0:
         clocks.start()
     pasta.pasta_profile_read(0, reset=True)

@@ -1,0 +1,50 @@
+"""The N > 1 path on one GPU: torchrun launches 2 ranks that share cuda:0 over gloo (NCCL
+refuses two ranks per GPU).  Checks the row-partitioned runner end to end (shards, kernel
+writes of owned rows, in-place all-gather) and bench.py's multi-rank code path (barrier,
+max-over-ranks timing, rank-0-only JSON line, reference arm)."""
+import json
+import os
+import socket
+import subprocess
+import sys
+
+import pytest
+
+pytestmark = pytest.mark.gpu
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _torchrun(args, env_extra=None, timeout=600):
+    env = dict(os.environ, **(env_extra or {}))
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
+           "--master-addr", "127.0.0.1", "--master-port", str(_port())] + args
+    return subprocess.run(cmd, cwd=ROOT, env=env, capture_output=True, text=True, timeout=timeout)
+
+
+def test_row_partitioned_two_ranks_gloo():
+    r = _torchrun([os.path.join(ROOT, "tests", "mp_rowpart_worker.py")])
+    assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-4000:]
+
+
+def test_bench_two_ranks_shared_gpu():
+    r = _torchrun(["bench.py", "--gpus", "2", "--config", "c4", "--steps", "3", "--warmup", "3",
+                   "--no-cpu-baseline"], {"PASTA_BENCH_SHARED_GPU": "1"})
+    assert r.returncode == 0, r.stderr[-4000:]
+    lines = [l for l in r.stdout.splitlines() if l.startswith("{")]
+    assert len(lines) == 1, r.stdout  # rank 0 only
+    d = json.loads(lines[0])
+    assert d["n_gpus"] == 2 and d["value"] > 0 and d["scaling"] == "strong"
+    assert "NCCL" in d["config"]["parallelism"] or "all-gather" in d["config"]["parallelism"]
+    r2 = _torchrun(["bench.py", "--impl", "reference", "--gpus", "2", "--config", "c1",
+                    "--steps", "2", "--warmup", "3", "--ref-sample", "2000"])
+    assert r2.returncode == 0, r2.stderr[-4000:]
+    lines = [l for l in r2.stdout.splitlines() if l.startswith("{")]
+    assert len(lines) == 1 and json.loads(lines[0])["impl"] == "reference"
