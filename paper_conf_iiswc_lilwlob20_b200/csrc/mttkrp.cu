@@ -22,6 +22,7 @@
 //     (one vector atomic per boundary, not per nonzero, cf. P:157/P:282 atomics).
 //   * No tensor cores: the path is a gather/scatter, not a dense contraction.
 #include <cstdlib>
+#include <type_traits>
 
 #include "internal.cuh"
 
@@ -602,6 +603,143 @@ __global__ void __launch_bounds__(kThreads) hicoo_heavy_kernel(const HArgs a) {
   }
 }
 
+// ---------------------------------------------------------------------------------------
+// COO MTTKRP with a shared-memory-staged nonzero stream (a6, default vector path).
+// Same work decomposition as mttkrp_kernel (warp chunk = G groups x `run` contiguous
+// nonzeros, 4-lane groups own 16-B column slices of every factor row), but the index/value
+// stream is copied global->shared by the whole warp with cp.async (LDGSTS, L1-bypassing
+// .cg, L2 evict_first policy: every 128-B line is consumed by one copy, so the stream never
+// needs to linger in L2 and does not displace power-law-hot factor rows), double-buffered
+// one stage (32 nonzeros per group) ahead of the gathers.
+template <int NO, int LPN, int WA>
+__global__ void __launch_bounds__(kThreads, 2) coo_staged_kernel(const KArgs a) {
+  constexpr int G = 32 / LPN;
+  constexpr int SG = 32;          // nonzeros per group per stage
+  constexpr int SW = G * SG;      // nonzeros per warp per stage
+  constexpr int NA = NO + 2;      // arrays: i_n, i_k (k != n), val
+  constexpr int U = 4;
+  extern __shared__ __align__(16) uint32_t stage_buf[];  // [warp][2][NA][SW]
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int g = lane / LPN, lig = lane % LPN;
+  uint32_t *wbuf = stage_buf + size_t(warp) * 2 * NA * SW;
+  const uint64_t w = uint64_t(blockIdx.x) * kWarpsPerCta + warp;
+  const uint64_t c0 = w * a.chunk;
+  if (c0 >= a.nnz) return;  // whole warp exits together
+  const uint64_t run = a.chunk / G;  // multiple of SG
+  const uint64_t x0 = c0 + uint64_t(g) * run;
+  const uint64_t x1 = (x0 + run < a.nnz) ? x0 + run : a.nnz;
+  const int nstages = int(run / SG);
+  const uint32_t R = a.R;
+  const uint32_t col = uint32_t(lig) * 4;
+  const Policies pol(a.cache_mode | 1u);  // the staged stream is always evict_first
+  const uint32_t *src[NA];
+  src[0] = a.irow;
+#pragma unroll
+  for (int j = 0; j < NO; ++j) src[1 + j] = a.io[j];
+  src[NA - 1] = reinterpret_cast<const uint32_t *>(a.val);
+
+  // issue the cp.async copies of stage s into buffer s & 1
+  auto issue_to = [&](int s, uint32_t *dst) {
+    for (int i = lane; i < SW / 4; i += 32) {  // 16-B chunks of one array
+      const int gi = i / (SG / 4), k = i % (SG / 4);
+      const uint64_t pos = c0 + uint64_t(gi) * run + uint64_t(s) * SG + uint64_t(k) * 4;
+      const int valid = pos >= a.nnz ? 0 : (a.nnz - pos >= 4 ? 16 : int(a.nnz - pos) * 4);
+#pragma unroll
+      for (int arr = 0; arr < NA; ++arr) {
+        const uint32_t d = smem_addr(dst + arr * SW + gi * SG + k * 4);
+        const uint32_t *sp = src[arr] + (valid ? pos : 0);
+        if (WA == 2) {
+          asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(d), "l"(sp), "r"(valid)
+                       : "memory");
+        } else {
+          asm volatile("cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, %2, %3;" ::"r"(d),
+                       "l"(sp), "r"(valid), "l"(pol.stream)
+                       : "memory");
+        }
+      }
+    }
+    asm volatile("cp.async.commit_group;" ::: "memory");
+  };
+  auto issue = [&](int s) {
+    if (WA == 1) {
+      if (s & 1) issue_to(s, wbuf + NA * SW); else issue_to(s, wbuf);
+    } else {
+      issue_to(s, wbuf + (s & 1) * NA * SW);
+    }
+  };
+
+  Vec<4> acc;
+#pragma unroll
+  for (int i = 0; i < 4; ++i) acc.v[i] = 0.f;
+  uint32_t cur = 0xFFFFFFFFu;
+  bool first = true;
+  const bool active = x0 < x1 && col < R;
+  issue(0);
+  for (int s = 0; s < nstages; ++s) {
+    if (s + 1 < nstages) {
+      issue(s + 1);
+      asm volatile("cp.async.wait_group 1;" ::: "memory");
+    } else {
+      asm volatile("cp.async.wait_group 0;" ::: "memory");
+    }
+    __syncwarp();
+    const uint32_t *buf = wbuf + (s & 1) * NA * SW + g * SG;
+    const uint64_t sx = x0 + uint64_t(s) * SG;  // first nonzero of this stage for the group
+    if (active && sx < x1) {
+      const int scnt = (x1 - sx) >= uint64_t(SG) ? SG : int(x1 - sx);
+#pragma unroll 1
+      for (int q = 0; q < scnt; q += U) {
+        const int cnt = (scnt - q) >= U ? U : scnt - q;
+        const uint4 r4 = *reinterpret_cast<const uint4 *>(buf + q);
+        const uint4 v4 = *reinterpret_cast<const uint4 *>(buf + (NA - 1) * SW + q);
+        uint32_t row[U] = {r4.x, r4.y, r4.z, r4.w};
+        float v[U] = {__uint_as_float(v4.x), __uint_as_float(v4.y), __uint_as_float(v4.z),
+                      __uint_as_float(v4.w)};
+        uint32_t idx[NO][U];
+#pragma unroll
+        for (int j = 0; j < NO; ++j) {
+          const uint4 i4 = *reinterpret_cast<const uint4 *>(buf + (1 + j) * SW + q);
+          idx[j][0] = i4.x; idx[j][1] = i4.y; idx[j][2] = i4.z; idx[j][3] = i4.w;
+        }
+        Vec<4> f[NO][U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+#pragma unroll
+          for (int j = 0; j < NO; ++j)
+            if (u < cnt) f[j][u] = ldg_vec<4>(a.Uo[j] + uint64_t(idx[j][u]) * R + col, pol.gather);
+        }
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+          if (u < cnt) {
+            Vec<4> t;
+#pragma unroll
+            for (int i = 0; i < 4; ++i) t.v[i] = v[u];
+#pragma unroll
+            for (int j = 0; j < NO; ++j) {
+#pragma unroll
+              for (int i = 0; i < 4; ++i) t.v[i] *= f[j][u].v[i];
+            }
+            if (row[u] == cur) {
+#pragma unroll
+              for (int i = 0; i < 4; ++i) acc.v[i] += t.v[i];
+            } else {
+              if (cur != 0xFFFFFFFFu) {
+                float *dst = a.out + uint64_t(cur) * R + col;
+                if (first) red_vec<4>(dst, acc, pol.out); else st_vec<4>(dst, acc, pol.out);
+                first = false;
+              }
+              cur = row[u];
+              acc = t;
+            }
+          }
+        }
+      }
+    }
+    __syncwarp();  // the buffer of stage s is refilled at stage s + 2
+  }
+  if (active && cur != 0xFFFFFFFFu) red_vec<4>(a.out + uint64_t(cur) * R + col, acc, pol.out);
+}
+
 template <int VW>
 __global__ void zero_rows_kernel(float *__restrict__ out, uint64_t n) {
   for (uint64_t e = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; e < n;
@@ -743,7 +881,42 @@ void launch_coo_mttkrp(const pasta_coo *x, uint32_t mode, const float *const *fa
   a.out = out;
   if (a.nnz == 0) return;
   ProfScope prof(kProfCoo, s);
-  dispatch<CooSrc>(a, vec4_ok(x->order, mode, factors, R, out), s);
+  const bool vec4 = vec4_ok(x->order, mode, factors, R, out);
+  const int staged = env_int("PASTA_COO_STAGED", 1);
+  const int no = int(x->order) - 1;
+  if (staged && vec4 && (R == 16 || R == 32) && (no == 2 || no == 3)) {
+    const int lpn = R == 16 ? 4 : 8;
+    const int G = 32 / lpn;
+    uint64_t run = uint64_t(env_int("PASTA_MTTKRP_RUN", 128));
+    run = run < 32 ? 32 : (run / 32) * 32;
+    a.chunk = uint64_t(G) * run;
+    a.cache_mode = uint32_t(env_int("PASTA_MTTKRP_CACHE", 0));
+    const size_t smem = size_t(kWarpsPerCta) * 2 * (no + 2) * (G * 32) * sizeof(uint32_t);
+    uint64_t nwarps = (a.nnz + a.chunk - 1) / a.chunk;
+    uint64_t nblk = (nwarps + kWarpsPerCta - 1) / kWarpsPerCta;
+    auto go = [&](auto kern) {
+      PASTA_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem)));
+      kern<<<unsigned(nblk), kThreads, smem, s>>>(a);
+      PASTA_LAUNCHED();
+    };
+    // WA 1 (default): one code path per buffer.  ptxas 12.9 turns the computed buffer
+    // offset into an [R+UR] LDGSTS operand that, combined with the L2 cache-policy
+    // descriptor, raises "illegal instruction" on sm_100a for some instantiations (observed
+    // with compute-sanitizer); WA 2 drops the L2 hint instead; WA 0 is the plain form.
+    const int wa = env_int("PASTA_STAGED_WA", 1);
+    auto pick = [&](auto tag) {
+      constexpr int W = decltype(tag)::value;
+      if (no == 2 && lpn == 4) go(coo_staged_kernel<2, 4, W>);
+      else if (no == 2) go(coo_staged_kernel<2, 8, W>);
+      else if (lpn == 4) go(coo_staged_kernel<3, 4, W>);
+      else go(coo_staged_kernel<3, 8, W>);
+    };
+    if (wa == 1) pick(std::integral_constant<int, 1>());
+    else if (wa == 2) pick(std::integral_constant<int, 2>());
+    else pick(std::integral_constant<int, 0>());
+    return;
+  }
+  dispatch<CooSrc>(a, vec4, s);
 }
 
 template <int NO>
