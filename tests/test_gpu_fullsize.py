@@ -81,3 +81,23 @@ def test_fullsize_generator_contains_oracle_prefix(env):
         assert gv[p].view(np.uint32) == ov[j].view(np.uint32)
         found += 1
     assert found == 200_000
+
+
+def test_fullsize_hicoo_conversion_and_mode_sort_bit_exact(env):
+    """Integer work at a BASELINE.json size (C4: 54M nonzeros, 4th order): the GPU COO->HiCOO
+    conversion (B = 128) and the mode-3 sort equal the oracle's qsort-based ones bit for bit."""
+    pasta, oracle, torch = env
+    cfg = si.CONFIGS["c4"]
+    dims, M = cfg["dims"], cfg["nnz"]
+    inds, vals = si.powerlaw_coo(dims, M, seed=cfg["seed"] + 5, dedup=False)
+    x = pasta.pasta_coo_from_arrays(dims, inds, vals)
+    h = pasta.pasta_hicoo_export(pasta.pasta_coo_to_hicoo(x, 7))
+    o = oracle.coo_to_hicoo(inds, vals, 7)
+    assert h["nblocks"] == o["nblocks"]
+    for key in ("bptr", "binds", "einds"):
+        assert np.array_equal(h[key], o[key]), key
+    assert np.array_equal(h["vals"].view(np.uint32), o["vals"].view(np.uint32))
+    del h, o
+    gi, gv = pasta.pasta_coo_export_mode(x, 3)
+    oi, ov = oracle.mode_sort(inds, vals, 3)
+    assert np.array_equal(gi, oi) and np.array_equal(gv.view(np.uint32), ov.view(np.uint32))

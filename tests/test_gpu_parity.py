@@ -337,3 +337,30 @@ def test_row_partitioned_runner_two_ranks_on_one_gpu(env):
             lo, hi = int(parts[r].bounds[n][r]), int(parts[r].bounds[n][r + 1])
             full[lo:hi] = outs[r][n][lo:hi]
         _check(full, ref, ab, f"rank-partitioned mode {n}")
+
+
+def test_torch_caching_allocator_hook(env):
+    """pasta_set_allocator: every libpasta device allocation goes through torch's caching
+    allocator (use_torch_allocator); results unchanged, memory visible to torch."""
+    pasta, oracle, torch = env
+    dims = (500, 400, 300)
+    inds, vals = si.powerlaw_coo(dims, 60_000, seed=2)
+    U = si.factors(dims, 16, seed=2)
+    Ud = _dev(torch, U)
+    torch.cuda.synchronize()
+    before = torch.cuda.memory_allocated()
+    pasta.use_torch_allocator()
+    try:
+        x = pasta.pasta_coo_from_arrays(dims, inds, vals)
+        h = pasta.pasta_coo_to_hicoo(x, 7)
+        g = pasta.pasta_gen_powerlaw((1000, 1000, 1000), 50_000, seed=3)
+        for n in range(3):
+            ref, ab = oracle.mttkrp(dims, inds, vals, n, U)
+            _check(pasta.pasta_mttkrp_coo(x, n, Ud), ref, ab, f"hooked coo mode {n}")
+            _check(pasta.pasta_mttkrp_hicoo(h, n, Ud), ref, ab, f"hooked hicoo mode {n}")
+        assert torch.cuda.memory_allocated() > before  # the handles' arrays live in torch's pool
+        del x, h, g
+        import gc
+        gc.collect()
+    finally:
+        pasta.pasta_set_allocator(None)
