@@ -120,8 +120,10 @@ pasta_status pasta_coo_to_hicoo(const pasta_coo *x, uint32_t block_bits, pasta_h
 
 /* Build (once; cached in the handle) the mode-`mode` working copy: for COO the nonzeros
  * stably sorted lexicographically by (i_mode, i_mode+1, ..., i_mode-1) (a2);
- * for HiCOO the blocks stably sorted by binds_mode and, inside each block, the entries
- * stably sorted by einds_mode (R#27).  Optional: MTTKRP prepares on first use. */
+ * for HiCOO (R#27) by default "row slices" (the entries of a block that share einds_mode,
+ * slices ordered by output row), or with PASTA_HICOO_LAYOUT=block the blocks stably sorted by
+ * binds_mode with entries by einds_mode (dense blocks then run one per CTA with TMA-staged
+ * factor tiles).  Optional: MTTKRP prepares on first use. */
 pasta_status pasta_coo_prepare(pasta_coo *x, uint32_t mode, void *stream);
 pasta_status pasta_hicoo_prepare(pasta_hicoo *h, uint32_t mode, void *stream);
 
@@ -167,6 +169,36 @@ pasta_status pasta_coo_partition(const pasta_coo *x, uint32_t mode, uint32_t npa
  * rows [row_lo, row_hi) of `out`. */
 pasta_status pasta_coo_shard(pasta_coo *x, uint32_t mode, uint32_t row_lo, uint32_t row_hi,
                              pasta_coo **out);
+
+/* ------------------------------------------------------- CP-ALS -------- */
+/* CANDECOMP/PARAFAC by alternating least squares around the MTTKRP: the paper's motivation
+ * for MTTKRP ("most computationally expensive kernel in CPD"; CPD listed as future work
+ * P:380).  The update is the textbook one of the paper's ref. [1] (Kolda & Bader).  All
+ * matrices are DEVICE memory; R <= 64 (EUNSUPPORTED otherwise).  Building blocks accumulate
+ * (+=) into fp64 outputs so that row-partitioned callers can all-reduce partial results. */
+
+/* G (R x R, fp64, row-major) += U^T U for U row-major [rows][R] fp32. */
+pasta_status pasta_gram(const float *U, uint64_t rows, uint32_t R, double *G, void *stream);
+/* U = M V^{-1} with V = Hadamard product of the `ngrams` R x R matrices grams[] (HOST array of
+ * DEVICE pointers; the grams of every mode but the updated one), inverted in fp64 (partial-
+ * pivot Gauss-Jordan, tiny ridge if singular); colsq[r] += sum_i U(i, r)^2 (fp64). */
+pasta_status pasta_cpals_solve(const float *M, uint64_t rows, uint32_t R, const double *const *grams,
+                               uint32_t ngrams, float *U, double *colsq, void *stream);
+/* lambda[r] = sqrt(colsq[r]) (1 where zero); U(:, r) /= lambda[r].  lambda: DEVICE fp64 [R]. */
+pasta_status pasta_normalize_columns(float *U, uint64_t rows, uint32_t R, const double *colsq,
+                                     double *lambda, void *stream);
+/* out += sum_{i, r} lambda[r] A(i, r) B(i, r)   (out: DEVICE fp64 scalar). */
+pasta_status pasta_weighted_inner(const float *A, const float *B, uint64_t rows, uint32_t R,
+                                  const double *lambda, double *out, void *stream);
+/* ||X||_F^2 = sum of squared values (HOST result). */
+pasta_status pasta_coo_norm2(const pasta_coo *x, double *out);
+/* Single-GPU CP-ALS: factors[k] (DEVICE [dims[k]][R], the initial guess on entry, the result
+ * on exit, columns normalised), lambda (HOST fp64 [R], out), fit_history (HOST fp64
+ * [max_iters], out: fit = 1 - ||X - [[lambda; U]]|| / ||X|| after each sweep over the modes),
+ * iters (out).  Stops when |fit - previous fit| < tol. */
+pasta_status pasta_cpals_coo(pasta_coo *x, uint32_t R, uint32_t max_iters, double tol,
+                             float *const *factors, double *lambda, double *fit_history,
+                             uint32_t *iters, void *stream);
 
 /* ------------------------------------------------------------ introspection ---------- */
 

@@ -22,7 +22,9 @@ __all__ = [
     "pasta_mttkrp_hicoo", "pasta_mttkrp_coo_allmodes_host", "pasta_coo_row_counts",
     "pasta_row_partition", "pasta_coo_partition", "pasta_coo_shard", "pasta_coo_info",
     "pasta_coo_export", "pasta_coo_export_mode", "pasta_hicoo_info", "pasta_hicoo_export",
-    "pasta_launch_count", "pasta_profile_enable", "pasta_profile_read",
+    "pasta_launch_count", "pasta_profile_enable", "pasta_profile_read", "pasta_gram",
+    "pasta_cpals_solve", "pasta_normalize_columns", "pasta_weighted_inner", "pasta_coo_norm2",
+    "pasta_cpals_coo",
 ]
 
 _u32p = C.POINTER(C.c_uint32)
@@ -370,3 +372,72 @@ def pasta_profile_read(which: int, reset: bool = True):
     n = C.c_uint64()
     check(lib().pasta_profile_read(which, C.byref(ms), C.byref(n), 1 if reset else 0))
     return ms.value, n.value
+
+
+# ----------------------------------------------------------------------------- CP-ALS
+def _dptr(t):
+    return C.c_void_p(t.data_ptr())
+
+
+def pasta_gram(U, G=None, stream=None):
+    """G (+)= U^T U in fp64 (R x R CUDA tensor; a fresh zero tensor when G is None)."""
+    import torch
+    R = int(U.shape[1])
+    if G is None:
+        G = torch.zeros((R, R), dtype=torch.float64, device=U.device)
+    check(lib().pasta_gram(_dptr(U), U.shape[0], R, _dptr(G), _stream_ptr(stream)))
+    return G
+
+
+def pasta_cpals_solve(M, grams, U=None, colsq=None, stream=None):
+    """U = M (Hadamard of grams)^-1, colsq += column sums of squares of U."""
+    import torch
+    rows, R = int(M.shape[0]), int(M.shape[1])
+    if U is None:
+        U = torch.empty_like(M)
+    if colsq is None:
+        colsq = torch.zeros(R, dtype=torch.float64, device=M.device)
+    gp = (C.c_void_p * max(len(grams), 1))(*[g.data_ptr() for g in grams])
+    check(lib().pasta_cpals_solve(_dptr(M), rows, R, gp, len(grams), _dptr(U), _dptr(colsq),
+                                  _stream_ptr(stream)))
+    return U, colsq
+
+
+def pasta_normalize_columns(U, colsq, lam=None, stream=None):
+    import torch
+    R = int(U.shape[1])
+    if lam is None:
+        lam = torch.empty(R, dtype=torch.float64, device=U.device)
+    check(lib().pasta_normalize_columns(_dptr(U), U.shape[0], R, _dptr(colsq), _dptr(lam),
+                                        _stream_ptr(stream)))
+    return lam
+
+
+def pasta_weighted_inner(A, B, lam, out=None, stream=None):
+    import torch
+    if out is None:
+        out = torch.zeros(1, dtype=torch.float64, device=A.device)
+    check(lib().pasta_weighted_inner(_dptr(A), _dptr(B), A.shape[0], int(A.shape[1]), _dptr(lam),
+                                     _dptr(out), _stream_ptr(stream)))
+    return out
+
+
+def pasta_coo_norm2(x: Coo) -> float:
+    v = C.c_double()
+    check(lib().pasta_coo_norm2(x.ptr, C.byref(v)))
+    return v.value
+
+
+def pasta_cpals_coo(x: Coo, factors, max_iters: int = 20, tol: float = 1e-5, stream=None):
+    """Single-GPU CP-ALS; `factors` (CUDA float32 [I_k, R], the initial guess) are updated in
+    place.  Returns (lambda float64[R], fit per sweep list, sweeps run)."""
+    R = int(factors[0].shape[1])
+    fp = (C.c_void_p * x.order)(*[f.data_ptr() for f in factors])
+    lam = np.zeros(R, np.float64)
+    fits = np.zeros(max(max_iters, 1), np.float64)
+    it = C.c_uint32()
+    check(lib().pasta_cpals_coo(x.ptr, R, max_iters, tol, fp,
+                                lam.ctypes.data_as(C.POINTER(C.c_double)),
+                                fits.ctypes.data_as(C.POINTER(C.c_double)), C.byref(it),
+                                _stream_ptr(stream)))
+    return lam, list(fits[: it.value]), it.value

@@ -72,6 +72,13 @@ SIGNATURES = {
     "pasta_hicoo_export": (_st, [_vp, _u64p, C.POINTER(_u32p), C.POINTER(_u8p), _f32p]),
     "pasta_coo_free": (None, [_vp]),
     "pasta_hicoo_free": (None, [_vp]),
+    "pasta_gram": (_st, [_vp, C.c_uint64, C.c_uint32, _vp, _vp]),
+    "pasta_cpals_solve": (_st, [_vp, C.c_uint64, C.c_uint32, C.POINTER(_vp), C.c_uint32, _vp, _vp, _vp]),
+    "pasta_normalize_columns": (_st, [_vp, C.c_uint64, C.c_uint32, _vp, _vp, _vp]),
+    "pasta_weighted_inner": (_st, [_vp, _vp, C.c_uint64, C.c_uint32, _vp, _vp, _vp]),
+    "pasta_coo_norm2": (_st, [_vp, C.POINTER(C.c_double)]),
+    "pasta_cpals_coo": (_st, [_vp, C.c_uint32, C.c_uint32, C.c_double, C.POINTER(_vp),
+                              C.POINTER(C.c_double), C.POINTER(C.c_double), _u32p, _vp]),
     "pasta_launch_count": (C.c_uint64, []),
     "pasta_profile_enable": (_st, [C.c_int]),
     "pasta_profile_read": (_st, [C.c_uint32, C.POINTER(C.c_double), _u64p, C.c_int]),

@@ -604,6 +604,133 @@ pasta_status pasta_coo_shard(pasta_coo *x, uint32_t mode, uint32_t row_lo, uint3
   API_END
 }
 
+// ---------------------------------------------------------------------------- CP-ALS
+static void require_R64(uint32_t R) {
+  require(R >= 1, "R must be >= 1");
+  if (R > 64) fail(PASTA_EUNSUPPORTED, "CP-ALS supports R <= 64");
+}
+
+pasta_status pasta_gram(const float *U, uint64_t rows, uint32_t R, double *G, void *stream) {
+  API_BEGIN
+  require((U || !rows) && G, "U/G is NULL");
+  require_R64(R);
+  launch_gram(U, rows, R, G, as_stream(stream));
+  API_END
+}
+
+pasta_status pasta_cpals_solve(const float *M, uint64_t rows, uint32_t R, const double *const *grams,
+                               uint32_t ngrams, float *U, double *colsq, void *stream) {
+  API_BEGIN
+  require((M && U) || !rows, "M/U is NULL");
+  require(colsq && (grams || !ngrams), "colsq/grams is NULL");
+  require_R64(R);
+  for (uint32_t k = 0; k < ngrams; ++k) require(grams[k] != nullptr, "grams[k] is NULL");
+  launch_solve(M, rows, R, grams, ngrams, U, colsq, as_stream(stream));
+  API_END
+}
+
+pasta_status pasta_normalize_columns(float *U, uint64_t rows, uint32_t R, const double *colsq,
+                                     double *lambda, void *stream) {
+  API_BEGIN
+  require((U || !rows) && colsq && lambda, "U/colsq/lambda is NULL");
+  require_R64(R);
+  launch_normalize(U, rows, R, colsq, lambda, as_stream(stream));
+  API_END
+}
+
+pasta_status pasta_weighted_inner(const float *A, const float *B, uint64_t rows, uint32_t R,
+                                  const double *lambda, double *out, void *stream) {
+  API_BEGIN
+  require(((A && B) || !rows) && lambda && out, "A/B/lambda/out is NULL");
+  require_R64(R);
+  launch_inner(A, B, rows, R, lambda, out, as_stream(stream));
+  API_END
+}
+
+pasta_status pasta_coo_norm2(const pasta_coo *x, double *out) {
+  API_BEGIN
+  require(x && out, "x/out is NULL");
+  check_device(x->device);
+  DevArray<double> d(1);
+  PASTA_CUDA(cudaMemset(d.p, 0, sizeof(double)));
+  launch_sumsq(x->val.p, x->nnz, d.p, nullptr);
+  PASTA_CUDA(cudaMemcpy(out, d.p, sizeof(double), cudaMemcpyDeviceToHost));
+  API_END
+}
+
+pasta_status pasta_cpals_coo(pasta_coo *x, uint32_t R, uint32_t max_iters, double tol,
+                             float *const *factors, double *lambda, double *fit_history,
+                             uint32_t *iters, void *stream) {
+  API_BEGIN
+  require(x && factors && lambda && (fit_history || !max_iters) && iters, "NULL argument");
+  require_R64(R);
+  const uint32_t N = x->order;
+  for (uint32_t k = 0; k < N; ++k) require(factors[k] != nullptr, "factors[k] is NULL");
+  require(N >= 2, "CP-ALS needs order >= 2");
+  check_device(x->device);
+  cudaStream_t s = as_stream(stream);
+  {
+    std::lock_guard<std::mutex> lk(x->mu);
+    for (uint32_t k = 0; k < N; ++k) coo_prepare_mode(x, k, s);
+  }
+  uint64_t maxd = 0;
+  for (uint32_t k = 0; k < N; ++k) maxd = x->dims[k] > maxd ? x->dims[k] : maxd;
+  DevArray<float> Mbuf(maxd * R, s);
+  DevArray<double> grams(uint64_t(N) * R * R, s), colsq(R, s), lam(R, s), scal(2, s);
+  auto G = [&](uint32_t k) { return grams.p + uint64_t(k) * R * R; };
+  PASTA_CUDA(cudaMemsetAsync(grams.p, 0, grams.bytes(), s));
+  for (uint32_t k = 0; k < N; ++k) launch_gram(factors[k], x->dims[k], R, G(k), s);
+  PASTA_CUDA(cudaMemsetAsync(scal.p, 0, scal.bytes(), s));
+  launch_sumsq(x->val.p, x->nnz, scal.p, s);
+  double normx2 = 0.0;
+  PASTA_CUDA(cudaMemcpyAsync(&normx2, scal.p, sizeof(double), cudaMemcpyDeviceToHost, s));
+  PASTA_CUDA(cudaStreamSynchronize(s));
+  std::vector<double> hg(uint64_t(N) * R * R), hl(R, 1.0);
+  double prev = 0.0;
+  uint32_t it = 0;
+  const float *cf[kMaxOrder];
+  for (uint32_t k = 0; k < N; ++k) cf[k] = factors[k];
+  for (; it < max_iters; ++it) {
+    for (uint32_t n = 0; n < N; ++n) {
+      launch_zero_rows(Mbuf.p, 0, x->dims[n], R, s);
+      launch_coo_mttkrp(x, n, cf, R, Mbuf.p, s);
+      const double *gl[kMaxOrder];
+      uint32_t ng = 0;
+      for (uint32_t k = 0; k < N; ++k)
+        if (k != n) gl[ng++] = G(k);
+      PASTA_CUDA(cudaMemsetAsync(colsq.p, 0, colsq.bytes(), s));
+      launch_solve(Mbuf.p, x->dims[n], R, gl, ng, factors[n], colsq.p, s);
+      launch_normalize(factors[n], x->dims[n], R, colsq.p, lam.p, s);
+      PASTA_CUDA(cudaMemsetAsync(G(n), 0, sizeof(double) * R * R, s));
+      launch_gram(factors[n], x->dims[n], R, G(n), s);
+    }
+    // fit from the last mode's MTTKRP (still in Mbuf) and the normalised factors
+    PASTA_CUDA(cudaMemsetAsync(scal.p + 1, 0, sizeof(double), s));
+    launch_inner(Mbuf.p, factors[N - 1], x->dims[N - 1], R, lam.p, scal.p + 1, s);
+    double inner = 0.0;
+    PASTA_CUDA(cudaMemcpyAsync(&inner, scal.p + 1, sizeof(double), cudaMemcpyDeviceToHost, s));
+    PASTA_CUDA(cudaMemcpyAsync(hg.data(), grams.p, grams.bytes(), cudaMemcpyDeviceToHost, s));
+    PASTA_CUDA(cudaMemcpyAsync(hl.data(), lam.p, lam.bytes(), cudaMemcpyDeviceToHost, s));
+    PASTA_CUDA(cudaStreamSynchronize(s));
+    double nxhat2 = 0.0;  // lambda^T (Hadamard_k G_k) lambda
+    for (uint32_t a = 0; a < R; ++a)
+      for (uint32_t b = 0; b < R; ++b) {
+        double v = hl[a] * hl[b];
+        for (uint32_t k = 0; k < N; ++k) v *= hg[uint64_t(k) * R * R + a * R + b];
+        nxhat2 += v;
+      }
+    const double resid2 = normx2 + nxhat2 - 2.0 * inner;
+    const double fit = normx2 > 0 ? 1.0 - std::sqrt(resid2 > 0 ? resid2 : 0.0) / std::sqrt(normx2) : 0.0;
+    fit_history[it] = fit;
+    const bool done = it > 0 && std::fabs(fit - prev) < tol;
+    prev = fit;
+    if (done) { ++it; break; }
+  }
+  for (uint32_t r = 0; r < R; ++r) lambda[r] = hl[r];
+  *iters = it;
+  API_END
+}
+
 // ---------------------------------------------------------------------------- introspection
 pasta_status pasta_coo_info(const pasta_coo *x, uint32_t *order, uint32_t *dims, uint64_t *nnz) {
   API_BEGIN

@@ -213,6 +213,14 @@ void launch_coo_mttkrp(const pasta_coo *x, uint32_t mode, const float *const *fa
                        float *out, cudaStream_t s);
 void launch_hicoo_mttkrp(const pasta_hicoo *h, uint32_t mode, const float *const *factors,
                          uint32_t R, float *out, cudaStream_t s);
+void launch_gram(const float *U, uint64_t rows, uint32_t R, double *G, cudaStream_t s);
+void launch_solve(const float *M, uint64_t rows, uint32_t R, const double *const *grams, uint32_t ngrams,
+                  float *U, double *colsq, cudaStream_t s);
+void launch_normalize(float *U, uint64_t rows, uint32_t R, const double *colsq, double *lambda,
+                      cudaStream_t s);
+void launch_inner(const float *A, const float *B, uint64_t rows, uint32_t R, const double *lambda,
+                  double *out, cudaStream_t s);
+void launch_sumsq(const float *v, uint64_t n, double *out, cudaStream_t s);
 void row_counts_device(const uint32_t *rows, uint64_t nnz, uint32_t nrows, uint64_t *counts_host,
                        cudaStream_t s);
 // first position x in the sorted array a[0..M) with a[x] >= v (device binary search).

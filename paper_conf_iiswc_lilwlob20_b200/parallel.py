@@ -71,3 +71,58 @@ class RowPartitionedMTTKRP:
         for w in works:
             w.wait()
         return self.out
+
+
+def _all_reduce(t):
+    import torch.distributed as dist
+    if dist.is_available() and dist.is_initialized() and dist.get_world_size() > 1:
+        dist.all_reduce(t)
+    return t
+
+
+class RowPartitionedCPALS(RowPartitionedMTTKRP):
+    """CP-ALS over row-partitioned MTTKRP: per mode n, each rank computes the
+    MTTKRP rows it owns, solves its rows of U_n = M V^-1 (V from the replicated R x R grams),
+    all-reduces the column sums of squares (lambda) and its partial gram, and all-gathers the
+    owned rows of U_n -- the step that makes the output all-gather necessary.
+    Every arithmetic step runs in libpasta kernels; only R-sized vectors and R x R matrices
+    cross the process group besides the gathered rows."""
+
+    def run(self, factors, max_iters=20, tol=1e-5):
+        import torch
+
+        from . import (pasta_coo_norm2, pasta_cpals_solve, pasta_gram, pasta_mttkrp_coo,
+                       pasta_normalize_columns, pasta_weighted_inner)
+        N, R = self.order, self.R
+        dev = factors[0].device
+        grams = [pasta_gram(u) for u in factors]  # factors are replicated: full grams locally
+        # ||X||^2: the mode-0 shards partition the nonzeros
+        normx2 = _all_reduce(torch.tensor([pasta_coo_norm2(self.shards[0])], dtype=torch.float64,
+                                          device=dev)).item()
+        lam = torch.ones(R, dtype=torch.float64, device=dev)
+        fits = []
+        for it in range(max_iters):
+            for n in range(N):
+                lo, hi = int(self.bounds[n][self.rank]), int(self.bounds[n][self.rank + 1])
+                M = pasta_mttkrp_coo(self.shards[n], n, factors, out=self.out[n])
+                others = [grams[k] for k in range(N) if k != n]
+                colsq = torch.zeros(R, dtype=torch.float64, device=dev)
+                pasta_cpals_solve(M[lo:hi], others, U=factors[n][lo:hi], colsq=colsq)
+                _all_reduce(colsq)
+                lam = pasta_normalize_columns(factors[n][lo:hi], colsq, lam=lam)
+                g = pasta_gram(factors[n][lo:hi])
+                grams[n] = _all_reduce(g)
+                if self.world > 1:
+                    gather_rows(factors[n], self.bounds[n])
+            lo, hi = int(self.bounds[N - 1][self.rank]), int(self.bounds[N - 1][self.rank + 1])
+            inner = _all_reduce(pasta_weighted_inner(self.out[N - 1][lo:hi],
+                                                     factors[N - 1][lo:hi], lam))
+            G = torch.ones((R, R), dtype=torch.float64, device=dev)
+            for g in grams:
+                G *= g
+            nxhat2 = float(lam @ G @ lam)
+            resid2 = max(normx2 + nxhat2 - 2.0 * float(inner.item()), 0.0)
+            fits.append(1.0 - (resid2 ** 0.5) / (normx2 ** 0.5) if normx2 > 0 else 0.0)
+            if it > 0 and abs(fits[-1] - fits[-2]) < tol:
+                break
+        return lam.cpu().numpy(), fits

@@ -48,3 +48,8 @@ def test_bench_two_ranks_shared_gpu():
     assert r2.returncode == 0, r2.stderr[-4000:]
     lines = [l for l in r2.stdout.splitlines() if l.startswith("{")]
     assert len(lines) == 1 and json.loads(lines[0])["impl"] == "reference"
+
+
+def test_row_partitioned_cpals_two_ranks_gloo():
+    r = _torchrun([os.path.join(ROOT, "tests", "mp_cpals_worker.py")])
+    assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-4000:]
