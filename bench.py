@@ -190,6 +190,7 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=10)
     ap.add_argument("--hicoo-steps", type=int, default=20)
+    ap.add_argument("--cpals-iters", type=int, default=5)
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3  # timing rule: >= 3 warm-up steps
@@ -355,6 +356,24 @@ def main():
                                   "mode_copies_all": round(t_hprep, 3)}}
         del h, houts
 
+    # NEXT-1: CP-ALS sweeps (each = MTTKRP + solve + normalise + gram for every mode)
+    cpals = None
+    if world == 1 and args.cpals_iters > 0:
+        Uc = [u.clone() for u in U]
+        pasta.pasta_cpals_coo(x, Uc, max_iters=1, tol=0.0)  # warm-up
+        Uc = [u.clone() for u in U]
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        lam_c, fits_c, it_c = pasta.pasta_cpals_coo(x, Uc, max_iters=args.cpals_iters, tol=0.0)
+        torch.cuda.synchronize()
+        c_ms = (time.perf_counter() - t0) * 1e3 / max(it_c, 1)
+        cpals = {"ms_per_sweep": round(c_ms, 3), "sweeps": it_c,
+                 "fit": [round(f, 6) for f in fits_c],
+                 "mttkrp_share": round(ms_per_step / c_ms, 3),
+                 "note": "pasta_cpals_coo from random U[0,1) factors; wall clock incl. the "
+                         "per-sweep fit read-back"}
+        del Uc
+
     if rank != 0:
         if world > 1:
             dist.destroy_process_group()
@@ -399,6 +418,7 @@ def main():
         "clocks": clk,
         "e2e": e2e,
         "hicoo": hicoo,
+        "cpals": cpals,
         "gpu_launches": launches,
         "cpu_baseline": cpu,
         "max_shard_nnz": per_launch_nnz,

@@ -117,10 +117,11 @@ class RowPartitionedCPALS(RowPartitionedMTTKRP):
             lo, hi = int(self.bounds[N - 1][self.rank]), int(self.bounds[N - 1][self.rank + 1])
             inner = _all_reduce(pasta_weighted_inner(self.out[N - 1][lo:hi],
                                                      factors[N - 1][lo:hi], lam))
-            G = torch.ones((R, R), dtype=torch.float64, device=dev)
+            G = np.ones((R, R))  # R x R host arithmetic: lambda^T (Hadamard_k G_k) lambda
             for g in grams:
-                G *= g
-            nxhat2 = float(lam @ G @ lam)
+                G *= g.cpu().numpy()
+            lh = lam.cpu().numpy()
+            nxhat2 = float(lh @ G @ lh)
             resid2 = max(normx2 + nxhat2 - 2.0 * float(inner.item()), 0.0)
             fits.append(1.0 - (resid2 ** 0.5) / (normx2 ** 0.5) if normx2 > 0 else 0.0)
             if it > 0 and abs(fits[-1] - fits[-2]) < tol:
