@@ -111,7 +111,18 @@ struct CooModeCopy {
   const float *val = nullptr;
   DevArray<uint32_t> own_inds[kMaxOrder];
   DevArray<float> own_val;
+  // Hot-row cache (coo_mark_hot): the most frequent rows of the gathered factors, packed into
+  // one contiguous buffer that fits the L2 budget for rank hot_R.  hot_inds[k] (k != mode)
+  // = inds[k] for cold entries, 0x80000000 | slot for hot ones (slot into hot_buf).
+  uint32_t hot_R = 0;       // 0: not marked
+  uint32_t hot_bucket = 0;  // rows with count bucket >= hot_bucket are hot
+  DevArray<uint32_t> hot_inds[kMaxOrder];
+  DevArray<uint32_t> hot_rows;          // slot -> factor row, factor k at [hot_base[k], +hot_cnt[k])
+  uint64_t hot_base[kMaxOrder] = {}, hot_cnt[kMaxOrder] = {}, hot_total = 0;
+  DevArray<float> hot_buf;              // hot_total x R, refilled from the factors every launch
 };
+
+constexpr int kCountBuckets = 256;  // 8 sub-buckets per octave of a row's nonzero count
 
 struct HicooModeCopy {
   bool ready = false;
@@ -156,6 +167,10 @@ struct pasta_coo {
   pasta::DevArray<float> stage_f[pasta::kMaxOrder];
   pasta::DevArray<float> stage_o[pasta::kMaxOrder];
   pasta::E2EStreams e2e;
+  // per-mode row nonzero counts (device u32) and their bucket histogram (host)
+  bool counts_ready[pasta::kMaxOrder] = {};
+  pasta::DevArray<uint32_t> row_count[pasta::kMaxOrder];
+  uint64_t count_hist[pasta::kMaxOrder][pasta::kCountBuckets] = {};
   std::mutex mu;
 };
 
@@ -221,6 +236,9 @@ void launch_normalize(float *U, uint64_t rows, uint32_t R, const double *colsq, 
 void launch_inner(const float *A, const float *B, uint64_t rows, uint32_t R, const double *lambda,
                   double *out, cudaStream_t s);
 void launch_sumsq(const float *v, uint64_t n, double *out, cudaStream_t s);
+void coo_mark_hot(pasta_coo *x, uint32_t mode, uint32_t R, cudaStream_t s);
+void launch_hot_fill(const CooModeCopy &mc, const float *const *factors, uint32_t order, uint32_t mode,
+                     uint32_t R, cudaStream_t s);
 void row_counts_device(const uint32_t *rows, uint64_t nnz, uint32_t nrows, uint64_t *counts_host,
                        cudaStream_t s);
 // first position x in the sorted array a[0..M) with a[x] >= v (device binary search).

@@ -63,6 +63,9 @@ struct KArgs {
   // L2 eviction-priority hints (bit 0: streams evict_first, bit 1: gathers evict_last,
   // bit 2: output stores / atomics evict_first); see Policies
   uint32_t cache_mode;
+  // io[] carry a hot flag in bit 31 (coo_mark_hot): hot entries hold a slot of hot_buf
+  uint32_t hot_marked;
+  const float *hot_buf;
 };
 
 // Per-thread L2 cache policies (createpolicy, sm_80+): the nonzero stream is touched once
@@ -611,8 +614,13 @@ __global__ void __launch_bounds__(kThreads) hicoo_heavy_kernel(const HArgs a) {
 // .cg, L2 evict_first policy: every 128-B line is consumed by one copy, so the stream never
 // needs to linger in L2 and does not displace power-law-hot factor rows), double-buffered
 // one stage (32 nonzeros per group) ahead of the gathers.
+// WA: 0/1/2 buffer-address forms (see the launcher); 3, 4, 5 are measurement probes that
+// decompose the kernel time (3: no output writes, 4: no factor gathers, 5: stream only).
 template <int NO, int LPN, int WA>
 __global__ void __launch_bounds__(kThreads, 2) coo_staged_kernel(const KArgs a) {
+  constexpr bool kGather = WA != 4 && WA != 5;
+  constexpr bool kWrite = WA != 3 && WA != 5;
+  constexpr int kBuf = (WA == 0 || WA == 2) ? WA : 1;
   constexpr int G = 32 / LPN;
   constexpr int SG = 32;          // nonzeros per group per stage
   constexpr int SW = G * SG;      // nonzeros per warp per stage
@@ -632,6 +640,8 @@ __global__ void __launch_bounds__(kThreads, 2) coo_staged_kernel(const KArgs a) 
   const uint32_t R = a.R;
   const uint32_t col = uint32_t(lig) * 4;
   const Policies pol(a.cache_mode | 1u);  // the staged stream is always evict_first
+  uint64_t pol_hot = pol.gather;
+  if (a.cache_mode & 8) asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol_hot));
   const uint32_t *src[NA];
   src[0] = a.irow;
 #pragma unroll
@@ -648,7 +658,7 @@ __global__ void __launch_bounds__(kThreads, 2) coo_staged_kernel(const KArgs a) 
       for (int arr = 0; arr < NA; ++arr) {
         const uint32_t d = smem_addr(dst + arr * SW + gi * SG + k * 4);
         const uint32_t *sp = src[arr] + (valid ? pos : 0);
-        if (WA == 2) {
+        if (kBuf == 2) {
           asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(d), "l"(sp), "r"(valid)
                        : "memory");
         } else {
@@ -661,7 +671,7 @@ __global__ void __launch_bounds__(kThreads, 2) coo_staged_kernel(const KArgs a) 
     asm volatile("cp.async.commit_group;" ::: "memory");
   };
   auto issue = [&](int s) {
-    if (WA == 1) {
+    if (kBuf == 1) {
       if (s & 1) issue_to(s, wbuf + NA * SW); else issue_to(s, wbuf);
     } else {
       issue_to(s, wbuf + (s & 1) * NA * SW);
@@ -705,8 +715,21 @@ __global__ void __launch_bounds__(kThreads, 2) coo_staged_kernel(const KArgs a) 
 #pragma unroll
         for (int u = 0; u < U; ++u) {
 #pragma unroll
-          for (int j = 0; j < NO; ++j)
-            if (u < cnt) f[j][u] = ldg_vec<4>(a.Uo[j] + uint64_t(idx[j][u]) * R + col, pol.gather);
+          for (int j = 0; j < NO; ++j) {
+            if (kGather) {
+              const float *base = a.Uo[j];
+              uint64_t gp = pol.gather;
+              if (a.hot_marked && (idx[j][u] >> 31)) {  // a row of the packed hot-row cache
+                base = a.hot_buf;
+                idx[j][u] &= 0x7FFFFFFFu;
+                gp = pol_hot;
+              }
+              if (u < cnt) f[j][u] = ldg_vec<4>(base + uint64_t(idx[j][u]) * R + col, gp);
+            } else {
+#pragma unroll
+              for (int i = 0; i < 4; ++i) f[j][u].v[i] = __uint_as_float(idx[j][u] | 0x3f800000u);
+            }
+          }
         }
 #pragma unroll
         for (int u = 0; u < U; ++u) {
@@ -725,7 +748,11 @@ __global__ void __launch_bounds__(kThreads, 2) coo_staged_kernel(const KArgs a) 
             } else {
               if (cur != 0xFFFFFFFFu) {
                 float *dst = a.out + uint64_t(cur) * R + col;
-                if (first) red_vec<4>(dst, acc, pol.out); else st_vec<4>(dst, acc, pol.out);
+                if (kWrite) {
+                  if (first) red_vec<4>(dst, acc, pol.out); else st_vec<4>(dst, acc, pol.out);
+                } else if (acc.v[0] == 1.2345e-30f) {
+                  st_vec<4>(dst, acc, pol.out);  // keeps the arithmetic live in probes
+                }
                 first = false;
               }
               cur = row[u];
@@ -737,7 +764,8 @@ __global__ void __launch_bounds__(kThreads, 2) coo_staged_kernel(const KArgs a) 
     }
     __syncwarp();  // the buffer of stage s is refilled at stage s + 2
   }
-  if (active && cur != 0xFFFFFFFFu) red_vec<4>(a.out + uint64_t(cur) * R + col, acc, pol.out);
+  if (active && cur != 0xFFFFFFFFu && (kWrite || acc.v[0] == 1.2345e-30f))
+    red_vec<4>(a.out + uint64_t(cur) * R + col, acc, pol.out);
 }
 
 template <int VW>
@@ -885,6 +913,27 @@ void launch_coo_mttkrp(const pasta_coo *x, uint32_t mode, const float *const *fa
   const int staged = env_int("PASTA_COO_STAGED", 1);
   const int no = int(x->order) - 1;
   if (staged && vec4 && (R == 16 || R == 32) && (no == 2 || no == 3)) {
+    // the hot-row cache pays only when the gathered factors do not fit in L2 already
+    static int l2 = 0;
+    if (!l2) {
+      int dev = 0;
+      cudaGetDevice(&dev);
+      cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, dev);
+      if (l2 <= 0) l2 = 126 << 20;
+    }
+    uint64_t gathered = 0;
+    for (uint32_t k = 0; k < x->order; ++k)
+      if (k != mode) gathered += uint64_t(x->dims[k]) * R * sizeof(float);
+    const bool want_hot = env_int("PASTA_HOT_FORCE", 0) || gathered > uint64_t(l2);
+    if (want_hot) coo_mark_hot(const_cast<pasta_coo *>(x), mode, R, s);
+    if (want_hot && mc.hot_R == R) {
+      a.hot_marked = 1;
+      a.hot_buf = mc.hot_buf.p;
+      int jj = 0;
+      for (uint32_t k = 0; k < x->order; ++k)
+        if (k != mode) a.io[jj++] = mc.hot_inds[k].p;
+      launch_hot_fill(mc, factors, x->order, mode, R, s);
+    }
     const int lpn = R == 16 ? 4 : 8;
     const int G = 32 / lpn;
     uint64_t run = uint64_t(env_int("PASTA_MTTKRP_RUN", 128));
@@ -894,9 +943,39 @@ void launch_coo_mttkrp(const pasta_coo *x, uint32_t mode, const float *const *fa
     const size_t smem = size_t(kWarpsPerCta) * 2 * (no + 2) * (G * 32) * sizeof(uint32_t);
     uint64_t nwarps = (a.nnz + a.chunk - 1) / a.chunk;
     uint64_t nblk = (nwarps + kWarpsPerCta - 1) / kWarpsPerCta;
+    // PASTA_HOT_PERSIST=1: launch with an L2 access-policy window marking the hot-row buffer
+    // persisting (within the device's persisting carve-out)
+    const bool persist = a.hot_marked && env_int("PASTA_HOT_PERSIST", 0);
     auto go = [&](auto kern) {
       PASTA_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem)));
-      kern<<<unsigned(nblk), kThreads, smem, s>>>(a);
+      if (!persist) {
+        kern<<<unsigned(nblk), kThreads, smem, s>>>(a);
+      } else {
+        static size_t carve = 0;
+        const size_t want = mc.hot_buf.bytes();
+        if (carve == 0) {
+          int dev = 0, maxp = 0;
+          cudaGetDevice(&dev);
+          cudaDeviceGetAttribute(&maxp, cudaDevAttrMaxPersistingL2CacheSize, dev);
+          carve = size_t(maxp);
+          PASTA_CUDA(cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, carve));
+        }
+        cudaLaunchConfig_t cfg = {};
+        cfg.gridDim = dim3(unsigned(nblk));
+        cfg.blockDim = dim3(kThreads);
+        cfg.dynamicSmemBytes = smem;
+        cfg.stream = s;
+        cudaLaunchAttribute attr[1];
+        attr[0].id = cudaLaunchAttributeAccessPolicyWindow;
+        attr[0].val.accessPolicyWindow.base_ptr = mc.hot_buf.p;
+        attr[0].val.accessPolicyWindow.num_bytes = want;
+        attr[0].val.accessPolicyWindow.hitRatio = want <= carve ? 1.0f : float(double(carve) / double(want));
+        attr[0].val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+        attr[0].val.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+        cfg.attrs = attr;
+        cfg.numAttrs = 1;
+        PASTA_CUDA(cudaLaunchKernelEx(&cfg, kern, a));
+      }
       PASTA_LAUNCHED();
     };
     // WA 1 (default): one code path per buffer.  ptxas 12.9 turns the computed buffer
@@ -913,6 +992,9 @@ void launch_coo_mttkrp(const pasta_coo *x, uint32_t mode, const float *const *fa
     };
     if (wa == 1) pick(std::integral_constant<int, 1>());
     else if (wa == 2) pick(std::integral_constant<int, 2>());
+    else if (wa == 3) pick(std::integral_constant<int, 3>());
+    else if (wa == 4) pick(std::integral_constant<int, 4>());
+    else if (wa == 5) pick(std::integral_constant<int, 5>());
     else pick(std::integral_constant<int, 0>());
     return;
   }

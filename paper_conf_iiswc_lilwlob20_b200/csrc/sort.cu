@@ -3,6 +3,10 @@
 // gathers, compaction, histograms.  Pre-processing trades for kernel time.
 #include <cub/cub.cuh>
 
+#include <cstdio>
+#include <cstdlib>
+#include <vector>
+
 #include "internal.cuh"
 
 namespace pasta {
@@ -248,6 +252,190 @@ bool is_lex_sorted_device(const uint32_t *const *inds, uint32_t order, uint64_t 
   PASTA_CUDA(cudaMemcpyAsync(&h, flag.p, sizeof(h), cudaMemcpyDeviceToHost, s));
   PASTA_CUDA(cudaStreamSynchronize(s));
   return h == 0;
+}
+
+}  // namespace pasta
+
+// ------------------------------------------------------------------------------------------
+// Frequency-aware L2 eviction priority for the COO factor gathers (see coo_mark_hot).
+namespace pasta {
+namespace {
+
+__device__ __host__ inline uint32_t count_bucket(uint32_t c) {
+  if (c == 0) return 0;
+  uint32_t e = 31 - __builtin_clz(c);
+  uint32_t m = e >= 3 ? (c >> (e - 3)) & 7u : (c << (3 - e)) & 7u;
+  return 8 * e + m;
+}
+
+__device__ inline uint32_t count_bucket_dev(uint32_t c) {
+  if (c == 0) return 0;
+  uint32_t e = 31 - __clz(c);
+  uint32_t m = e >= 3 ? (c >> (e - 3)) & 7u : (c << (3 - e)) & 7u;
+  return 8 * e + m;
+}
+
+__global__ void count_rows_kernel(const uint32_t *__restrict__ rows, uint64_t M, uint32_t *__restrict__ cnt) {
+  for (uint64_t x = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; x < M;
+       x += uint64_t(gridDim.x) * blockDim.x)
+    atomicAdd(&cnt[rows[x]], 1u);
+}
+
+__global__ void bucket_hist_kernel(const uint32_t *__restrict__ cnt, uint64_t n,
+                                   unsigned long long *__restrict__ hist) {
+  __shared__ unsigned long long h[kCountBuckets];
+  for (int b = threadIdx.x; b < kCountBuckets; b += blockDim.x) h[b] = 0;
+  __syncthreads();
+  for (uint64_t i = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; i < n;
+       i += uint64_t(gridDim.x) * blockDim.x)
+    if (cnt[i]) atomicAdd(&h[count_bucket_dev(cnt[i])], 1ull);
+  __syncthreads();
+  for (int b = threadIdx.x; b < kCountBuckets; b += blockDim.x)
+    if (h[b]) atomicAdd(&hist[b], h[b]);
+}
+
+__global__ void hot_flag_kernel(const uint32_t *__restrict__ cnt, uint64_t n, uint32_t hot_bucket,
+                                uint8_t *__restrict__ flag) {
+  for (uint64_t i = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; i < n;
+       i += uint64_t(gridDim.x) * blockDim.x)
+    flag[i] = cnt[i] && count_bucket_dev(cnt[i]) >= hot_bucket;
+}
+
+__global__ void slot_map_kernel(const uint32_t *__restrict__ rows, uint64_t nh, uint64_t base,
+                                uint32_t *__restrict__ slot_of, uint32_t *__restrict__ hot_rows) {
+  for (uint64_t s = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; s < nh;
+       s += uint64_t(gridDim.x) * blockDim.x) {
+    slot_of[rows[s]] = uint32_t(base + s);
+    hot_rows[base + s] = rows[s];
+  }
+}
+
+__global__ void mark_hot_kernel(const uint32_t *__restrict__ src, const uint32_t *__restrict__ slot_of,
+                                uint64_t M, uint32_t *__restrict__ dst) {
+  for (uint64_t x = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; x < M;
+       x += uint64_t(gridDim.x) * blockDim.x) {
+    const uint32_t v = src[x];
+    const uint32_t sl = __ldg(slot_of + v);
+    dst[x] = sl != 0xFFFFFFFFu ? (0x80000000u | sl) : v;
+  }
+}
+
+// hot_buf[s][:] = U[hot_rows[s]][:] for the slots [base, base + n) of one factor (float4)
+__global__ void hot_fill_kernel(const float4 *__restrict__ U, const uint32_t *__restrict__ hot_rows,
+                                uint64_t base, uint64_t n, uint32_t r4, float4 *__restrict__ buf) {
+  for (uint64_t e = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; e < n * r4;
+       e += uint64_t(gridDim.x) * blockDim.x) {
+    const uint64_t s = e / r4, c = e % r4;
+    buf[(base + s) * r4 + c] = __ldg(U + uint64_t(__ldg(hot_rows + base + s)) * r4 + c);
+  }
+}
+
+unsigned grid8(uint64_t n) {
+  uint64_t b = (n + 256 * 8 - 1) / (256 * 8);
+  if (b < 1) b = 1;
+  if (b > (1u << 30)) b = 1u << 30;
+  return unsigned(b);
+}
+
+}  // namespace
+
+// Hot-row cache for the COO factor gathers.  The most frequent rows of the gathered factors
+// (row nonzero counts, bucketed), as many as fit PASTA_HOT_MB (default 64 MB of the 126 MB
+// L2) at R*4 bytes per row, get contiguous slots of one buffer that is refilled from the
+// factors before every launch; the per-mode index copies point hot entries at their slot
+// (bit 31 set).  Packed hot rows fill whole L2 lines and stay resident, where scattered ones
+// share lines with cold neighbours and are evicted by the cold-row and stream traffic: L2
+// turns from LRU over scattered rows into a frequency-based cache for the power-law gathers
+// (cache reuse is why MTTKRP beats its DRAM roofline).  Needs dims < 2^31.
+void coo_mark_hot(pasta_coo *x, uint32_t mode, uint32_t R, cudaStream_t s) {
+  CooModeCopy &mc = x->mc[mode];
+  if (mc.hot_R == R) return;
+  const char *env = getenv("PASTA_HOT_MB");
+  const double hot_mb = (env && *env) ? atof(env) : 64.0;
+  const uint32_t N = x->order;
+  const uint64_t M = x->nnz;
+  for (uint32_t k = 0; k < N; ++k)
+    if (x->dims[k] >= 0x80000000u) return;
+  if (hot_mb <= 0 || M == 0) return;
+  for (uint32_t k = 0; k < N; ++k) {
+    if (k == mode || x->counts_ready[k]) continue;
+    x->row_count[k].alloc(x->dims[k], s);
+    PASTA_CUDA(cudaMemsetAsync(x->row_count[k].p, 0, x->row_count[k].bytes(), s));
+    count_rows_kernel<<<grid8(M), 256, 0, s>>>(x->inds[k].p, M, x->row_count[k].p);
+    PASTA_LAUNCHED();
+    DevArray<unsigned long long> h(kCountBuckets, s);
+    PASTA_CUDA(cudaMemsetAsync(h.p, 0, h.bytes(), s));
+    bucket_hist_kernel<<<grid8(x->dims[k]), 256, 0, s>>>(x->row_count[k].p, x->dims[k], h.p);
+    PASTA_LAUNCHED();
+    PASTA_CUDA(cudaMemcpyAsync(x->count_hist[k], h.p, h.bytes(), cudaMemcpyDeviceToHost, s));
+    PASTA_CUDA(cudaStreamSynchronize(s));
+    x->counts_ready[k] = true;
+  }
+  // smallest bucket b* such that the rows with bucket >= b* of every gathered factor fit
+  const double budget_rows = hot_mb * 1048576.0 / (double(R) * 4.0);
+  uint32_t hb = kCountBuckets;
+  double acc = 0.0;
+  for (int b = kCountBuckets - 1; b >= 1; --b) {
+    double add = 0.0;
+    for (uint32_t k = 0; k < N; ++k)
+      if (k != mode) add += double(x->count_hist[k][b]);
+    if (acc + add > budget_rows) break;
+    acc += add;
+    hb = uint32_t(b);
+  }
+  // hot rows of each gathered factor -> contiguous slots of one buffer
+  uint64_t total = 0;
+  std::vector<DevArray<uint32_t>> lists(N);
+  for (uint32_t k = 0; k < N; ++k) {
+    mc.hot_base[k] = total;
+    mc.hot_cnt[k] = 0;
+    if (k == mode) continue;
+    DevArray<uint8_t> flag(x->dims[k], s);
+    hot_flag_kernel<<<grid8(x->dims[k]), 256, 0, s>>>(x->row_count[k].p, x->dims[k], hb, flag.p);
+    PASTA_LAUNCHED();
+    mc.hot_cnt[k] = select_flagged(flag.p, x->dims[k], lists[k], s);
+    total += mc.hot_cnt[k];
+  }
+  mc.hot_total = total;
+  mc.hot_rows.alloc(total ? total : 1, s);
+  mc.hot_buf.alloc((total ? total : 1) * R, s);
+  for (uint32_t k = 0; k < N; ++k) {
+    if (k == mode) continue;
+    DevArray<uint32_t> slot_of(x->dims[k], s);
+    PASTA_CUDA(cudaMemsetAsync(slot_of.p, 0xFF, slot_of.bytes(), s));
+    if (mc.hot_cnt[k]) {
+      slot_map_kernel<<<grid8(mc.hot_cnt[k]), 256, 0, s>>>(lists[k].p, mc.hot_cnt[k], mc.hot_base[k],
+                                                          slot_of.p, mc.hot_rows.p);
+      PASTA_LAUNCHED();
+    }
+    if (mc.hot_inds[k].n != M) mc.hot_inds[k].alloc(M, s);
+    mark_hot_kernel<<<grid8(M), 256, 0, s>>>(mc.inds[k], slot_of.p, M, mc.hot_inds[k].p);
+    PASTA_LAUNCHED();
+    PASTA_CUDA(cudaStreamSynchronize(s));  // slot_of is released at scope exit
+  }
+  mc.hot_bucket = hb;
+  mc.hot_R = R;
+  if (getenv("PASTA_DEBUG")) {
+    fprintf(stderr, "[pasta] hot cache mode %u R %u: budget %.0f rows, bucket >= %u, %llu hot rows (",
+            mode, R, budget_rows, hb, (unsigned long long)total);
+    for (uint32_t k = 0; k < N; ++k)
+      if (k != mode) fprintf(stderr, " k%u:%llu", k, (unsigned long long)mc.hot_cnt[k]);
+    fprintf(stderr, " )\n");
+  }
+}
+
+void launch_hot_fill(const CooModeCopy &mc, const float *const *factors, uint32_t order, uint32_t mode,
+                     uint32_t R, cudaStream_t s) {
+  for (uint32_t k = 0; k < order; ++k) {
+    if (k == mode || mc.hot_cnt[k] == 0) continue;
+    const uint64_t n = mc.hot_cnt[k] * (R / 4);
+    uint64_t g = (n + 255) / 256;
+    if (g > 148 * 32) g = 148 * 32;
+    hot_fill_kernel<<<unsigned(g), 256, 0, s>>>(reinterpret_cast<const float4 *>(factors[k]), mc.hot_rows.p,
+                                                mc.hot_base[k], mc.hot_cnt[k], R / 4,
+                                                reinterpret_cast<float4 *>(mc.hot_buf.p));
+    PASTA_LAUNCHED();
+  }
 }
 
 }  // namespace pasta

@@ -276,12 +276,15 @@ def test_profile_and_launch_counters(env):
     pasta.pasta_profile_read(0, reset=True)
     pasta.pasta_profile_enable(True)
     n0 = pasta.pasta_launch_count()
-    for _ in range(3):
+    pasta.pasta_mttkrp_coo(x, 0, Ud)
+    per_call = pasta.pasta_launch_count() - n0  # zero-fill (+ hot-row fills) + MTTKRP
+    for _ in range(2):
         pasta.pasta_mttkrp_coo(x, 0, Ud)
     ms, n = pasta.pasta_profile_read(0, reset=True)
     pasta.pasta_profile_enable(False)
     assert n == 3 and ms > 0
-    assert pasta.pasta_launch_count() - n0 == 6  # zero-fill + MTTKRP per call
+    assert 2 <= per_call <= 2 + len(dims) - 1
+    assert pasta.pasta_launch_count() - n0 == 3 * per_call
 
 
 def test_errors_on_device(env):
@@ -364,3 +367,29 @@ def test_torch_caching_allocator_hook(env):
         gc.collect()
     finally:
         pasta.pasta_set_allocator(None)
+
+
+@pytest.mark.parametrize("hot_mb", ["0.05", "1"])
+def test_coo_hot_row_cache_forced(env, hot_mb, monkeypatch):
+    """The packed hot-row cache (coo_mark_hot) is enabled automatically only when the gathered
+    factors exceed L2; force it on small tensors (tiny budgets so that hot and cold rows mix)."""
+    pasta, oracle, torch = env
+    monkeypatch.setenv("PASTA_HOT_FORCE", "1")
+    monkeypatch.setenv("PASTA_HOT_MB", hot_mb)
+    for dims, nnz, R in [((3000, 2000, 4000), 120_000, 16), ((300, 400, 500, 60), 80_000, 32),
+                         ((5000, 3000, 2000), 0, 16)]:
+        if nnz:
+            inds, vals = si.powerlaw_coo(dims, nnz, seed=nnz + R)
+        else:
+            inds, vals = si.hot_row_coo(dims, 300_000, 50_000, seed=4, mode=1, hot_row=0)
+        U = si.factors(dims, R, seed=R)
+        Ud = _dev(torch, U)
+        x = pasta.pasta_coo_from_arrays(dims, inds, vals)
+        for n in range(len(dims)):
+            ref, ab = oracle.mttkrp(dims, inds, vals, n, U)
+            _check(pasta.pasta_mttkrp_coo(x, n, Ud), ref, ab, f"hot cache {dims} R={R} mode {n}")
+        # factors change between calls (CP-ALS): the cache is refilled every launch
+        Ud2 = [u * 0.5 for u in Ud]
+        U2 = [u.cpu().numpy() for u in Ud2]
+        ref, ab = oracle.mttkrp(dims, inds, vals, 0, U2)
+        _check(pasta.pasta_mttkrp_coo(x, 0, Ud2), ref, ab, "hot cache refill")
