@@ -617,10 +617,10 @@ __global__ void __launch_bounds__(kThreads) hicoo_heavy_kernel(const HArgs a) {
 // WA: 0/1/2 buffer-address forms (see the launcher); 3, 4, 5 are measurement probes that
 // decompose the kernel time (3: no output writes, 4: no factor gathers, 5: stream only).
 template <int NO, int LPN, int WA>
-__global__ void __launch_bounds__(kThreads, 2) coo_staged_kernel(const KArgs a) {
+__global__ void __launch_bounds__(kThreads, WA == 6 ? 3 : 2) coo_staged_kernel(const KArgs a) {
   constexpr bool kGather = WA != 4 && WA != 5;
   constexpr bool kWrite = WA != 3 && WA != 5;
-  constexpr int kBuf = (WA == 0 || WA == 2) ? WA : 1;
+  constexpr int kBuf = (WA == 0 || WA == 2) ? WA : 1;  // 6: form 1 with 3 CTAs per SM
   constexpr int G = 32 / LPN;
   constexpr int SG = 32;          // nonzeros per group per stage
   constexpr int SW = G * SG;      // nonzeros per warp per stage
@@ -995,6 +995,7 @@ void launch_coo_mttkrp(const pasta_coo *x, uint32_t mode, const float *const *fa
     else if (wa == 3) pick(std::integral_constant<int, 3>());
     else if (wa == 4) pick(std::integral_constant<int, 4>());
     else if (wa == 5) pick(std::integral_constant<int, 5>());
+    else if (wa == 6) pick(std::integral_constant<int, 6>());
     else pick(std::integral_constant<int, 0>());
     return;
   }
