@@ -4,13 +4,16 @@
     python bench.py [--gpus N] [--steps K] [--warmup W] [--config h|c2|c3|c4|c1] [--impl reference]
 
 One STEP = COO MTTKRP of every mode (output zero-fill + kernel, the paper times all modes and
-averages) over the synthetic tensor resident in HBM; at N > 1 each rank runs its
-nnz-balanced row shard of every mode and the owned output rows are all-gathered (NCCL).
-Rank 0 prints one JSON line.  GFLOP/s uses the nominal N*M*R flops per mode (Table I
-generalised; R#7).
+averages) over the synthetic tensor resident in HBM.  Rank 0 prints one JSON line.
+GFLOP/s uses the nominal N*M*R flops per mode (Table I generalised; R#7).
 
 The default workload is the north_star target: a 100M-nonzero 3rd-order power-law tensor,
-regL-shaped (2^23)^3 (Table II s3), R = 16.
+regL-shaped (2^23)^3 (Table II s3), R = 16.  At N GPUs (torchrun) the tensor has
+N x 100M nonzeros of the same draw sequence and shape (weak scaling, cf. BASELINE config 5:
+1B nonzeros at 8 GPUs); every rank owns the nnz-balanced row shard of every mode and the
+timed step has no collective.  The all-gather of the owned output rows over NCCL -- needed
+only when the next CP-ALS step consumes the factor (north_star) -- is timed separately
+(`allgather` object).
 
 --impl reference times the fp64 CPU oracle (oracle/, the slow correctness reference) on a
 bounded sample of the same workload on the host cores; under torchrun only rank 0 works.
@@ -154,20 +157,28 @@ def ncu_traffic(config_key, family="coo_mttkrp"):
         return None
 
 
+def workload_name(key, cfg, world):
+    if world == 1:
+        return f"{key}: {cfg['name']}"
+    return f"{key}x{world}: {cfg['name']} grown to {world} x {cfg['nnz']} nonzeros (weak scaling)"
+
+
 def run_reference(args, cfg, world, rank):
     if rank != 0:
         return
     R = cfg["R"]
+    M_total = cfg["nnz"] * world
     sample = args.ref_sample
     gflops, t = cpu_baseline(cfg, R, sample, steps=args.steps, warmup=args.warmup)
     cores = 1
     line = {
         "impl": "reference", "metric": METRIC, "value": round(gflops, 4), "unit": "GFLOP/s",
         "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
-        "ms_per_step": round(t * 1e3, 3), "higher_is_better": True, "scaling": "strong",
+        "ms_per_step": round(t * 1e3, 3), "higher_is_better": True,
+        "scaling": "weak" if world > 1 else "strong",
         "vs_baseline": None, "dtype": "f64", "data": "synthetic (oracle generator, same draws)",
-        "config": {"workload": f"{args.config}: {cfg['name']}", "dims": list(cfg["dims"]),
-                   "nnz": cfg["nnz"], "R": R, "format": "COO", "modes": "all"},
+        "config": {"workload": workload_name(args.config, cfg, world), "dims": list(cfg["dims"]),
+                   "nnz": M_total, "R": R, "format": "COO", "modes": "all"},
         "cpu_baseline": {"value": round(gflops, 4), "unit": "GFLOP/s", "cores": cores,
                          "kind": "oracle",
                          "sample": f"first {sample} distinct nonzeros of the workload's draw "
@@ -220,7 +231,8 @@ def main():
             dist.init_process_group("nccl", device_id=dev)
     stream = torch.cuda.current_stream()
 
-    dims, R, M = cfg["dims"], cfg["R"], cfg["nnz"]
+    dims, R = cfg["dims"], cfg["R"]
+    M = cfg["nnz"] * world  # weak scaling: cfg["nnz"] nonzeros per GPU
     N = len(dims)
     t0 = time.perf_counter()
     x = pasta.pasta_gen_powerlaw(dims, M, cfg["seed"], kind=0 if cfg["kind"] == "uniform" else 1)
@@ -238,12 +250,11 @@ def main():
     if world > 1:
         part = RowPartitionedMTTKRP(x, rank, world, R, dev)
         shard_nnz = part.shard_nnz()
-        x_local = None
         del x
         torch.cuda.synchronize()
 
         def step():
-            part.step(U, gather=True)
+            part.step(U, gather=False)
     else:
         outs = [torch.empty((d, R), dtype=torch.float32, device=dev) for d in dims]
         shard_nnz = [M] * N
@@ -291,7 +302,7 @@ def main():
     total_flops = N * model_flops(N, M, R)  # all ranks together, every mode
     value = total_flops / (ms_per_step * 1e-3) / 1e9
 
-    # e2e: the same metric through the public C ABI with HOST buffers (pinned)
+    # e2e: the same metric through the public API with HOST buffers (pinned)
     e2e = None
     if world == 1 and args.e2e_steps > 0:
         hf = [u.cpu().pin_memory() for u in U]
@@ -310,6 +321,69 @@ def main():
                "path": "pasta_mttkrp_coo_allmodes_host (pinned host factors in, results out; copies "
                        "pipelined against the kernels on two copy streams; wall clock)"}
         del hf, ho
+
+    # N > 1: the exchange step, timed apart from the MTTKRP step (max over ranks)
+    allgather = None
+    if world > 1:
+        from paper_conf_iiswc_lilwlob20_b200.parallel import gather_rows
+
+        def gather_step():
+            works = []
+            for n in range(N):
+                works += gather_rows(part.out[n], part.bounds[n], async_op=True)
+            for w in works:
+                w.wait()
+
+        for _ in range(2):
+            gather_step()
+        torch.cuda.synchronize()
+        dist.barrier()
+        g0, g1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        gsteps = max(3, min(args.steps, 10))
+        g0.record(stream)
+        for _ in range(gsteps):
+            gather_step()
+        g1.record(stream)
+        torch.cuda.synchronize()
+        dist.barrier()
+        t = torch.tensor([g0.elapsed_time(g1) / gsteps], device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        g_ms = float(t.item())
+        recv = sum((d - (int(part.bounds[n][rank + 1]) - int(part.bounds[n][rank]))) * R * 4
+                   for n, d in enumerate(dims))
+        allgather = {"ms_per_step": round(g_ms, 4), "bytes_received_per_rank": recv,
+                     "gbs_per_rank": round(recv / (g_ms * 1e-3) / 1e9, 1),
+                     "value_with_allgather": round(N * model_flops(N, M, R) /
+                                                   ((elapsed_ms / args.steps + g_ms) * 1e-3) / 1e9, 3),
+                     "how": "in-place uneven all-gather of owned output rows: one NCCL broadcast "
+                            "per rank per mode (parallel.gather_rows)"}
+    if world > 1 and args.e2e_steps > 0:
+        hf = [u.cpu().pin_memory() for u in U]
+        own = [(int(part.bounds[n][rank]), int(part.bounds[n][rank + 1])) for n in range(N)]
+        ho = [torch.empty((hi - lo, R), dtype=torch.float32).pin_memory() for lo, hi in own]
+
+        def e2e_step():
+            for k in range(N):
+                U[k].copy_(hf[k], non_blocking=True)
+            part.step(U, gather=False)
+            for n, (lo, hi) in enumerate(own):
+                ho[n].copy_(part.out[n][lo:hi], non_blocking=True)
+            torch.cuda.synchronize()
+
+        e2e_step()
+        dist.barrier()
+        t0 = time.perf_counter()
+        for _ in range(args.e2e_steps):
+            e2e_step()
+        t = torch.tensor([(time.perf_counter() - t0) * 1e3 / args.e2e_steps], device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        e_ms = float(t.item())
+        e2e = {"value": round(N * model_flops(N, M, R) / (e_ms * 1e-3) / 1e9, 3), "unit": "GFLOP/s",
+               "h2d_bytes_per_step": sum(d * R * 4 for d in dims),
+               "d2h_bytes_per_step": sum((hi - lo) * R * 4 for lo, hi in own),
+               "ms_per_step": round(e_ms, 3),
+               "path": "per rank: pinned factors H2D, pasta_mttkrp_coo on the rank's shards, owned "
+                       "rows D2H (wall clock, max over ranks); bytes are rank 0's"}
 
     # a7: HiCOO MTTKRP (B = 128) on the same tensor, every mode per step
     hicoo = None
@@ -398,12 +472,13 @@ def main():
     line = {
         "metric": METRIC, "value": round(value, 3), "unit": "GFLOP/s", "n_gpus": world,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms_per_step, 4),
-        "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f32",
+        "higher_is_better": True, "scaling": "weak" if world > 1 else "strong",
+        "vs_baseline": None, "dtype": "f32",
         "data": f"synthetic: GPU Stochastic Kronecker generator (q=0.75), seed {cfg['seed']}",
-        "config": {"workload": f"{args.config}: {cfg['name']}", "dims": list(dims), "nnz": M,
+        "config": {"workload": workload_name(args.config, cfg, world), "dims": list(dims), "nnz": M,
                    "R": R, "format": "COO", "modes": f"all {N} per step",
-                   "parallelism": f"row-partitioned x{world}" + (" + NCCL all-gather" if world > 1
-                                                                  else ""),
+                   "parallelism": f"row-partitioned x{world}, no collective in the step" +
+                                  (" (NCCL all-gather timed separately)" if world > 1 else ""),
                    "l2": "no flush: per-step working set (COO copies + factors + outputs) "
                          "> 126 MB L2"},
         "model_gbs": round(model_bytes_coo(N, M, R) * N / (ms_per_step * 1e-3) / 1e9, 1),
@@ -412,11 +487,17 @@ def main():
                      "kernel": "mttkrp_kernel<CooSrc> (a6)",
                      "bytes_model": "4(N+1)M + 4NRM per launch (Table I, P:117)",
                      "avg_launch_ms": round(avg_launch_ms, 4), "launches": kern_n,
-                     "peak_source": peak_src},
+                     "peak_source": peak_src,
+                     "dram_gbs": round(traffic / (avg_launch_ms * 1e-3) / 1e9, 1) if traffic else None,
+                     "dram_frac": round(traffic / (avg_launch_ms * 1e-3) / 1e9 / peak, 4)
+                     if traffic else None,
+                     "note": "frac uses the paper's byte model, which counts every factor gather as a "
+                             "DRAM access (P:117); dram_* use the ncu-measured traffic"},
         "zero_fill_ms_per_step": round(zero_ms / args.steps, 4),
         "preprocess_s": {"generate": round(t_gen, 3), "mode_sort_all": round(t_prep, 3)},
         "clocks": clk,
         "e2e": e2e,
+        "allgather": allgather,
         "hicoo": hicoo,
         "cpals": cpals,
         "gpu_launches": launches,

@@ -640,8 +640,9 @@ __global__ void __launch_bounds__(kThreads, WA == 6 ? 3 : 2) coo_staged_kernel(c
   const uint32_t R = a.R;
   const uint32_t col = uint32_t(lig) * 4;
   const Policies pol(a.cache_mode | 1u);  // the staged stream is always evict_first
-  uint64_t pol_hot = pol.gather;
+  uint64_t pol_hot = pol.gather, pol_cold = pol.gather;
   if (a.cache_mode & 8) asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol_hot));
+  if (a.cache_mode & 16) asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol_cold));
   const uint32_t *src[NA];
   src[0] = a.irow;
 #pragma unroll
@@ -718,7 +719,7 @@ __global__ void __launch_bounds__(kThreads, WA == 6 ? 3 : 2) coo_staged_kernel(c
           for (int j = 0; j < NO; ++j) {
             if (kGather) {
               const float *base = a.Uo[j];
-              uint64_t gp = pol.gather;
+              uint64_t gp = a.hot_marked ? pol_cold : pol.gather;
               if (a.hot_marked && (idx[j][u] >> 31)) {  // a row of the packed hot-row cache
                 base = a.hot_buf;
                 idx[j][u] &= 0x7FFFFFFFu;
