@@ -200,6 +200,23 @@ pasta_status pasta_cpals_coo(pasta_coo *x, uint32_t R, uint32_t max_iters, doubl
                              float *const *factors, double *lambda, double *fit_history,
                              uint32_t *iters, void *stream);
 
+/* ------------------------------------------------- TTV / TTM --------- */
+/* Tensor-times-vector (Eq. 1) and tensor-times-matrix (Eq. 2) in mode `mode`.
+ * The result is semi-sparse (sCOO): one dense vector of length R per mode-n fiber of X
+ * (sparse-dense property), fibers in lexicographic order of their coordinates over the
+ * modes k != mode.  The fibers are pre-processed once per mode and cached. */
+
+/* Build (cached) the mode-`mode` fibers; *nfibers = M_F. */
+pasta_status pasta_coo_fibers(pasta_coo *x, uint32_t mode, uint64_t *nfibers, void *stream);
+/* Copy the fiber coordinates to HOST buffers: inds[k] (k != mode) gets M_F uint32; inds[mode]
+ * is not touched (may be NULL). */
+pasta_status pasta_coo_fiber_export(pasta_coo *x, uint32_t mode, uint32_t *const *inds);
+/* out (DEVICE [M_F][R], OVERWRITTEN) = X x_mode U with U DEVICE row-major [dims[mode]][R]. */
+pasta_status pasta_ttm_coo(pasta_coo *x, uint32_t mode, const float *U, uint32_t R, float *out,
+                           void *stream);
+/* out (DEVICE [M_F]) = X x_mode v with v DEVICE [dims[mode]] (TTM with R = 1). */
+pasta_status pasta_ttv_coo(pasta_coo *x, uint32_t mode, const float *v, float *out, void *stream);
+
 /* ------------------------------------------------------------ introspection ---------- */
 
 pasta_status pasta_coo_info(const pasta_coo *x, uint32_t *order, uint32_t *dims,

@@ -63,6 +63,9 @@ def _L():
         lib.oracle_coo_to_hicoo.argtypes = [C.c_uint32, C.c_uint64, C.POINTER(_u32p), _f32p,
                                             C.c_uint32, _u64p, C.POINTER(_u32p), C.POINTER(_u8p),
                                             _f32p]
+        lib.oracle_ttm.restype = C.c_int64
+        lib.oracle_ttm.argtypes = [C.c_uint32, _u32p, C.c_uint64, C.POINTER(_u32p), _f32p, C.c_uint32,
+                                   _f32p, C.c_uint32, C.POINTER(_u32p), _f64p, _f64p]
         lib.oracle_gen_powerlaw.restype = C.c_int
         lib.oracle_gen_powerlaw.argtypes = [C.c_uint32, _u32p, C.c_uint64, C.c_uint64, _f64p,
                                             C.c_double, C.c_float, C.c_float, C.POINTER(_u32p),
@@ -221,3 +224,29 @@ def gen_powerlaw(dims, nnz, seed, initiator=None, q=0.75, val_lo=-1.0, val_hi=1.
     if rc != 0:
         raise ValueError(f"oracle_gen_powerlaw failed rc={rc}")
     return np.stack([o[:nnz] for o in outs]), ov[:nnz].copy()
+
+
+def ttm(dims, inds, vals, mode, U):
+    """O-TTM (Eq. 2): semi-sparse result over the mode-n fibers of X.
+    Returns (fiber_inds u32[N][F] with row `mode` zero, Y f64[F, R], sum|terms| f64[F, R])."""
+    dims, inds, vals = _prep(dims, inds, vals)
+    order, M = inds.shape
+    U = np.ascontiguousarray(U, dtype=np.float32)
+    if U.ndim == 1:
+        U = U.reshape(-1, 1)
+    R = U.shape[1]
+    rows = [np.ascontiguousarray(inds[k]) for k in range(order)]
+    fib = [np.zeros(max(M, 1), np.uint32) for _ in range(order)]
+    y = np.zeros((max(M, 1), R), np.float64)
+    ya = np.zeros_like(y)
+    nf = _L().oracle_ttm(order, _ptr(dims, _u32p), M, _ptr_list(rows, _u32p), _ptr(vals, _f32p), mode,
+                         _ptr(U, _f32p), R, _ptr_list(fib, _u32p), _ptr(y, _f64p), _ptr(ya, _f64p))
+    if nf < 0:
+        raise ValueError("oracle_ttm: invalid arguments")
+    return np.stack([f[:nf] for f in fib]), y[:nf].copy(), ya[:nf].copy()
+
+
+def ttv(dims, inds, vals, mode, v):
+    """O-TTV (Eq. 1): TTM with a single column u = v."""
+    f, y, ya = ttm(dims, inds, vals, mode, np.asarray(v, np.float32).reshape(-1, 1))
+    return f, y[:, 0].copy(), ya[:, 0].copy()

@@ -362,3 +362,63 @@ int oracle_gen_powerlaw(uint32_t order, const uint32_t *dims, uint64_t nnz, uint
         if (D > cap) D = cap;
     }
 }
+
+/* ------------------------------------------------------------------------- */
+/* O-TTM / O-TTV: Eq. 2 and Eq. 1 over nonzeros: */
+/*   y(i_1..i_{n-1}, r, i_{n+1}..i_N) = sum_{i_n} x(..., i_n, ...) u(i_n, r)  */
+/* The output is semi-sparse (sCOO): one dense length-R vector per      */
+/* mode-n fiber of X (the sparse-dense property).  Fibers are emitted   */
+/* in lexicographic order of their coordinates (modes k != n, ascending k);   */
+/* TTV is the R = 1 case with u = v.  fiber_inds: order arrays (capacity nnz, */
+/* the mode-n array is left untouched); y, yabs: capacity nnz * R (fp64).      */
+/* Returns the number of fibers, or -1 on invalid arguments.                  */
+/* ------------------------------------------------------------------------- */
+static uint32_t g_fib_mode;
+static int cmp_fiber_then_n(const void *pa, const void *pb)
+{
+    uint64_t a = *(const uint64_t *)pa, b = *(const uint64_t *)pb;
+    for (uint32_t k = 0; k < g_order; ++k) {
+        if (k == g_fib_mode) continue;
+        uint32_t va = g_inds[k][a], vb = g_inds[k][b];
+        if (va != vb) return va < vb ? -1 : 1;
+    }
+    uint32_t va = g_inds[g_fib_mode][a], vb = g_inds[g_fib_mode][b];
+    if (va != vb) return va < vb ? -1 : 1;
+    return a < b ? -1 : (a > b ? 1 : 0);
+}
+
+int64_t oracle_ttm(uint32_t order, const uint32_t *dims, uint64_t nnz, const uint32_t *const *inds,
+                   const float *vals, uint32_t mode, const float *U, uint32_t R,
+                   uint32_t *const *fiber_inds, double *y, double *yabs)
+{
+    if (order < 1 || order > ORACLE_MAX_ORDER || mode >= order || R < 1) return -1;
+    (void)dims;
+    uint64_t *perm = (uint64_t *)malloc((nnz ? nnz : 1) * sizeof(uint64_t));
+    if (!perm) return -2;
+    for (uint64_t x = 0; x < nnz; ++x) perm[x] = x;
+    g_order = order; g_inds = inds; g_fib_mode = mode;
+    qsort(perm, nnz, sizeof(uint64_t), cmp_fiber_then_n);
+    int64_t nf = 0;
+    for (uint64_t q = 0; q < nnz; ++q) {
+        uint64_t x = perm[q];
+        int new_fiber = (q == 0);
+        if (!new_fiber) {
+            uint64_t p = perm[q - 1];
+            for (uint32_t k = 0; k < order; ++k)
+                if (k != mode && inds[k][x] != inds[k][p]) new_fiber = 1;
+        }
+        if (new_fiber) {
+            for (uint32_t k = 0; k < order; ++k)
+                if (k != mode) fiber_inds[k][nf] = inds[k][x];
+            for (uint32_t r = 0; r < R; ++r) { y[nf * R + r] = 0.0; yabs[nf * R + r] = 0.0; }
+            ++nf;
+        }
+        for (uint32_t r = 0; r < R; ++r) {
+            double t = (double)vals[x] * (double)U[(uint64_t)inds[mode][x] * R + r];
+            y[(nf - 1) * R + r] += t;
+            yabs[(nf - 1) * R + r] += fabs(t);
+        }
+    }
+    free(perm);
+    return nf;
+}

@@ -24,7 +24,8 @@ __all__ = [
     "pasta_coo_export", "pasta_coo_export_mode", "pasta_hicoo_info", "pasta_hicoo_export",
     "pasta_launch_count", "pasta_profile_enable", "pasta_profile_read", "pasta_gram",
     "pasta_cpals_solve", "pasta_normalize_columns", "pasta_weighted_inner", "pasta_coo_norm2",
-    "pasta_cpals_coo",
+    "pasta_cpals_coo", "pasta_coo_fibers", "pasta_coo_fiber_export", "pasta_ttm_coo",
+    "pasta_ttv_coo",
 ]
 
 _u32p = C.POINTER(C.c_uint32)
@@ -441,3 +442,43 @@ def pasta_cpals_coo(x: Coo, factors, max_iters: int = 20, tol: float = 1e-5, str
                                 fits.ctypes.data_as(C.POINTER(C.c_double)), C.byref(it),
                                 _stream_ptr(stream)))
     return lam, list(fits[: it.value]), it.value
+
+
+# ----------------------------------------------------------------------------- TTV / TTM
+def pasta_coo_fibers(x: Coo, mode: int, stream=None) -> int:
+    """Number of mode-`mode` fibers M_F (built once, cached)."""
+    nf = C.c_uint64()
+    check(lib().pasta_coo_fibers(x.ptr, mode, C.byref(nf), _stream_ptr(stream)))
+    return nf.value
+
+
+def pasta_coo_fiber_export(x: Coo, mode: int) -> np.ndarray:
+    """Fiber coordinates u32 [N, M_F] (row `mode` is zero)."""
+    nf = pasta_coo_fibers(x, mode)
+    arrs = [np.zeros(max(nf, 1), np.uint32) for _ in range(x.order)]
+    p = (_u32p * x.order)(*[_np_ptr(a, _u32p) for a in arrs])
+    check(lib().pasta_coo_fiber_export(x.ptr, mode, p))
+    return np.stack([a[:nf] for a in arrs])
+
+
+def pasta_ttm_coo(x: Coo, mode: int, U, out=None, stream=None):
+    """Semi-sparse TTM (Eq. 2): values [M_F, R] on the mode-`mode` fibers."""
+    import torch
+    R = int(U.shape[1])
+    nf = pasta_coo_fibers(x, mode, stream)
+    if out is None:
+        out = torch.empty((nf, R), dtype=torch.float32, device=U.device)
+    check(lib().pasta_ttm_coo(x.ptr, mode, C.c_void_p(U.data_ptr()), R, C.c_void_p(out.data_ptr()),
+                              _stream_ptr(stream)))
+    return out
+
+
+def pasta_ttv_coo(x: Coo, mode: int, v, out=None, stream=None):
+    """Semi-sparse TTV (Eq. 1): values [M_F] on the mode-`mode` fibers."""
+    import torch
+    nf = pasta_coo_fibers(x, mode, stream)
+    if out is None:
+        out = torch.empty(nf, dtype=torch.float32, device=v.device)
+    check(lib().pasta_ttv_coo(x.ptr, mode, C.c_void_p(v.data_ptr()), C.c_void_p(out.data_ptr()),
+                              _stream_ptr(stream)))
+    return out

@@ -79,6 +79,10 @@ SIGNATURES = {
     "pasta_coo_norm2": (_st, [_vp, C.POINTER(C.c_double)]),
     "pasta_cpals_coo": (_st, [_vp, C.c_uint32, C.c_uint32, C.c_double, C.POINTER(_vp),
                               C.POINTER(C.c_double), C.POINTER(C.c_double), _u32p, _vp]),
+    "pasta_coo_fibers": (_st, [_vp, C.c_uint32, _u64p, _vp]),
+    "pasta_coo_fiber_export": (_st, [_vp, C.c_uint32, C.POINTER(_u32p)]),
+    "pasta_ttm_coo": (_st, [_vp, C.c_uint32, _vp, C.c_uint32, _vp, _vp]),
+    "pasta_ttv_coo": (_st, [_vp, C.c_uint32, _vp, _vp, _vp]),
     "pasta_launch_count": (C.c_uint64, []),
     "pasta_profile_enable": (_st, [C.c_int]),
     "pasta_profile_read": (_st, [C.c_uint32, C.POINTER(C.c_double), _u64p, C.c_int]),

@@ -162,6 +162,10 @@ static std::unique_ptr<pasta_coo> coo_upload(uint32_t order, const uint32_t *dim
   return x;
 }
 
+pasta_coo::~pasta_coo() {
+  for (auto *f : fib) delete f;
+}
+
 namespace pasta {
 
 void coo_prepare_mode(pasta_coo *x, uint32_t mode, cudaStream_t s) {
@@ -729,6 +733,63 @@ pasta_status pasta_cpals_coo(pasta_coo *x, uint32_t R, uint32_t max_iters, doubl
   for (uint32_t r = 0; r < R; ++r) lambda[r] = hl[r];
   *iters = it;
   API_END
+}
+
+// ---------------------------------------------------------------------------- TTV / TTM
+pasta_status pasta_coo_fibers(pasta_coo *x, uint32_t mode, uint64_t *nfibers, void *stream) {
+  API_BEGIN
+  require(x && nfibers, "x/nfibers is NULL");
+  require(mode < x->order, "mode >= order");
+  check_device(x->device);
+  std::lock_guard<std::mutex> lk(x->mu);
+  coo_build_fibers(x, mode, as_stream(stream));
+  *nfibers = x->fib[mode]->nf;
+  API_END
+}
+
+pasta_status pasta_coo_fiber_export(pasta_coo *x, uint32_t mode, uint32_t *const *inds) {
+  API_BEGIN
+  require(x && inds, "x/inds is NULL");
+  require(mode < x->order, "mode >= order");
+  check_device(x->device);
+  {
+    std::lock_guard<std::mutex> lk(x->mu);
+    coo_build_fibers(x, mode, nullptr);
+  }
+  const FiberCopy &f = *x->fib[mode];
+  for (uint32_t k = 0; k < x->order; ++k) {
+    if (k == mode || !f.nf) continue;
+    require(inds[k] != nullptr, "inds[k] is NULL for a mode k != mode");
+    PASTA_CUDA(cudaMemcpy(inds[k], f.finds[k].p, f.nf * sizeof(uint32_t), cudaMemcpyDeviceToHost));
+  }
+  API_END
+}
+
+pasta_status pasta_ttm_coo(pasta_coo *x, uint32_t mode, const float *U, uint32_t R, float *out,
+                           void *stream) {
+  API_BEGIN
+  require(x && U && out, "x/U/out is NULL");
+  require(mode < x->order, "mode >= order");
+  require(R >= 1, "R must be >= 1");
+  check_device(x->device);
+  cudaStream_t s = as_stream(stream);
+  if (!x->fib[mode]) {
+    std::lock_guard<std::mutex> lk(x->mu);
+    coo_build_fibers(x, mode, s);
+  }
+  FiberCopy &f = *x->fib[mode];
+  if (!f.mat.mc[0].ready) {
+    std::lock_guard<std::mutex> lk(f.mat.mu);
+    coo_prepare_mode(&f.mat, 0, s);
+  }
+  launch_zero_rows(out, 0, f.nf, R, s);
+  const float *fac[2] = {nullptr, U};
+  launch_coo_mttkrp(&f.mat, 0, fac, R, out, s);
+  API_END
+}
+
+pasta_status pasta_ttv_coo(pasta_coo *x, uint32_t mode, const float *v, float *out, void *stream) {
+  return pasta_ttm_coo(x, mode, v, 1, out, stream);
 }
 
 // ---------------------------------------------------------------------------- introspection

@@ -151,6 +151,13 @@ struct HicooModeCopy {
 
 }  // namespace pasta
 
+namespace pasta {
+// Mode-n fibers of a COO tensor (TTV/TTM): nonzeros sorted by the other modes
+// then i_n; `mat` is the order-2 COO (fiber id, i_n) with the same values, so that
+// TTM = mode-0 MTTKRP of `mat` with the single factor U (Eq. 2 = Eq. 3 on the fiberised matrix).
+struct FiberCopy;
+}  // namespace pasta
+
 struct pasta_coo {
   uint32_t order = 0;
   uint32_t dims[pasta::kMaxOrder] = {};
@@ -171,6 +178,8 @@ struct pasta_coo {
   bool counts_ready[pasta::kMaxOrder] = {};
   pasta::DevArray<uint32_t> row_count[pasta::kMaxOrder];
   uint64_t count_hist[pasta::kMaxOrder][pasta::kCountBuckets] = {};
+  pasta::FiberCopy *fib[pasta::kMaxOrder] = {};
+  ~pasta_coo();
   std::mutex mu;
 };
 
@@ -190,6 +199,12 @@ struct pasta_hicoo {
 };
 
 namespace pasta {
+
+struct FiberCopy {
+  uint64_t nf = 0;
+  pasta::DevArray<uint32_t> finds[kMaxOrder];  // fiber coordinates (k != mode), nf each
+  pasta_coo mat;                               // order 2: (fiber id, i_mode), lex sorted
+};
 
 inline uint32_t ceil_log2(uint64_t v) {
   uint32_t l = 0;
@@ -237,6 +252,7 @@ void launch_inner(const float *A, const float *B, uint64_t rows, uint32_t R, con
                   double *out, cudaStream_t s);
 void launch_sumsq(const float *v, uint64_t n, double *out, cudaStream_t s);
 void coo_mark_hot(pasta_coo *x, uint32_t mode, uint32_t R, cudaStream_t s);
+void coo_build_fibers(pasta_coo *x, uint32_t mode, cudaStream_t s);
 void launch_hot_fill(const CooModeCopy &mc, const float *const *factors, uint32_t order, uint32_t mode,
                      uint32_t R, cudaStream_t s);
 void row_counts_device(const uint32_t *rows, uint64_t nnz, uint32_t nrows, uint64_t *counts_host,

@@ -1,0 +1,59 @@
+"""TTV / TTM on the GPU against the oracle (Eq. 1, Eq. 2):
+fibers bit-exact, values within 1e-4 * sum|terms| + 1e-6."""
+import numpy as np
+import pytest
+
+import synth_inputs as si
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def env(oracle_mod):
+    import torch
+
+    import paper_conf_iiswc_lilwlob20_b200 as pasta
+    assert torch.cuda.is_available()
+    torch.cuda.set_device(0)
+    return pasta, oracle_mod, torch
+
+
+@pytest.mark.parametrize("dims,nnz,R", [((300, 200, 500), 50_013, 16), ((60, 70, 80, 90), 40_007, 8),
+                                        ((1000, 900), 30_001, 3), ((4096, 4096, 4096), 200_000, 32)])
+def test_ttm_and_ttv_match_oracle(env, dims, nnz, R):
+    pasta, oracle, torch = env
+    inds, vals = si.powerlaw_coo(dims, nnz, seed=nnz)
+    x = pasta.pasta_coo_from_arrays(dims, inds, vals)
+    for n in range(len(dims)):
+        U = si.factors([dims[n]], R, seed=n + R)[0]
+        fib, Y, Ya = oracle.ttm(dims, inds, vals, n, U)
+        assert pasta.pasta_coo_fibers(x, n) == fib.shape[1]
+        gf = pasta.pasta_coo_fiber_export(x, n)
+        for k in range(len(dims)):
+            if k != n:
+                np.testing.assert_array_equal(gf[k], fib[k])
+        got = pasta.pasta_ttm_coo(x, n, torch.from_numpy(U).cuda()).cpu().numpy().astype(np.float64)
+        assert np.all(np.abs(got - Y) <= 1e-4 * Ya + 1e-6), (dims, n)
+        v = U[:, 0].copy()
+        fv, yv, yva = oracle.ttv(dims, inds, vals, n, v)
+        gv = pasta.pasta_ttv_coo(x, n, torch.from_numpy(v).cuda()).cpu().numpy().astype(np.float64)
+        assert np.all(np.abs(gv - yv) <= 1e-4 * yva + 1e-6)
+
+
+def test_ttm_hot_fiber_and_empty(env):
+    pasta, oracle, torch = env
+    dims = (50, 4000, 30)
+    # one mode-1 fiber holds 3000 nonzeros (all of (i0=7, i2=3) with distinct i1)
+    i1 = np.random.default_rng(0).choice(4000, 3000, replace=False).astype(np.uint32)
+    hot = np.stack([np.full(3000, 7, np.uint32), i1, np.full(3000, 3, np.uint32)])
+    rest, _ = si.uniform_coo(dims, 5000, seed=2)
+    keep = ~((rest[0] == 7) & (rest[2] == 3))
+    inds = np.ascontiguousarray(np.concatenate([hot, rest[:, keep]], axis=1))
+    vals = np.random.default_rng(1).uniform(-1, 1, inds.shape[1]).astype(np.float32)
+    x = pasta.pasta_coo_from_arrays(dims, inds, vals)
+    U = si.factors([dims[1]], 16, seed=3)[0]
+    fib, Y, Ya = oracle.ttm(dims, inds, vals, 1, U)
+    got = pasta.pasta_ttm_coo(x, 1, torch.from_numpy(U).cuda()).cpu().numpy().astype(np.float64)
+    assert np.all(np.abs(got - Y) <= 1e-4 * Ya + 1e-6)
+    e = pasta.pasta_coo_from_arrays(dims, np.zeros((3, 0), np.uint32), np.zeros(0, np.float32))
+    assert pasta.pasta_coo_fibers(e, 0) == 0
