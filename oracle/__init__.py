@@ -63,6 +63,15 @@ def _L():
         lib.oracle_coo_to_hicoo.argtypes = [C.c_uint32, C.c_uint64, C.POINTER(_u32p), _f32p,
                                             C.c_uint32, _u64p, C.POINTER(_u32p), C.POINTER(_u8p),
                                             _f32p]
+        lib.oracle_coo_to_ghicoo.restype = C.c_int64
+        lib.oracle_coo_to_ghicoo.argtypes = [C.c_uint32, C.c_uint64, C.POINTER(_u32p), _f32p,
+                                             C.c_uint32, C.c_uint32, _u64p, C.POINTER(_u32p),
+                                             C.POINTER(_u8p), C.POINTER(_u32p), _f32p]
+        lib.oracle_mttkrp_ghicoo.restype = C.c_int
+        lib.oracle_mttkrp_ghicoo.argtypes = [C.c_uint32, _u32p, C.c_uint32, C.c_uint32, C.c_uint64,
+                                             _u64p, C.POINTER(_u32p), C.POINTER(_u8p),
+                                             C.POINTER(_u32p), _f32p, C.c_uint32,
+                                             C.POINTER(_f32p), C.c_uint32, _f64p, _f64p]
         lib.oracle_ttm.restype = C.c_int64
         lib.oracle_ttm.argtypes = [C.c_uint32, _u32p, C.c_uint64, C.POINTER(_u32p), _f32p, C.c_uint32,
                                    _f32p, C.c_uint32, C.POINTER(_u32p), _f64p, _f64p]
@@ -205,6 +214,63 @@ def coo_to_hicoo(inds, vals, block_bits=7):
         "einds": np.stack([e[:M] for e in einds]),
         "vals": ov[:M].copy(),
     }
+
+
+def coo_to_ghicoo(inds, vals, block_bits, cmask):
+    """O-gHiCOO conversion (Fig. 2(b); R#29): modes with bit k of ``cmask`` set are
+    blocked as in HiCOO, the others stay COO.  Returns a dict with ``bptr`` u64[n_b+1],
+    ``binds`` / ``einds`` (lists, None for uncompressed modes), ``uinds`` (list, None for
+    compressed modes), ``vals``."""
+    inds = np.ascontiguousarray(inds, dtype=np.uint32)
+    vals = np.ascontiguousarray(vals, dtype=np.float32)
+    order, M = inds.shape
+    rows = [np.ascontiguousarray(inds[k]) for k in range(order)]
+    bptr = np.zeros(M + 1, np.uint64)
+    binds = [np.zeros(max(M, 1), np.uint32) for _ in range(order)]
+    einds = [np.zeros(max(M, 1), np.uint8) for _ in range(order)]
+    uinds = [np.zeros(max(M, 1), np.uint32) for _ in range(order)]
+    ov = np.zeros(max(M, 1), np.float32)
+    nb = _L().oracle_coo_to_ghicoo(order, M, _ptr_list(rows, _u32p), _ptr(vals, _f32p),
+                                   block_bits, cmask, _ptr(bptr, _u64p), _ptr_list(binds, _u32p),
+                                   _ptr_list(einds, _u8p), _ptr_list(uinds, _u32p),
+                                   _ptr(ov, _f32p))
+    if nb < 0:
+        raise ValueError("oracle_coo_to_ghicoo: invalid arguments")
+    comp = [bool((cmask >> k) & 1) for k in range(order)]
+    return {
+        "order": order, "block_bits": block_bits, "cmask": cmask, "nblocks": int(nb), "nnz": M,
+        "bptr": bptr[: nb + 1].copy(),
+        "binds": [binds[k][:nb].copy() if comp[k] else None for k in range(order)],
+        "einds": [einds[k][:M].copy() if comp[k] else None for k in range(order)],
+        "uinds": [None if comp[k] else uinds[k][:M].copy() for k in range(order)],
+        "vals": ov[:M].copy(),
+    }
+
+
+def mttkrp_ghicoo(dims, g, mode, factors, R=None):
+    """O-gHiCOO-MTTKRP: Alg. 3 rebasing the compressed modes only (R#29)."""
+    dims = np.ascontiguousarray(dims, dtype=np.uint32)
+    order = dims.shape[0]
+    if R is None:
+        R = next(f.shape[1] for k, f in enumerate(factors) if k != mode and f is not None)
+    fl = _factor_list(order, mode, factors, R)
+    Mref = np.zeros((int(dims[mode]), R), np.float64)
+    Aref = np.zeros_like(Mref)
+    dummy32 = np.zeros(1, np.uint32)
+    dummy8 = np.zeros(1, np.uint8)
+    binds = [np.ascontiguousarray(b) if b is not None else dummy32 for b in g["binds"]]
+    einds = [np.ascontiguousarray(e) if e is not None else dummy8 for e in g["einds"]]
+    uinds = [np.ascontiguousarray(u) if u is not None else dummy32 for u in g["uinds"]]
+    bptr = np.ascontiguousarray(g["bptr"], dtype=np.uint64)
+    vals = np.ascontiguousarray(g["vals"], dtype=np.float32)
+    rc = _L().oracle_mttkrp_ghicoo(order, _ptr(dims, _u32p), g["block_bits"], g["cmask"],
+                                   g["nblocks"], _ptr(bptr, _u64p), _ptr_list(binds, _u32p),
+                                   _ptr_list(einds, _u8p), _ptr_list(uinds, _u32p),
+                                   _ptr(vals, _f32p), mode, _ptr_list(fl, _f32p), R,
+                                   _ptr(Mref, _f64p), _ptr(Aref, _f64p))
+    if rc != 0:
+        raise ValueError("oracle_mttkrp_ghicoo: invalid arguments")
+    return Mref, Aref
 
 
 def gen_powerlaw(dims, nnz, seed, initiator=None, q=0.75, val_lo=-1.0, val_hi=1.0):

@@ -422,3 +422,113 @@ int64_t oracle_ttm(uint32_t order, const uint32_t *dims, uint64_t nnz, const uin
     free(perm);
     return nf;
 }
+
+/* ------------------------------------------------------------------------- */
+/* O-gHiCOO conversion (Fig. 2(b); R#29):           */
+/* "pick which modes to be compressed in units of blocks for HiCOO and which  */
+/* stay in COO format".  cmask bit k set <=> mode k is compressed (blocked).  */
+/*  1. sort nonzeros by the Morton order of the COMPRESSED modes' coordinates */
+/*     (same level-major convention as HiCOO, R#13, restricted to those       */
+/*     modes), ties by the uncompressed coordinates in ascending mode order   */
+/*     (lexicographic), then by input position (stable);                      */
+/*  2. scan: a new block starts where (i_k >> b) differs for a compressed k;  */
+/*  3. emit bptr (u64), binds_k (u32) and einds_k (u8) for compressed k, the  */
+/*     full coordinate inds_k (u32, as in COO) for uncompressed k, and val.   */
+/* cmask = all modes is HiCOO; cmask = {0} is the mode-0 lexicographic order. */
+/* Arrays of the other kind are left untouched.  Returns n_b or -1.           */
+/* ------------------------------------------------------------------------- */
+static uint32_t g_cmask;
+static int cmp_ghicoo(const void *pa, const void *pb)
+{
+    uint64_t a = *(const uint64_t *)pa, b = *(const uint64_t *)pb;
+    int best = -1;
+    uint32_t best_x = 0;
+    for (uint32_t k = 0; k < g_order; ++k) {
+        if (!((g_cmask >> k) & 1u)) continue;
+        uint32_t x = g_inds[k][a] ^ g_inds[k][b];
+        if (msb_less(best_x, x)) { best = (int)k; best_x = x; }
+    }
+    if (best >= 0) {
+        uint32_t va = g_inds[best][a], vb = g_inds[best][b];
+        return va < vb ? -1 : 1;
+    }
+    for (uint32_t k = 0; k < g_order; ++k) {
+        if ((g_cmask >> k) & 1u) continue;
+        uint32_t va = g_inds[k][a], vb = g_inds[k][b];
+        if (va != vb) return va < vb ? -1 : 1;
+    }
+    return a < b ? -1 : (a > b ? 1 : 0);
+}
+
+int64_t oracle_coo_to_ghicoo(uint32_t order, uint64_t nnz, const uint32_t *const *inds,
+                             const float *vals, uint32_t block_bits, uint32_t cmask,
+                             uint64_t *bptr, uint32_t *const *binds, uint8_t *const *einds,
+                             uint32_t *const *uinds, float *out_vals)
+{
+    if (order < 1 || order > ORACLE_MAX_ORDER || block_bits < 1 || block_bits > 8) return -1;
+    if (cmask == 0 || (cmask >> order) != 0) return -1;
+    uint64_t *perm = (uint64_t *)malloc((nnz ? nnz : 1) * sizeof(uint64_t));
+    if (!perm) return -2;
+    for (uint64_t x = 0; x < nnz; ++x) perm[x] = x;
+    g_order = order; g_inds = inds; g_cmask = cmask;
+    qsort(perm, nnz, sizeof(uint64_t), cmp_ghicoo);
+    uint32_t emask = (1u << block_bits) - 1u;
+    int64_t nb = 0;
+    for (uint64_t x = 0; x < nnz; ++x) {
+        uint64_t p = perm[x];
+        int new_block = (x == 0);
+        if (!new_block) {
+            uint64_t q = perm[x - 1];
+            for (uint32_t k = 0; k < order; ++k)
+                if (((cmask >> k) & 1u) && (inds[k][p] >> block_bits) != (inds[k][q] >> block_bits))
+                    new_block = 1;
+        }
+        if (new_block) {
+            bptr[nb] = x;
+            for (uint32_t k = 0; k < order; ++k)
+                if ((cmask >> k) & 1u) binds[k][nb] = inds[k][p] >> block_bits;
+            ++nb;
+        }
+        for (uint32_t k = 0; k < order; ++k) {
+            if ((cmask >> k) & 1u) einds[k][x] = (uint8_t)(inds[k][p] & emask);
+            else uinds[k][x] = inds[k][p];
+        }
+        out_vals[x] = vals[p];
+    }
+    bptr[nb] = nnz;
+    free(perm);
+    return nb;
+}
+
+/* O-gHiCOO-MTTKRP: Alg. 3 with the block rebasing applied to the     */
+/* compressed modes only: i_k = binds_k(b)*B + einds_k(x) if k is compressed, */
+/* else i_k = inds_k(x); then the accumulation of O-MTTKRP.                   */
+int oracle_mttkrp_ghicoo(uint32_t order, const uint32_t *dims, uint32_t block_bits, uint32_t cmask,
+                         uint64_t nblocks, const uint64_t *bptr, const uint32_t *const *binds,
+                         const uint8_t *const *einds, const uint32_t *const *uinds,
+                         const float *vals, uint32_t mode, const float *const *factors,
+                         uint32_t R, double *Mref, double *Aref)
+{
+    if (order < 1 || order > ORACLE_MAX_ORDER || mode >= order || R < 1) return -1;
+    uint64_t B = 1ull << block_bits;
+    uint64_t rows = dims[mode];
+    uint64_t ik[ORACLE_MAX_ORDER];
+    for (uint64_t e = 0; e < rows * R; ++e) { Mref[e] = 0.0; Aref[e] = 0.0; }
+    for (uint64_t b = 0; b < nblocks; ++b) {
+        for (uint64_t x = bptr[b]; x < bptr[b + 1]; ++x) {
+            for (uint32_t k = 0; k < order; ++k)
+                ik[k] = ((cmask >> k) & 1u) ? (uint64_t)binds[k][b] * B + einds[k][x]
+                                            : (uint64_t)uinds[k][x];
+            for (uint32_t r = 0; r < R; ++r) {
+                double t = (double)vals[x];
+                for (uint32_t k = 0; k < order; ++k) {
+                    if (k == mode) continue;
+                    t *= (double)factors[k][ik[k] * R + r];
+                }
+                Mref[ik[mode] * R + r] += t;
+                Aref[ik[mode] * R + r] += fabs(t);
+            }
+        }
+    }
+    return 0;
+}
