@@ -72,6 +72,10 @@ def _L():
                                              _u64p, C.POINTER(_u32p), C.POINTER(_u8p),
                                              C.POINTER(_u32p), _f32p, C.c_uint32,
                                              C.POINTER(_f32p), C.c_uint32, _f64p, _f64p]
+        lib.oracle_gen_slice_powerlaw.restype = C.c_int
+        lib.oracle_gen_slice_powerlaw.argtypes = [C.c_uint32, _u32p, C.c_uint64, C.c_uint64,
+                                                  C.c_double, C.c_float, C.c_float,
+                                                  C.POINTER(_u32p), _f32p]
         lib.oracle_ttm.restype = C.c_int64
         lib.oracle_ttm.argtypes = [C.c_uint32, _u32p, C.c_uint64, C.POINTER(_u32p), _f32p, C.c_uint32,
                                    _f32p, C.c_uint32, C.POINTER(_u32p), _f64p, _f64p]
@@ -289,6 +293,20 @@ def gen_powerlaw(dims, nnz, seed, initiator=None, q=0.75, val_lo=-1.0, val_hi=1.
                                   _ptr_list(outs, _u32p), _ptr(ov, _f32p))
     if rc != 0:
         raise ValueError(f"oracle_gen_powerlaw failed rc={rc}")
+    return np.stack([o[:nnz] for o in outs]), ov[:nnz].copy()
+
+
+def gen_slice_powerlaw(dims, nnz, seed, alpha=1.0, val_lo=-1.0, val_hi=1.0):
+    """FireHose-style slice power-law generator (R#30): every mode index drawn
+    independently from P(i) ~ (i+1)^-alpha.  Returns (inds u32[N][M] lexicographic, vals)."""
+    dims = np.ascontiguousarray(dims, dtype=np.uint32)
+    order = dims.shape[0]
+    outs = [np.zeros(max(nnz, 1), np.uint32) for _ in range(order)]
+    ov = np.zeros(max(nnz, 1), np.float32)
+    rc = _L().oracle_gen_slice_powerlaw(order, _ptr(dims, _u32p), nnz, seed, alpha, val_lo, val_hi,
+                                        _ptr_list(outs, _u32p), _ptr(ov, _f32p))
+    if rc != 0:
+        raise ValueError(f"oracle_gen_slice_powerlaw failed rc={rc}")
     return np.stack([o[:nnz] for o in outs]), ov[:nnz].copy()
 
 

@@ -270,45 +270,13 @@ static int cmp_draw_d(const void *pa, const void *pb)
     return a->d < b->d ? -1 : (a->d > b->d ? 1 : 0);
 }
 
-int oracle_gen_powerlaw(uint32_t order, const uint32_t *dims, uint64_t nnz, uint64_t seed,
-                        const double *initiator, double q, float val_lo, float val_hi,
-                        uint32_t *const *out_inds, float *out_vals)
+/* Common tail of both generators: D draws produced by draw(), invalid ones    */
+/* stripped, the first nnz distinct coordinates in draw order kept, emitted in */
+/* lexicographic order with value lo + (hi - lo) * u(d_first, 0xFFFF).        */
+typedef int (*draw_fn)(const void *ctx, uint64_t d, uint32_t *c);
+static int gen_common(uint32_t order, uint64_t nnz, uint64_t key, draw_fn draw, const void *ctx,
+                      float val_lo, float val_hi, uint32_t *const *out_inds, float *out_vals)
 {
-    if (order < 1 || order > ORACLE_MAX_ORDER) return -1;
-    uint32_t ncell = 1u << order;
-    double table[1u << ORACLE_MAX_ORDER], cum[1u << ORACLE_MAX_ORDER];
-    if (initiator) {
-        for (uint32_t c = 0; c < ncell; ++c) table[c] = initiator[c];
-    } else {
-        if (!(q > 0.0 && q < 1.0)) q = 0.75;
-        for (uint32_t c = 0; c < ncell; ++c) {
-            double p = 1.0;
-            for (uint32_t k = 0; k < order; ++k) p = p * (((c >> k) & 1u) ? (1.0 - q) : q);
-            table[c] = p;
-        }
-    }
-    double run = 0.0;
-    uint32_t last_pos = 0;
-    for (uint32_t c = 0; c < ncell; ++c) {
-        if (table[c] < 0.0) return -1;
-        run = run + table[c];
-        cum[c] = run;
-        if (table[c] > 0.0) last_pos = c;
-    }
-    if (!(run > 0.0)) return -1;
-    uint32_t L[ORACLE_MAX_ORDER], Lmax = 0;
-    double cells = 1.0;
-    for (uint32_t k = 0; k < order; ++k) {
-        if (dims[k] < 1) return -1;
-        uint32_t l = 0;
-        while (l < 32 && ((uint64_t)1 << l) < dims[k]) ++l;
-        L[k] = l;
-        if (l > Lmax) Lmax = l;
-        cells *= (double)dims[k];
-    }
-    if ((double)nnz > cells) return -1;
-    uint64_t key = mix64(seed ^ 0x5851F42D4C957F2Dull);
-
     uint64_t D = nnz + nnz / 16 + 4096;
     uint64_t cap = 64 * nnz + (1ull << 22);
     for (;;) {
@@ -319,17 +287,7 @@ int oracle_gen_powerlaw(uint32_t order, const uint32_t *dims, uint64_t nnz, uint
             draw_rec r;
             memset(&r, 0, sizeof(r));
             r.d = d;
-            for (uint32_t l = 0; l < Lmax; ++l) {
-                double u = gen_uniform(key, d, l) * run;
-                uint32_t cell = last_pos;
-                for (uint32_t c = 0; c < ncell; ++c)
-                    if (u < cum[c]) { cell = c; break; }
-                for (uint32_t k = 0; k < order; ++k)
-                    if (l < L[k]) r.c[k] |= ((cell >> k) & 1u) << l;
-            }
-            int ok = 1;
-            for (uint32_t k = 0; k < order; ++k) if (r.c[k] >= dims[k]) ok = 0;
-            if (ok) rec[nvalid++] = r;
+            if (draw(ctx, d, r.c)) rec[nvalid++] = r;
         }
         g_gen_order = order;
         qsort(rec, nvalid, sizeof(draw_rec), cmp_draw_coords_then_d);
@@ -361,6 +319,141 @@ int oracle_gen_powerlaw(uint32_t order, const uint32_t *dims, uint64_t nnz, uint
         D = D + D / 2 + 2 * (nnz - nuniq) + 4096; /* geometric growth */
         if (D > cap) D = cap;
     }
+}
+
+typedef struct {
+    uint32_t order, ncell, last_pos, Lmax;
+    uint32_t L[ORACLE_MAX_ORDER];
+    const uint32_t *dims;
+    const double *cum;
+    double run;
+    uint64_t key;
+} kron_ctx;
+
+static int kron_draw(const void *vctx, uint64_t d, uint32_t *c)
+{
+    const kron_ctx *x = (const kron_ctx *)vctx;
+    for (uint32_t l = 0; l < x->Lmax; ++l) {
+        double u = gen_uniform(x->key, d, l) * x->run;
+        uint32_t cell = x->last_pos;
+        for (uint32_t j = 0; j < x->ncell; ++j)
+            if (u < x->cum[j]) { cell = j; break; }
+        for (uint32_t k = 0; k < x->order; ++k)
+            if (l < x->L[k]) c[k] |= ((cell >> k) & 1u) << l;
+    }
+    for (uint32_t k = 0; k < x->order; ++k) if (c[k] >= x->dims[k]) return 0;
+    return 1;
+}
+
+int oracle_gen_powerlaw(uint32_t order, const uint32_t *dims, uint64_t nnz, uint64_t seed,
+                        const double *initiator, double q, float val_lo, float val_hi,
+                        uint32_t *const *out_inds, float *out_vals)
+{
+    if (order < 1 || order > ORACLE_MAX_ORDER) return -1;
+    uint32_t ncell = 1u << order;
+    double table[1u << ORACLE_MAX_ORDER], cum[1u << ORACLE_MAX_ORDER];
+    if (initiator) {
+        for (uint32_t c = 0; c < ncell; ++c) table[c] = initiator[c];
+    } else {
+        if (!(q > 0.0 && q < 1.0)) q = 0.75;
+        for (uint32_t c = 0; c < ncell; ++c) {
+            double p = 1.0;
+            for (uint32_t k = 0; k < order; ++k) p = p * (((c >> k) & 1u) ? (1.0 - q) : q);
+            table[c] = p;
+        }
+    }
+    double run = 0.0;
+    uint32_t last_pos = 0;
+    for (uint32_t c = 0; c < ncell; ++c) {
+        if (table[c] < 0.0) return -1;
+        run = run + table[c];
+        cum[c] = run;
+        if (table[c] > 0.0) last_pos = c;
+    }
+    if (!(run > 0.0)) return -1;
+    kron_ctx ctx;
+    memset(&ctx, 0, sizeof(ctx));
+    double cells = 1.0;
+    for (uint32_t k = 0; k < order; ++k) {
+        if (dims[k] < 1) return -1;
+        uint32_t l = 0;
+        while (l < 32 && ((uint64_t)1 << l) < dims[k]) ++l;
+        ctx.L[k] = l;
+        if (l > ctx.Lmax) ctx.Lmax = l;
+        cells *= (double)dims[k];
+    }
+    if ((double)nnz > cells) return -1;
+    ctx.order = order; ctx.ncell = ncell; ctx.last_pos = last_pos;
+    ctx.dims = dims; ctx.cum = cum; ctx.run = run;
+    ctx.key = mix64(seed ^ 0x5851F42D4C957F2Dull);
+    return gen_common(order, nnz, ctx.key, kron_draw, &ctx, val_lo, val_hi, out_inds, out_vals);
+}
+
+/* ------------------------------------------------------------------------- */
+/* Slice power-law generator (FireHose-style;    */
+/* R#30).  "combines graphs together to form slices of a hypergraph ... when  */
+/* repeated on an (N-1)th-order tensor, will generate a sparse tensor with N  */
+/* modes": every mode index is drawn independently from the discrete power   */
+/* law P(i) ~ (i+1)^(-alpha), i < I_k, so each slice is a power-law graph     */
+/* (no clustering) and slices are combined the same way.               */
+/* Table: w_i = pow(i+1, -alpha), cum_i = running fp64 sum (i ascending).     */
+/* Draw d, mode k: u = u(d, k) * cum_{I_k-1}; i_k = the first i with         */
+/* u < cum_i (binary search), else I_k - 1.  Then gen_common.                 */
+/* ------------------------------------------------------------------------- */
+typedef struct {
+    uint32_t order;
+    const uint32_t *dims;
+    double *cum[ORACLE_MAX_ORDER];
+    uint64_t key;
+} slice_ctx;
+
+static int slice_draw(const void *vctx, uint64_t d, uint32_t *c)
+{
+    const slice_ctx *x = (const slice_ctx *)vctx;
+    for (uint32_t k = 0; k < x->order; ++k) {
+        const double *cum = x->cum[k];
+        uint32_t I = x->dims[k];
+        double u = gen_uniform(x->key, d, k) * cum[I - 1];
+        uint32_t lo = 0, hi = I; /* first i in [lo, hi) with u < cum[i]; hi = none */
+        while (lo < hi) {
+            uint32_t mid = lo + (hi - lo) / 2;
+            if (u < cum[mid]) hi = mid; else lo = mid + 1;
+        }
+        c[k] = lo < I ? lo : I - 1;
+    }
+    return 1;
+}
+
+int oracle_gen_slice_powerlaw(uint32_t order, const uint32_t *dims, uint64_t nnz, uint64_t seed,
+                              double alpha, float val_lo, float val_hi,
+                              uint32_t *const *out_inds, float *out_vals)
+{
+    if (order < 1 || order > ORACLE_MAX_ORDER || !(alpha >= 0.0 && alpha <= 8.0)) return -1;
+    slice_ctx ctx;
+    memset(&ctx, 0, sizeof(ctx));
+    double cells = 1.0;
+    for (uint32_t k = 0; k < order; ++k) {
+        if (dims[k] < 1) return -1;
+        cells *= (double)dims[k];
+    }
+    if ((double)nnz > cells) return -1;
+    int rc = 0;
+    for (uint32_t k = 0; k < order && rc == 0; ++k) {
+        ctx.cum[k] = (double *)malloc((size_t)dims[k] * sizeof(double));
+        if (!ctx.cum[k]) { rc = -2; break; }
+        double run = 0.0;
+        for (uint32_t i = 0; i < dims[k]; ++i) {
+            run = run + pow((double)i + 1.0, -alpha);
+            ctx.cum[k][i] = run;
+        }
+    }
+    if (rc == 0) {
+        ctx.order = order; ctx.dims = dims;
+        ctx.key = mix64(seed ^ 0x5851F42D4C957F2Dull);
+        rc = gen_common(order, nnz, ctx.key, slice_draw, &ctx, val_lo, val_hi, out_inds, out_vals);
+    }
+    for (uint32_t k = 0; k < order; ++k) free(ctx.cum[k]);
+    return rc;
 }
 
 /* ------------------------------------------------------------------------- */
