@@ -385,11 +385,11 @@ def main():
                "path": "per rank: pinned factors H2D, pasta_mttkrp_coo on the rank's shards, owned "
                        "rows D2H (wall clock, max over ranks); bytes are rank 0's"}
 
-    # a7: HiCOO MTTKRP (B = 128) on the same tensor, every mode per step
-    hicoo = None
-    if world == 1 and args.hicoo_steps > 0:
+    # a7: HiCOO MTTKRP (B = 128) on the same tensor, every mode per step; NEXT-2: the
+    # same on the gHiCOO form with the storage-minimising mask
+    def time_blocked(make, label):
         t0 = time.perf_counter()
-        h = pasta.pasta_coo_to_hicoo(x, 7)
+        h = make()
         torch.cuda.synchronize()
         t_conv = time.perf_counter() - t0
         t0 = time.perf_counter()
@@ -414,21 +414,32 @@ def main():
         pasta.pasta_profile_enable(False)
         hk_ms, hk_n = pasta.pasta_profile_read(1, reset=True)
         h_ms = h0.elapsed_time(h1) / args.hicoo_steps
-        hb = model_bytes_hicoo(N, M, h.nblocks, R)
+        nc = bin(h.cmask).count("1")
+        if nc == N:
+            hb = model_bytes_hicoo(N, M, h.nblocks, R)
+            bm = "(N+4)M + (8+4N)n_b + 4NR min(n_b B, M) per launch"
+        else:  # gHiCOO stream + the COO upper bound for the gathers (R#29)
+            hb = (nc + 4 * (N - nc) + 4) * M + (8 + 4 * nc) * h.nblocks + 4 * N * R * M
+            bm = "(N_c + 4N_u + 4)M + (8+4N_c)n_b + 4NRM per launch"
         peak_h, _ = load_peaks()
         ach = hb / (hk_ms / max(hk_n, 1) * 1e-3) / 1e9
-        hicoo = {"value": round(total_flops / (h_ms * 1e-3) / 1e9, 3), "unit": "GFLOP/s",
-                 "ms_per_step": round(h_ms, 4), "nblocks": h.nblocks, "block": 128,
-                 "nnz_per_block": round(M / max(h.nblocks, 1), 3),
-                 "roofline": {"bound": "hbm", "achieved": round(ach, 1), "peak": peak_h,
-                              "unit": "GB/s", "frac": round(ach / peak_h, 4),
-                              "traffic": ncu_traffic(args.config, "hicoo_mttkrp"),
-                              "kernel": "mttkrp_kernel<HicooRowSrc> (a7, row-slice layout)",
-                              "bytes_model": "(N+4)M + (8+4N)n_b + 4NR min(n_b B, M) per launch",
-                              "avg_launch_ms": round(hk_ms / max(hk_n, 1), 4)},
-                 "preprocess_s": {"coo_to_hicoo": round(t_conv, 3),
-                                  "mode_copies_all": round(t_hprep, 3)}}
+        res = {"value": round(total_flops / (h_ms * 1e-3) / 1e9, 3), "unit": "GFLOP/s",
+               "ms_per_step": round(h_ms, 4), "nblocks": h.nblocks, "block": 128,
+               "cmask": h.cmask, "nnz_per_block": round(M / max(h.nblocks, 1), 3),
+               "roofline": {"bound": "hbm", "achieved": round(ach, 1), "peak": peak_h,
+                            "unit": "GB/s", "frac": round(ach / peak_h, 4),
+                            "traffic": ncu_traffic(args.config, label + "_mttkrp"),
+                            "kernel": f"mttkrp_kernel<HicooRowSrc> ({label}, row-slice layout)",
+                            "bytes_model": bm,
+                            "avg_launch_ms": round(hk_ms / max(hk_n, 1), 4)},
+               "preprocess_s": {"convert": round(t_conv, 3), "mode_copies_all": round(t_hprep, 3)}}
         del h, houts
+        return res
+
+    hicoo = ghicoo = None
+    if world == 1 and args.hicoo_steps > 0:
+        hicoo = time_blocked(lambda: pasta.pasta_coo_to_hicoo(x, 7), "hicoo")
+        ghicoo = time_blocked(lambda: pasta.pasta_coo_to_ghicoo(x, 7, 0), "ghicoo")
 
     # NEXT-1: CP-ALS sweeps (each = MTTKRP + solve + normalise + gram for every mode)
     cpals = None
@@ -484,7 +495,7 @@ def main():
         "model_gbs": round(model_bytes_coo(N, M, R) * N / (ms_per_step * 1e-3) / 1e9, 1),
         "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
                      "frac": round(achieved / peak, 4), "traffic": traffic,
-                     "kernel": "mttkrp_kernel<CooSrc> (a6)",
+                     "kernel": "coo_staged_kernel (a6, csrc/mttkrp.cu)",
                      "bytes_model": "4(N+1)M + 4NRM per launch (Table I, P:117)",
                      "avg_launch_ms": round(avg_launch_ms, 4), "launches": kern_n,
                      "peak_source": peak_src,
@@ -499,6 +510,7 @@ def main():
         "e2e": e2e,
         "allgather": allgather,
         "hicoo": hicoo,
+        "ghicoo": ghicoo,
         "cpals": cpals,
         "gpu_launches": launches,
         "cpu_baseline": cpu,

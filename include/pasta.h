@@ -118,6 +118,29 @@ pasta_status pasta_gen_powerlaw(uint32_t order, const uint32_t *dims, uint64_t n
  * with the oracle's conversion.  Runs on the GPU. */
 pasta_status pasta_coo_to_hicoo(const pasta_coo *x, uint32_t block_bits, pasta_hicoo **out);
 
+/* gHiCOO conversion (Fig. 2(b); R#29): "pick which modes to be
+ * compressed in units of blocks for HiCOO and which stay in COO format", for hypersparse
+ * tensors whose HiCOO blocks hold one or few nonzeros.  Bit k of `cmask`
+ * set <=> mode k is blocked (binds_k u32 per block, einds_k u8 per nonzero); the other modes
+ * keep their u32 coordinates per nonzero (uinds_k).  Order: Morton order (R#13) of the
+ * compressed modes' coordinates, ties lexicographic over the uncompressed modes in ascending
+ * mode order, then canonical position; a block starts where i_k >> b changes for a
+ * compressed k.  cmask = all modes is exactly pasta_coo_to_hicoo; cmask = 0 picks the mask
+ * with pasta_ghicoo_auto_mask.  Bit-exact with the oracle's conversion.  The result is a
+ * pasta_hicoo handle: pasta_mttkrp_hicoo / pasta_hicoo_prepare / pasta_hicoo_info accept it
+ * (row-slice layout; an uncompressed target mode makes a slice = the entries of one block
+ * that share i_mode).  Errors: EINVAL (NULL, block_bits outside 1..8, cmask bits >= order). */
+pasta_status pasta_coo_to_ghicoo(const pasta_coo *x, uint32_t block_bits, uint32_t cmask,
+                                 pasta_hicoo **out);
+/* Hypersparse-aware mode choice for gHiCOO: the mask minimising the gHiCOO storage
+ *   bytes(mask) = (N_c + 4 N_u + 4) M + (8 + 4 N_c) n_b(mask)
+ * (Table I's HiCOO storage, generalised; N_c / N_u compressed / uncompressed modes,
+ * n_b(mask) = number of distinct (i_k >> b, k in mask) keys, counted on the GPU).  Exhaustive
+ * over all non-empty masks for order <= 4 (ties -> smallest mask value), greedy forward
+ * selection from the best single mode above.  `bytes` (may be NULL) receives the minimum. */
+pasta_status pasta_ghicoo_auto_mask(const pasta_coo *x, uint32_t block_bits, uint32_t *cmask,
+                                    uint64_t *bytes);
+
 /* Build (once; cached in the handle) the mode-`mode` working copy: for COO the nonzeros
  * stably sorted lexicographically by (i_mode, i_mode+1, ..., i_mode-1) (a2);
  * for HiCOO (R#27) by default "row slices" (the entries of a block that share einds_mode,
@@ -232,6 +255,14 @@ pasta_status pasta_hicoo_info(const pasta_hicoo *h, uint32_t *order, uint32_t *d
  * binds: `order` pointers to nblocks uint32, einds: `order` pointers to nnz uint8, vals. */
 pasta_status pasta_hicoo_export(const pasta_hicoo *h, uint64_t *bptr, uint32_t *const *binds,
                                 uint8_t *const *einds, float *vals);
+/* gHiCOO: the compression mask of a handle (all bits for a HiCOO handle). */
+pasta_status pasta_ghicoo_info(const pasta_hicoo *h, uint32_t *cmask);
+/* Copy the canonical gHiCOO arrays to HOST buffers: bptr[nblocks+1]; for compressed modes
+ * binds[k] (nblocks u32) and einds[k] (nnz u8); for uncompressed modes uinds[k] (nnz u32).
+ * NULL array pointers (or NULL entries) are skipped.  pasta_hicoo_export rejects (EINVAL) a
+ * handle that is not fully compressed. */
+pasta_status pasta_ghicoo_export(const pasta_hicoo *h, uint64_t *bptr, uint32_t *const *binds,
+                                 uint8_t *const *einds, uint32_t *const *uinds, float *vals);
 void pasta_coo_free(pasta_coo *x);
 void pasta_hicoo_free(pasta_hicoo *h);
 

@@ -65,6 +65,9 @@ class Hicoo:
         self._p = C.c_void_p(ptr)
         info = pasta_hicoo_info(self)
         self.order, self.dims, self.block_bits, self.nblocks, self.nnz = info
+        cm = C.c_uint32()
+        check(lib().pasta_ghicoo_info(self._p, C.byref(cm)))
+        self.cmask = cm.value  # gHiCOO compression mask (all bits: HiCOO)
 
     @property
     def ptr(self):
@@ -189,6 +192,22 @@ def pasta_coo_to_hicoo(x: Coo, block_bits: int = 7) -> Hicoo:
     out = C.c_void_p()
     check(lib().pasta_coo_to_hicoo(x.ptr, block_bits, C.byref(out)))
     return Hicoo(out.value)
+
+
+def pasta_coo_to_ghicoo(x: Coo, block_bits: int = 7, cmask: int = 0) -> Hicoo:
+    """gHiCOO: modes with bit k of ``cmask`` blocked, the rest kept as COO
+    coordinates; ``cmask = 0`` lets the library pick (:func:`pasta_ghicoo_auto_mask`)."""
+    out = C.c_void_p()
+    check(lib().pasta_coo_to_ghicoo(x.ptr, block_bits, cmask, C.byref(out)))
+    return Hicoo(out.value)
+
+
+def pasta_ghicoo_auto_mask(x: Coo, block_bits: int = 7):
+    """(cmask, bytes): the storage-minimising gHiCOO mask and its storage in bytes."""
+    cm = C.c_uint32()
+    nbytes = C.c_uint64()
+    check(lib().pasta_ghicoo_auto_mask(x.ptr, block_bits, C.byref(cm), C.byref(nbytes)))
+    return cm.value, nbytes.value
 
 
 def pasta_coo_prepare(x: Coo, mode: int, stream=None) -> None:
@@ -355,6 +374,27 @@ def pasta_hicoo_export(h: Hicoo) -> dict:
     check(lib().pasta_hicoo_export(h.ptr, _np_ptr(bptr, _u64p), bp, ep, _np_ptr(vals, _f32p)))
     return {"order": N, "block_bits": h.block_bits, "nblocks": nb, "nnz": M, "bptr": bptr,
             "binds": np.stack([b[:nb] for b in binds]), "einds": np.stack([e[:M] for e in einds]),
+            "vals": vals[:M].copy()}
+
+
+def pasta_ghicoo_export(h: Hicoo) -> dict:
+    """Canonical gHiCOO arrays (lists indexed by mode; None where a mode has no such array)."""
+    nb, M, N, cm = h.nblocks, h.nnz, h.order, h.cmask
+    comp = [bool((cm >> k) & 1) for k in range(N)]
+    bptr = np.zeros(nb + 1, np.uint64)
+    binds = [np.zeros(max(nb, 1), np.uint32) if comp[k] else None for k in range(N)]
+    einds = [np.zeros(max(M, 1), np.uint8) if comp[k] else None for k in range(N)]
+    uinds = [None if comp[k] else np.zeros(max(M, 1), np.uint32) for k in range(N)]
+    bp = (_u32p * N)(*[_np_ptr(b, _u32p) if b is not None else None for b in binds])
+    ep = (_u8p * N)(*[_np_ptr(e, _u8p) if e is not None else None for e in einds])
+    up = (_u32p * N)(*[_np_ptr(u, _u32p) if u is not None else None for u in uinds])
+    vals = np.zeros(max(M, 1), np.float32)
+    check(lib().pasta_ghicoo_export(h.ptr, _np_ptr(bptr, _u64p), bp, ep, up, _np_ptr(vals, _f32p)))
+    return {"order": N, "block_bits": h.block_bits, "cmask": cm, "nblocks": nb, "nnz": M,
+            "bptr": bptr,
+            "binds": [b[:nb] if b is not None else None for b in binds],
+            "einds": [e[:M] if e is not None else None for e in einds],
+            "uinds": [u[:M] if u is not None else None for u in uinds],
             "vals": vals[:M].copy()}
 
 

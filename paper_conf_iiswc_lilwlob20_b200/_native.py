@@ -56,6 +56,10 @@ SIGNATURES = {
     "pasta_gen_powerlaw": (_st, [C.c_uint32, _u32p, C.c_uint64, C.c_uint64, C.POINTER(GenParams),
                                  C.POINTER(_vp)]),
     "pasta_coo_to_hicoo": (_st, [_vp, C.c_uint32, C.POINTER(_vp)]),
+    "pasta_coo_to_ghicoo": (_st, [_vp, C.c_uint32, C.c_uint32, C.POINTER(_vp)]),
+    "pasta_ghicoo_auto_mask": (_st, [_vp, C.c_uint32, _u32p, _u64p]),
+    "pasta_ghicoo_info": (_st, [_vp, _u32p]),
+    "pasta_ghicoo_export": (_st, [_vp, _u64p, C.POINTER(_u32p), C.POINTER(_u8p), C.POINTER(_u32p), _f32p]),
     "pasta_coo_prepare": (_st, [_vp, C.c_uint32, _vp]),
     "pasta_hicoo_prepare": (_st, [_vp, C.c_uint32, _vp]),
     "pasta_mttkrp_coo": (_st, [_vp, C.c_uint32, C.POINTER(_vp), C.c_uint32, _vp, _vp]),

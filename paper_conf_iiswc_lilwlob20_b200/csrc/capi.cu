@@ -402,6 +402,78 @@ pasta_status pasta_coo_to_hicoo(const pasta_coo *x, uint32_t block_bits, pasta_h
   h->order = x->order;
   for (uint32_t k = 0; k < x->order; ++k) h->dims[k] = x->dims[k];
   h->block_bits = block_bits;
+  h->cmask = (1u << x->order) - 1u;
+  h->device = x->device;
+  coo_to_hicoo_device(x, h.get(), nullptr);
+  *out = h.release();
+  API_END
+}
+
+// gHiCOO storage in bytes (R#29): per nonzero 1 B per compressed mode, 4 B per uncompressed
+// mode, 4 B value; per block 8 B bptr + 4 B binds per compressed mode.
+static uint64_t ghicoo_bytes(uint32_t order, uint32_t cmask, uint64_t M, uint64_t nb) {
+  uint32_t nc = uint32_t(__builtin_popcount(cmask)), nu = order - nc;
+  return (uint64_t(nc) + 4ull * nu + 4ull) * M + (8ull + 4ull * nc) * nb;
+}
+
+static uint32_t choose_ghicoo_mask(const pasta_coo *x, uint32_t block_bits, uint64_t *bytes) {
+  const uint32_t N = x->order;
+  const uint32_t full = (1u << N) - 1u;
+  uint32_t best = full;
+  uint64_t best_b = ~0ull;
+  auto cost = [&](uint32_t m) {
+    return ghicoo_bytes(N, m, x->nnz, count_blocks_device(x, block_bits, m, nullptr));
+  };
+  if (N <= 4) {  // exhaustive, ascending mask value; strict improvement keeps the smallest mask
+    for (uint32_t m = 1; m <= full; ++m) {
+      uint64_t c = cost(m);
+      if (c < best_b) { best_b = c; best = m; }
+    }
+  } else {  // greedy forward selection from the best single mode
+    for (uint32_t k = 0; k < N; ++k) {
+      uint64_t c = cost(1u << k);
+      if (c < best_b) { best_b = c; best = 1u << k; }
+    }
+    for (bool grew = true; grew;) {
+      grew = false;
+      uint32_t cand = best;
+      uint64_t cand_b = best_b;
+      for (uint32_t k = 0; k < N; ++k) {
+        if ((best >> k) & 1u) continue;
+        uint64_t c = cost(best | (1u << k));
+        if (c < cand_b) { cand_b = c; cand = best | (1u << k); }
+      }
+      if (cand != best) { best = cand; best_b = cand_b; grew = true; }
+    }
+  }
+  if (bytes) *bytes = best_b;
+  return best;
+}
+
+pasta_status pasta_ghicoo_auto_mask(const pasta_coo *x, uint32_t block_bits, uint32_t *cmask,
+                                    uint64_t *bytes) {
+  API_BEGIN
+  require(x && cmask, "x/cmask is NULL");
+  require(block_bits >= 1 && block_bits <= 8, "block_bits must be in 1..8 (8-bit element indices, P:181)");
+  check_device(x->device);
+  *cmask = choose_ghicoo_mask(x, block_bits, bytes);
+  API_END
+}
+
+pasta_status pasta_coo_to_ghicoo(const pasta_coo *x, uint32_t block_bits, uint32_t cmask,
+                                 pasta_hicoo **out) {
+  API_BEGIN
+  require(x && out, "x/out is NULL");
+  *out = nullptr;
+  require(block_bits >= 1 && block_bits <= 8, "block_bits must be in 1..8 (8-bit element indices, P:181)");
+  require((cmask >> x->order) == 0, "cmask has bits >= order");
+  check_device(x->device);
+  if (cmask == 0) cmask = choose_ghicoo_mask(x, block_bits, nullptr);
+  auto h = std::make_unique<pasta_hicoo>();
+  h->order = x->order;
+  for (uint32_t k = 0; k < x->order; ++k) h->dims[k] = x->dims[k];
+  h->block_bits = block_bits;
+  h->cmask = cmask;
   h->device = x->device;
   coo_to_hicoo_device(x, h.get(), nullptr);
   *out = h.release();
@@ -849,10 +921,38 @@ pasta_status pasta_hicoo_info(const pasta_hicoo *h, uint32_t *order, uint32_t *d
   API_END
 }
 
+pasta_status pasta_ghicoo_info(const pasta_hicoo *h, uint32_t *cmask) {
+  API_BEGIN
+  require(h && cmask, "h/cmask is NULL");
+  *cmask = h->cmask;
+  API_END
+}
+
+pasta_status pasta_ghicoo_export(const pasta_hicoo *h, uint64_t *bptr, uint32_t *const *binds,
+                                 uint8_t *const *einds, uint32_t *const *uinds, float *vals) {
+  API_BEGIN
+  require(h != nullptr, "h is NULL");
+  check_device(h->device);
+  if (bptr) PASTA_CUDA(cudaMemcpy(bptr, h->bptr.p, (h->nblocks + 1) * 8, cudaMemcpyDeviceToHost));
+  for (uint32_t k = 0; k < h->order; ++k) {
+    if ((h->cmask >> k) & 1u) {
+      if (binds && binds[k] && h->nblocks)
+        PASTA_CUDA(cudaMemcpy(binds[k], h->binds[k].p, h->nblocks * 4, cudaMemcpyDeviceToHost));
+      if (einds && einds[k] && h->nnz)
+        PASTA_CUDA(cudaMemcpy(einds[k], h->einds[k].p, h->nnz, cudaMemcpyDeviceToHost));
+    } else if (uinds && uinds[k] && h->nnz) {
+      PASTA_CUDA(cudaMemcpy(uinds[k], h->uinds[k].p, h->nnz * 4, cudaMemcpyDeviceToHost));
+    }
+  }
+  if (vals && h->nnz) PASTA_CUDA(cudaMemcpy(vals, h->val.p, h->nnz * 4, cudaMemcpyDeviceToHost));
+  API_END
+}
+
 pasta_status pasta_hicoo_export(const pasta_hicoo *h, uint64_t *bptr, uint32_t *const *binds,
                                 uint8_t *const *einds, float *vals) {
   API_BEGIN
   require(h != nullptr, "h is NULL");
+  require(h->cmask == (1u << h->order) - 1u, "gHiCOO handle: use pasta_ghicoo_export");
   check_device(h->device);
   if (bptr) PASTA_CUDA(cudaMemcpy(bptr, h->bptr.p, (h->nblocks + 1) * 8, cudaMemcpyDeviceToHost));
   for (uint32_t k = 0; k < h->order; ++k) {

@@ -80,6 +80,13 @@ __global__ void gather_binds_kernel(const uint32_t *__restrict__ binds_n, const 
     out[x] = binds_n[blk[x]];
 }
 
+__global__ void shift_u32_kernel(const uint32_t *__restrict__ in, uint64_t M, uint32_t sh,
+                                 uint32_t *__restrict__ out) {
+  for (uint64_t x = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; x < M;
+       x += uint64_t(gridDim.x) * blockDim.x)
+    out[x] = in[x] >> sh;
+}
+
 __global__ void u8_to_u32_kernel(const uint8_t *__restrict__ in, uint64_t M, uint32_t *__restrict__ out) {
   for (uint64_t x = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; x < M;
        x += uint64_t(gridDim.x) * blockDim.x)
@@ -131,6 +138,8 @@ struct SliceOut {
   const uint32_t *binds[kMaxOrder];
   uint32_t *base[kMaxOrder];
   uint32_t order, mode, bbits;
+  uint32_t cmask;  // gHiCOO: only compressed modes have block bases; an uncompressed mode's
+                   // row comes in full (enp = i_mode)
 };
 
 __global__ void slice_emit_kernel(SliceOut o, const uint32_t *__restrict__ starts, uint64_t nsb, uint64_t M,
@@ -142,9 +151,9 @@ __global__ void slice_emit_kernel(SliceOut o, const uint32_t *__restrict__ start
     uint32_t x = starts[j];
     uint32_t b = blkp[x];
     sbptr[j] = x;
-    sbrow[j] = (o.binds[o.mode][b] << o.bbits) + enp[x];
+    sbrow[j] = ((o.cmask >> o.mode) & 1u) ? (o.binds[o.mode][b] << o.bbits) + enp[x] : enp[x];
     for (uint32_t k = 0; k < o.order; ++k)
-      if (k != o.mode) o.base[k][j] = o.binds[k][b] << o.bbits;
+      if (k != o.mode && ((o.cmask >> k) & 1u)) o.base[k][j] = o.binds[k][b] << o.bbits;
   }
 }
 
@@ -160,25 +169,40 @@ __global__ void sched_counts_kernel(const uint64_t *__restrict__ bptr, const uin
 
 }  // namespace
 
+// COO -> HiCOO / gHiCOO.  HiCOO (cmask = all modes): Morton order of the full coordinates.
+// gHiCOO (R#29): stable lexicographic sort by the uncompressed modes first, then a
+// stable Morton sort by the compressed modes, which gives Morton order of the compressed
+// coordinates with ties in lexicographic order of the uncompressed ones; blocks split where
+// (i_k >> b) changes for a compressed k; uncompressed modes keep their u32 coordinates.
 void coo_to_hicoo_device(const pasta_coo *x, pasta_hicoo *h, cudaStream_t s) {
   const uint32_t N = x->order;
   const uint64_t M = x->nnz;
   const uint32_t bb = h->block_bits;
-  uint32_t Lm = 0;
-  for (uint32_t k = 0; k < N; ++k) Lm = ceil_log2(x->dims[k]) > Lm ? ceil_log2(x->dims[k]) : Lm;
+  const uint32_t cmask = h->cmask;
+  uint32_t Lm = 0, nc = 0, nu = 0;
+  const uint32_t *comp[kMaxOrder], *unc[kMaxOrder];
+  uint32_t ubits[kMaxOrder];
+  for (uint32_t k = 0; k < N; ++k) {
+    if ((cmask >> k) & 1u) {
+      comp[nc++] = x->inds[k].p;
+      if (ceil_log2(x->dims[k]) > Lm) Lm = ceil_log2(x->dims[k]);
+    } else {
+      ubits[nu] = ceil_log2(x->dims[k]);
+      unc[nu++] = x->inds[k].p;
+    }
+  }
   DevArray<uint32_t> perm(M, s);
   iota_u32(perm.p, M, s);
-  const uint32_t *canon[kMaxOrder];
-  for (uint32_t k = 0; k < N; ++k) canon[k] = x->inds[k].p;
-  morton_sort(canon, N, Lm, perm, M, s);
+  if (nu) lexsort(unc, ubits, int(nu), perm, M, s);
+  morton_sort(comp, nc, Lm, perm, M, s);
 
   DevArray<uint32_t> sc[kMaxOrder];
   Coords co{};
-  co.order = N;
+  co.order = 0;
   for (uint32_t k = 0; k < N; ++k) {
     sc[k].alloc(M, s);
-    gather_u32(canon[k], perm.p, sc[k].p, M, s);
-    co.c[k] = sc[k].p;
+    gather_u32(x->inds[k].p, perm.p, sc[k].p, M, s);
+    if ((cmask >> k) & 1u) co.c[co.order++] = sc[k].p;
   }
   uint64_t nb = 0;
   DevArray<uint32_t> starts;
@@ -195,13 +219,19 @@ void coo_to_hicoo_device(const pasta_coo *x, pasta_hicoo *h, cudaStream_t s) {
     uint64_t zero = 0;
     PASTA_CUDA(cudaMemcpyAsync(h->bptr.p, &zero, sizeof(zero), cudaMemcpyHostToDevice, s));
   }
+  bool bptr_written = false;
   for (uint32_t k = 0; k < N; ++k) {
+    if (!((cmask >> k) & 1u)) {
+      h->uinds[k] = std::move(sc[k]);  // full coordinates, already in gHiCOO order
+      continue;
+    }
     h->binds[k].alloc(nb, s);
     h->einds[k].alloc(M, s);
     if (M) {
       emit_blocks_kernel<<<grid_for(nb + 1), kThreads, 0, s>>>(starts.p, nb, M, sc[k].p, bb, h->bptr.p,
-                                                             h->binds[k].p, k == 0);
+                                                             h->binds[k].p, !bptr_written);
       PASTA_LAUNCHED();
+      bptr_written = true;
       emit_einds_kernel<<<grid_for(M), kThreads, 0, s>>>(sc[k].p, M, (1u << bb) - 1u, h->einds[k].p);
       PASTA_LAUNCHED();
     }
@@ -209,6 +239,42 @@ void coo_to_hicoo_device(const pasta_coo *x, pasta_hicoo *h, cudaStream_t s) {
   h->val.alloc(M, s);
   gather_f32(x->val.p, perm.p, h->val.p, M, s);
   PASTA_CUDA(cudaStreamSynchronize(s));
+}
+
+uint64_t count_blocks_device(const pasta_coo *x, uint32_t block_bits, uint32_t cmask, cudaStream_t s) {
+  const uint64_t M = x->nnz;
+  if (M == 0) return 0;
+  const uint32_t N = x->order;
+  DevArray<uint32_t> keys[kMaxOrder];
+  const uint32_t *comps[kMaxOrder];
+  uint32_t bits[kMaxOrder];
+  int nc = 0;
+  Coords co{};
+  for (uint32_t k = 0; k < N; ++k) {
+    if (!((cmask >> k) & 1u)) continue;
+    keys[nc].alloc(M, s);
+    shift_u32_kernel<<<grid_for(M), kThreads, 0, s>>>(x->inds[k].p, M, block_bits, keys[nc].p);
+    PASTA_LAUNCHED();
+    comps[nc] = keys[nc].p;
+    uint32_t l = ceil_log2(x->dims[k]);
+    bits[nc] = l > block_bits ? l - block_bits : 0;
+    ++nc;
+  }
+  DevArray<uint32_t> perm(M, s);
+  iota_u32(perm.p, M, s);
+  lexsort(comps, bits, nc, perm, M, s);
+  DevArray<uint32_t> sk[kMaxOrder];
+  for (int c = 0; c < nc; ++c) {
+    sk[c].alloc(M, s);
+    gather_u32(keys[c].p, perm.p, sk[c].p, M, s);
+    co.c[c] = sk[c].p;
+  }
+  co.order = uint32_t(nc);
+  DevArray<uint8_t> flag(M, s);
+  block_flag_kernel<<<grid_for(M), kThreads, 0, s>>>(co, 0, M, flag.p);
+  PASTA_LAUNCHED();
+  DevArray<uint32_t> starts;
+  return select_flagged(flag.p, M, starts, s);
 }
 
 // Per-mode copy (R#27): blocks stably sorted by (light, binds_mode), entries inside a block
@@ -220,9 +286,12 @@ static void hicoo_prepare_rowslice(pasta_hicoo *h, uint32_t mode, cudaStream_t s
   const uint32_t N = h->order;
   const uint64_t M = h->nnz, nb = h->nblocks;
   const uint32_t bb = h->block_bits;
+  auto comp = [&](uint32_t k) { return ((h->cmask >> k) & 1u) != 0; };
   mc.layout = 0;
-  for (uint32_t k = 0; k < N; ++k)
-    if (k != mode) mc.einds[k].alloc(M, s);
+  for (uint32_t k = 0; k < N; ++k) {
+    if (k == mode) continue;
+    if (comp(k)) mc.einds[k].alloc(M, s); else mc.uinds[k].alloc(M, s);
+  }
   mc.val.alloc(M, s);
   if (M == 0) {
     mc.nsb = 0;
@@ -233,26 +302,41 @@ static void hicoo_prepare_rowslice(pasta_hicoo *h, uint32_t mode, cudaStream_t s
     mc.ready = true;
     return;
   }
-  // entry order: (binds_mode[blk], einds_mode, blk); ties keep Morton order (stable)
-  DevArray<uint32_t> blk(M, s), c0(M, s), en(M, s);
+  // entry order: (output row, blk), the row as (binds_mode[blk], einds_mode) when the mode is
+  // compressed, else the full i_mode (gHiCOO); ties keep the canonical order (stable)
+  DevArray<uint32_t> blk(M, s), c0, en;
   entry_block_kernel<<<grid_for(M), kThreads, 0, s>>>(h->bptr.p, nb, M, blk.p);
   PASTA_LAUNCHED();
-  gather_binds_kernel<<<grid_for(M), kThreads, 0, s>>>(h->binds[mode].p, blk.p, M, c0.p);
-  PASTA_LAUNCHED();
-  u8_to_u32_kernel<<<grid_for(M), kThreads, 0, s>>>(h->einds[mode].p, M, en.p);
-  PASTA_LAUNCHED();
-  uint64_t nbr = (uint64_t(h->dims[mode]) + (1ull << bb) - 1) >> bb;
-  const uint32_t *comps[3] = {c0.p, en.p, blk.p};
-  uint32_t bits[3] = {ceil_log2(nbr), bb, ceil_log2(nb)};
   DevArray<uint32_t> perm(M, s);
   iota_u32(perm.p, M, s);
-  lexsort(comps, bits, 3, perm, M, s);
-  c0.reset();
+  const uint32_t *en_src;
+  if (comp(mode)) {
+    c0.alloc(M, s);
+    en.alloc(M, s);
+    gather_binds_kernel<<<grid_for(M), kThreads, 0, s>>>(h->binds[mode].p, blk.p, M, c0.p);
+    PASTA_LAUNCHED();
+    u8_to_u32_kernel<<<grid_for(M), kThreads, 0, s>>>(h->einds[mode].p, M, en.p);
+    PASTA_LAUNCHED();
+    uint64_t nbr = (uint64_t(h->dims[mode]) + (1ull << bb) - 1) >> bb;
+    const uint32_t *comps[3] = {c0.p, en.p, blk.p};
+    uint32_t bits[3] = {ceil_log2(nbr), bb, ceil_log2(nb)};
+    lexsort(comps, bits, 3, perm, M, s);
+    c0.reset();
+    en_src = en.p;
+  } else {
+    const uint32_t *comps[2] = {h->uinds[mode].p, blk.p};
+    uint32_t bits[2] = {ceil_log2(h->dims[mode]), ceil_log2(nb)};
+    lexsort(comps, bits, 2, perm, M, s);
+    en_src = h->uinds[mode].p;
+  }
   DevArray<uint32_t> blkp(M, s), enp(M, s);
   gather_u32(blk.p, perm.p, blkp.p, M, s);
-  gather_u32(en.p, perm.p, enp.p, M, s);
-  for (uint32_t k = 0; k < N; ++k)
-    if (k != mode) gather_u8(h->einds[k].p, perm.p, mc.einds[k].p, M, s);
+  gather_u32(en_src, perm.p, enp.p, M, s);
+  for (uint32_t k = 0; k < N; ++k) {
+    if (k == mode) continue;
+    if (comp(k)) gather_u8(h->einds[k].p, perm.p, mc.einds[k].p, M, s);
+    else gather_u32(h->uinds[k].p, perm.p, mc.uinds[k].p, M, s);
+  }
   gather_f32(h->val.p, perm.p, mc.val.p, M, s);
   DevArray<uint8_t> flag(M, s);
   slice_flag_kernel<<<grid_for(M), kThreads, 0, s>>>(blkp.p, enp.p, M, flag.p);
@@ -265,9 +349,10 @@ static void hicoo_prepare_rowslice(pasta_hicoo *h, uint32_t mode, cudaStream_t s
   o.order = N;
   o.mode = mode;
   o.bbits = bb;
+  o.cmask = h->cmask;
   for (uint32_t k = 0; k < N; ++k) {
     o.binds[k] = h->binds[k].p;
-    if (k != mode) {
+    if (k != mode && comp(k)) {
       mc.sbbase[k].alloc(mc.nsb, s);
       o.base[k] = mc.sbbase[k].p;
     }
@@ -283,7 +368,8 @@ void hicoo_prepare_mode(pasta_hicoo *h, uint32_t mode, cudaStream_t s) {
   HicooModeCopy &mc = h->mc[mode];
   if (mc.ready) return;
   const char *lay = getenv("PASTA_HICOO_LAYOUT");
-  if (!(lay && std::string(lay) == "block")) return hicoo_prepare_rowslice(h, mode, s);
+  const bool full = h->cmask == (1u << h->order) - 1u;  // the block layout needs every mode blocked
+  if (!full || !(lay && std::string(lay) == "block")) return hicoo_prepare_rowslice(h, mode, s);
   mc.layout = 1;
   const uint32_t N = h->order;
   const uint64_t M = h->nnz, nb = h->nblocks;

@@ -146,7 +146,8 @@ struct HicooModeCopy {
   uint64_t nsb = 0;
   DevArray<uint64_t> sbptr;              // nsb + 1
   DevArray<uint32_t> sbrow;              // nsb: output row of the slice
-  DevArray<uint32_t> sbbase[kMaxOrder];  // nsb each (k != mode): binds_k << block_bits
+  DevArray<uint32_t> sbbase[kMaxOrder];  // nsb each (k != mode, k compressed): binds_k << block_bits
+  DevArray<uint32_t> uinds[kMaxOrder];   // gHiCOO: nnz each (k != mode, k uncompressed): i_k
 };
 
 }  // namespace pasta
@@ -187,12 +188,16 @@ struct pasta_hicoo {
   uint32_t order = 0;
   uint32_t dims[pasta::kMaxOrder] = {};
   uint32_t block_bits = 7;
+  // gHiCOO (R#29): bit k set <=> mode k is blocked (binds_k, einds_k); the
+  // other modes keep full u32 coordinates (uinds_k).  HiCOO = all bits set.
+  uint32_t cmask = 0;
   uint64_t nblocks = 0;
   uint64_t nnz = 0;
   int device = 0;
   pasta::DevArray<uint64_t> bptr;
   pasta::DevArray<uint32_t> binds[pasta::kMaxOrder];
   pasta::DevArray<uint8_t> einds[pasta::kMaxOrder];
+  pasta::DevArray<uint32_t> uinds[pasta::kMaxOrder];
   pasta::DevArray<float> val;
   pasta::HicooModeCopy mc[pasta::kMaxOrder];
   std::mutex mu;
@@ -236,7 +241,9 @@ void coo_prepare_mode(pasta_coo *x, uint32_t mode, cudaStream_t s);
 void hicoo_prepare_mode(pasta_hicoo *h, uint32_t mode, cudaStream_t s);
 void gen_powerlaw_device(pasta_coo *x, uint64_t seed, const double *table, uint32_t ncell,
                          float val_lo, float val_hi, cudaStream_t s);
-void coo_to_hicoo_device(const pasta_coo *x, pasta_hicoo *h, cudaStream_t s);
+void coo_to_hicoo_device(const pasta_coo *x, pasta_hicoo *h, cudaStream_t s);  // honours h->cmask
+// number of distinct block keys (i_k >> block_bits, k in cmask) of a COO tensor
+uint64_t count_blocks_device(const pasta_coo *x, uint32_t block_bits, uint32_t cmask, cudaStream_t s);
 
 void launch_zero_rows(float *out, uint64_t row_lo, uint64_t row_hi, uint32_t R, cudaStream_t s);
 void launch_coo_mttkrp(const pasta_coo *x, uint32_t mode, const float *const *factors, uint32_t R,

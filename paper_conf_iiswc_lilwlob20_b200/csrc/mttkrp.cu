@@ -57,6 +57,9 @@ struct KArgs {
   uint64_t nsb;
   const uint32_t *sbrow;
   const uint32_t *sbbase[kMaxOrder - 1];
+  // gHiCOO (R#29): bit j set <=> other-mode slot j is uncompressed: its u32 coordinates come
+  // from io[j] (no slice base); clear -> 8-bit element index eo[j] + slice base
+  uint32_t wide;
   // factors of the other modes (ascending k), output
   const float *Uo[kMaxOrder - 1];
   float *out;
@@ -265,6 +268,9 @@ struct HicooSrc {
 // einds_n; slices are ordered by output row, so rows are globally sorted as in COO.  Per
 // entry only the 8-bit element indices of the other modes and the value are streamed; the
 // row and the other-mode block bases (Alg. 3's rebased pointers) come per slice.
+// gHiCOO (R#29): an uncompressed other mode streams its u32 coordinate instead
+// (KArgs::wide), an uncompressed target mode makes a slice = the entries of a block sharing
+// i_n.  The wide test is warp-uniform.
 template <int NO, int U>
 struct HicooRowSrc {
   static constexpr bool kSortedRows = true;
@@ -276,6 +282,7 @@ struct HicooRowSrc {
   uint32_t srow, nrow;
   uint32_t base[NOA], nbase[NOA];
   int no;
+  uint32_t wide;
   uint64_t pol;
   __device__ __forceinline__ void load_next(const KArgs &a) {
     const uint64_t n1 = sb + 1 < a.nsb ? sb + 1 : sb;  // clamp: never read past the end
@@ -283,7 +290,7 @@ struct HicooRowSrc {
     nrow = __ldg(a.sbrow + n1);
 #pragma unroll
     for (int j = 0; j < NOA; ++j)
-      if (j < no) nbase[j] = __ldg(a.sbbase[j] + n1);
+      if (j < no) nbase[j] = ((wide >> j) & 1u) ? 0u : __ldg(a.sbbase[j] + n1);
   }
   __device__ __forceinline__ void advance(const KArgs &a) {
     ++sb;
@@ -296,6 +303,7 @@ struct HicooRowSrc {
   __device__ __forceinline__ void init(const KArgs &a, uint64_t x0, uint64_t p) {
     pol = p;
     no = int(a.order) - 1;
+    wide = a.wide;
     uint64_t lo = 0, hi = a.nsb;  // last slice with sbptr[sb] <= x0
     while (hi - lo > 1) {
       uint64_t mid = (lo + hi) / 2;
@@ -306,7 +314,7 @@ struct HicooRowSrc {
     srow = __ldg(a.sbrow + sb);
 #pragma unroll
     for (int j = 0; j < NOA; ++j)
-      if (j < no) base[j] = __ldg(a.sbbase[j] + sb);
+      if (j < no) base[j] = ((wide >> j) & 1u) ? 0u : __ldg(a.sbbase[j] + sb);
     load_next(a);
   }
   __device__ __forceinline__ void load(const KArgs &a, uint64_t x, int cnt, uint32_t (&row)[U],
@@ -321,9 +329,14 @@ struct HicooRowSrc {
 #pragma unroll
         for (int j = 0; j < NOA; ++j) {
           if (j < no) {
-            uint32_t e = ld_stream_u32(a.eo[j] + x + q, pol);
-            ej[j][q] = e & 0xff; ej[j][q + 1] = (e >> 8) & 0xff; ej[j][q + 2] = (e >> 16) & 0xff;
-            ej[j][q + 3] = e >> 24;
+            if ((wide >> j) & 1u) {
+              uint4 i4 = ld_stream_u4(a.io[j] + x + q, pol);
+              ej[j][q] = i4.x; ej[j][q + 1] = i4.y; ej[j][q + 2] = i4.z; ej[j][q + 3] = i4.w;
+            } else {
+              uint32_t e = ld_stream_u32(a.eo[j] + x + q, pol);
+              ej[j][q] = e & 0xff; ej[j][q + 1] = (e >> 8) & 0xff; ej[j][q + 2] = (e >> 16) & 0xff;
+              ej[j][q + 3] = e >> 24;
+            }
           }
         }
       }
@@ -334,7 +347,7 @@ struct HicooRowSrc {
           v[u] = __ldg(a.val + x + u);
 #pragma unroll
           for (int j = 0; j < NOA; ++j)
-            if (j < no) ej[j][u] = __ldg(a.eo[j] + x + u);
+            if (j < no) ej[j][u] = ((wide >> j) & 1u) ? __ldg(a.io[j] + x + u) : uint32_t(__ldg(a.eo[j] + x + u));
         }
       }
     }
@@ -1036,8 +1049,13 @@ void launch_hicoo_mttkrp(const pasta_hicoo *h, uint32_t mode, const float *const
     int j = 0;
     for (uint32_t k = 0; k < h->order; ++k) {
       if (k == mode) continue;
-      a.sbbase[j] = mc.sbbase[k].p;
-      a.eo[j] = mc.einds[k].p;
+      if ((h->cmask >> k) & 1u) {
+        a.sbbase[j] = mc.sbbase[k].p;
+        a.eo[j] = mc.einds[k].p;
+      } else {
+        a.io[j] = mc.uinds[k].p;
+        a.wide |= 1u << j;
+      }
       a.Uo[j] = factors[k];
       ++j;
     }

@@ -23,12 +23,16 @@ def main():
     ap.add_argument("--formats", default="coo")
     ap.add_argument("--reps", type=int, default=10)
     ap.add_argument("--caches", default="0")
+    ap.add_argument("--cmask", type=int, default=0, help="gHiCOO mask (0 = auto)")
     args = ap.parse_args()
     cfg = si.CONFIGS[args.config]
     dims, R, M = cfg["dims"], cfg["R"], cfg["nnz"]
     x = pasta.pasta_gen_powerlaw(dims, M, cfg["seed"], kind=0 if cfg["kind"] == "uniform" else 1)
     fmts = args.formats.split(",")
     h = pasta.pasta_coo_to_hicoo(x, 7) if "hicoo" in fmts else None
+    gh = pasta.pasta_coo_to_ghicoo(x, 7, args.cmask) if "ghicoo" in fmts else None
+    if gh is not None:
+        print(json.dumps({"ghicoo_cmask": gh.cmask, "ghicoo_nblocks": gh.nblocks}), flush=True)
     g = torch.Generator(device="cuda")
     g.manual_seed(1)
     U = [torch.rand((d, R), generator=g, device="cuda") for d in dims]
@@ -36,7 +40,8 @@ def main():
     if h is not None:
         print(json.dumps({"hicoo_nblocks": h.nblocks, "nnz": h.nnz}), flush=True)
     for fmt in fmts:
-        fn, t = (pasta.pasta_mttkrp_coo, x) if fmt == "coo" else (pasta.pasta_mttkrp_hicoo, h)
+        fn, t = {"coo": (pasta.pasta_mttkrp_coo, x), "hicoo": (pasta.pasta_mttkrp_hicoo, h),
+                 "ghicoo": (pasta.pasta_mttkrp_hicoo, gh)}[fmt]
         which = 0 if fmt == "coo" else 1
         for n in range(len(dims)):
             fn(t, n, U, out=outs[n])  # prepare
