@@ -76,6 +76,13 @@ def _L():
         lib.oracle_gen_slice_powerlaw.argtypes = [C.c_uint32, _u32p, C.c_uint64, C.c_uint64,
                                                   C.c_double, C.c_float, C.c_float,
                                                   C.POINTER(_u32p), _f32p]
+        lib.oracle_ts.restype = C.c_int
+        lib.oracle_ts.argtypes = [C.c_uint64, _f32p, C.c_uint32, C.c_float, _f32p]
+        lib.oracle_tew_same.restype = C.c_int
+        lib.oracle_tew_same.argtypes = [C.c_uint64, _f32p, _f32p, C.c_uint32, _f32p]
+        lib.oracle_tew_merge.restype = C.c_int64
+        lib.oracle_tew_merge.argtypes = [C.c_uint32, C.c_uint64, C.POINTER(_u32p), _f32p, C.c_uint64,
+                                         C.POINTER(_u32p), _f32p, C.c_uint32, C.POINTER(_u32p), _f32p]
         lib.oracle_ttm.restype = C.c_int64
         lib.oracle_ttm.argtypes = [C.c_uint32, _u32p, C.c_uint64, C.POINTER(_u32p), _f32p, C.c_uint32,
                                    _f32p, C.c_uint32, C.POINTER(_u32p), _f64p, _f64p]
@@ -334,3 +341,49 @@ def ttv(dims, inds, vals, mode, v):
     """O-TTV (Eq. 1): TTM with a single column u = v."""
     f, y, ya = ttm(dims, inds, vals, mode, np.asarray(v, np.float32).reshape(-1, 1))
     return f, y[:, 0].copy(), ya[:, 0].copy()
+
+
+OPS = {"add": 0, "sub": 1, "mul": 2, "div": 3}
+
+
+def ts(vals, op, s):
+    """O-TS: vals op s, each result rounded once to fp32."""
+    vals = np.ascontiguousarray(vals, dtype=np.float32)
+    out = np.empty_like(vals)
+    if _L().oracle_ts(vals.shape[0], _ptr(vals, _f32p), OPS[op], float(s), _ptr(out, _f32p)) != 0:
+        raise ValueError("oracle_ts: invalid arguments")
+    return out
+
+
+def tew_same(a, b, op):
+    """O-TEW for identical patterns: a op b element by element."""
+    a = np.ascontiguousarray(a, dtype=np.float32)
+    b = np.ascontiguousarray(b, dtype=np.float32)
+    assert a.shape == b.shape
+    out = np.empty_like(a)
+    if _L().oracle_tew_same(a.shape[0], _ptr(a, _f32p), _ptr(b, _f32p), OPS[op], _ptr(out, _f32p)) != 0:
+        raise ValueError("oracle_tew_same: invalid arguments")
+    return out
+
+
+def tew_merge(ix, vx, iy, vy, op):
+    """O-TEW for different patterns (R#31): union (add/sub) or intersection (mul/div),
+    lexicographic output.  Returns (inds u32[N][nz], vals f32[nz])."""
+    ix = np.ascontiguousarray(ix, dtype=np.uint32)
+    iy = np.ascontiguousarray(iy, dtype=np.uint32)
+    vx = np.ascontiguousarray(vx, dtype=np.float32)
+    vy = np.ascontiguousarray(vy, dtype=np.float32)
+    order = ix.shape[0]
+    T = vx.shape[0] + vy.shape[0]
+    rx = [np.ascontiguousarray(ix[k]) for k in range(order)]
+    ry = [np.ascontiguousarray(iy[k]) for k in range(order)]
+    outs = [np.zeros(max(T, 1), np.uint32) for _ in range(order)]
+    ov = np.zeros(max(T, 1), np.float32)
+    nz = _L().oracle_tew_merge(order, vx.shape[0], _ptr_list(rx, _u32p), _ptr(vx, _f32p), vy.shape[0],
+                               _ptr_list(ry, _u32p), _ptr(vy, _f32p), OPS[op],
+                               _ptr_list(outs, _u32p), _ptr(ov, _f32p))
+    if nz == -4:
+        raise ValueError("oracle_tew_merge: repeated coordinate inside one input")
+    if nz < 0:
+        raise ValueError("oracle_tew_merge: invalid arguments")
+    return np.stack([o[:nz] for o in outs]), ov[:nz].copy()

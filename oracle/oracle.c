@@ -625,3 +625,91 @@ int oracle_mttkrp_ghicoo(uint32_t order, const uint32_t *dims, uint32_t block_bi
     }
     return 0;
 }
+
+/* ------------------------------------------------------------------------- */
+/* O-TS / O-TEW.  The paper fixes single precision   */
+/* (P:109): each result is the fp64 operation rounded once to fp32, which    */
+/* equals the correctly rounded fp32 operation (53 >= 2*24 + 2).             */
+/*   op: 0 add, 1 sub, 2 mul, 3 div.                                          */
+/* ------------------------------------------------------------------------- */
+static float ew_apply(uint32_t op, float a, float b)
+{
+    double x = (double)a, y = (double)b, z;
+    if (op == 0) z = x + y;
+    else if (op == 1) z = x - y;
+    else if (op == 2) z = x * y;
+    else z = x / y;
+    return (float)z;
+}
+
+/* TS: out[i] = vals[i] op s. */
+int oracle_ts(uint64_t n, const float *vals, uint32_t op, float s, float *out)
+{
+    if (op > 3) return -1;
+    for (uint64_t i = 0; i < n; ++i) out[i] = ew_apply(op, vals[i], s);
+    return 0;
+}
+
+/* TEW with identical non-zero patterns: out[i] = a[i] op b[i]. */
+int oracle_tew_same(uint64_t n, const float *a, const float *b, uint32_t op, float *out)
+{
+    if (op > 3) return -1;
+    for (uint64_t i = 0; i < n; ++i) out[i] = ew_apply(op, a[i], b[i]);
+    return 0;
+}
+
+/* TEW with different patterns (R#31): Z(c) = X(c) op Y(c) over the union of  */
+/* the patterns for add/sub (a missing operand: z = x, or z = 0 - y) and over their */
+/* intersection for mul/div; output in lexicographic order.  Entries of X and Y are */
+/* merged by sorting (coords, source); a coordinate repeated inside one input is an */
+/* error (-4).  Returns the output nnz (capacity Mx + My), or < 0.                  */
+typedef struct { uint32_t c[ORACLE_MAX_ORDER]; int src; float v; } ew_rec;
+static uint32_t g_ew_order;
+static int cmp_ew(const void *pa, const void *pb)
+{
+    const ew_rec *a = (const ew_rec *)pa, *b = (const ew_rec *)pb;
+    for (uint32_t k = 0; k < g_ew_order; ++k)
+        if (a->c[k] != b->c[k]) return a->c[k] < b->c[k] ? -1 : 1;
+    return a->src - b->src;
+}
+
+int64_t oracle_tew_merge(uint32_t order, uint64_t Mx, const uint32_t *const *ix, const float *vx,
+                         uint64_t My, const uint32_t *const *iy, const float *vy, uint32_t op,
+                         uint32_t *const *out_inds, float *out_vals)
+{
+    if (order < 1 || order > ORACLE_MAX_ORDER || op > 3) return -1;
+    uint64_t T = Mx + My;
+    ew_rec *r = (ew_rec *)malloc((T ? T : 1) * sizeof(ew_rec));
+    if (!r) return -2;
+    for (uint64_t i = 0; i < T; ++i) {
+        memset(&r[i], 0, sizeof(ew_rec));
+        for (uint32_t k = 0; k < order; ++k) r[i].c[k] = i < Mx ? ix[k][i] : iy[k][i - Mx];
+        r[i].src = i < Mx ? 0 : 1;
+        r[i].v = i < Mx ? vx[i] : vy[i - Mx];
+    }
+    g_ew_order = order;
+    qsort(r, T, sizeof(ew_rec), cmp_ew);
+    int64_t nz = 0;
+    uint64_t i = 0;
+    while (i < T) {
+        uint64_t j = i + 1;
+        while (j < T && memcmp(r[i].c, r[j].c, sizeof(r[i].c)) == 0) ++j; /* same coordinate */
+        if (j - i > 2 || (j - i == 2 && r[i].src == r[i + 1].src)) { free(r); return -4; }
+        int hx = r[i].src == 0 || (j - i == 2);
+        int hy = r[j - 1].src == 1;
+        float xv = r[i].src == 0 ? r[i].v : 0.0f, yv = r[j - 1].src == 1 ? r[j - 1].v : 0.0f;
+        int keep = (op <= 1) ? 1 : (hx && hy);
+        if (keep) {
+            float z;
+            if (hx && hy) z = ew_apply(op, xv, yv);
+            else if (hx) z = xv;
+            else z = (op == 1) ? ew_apply(1, 0.0f, yv) : yv;
+            for (uint32_t k = 0; k < order; ++k) out_inds[k][nz] = r[i].c[k];
+            out_vals[nz] = z;
+            ++nz;
+        }
+        i = j;
+    }
+    free(r);
+    return nz;
+}
