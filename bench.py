@@ -202,6 +202,7 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=10)
     ap.add_argument("--hicoo-steps", type=int, default=20)
     ap.add_argument("--cpals-iters", type=int, default=5)
+    ap.add_argument("--ew-steps", type=int, default=20)
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3  # timing rule: >= 3 warm-up steps
@@ -459,6 +460,37 @@ def main():
                          "per-sweep fit read-back"}
         del Uc
 
+    # NEXT-4: TS and same-pattern TEW on the tensor's value array (Table I: TS 8M bytes, TEW
+    # 12M bytes, M flops) -- the streaming kernels that bound the HBM roofline
+    ew = None
+    if world == 1 and args.ew_steps > 0:
+        vals = torch.empty(M, dtype=torch.float32, device=dev)
+        vals.uniform_(-1.0, 1.0)
+        other = torch.empty_like(vals)
+        dst = torch.empty_like(vals)
+        peak_e, _ = load_peaks()
+        ew = {}
+        for name, fn, nbytes in (
+                ("ts_mul", lambda: pasta.pasta_ts(vals, "mul", 0.5, out=dst), 8 * M),
+                ("tew_add", lambda: pasta.pasta_tew(vals, other, "add", out=dst), 12 * M)):
+            for _ in range(3):
+                fn()
+            torch.cuda.synchronize()
+            pasta.pasta_profile_read(3, reset=True)
+            pasta.pasta_profile_enable(True)
+            for _ in range(args.ew_steps):
+                fn()
+            torch.cuda.synchronize()
+            pasta.pasta_profile_enable(False)
+            e_ms, e_n = pasta.pasta_profile_read(3, reset=True)
+            avg = e_ms / max(e_n, 1)
+            gbs = nbytes / (avg * 1e-3) / 1e9
+            ew[name] = {"ms": round(avg, 4), "GFLOP/s": round(M / (avg * 1e-3) / 1e9, 1),
+                        "roofline": {"bound": "hbm", "achieved": round(gbs, 1), "peak": peak_e,
+                                     "unit": "GB/s", "frac": round(gbs / peak_e, 4),
+                                     "bytes_model": "TS 8M / TEW 12M per launch (Table I, P:117)"}}
+        del vals, other, dst
+
     if rank != 0:
         if world > 1:
             dist.destroy_process_group()
@@ -512,6 +544,7 @@ def main():
         "hicoo": hicoo,
         "ghicoo": ghicoo,
         "cpals": cpals,
+        "ew": ew,
         "gpu_launches": launches,
         "cpu_baseline": cpu,
         "max_shard_nnz": per_launch_nnz,

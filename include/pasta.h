@@ -88,12 +88,13 @@ pasta_status pasta_coo_from_arrays(uint32_t order, const uint32_t *dims, uint64_
 /* Synthetic tensor generator parameters (R#19-R#23). */
 typedef struct {
     uint32_t kind;            /* 0 uniform (q = 0.5), 1 Stochastic Kronecker (default),
-                                 2 FireHose slice power law (not implemented: EUNSUPPORTED) */
+                                 2 FireHose-style slice power law (R#30)                     */
     const double *initiator;  /* 2^order non-negative cell weights, cell c sets bit k of mode
                                  k's index to (c >> k) & 1; NULL -> product form from q     */
     double q;                 /* product-form P(bit = 0) per mode per level; 0 -> 0.75      */
     uint32_t permute;         /* must be 0 (random relabelling: EUNSUPPORTED)                */
     float val_lo, val_hi;     /* values uniform in [val_lo, val_hi); both 0 -> [-1, 1)       */
+    double alpha;             /* kind 2: power-law exponent in (0, 8]; 0 -> 1.0              */
 } pasta_gen_params;
 
 /* Stochastic Kronecker tensor by ball dropping (R#20-R#21): draw d chooses, at each
@@ -103,8 +104,18 @@ typedef struct {
  * of i_k; draws with any i_k >= I_k are stripped.  The tensor is the first `nnz` distinct
  * coordinates in draw order, each with value lo + (hi - lo) * u(d_first, 0xFFFF) (fp64,
  * rounded to fp32), stored in lexicographic (i_0, ..., i_{N-1}) order.  Runs on the GPU.
- * Errors: EINVAL (order, dims, nnz > prod dims, bad initiator), ERANGE (more than 2^32-2
- * draws would be needed), EUNSUPPORTED (kind 2, permute). */
+ *
+ * kind 2 -- slice power law, the FireHose-style generator of the irregular tensors (P:225,
+ * P:229, Table II s4-s6/s10-s15; R#30): "combines graphs together to form
+ * slices ... repeated on an (N-1)th-order tensor"; every mode index is drawn independently
+ * from P(i) ~ (i+1)^-alpha, i < I_k, so each slice is a power-law graph without clustering
+ * (P:229).  Table: w_i = pow(i + 1, -alpha), cum_i = running fp64 sum over ascending i
+ * (computed on the host).  Draw d, mode k: u = u(d, k) * cum_{I_k - 1} (fp64 product);
+ * i_k = the first i with u < cum_i, else I_k - 1.  No draw is stripped; the tensor is the
+ * first `nnz` distinct coordinates in draw order with the values of kind 1, lexicographic.
+ * dims <= 2^27 per mode (ERANGE otherwise).
+ * Errors: EINVAL (order, dims, nnz > prod dims, bad initiator, alpha), ERANGE (more than
+ * 2^32-2 draws would be needed), EUNSUPPORTED (permute). */
 pasta_status pasta_gen_powerlaw(uint32_t order, const uint32_t *dims, uint64_t nnz,
                                 uint64_t seed, const pasta_gen_params *params,
                                 pasta_coo **out);
@@ -240,6 +251,33 @@ pasta_status pasta_ttm_coo(pasta_coo *x, uint32_t mode, const float *U, uint32_t
 /* out (DEVICE [M_F]) = X x_mode v with v DEVICE [dims[mode]] (TTM with R = 1). */
 pasta_status pasta_ttv_coo(pasta_coo *x, uint32_t mode, const float *v, float *out, void *stream);
 
+/* ------------------------------------------------------- TEW / TS ---- */
+
+/* Element-wise operators: z = x op y. */
+enum { PASTA_OP_ADD = 0, PASTA_OP_SUB = 1, PASTA_OP_MUL = 2, PASTA_OP_DIV = 3 };
+
+/* Tensor-scalar (TS) on a value array: out[i] = vals[i] op s, i < n, IEEE fp32
+ * (correctly rounded, division included).  DEVICE arrays (out may equal vals).  Async on
+ * `stream`.  Table I: M flops, 8M bytes. */
+pasta_status pasta_ts(const float *vals, uint64_t n, uint32_t op, float s, float *out, void *stream);
+/* Tensor element-wise (TEW) of two tensors with the same non-zero pattern, on their
+ * value arrays: out[i] = a[i] op b[i].  DEVICE arrays.  Table I: M flops, 12M bytes. */
+pasta_status pasta_tew(const float *a, const float *b, uint64_t n, uint32_t op, float *out,
+                       void *stream);
+/* Device pointer to the canonical value array of `x` (library-owned, valid until free). */
+pasta_status pasta_coo_values(const pasta_coo *x, float **vals);
+/* Y = X op s (TS) as a new tensor: the output indices are copied in pre-processing (the
+ * output pattern is the input's), then the values come from pasta_ts. */
+pasta_status pasta_coo_ts(const pasta_coo *x, uint32_t op, float s, pasta_coo **out);
+/* Z = X op Y (TEW) for tensors of the same order and shape.  Same pattern (same
+ * canonical index arrays, checked on the GPU): Z has X's pattern and z_i = x_i op y_i.
+ * Different patterns (R#31): the output pattern is predicted from a merge of both mode-0
+ * lexicographic index lists -- the union for add/sub (a missing operand contributes
+ * nothing: z = x, or z = 0 - y), the intersection for mul/div -- and Z is stored in
+ * lexicographic order.  Errors: EINVAL (order/shape mismatch, a repeated coordinate inside
+ * one input in the merge case), ERANGE (more than 2^32-2 merged entries). */
+pasta_status pasta_coo_tew(pasta_coo *x, pasta_coo *y, uint32_t op, pasta_coo **out);
+
 /* ------------------------------------------------------------ introspection ---------- */
 
 pasta_status pasta_coo_info(const pasta_coo *x, uint32_t *order, uint32_t *dims,
@@ -273,7 +311,7 @@ uint64_t pasta_launch_count(void);
 /* When enabled, every MTTKRP main-kernel launch is bracketed by CUDA events recorded on
  * its own stream.  pasta_profile_read synchronises those events and returns the summed
  * device time (ms) and the launch count of kernel family `which` (0 = COO MTTKRP,
- * 1 = HiCOO MTTKRP, 2 = output zero-fill), then clears the record if `reset`. */
+ * 1 = HiCOO MTTKRP, 2 = output zero-fill, 3 = TEW/TS), then clears the record if `reset`. */
 pasta_status pasta_profile_enable(int on);
 pasta_status pasta_profile_read(uint32_t which, double *total_ms, uint64_t *launches,
                                 int reset);

@@ -25,7 +25,8 @@ __all__ = [
     "pasta_launch_count", "pasta_profile_enable", "pasta_profile_read", "pasta_gram",
     "pasta_cpals_solve", "pasta_normalize_columns", "pasta_weighted_inner", "pasta_coo_norm2",
     "pasta_cpals_coo", "pasta_coo_fibers", "pasta_coo_fiber_export", "pasta_ttm_coo",
-    "pasta_ttv_coo",
+    "pasta_ttv_coo", "pasta_coo_to_ghicoo", "pasta_ghicoo_auto_mask", "pasta_ghicoo_export",
+    "pasta_ts", "pasta_tew", "pasta_coo_values_ptr", "pasta_coo_ts", "pasta_coo_tew", "OPS",
 ]
 
 _u32p = C.POINTER(C.c_uint32)
@@ -171,11 +172,13 @@ def pasta_coo_from_arrays(dims: Sequence[int], inds: np.ndarray, vals: np.ndarra
 
 def pasta_gen_powerlaw(dims: Sequence[int], nnz: int, seed: int, kind: int = 1,
                        initiator: Optional[Sequence[float]] = None, q: float = 0.0,
-                       val_lo: float = -1.0, val_hi: float = 1.0, permute: int = 0) -> Coo:
-    """Stochastic Kronecker tensor on the GPU; see include/pasta.h."""
+                       val_lo: float = -1.0, val_hi: float = 1.0, permute: int = 0,
+                       alpha: float = 0.0) -> Coo:
+    """Synthetic tensor on the GPU: kind 1 Stochastic Kronecker, kind 0 uniform,
+    kind 2 slice power law with exponent ``alpha``; see include/pasta.h."""
     dims_a = np.ascontiguousarray(dims, dtype=np.uint32)
     p = GenParams()
-    p.kind, p.q, p.permute, p.val_lo, p.val_hi = kind, q, permute, val_lo, val_hi
+    p.kind, p.q, p.permute, p.val_lo, p.val_hi, p.alpha = kind, q, permute, val_lo, val_hi, alpha
     keep = None
     if initiator is not None:
         keep = np.ascontiguousarray(initiator, dtype=np.float64)
@@ -522,3 +525,63 @@ def pasta_ttv_coo(x: Coo, mode: int, v, out=None, stream=None):
     check(lib().pasta_ttv_coo(x.ptr, mode, C.c_void_p(v.data_ptr()), C.c_void_p(out.data_ptr()),
                               _stream_ptr(stream)))
     return out
+
+
+# ----------------------------------------------------------------------------- TEW / TS
+OPS = {"add": 0, "sub": 1, "mul": 2, "div": 3}
+
+
+def _op(op):
+    return OPS[op] if isinstance(op, str) else int(op)
+
+
+def _f32_cuda(t, name):
+    import torch
+    if not (isinstance(t, torch.Tensor) and t.is_cuda and t.dtype == torch.float32 and t.is_contiguous()):
+        raise PastaError(-1, f"{name} must be a contiguous float32 CUDA tensor")
+
+
+def pasta_ts(vals, op, s: float, out=None, stream=None):
+    """TS on a value tensor: out = vals op s (IEEE fp32)."""
+    import torch
+    _f32_cuda(vals, "vals")
+    if out is None:
+        out = torch.empty_like(vals)
+    _f32_cuda(out, "out")
+    check(lib().pasta_ts(C.c_void_p(vals.data_ptr()), vals.numel(), _op(op), float(s),
+                         C.c_void_p(out.data_ptr()), _stream_ptr(stream)))
+    return out
+
+
+def pasta_tew(a, b, op, out=None, stream=None):
+    """Same-pattern TEW on value tensors: out = a op b."""
+    import torch
+    _f32_cuda(a, "a")
+    _f32_cuda(b, "b")
+    if a.numel() != b.numel():
+        raise PastaError(-1, "a and b differ in length")
+    if out is None:
+        out = torch.empty_like(a)
+    _f32_cuda(out, "out")
+    check(lib().pasta_tew(C.c_void_p(a.data_ptr()), C.c_void_p(b.data_ptr()), a.numel(), _op(op),
+                          C.c_void_p(out.data_ptr()), _stream_ptr(stream)))
+    return out
+
+
+def pasta_coo_values_ptr(x: Coo) -> int:
+    """Device address of x's canonical value array (library-owned)."""
+    p = C.c_void_p()
+    check(lib().pasta_coo_values(x.ptr, C.byref(p)))
+    return p.value or 0
+
+
+def pasta_coo_ts(x: Coo, op, s: float) -> Coo:
+    out = C.c_void_p()
+    check(lib().pasta_coo_ts(x.ptr, _op(op), float(s), C.byref(out)))
+    return Coo(out.value)
+
+
+def pasta_coo_tew(x: Coo, y: Coo, op) -> Coo:
+    out = C.c_void_p()
+    check(lib().pasta_coo_tew(x.ptr, y.ptr, _op(op), C.byref(out)))
+    return Coo(out.value)

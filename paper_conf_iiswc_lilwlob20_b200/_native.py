@@ -26,7 +26,8 @@ class PastaError(RuntimeError):
 
 class GenParams(C.Structure):
     _fields_ = [("kind", C.c_uint32), ("initiator", C.POINTER(C.c_double)), ("q", C.c_double),
-                ("permute", C.c_uint32), ("val_lo", C.c_float), ("val_hi", C.c_float)]
+                ("permute", C.c_uint32), ("val_lo", C.c_float), ("val_hi", C.c_float),
+                ("alpha", C.c_double)]
 
 
 ALLOC_FN = C.CFUNCTYPE(C.c_void_p, C.c_size_t, C.c_void_p, C.c_void_p)
@@ -69,6 +70,11 @@ SIGNATURES = {
     "pasta_row_partition": (_st, [C.c_uint32, _u64p, C.c_uint32, _u32p]),
     "pasta_coo_partition": (_st, [_vp, C.c_uint32, C.c_uint32, _u32p]),
     "pasta_coo_shard": (_st, [_vp, C.c_uint32, C.c_uint32, C.c_uint32, C.POINTER(_vp)]),
+    "pasta_ts": (_st, [_vp, C.c_uint64, C.c_uint32, C.c_float, _vp, _vp]),
+    "pasta_tew": (_st, [_vp, _vp, C.c_uint64, C.c_uint32, _vp, _vp]),
+    "pasta_coo_values": (_st, [_vp, C.POINTER(_vp)]),
+    "pasta_coo_ts": (_st, [_vp, C.c_uint32, C.c_float, C.POINTER(_vp)]),
+    "pasta_coo_tew": (_st, [_vp, _vp, C.c_uint32, C.POINTER(_vp)]),
     "pasta_coo_info": (_st, [_vp, _u32p, _u32p, _u64p]),
     "pasta_coo_export": (_st, [_vp, C.POINTER(_u32p), _f32p]),
     "pasta_coo_export_mode": (_st, [_vp, C.c_uint32, C.POINTER(_u32p), _f32p]),

@@ -343,15 +343,32 @@ pasta_status pasta_gen_powerlaw(uint32_t order, const uint32_t *dims, uint64_t n
   require(out != nullptr, "out is NULL");
   *out = nullptr;
   validate_dims(order, dims);
-  pasta_gen_params p{1, nullptr, 0.0, 0, 0.f, 0.f};
+  pasta_gen_params p{1, nullptr, 0.0, 0, 0.f, 0.f, 0.0};
   if (params) p = *params;
-  if (p.kind == 2) fail(PASTA_EUNSUPPORTED, "FireHose slice power-law generator (kind 2) is not implemented");
-  require(p.kind <= 1, "unknown generator kind");
+  require(p.kind <= 2, "unknown generator kind");
   if (p.permute) fail(PASTA_EUNSUPPORTED, "label permutation is not implemented");
   double cells = 1.0;
   for (uint32_t k = 0; k < order; ++k) cells *= double(dims[k]);
   require(double(nnz) <= cells, "nnz exceeds the number of cells");
   if (nnz > 0xFFFFFFFEull) fail(PASTA_ERANGE, "more than 2^32-2 nonzeros");
+  if (p.kind == 2) {
+    const double alpha = p.alpha == 0.0 ? 1.0 : p.alpha;
+    require(alpha > 0.0 && alpha <= 8.0, "alpha must be in (0, 8] (0 selects the default 1.0)");
+    for (uint32_t k = 0; k < order; ++k)
+      if (dims[k] > (1u << 27)) fail(PASTA_ERANGE, "slice power law: dims above 2^27 (weight table)");
+    float lo = p.val_lo, hi = p.val_hi;
+    if (lo == 0.f && hi == 0.f) { lo = -1.f; hi = 1.f; }
+    require(lo < hi, "val_lo must be < val_hi");
+    auto x = std::make_unique<pasta_coo>();
+    x->order = order;
+    for (uint32_t k = 0; k < order; ++k) x->dims[k] = dims[k];
+    x->nnz = nnz;
+    x->device = current_device();
+    gen_powerlaw_device(x.get(), seed, nullptr, 0, lo, hi, nullptr, alpha);
+    x->lex_sorted = true;
+    *out = x.release();
+    return PASTA_OK;
+  }
   const uint32_t ncell = 1u << order;
   double table[1 << kMaxOrder];
   if (p.kind == 0) {
@@ -865,6 +882,73 @@ pasta_status pasta_ttv_coo(pasta_coo *x, uint32_t mode, const float *v, float *o
 }
 
 // ---------------------------------------------------------------------------- introspection
+// ---------------------------------------------------------------------------- TEW / TS
+pasta_status pasta_ts(const float *vals, uint64_t n, uint32_t op, float s, float *out, void *stream) {
+  API_BEGIN
+  require(op <= PASTA_OP_DIV, "op must be PASTA_OP_ADD/SUB/MUL/DIV");
+  require(n == 0 || (vals && out), "vals/out is NULL");
+  launch_ts(op, vals, s, out, n, as_stream(stream));
+  API_END
+}
+
+pasta_status pasta_tew(const float *a, const float *b, uint64_t n, uint32_t op, float *out, void *stream) {
+  API_BEGIN
+  require(op <= PASTA_OP_DIV, "op must be PASTA_OP_ADD/SUB/MUL/DIV");
+  require(n == 0 || (a && b && out), "a/b/out is NULL");
+  launch_tew(op, a, b, out, n, as_stream(stream));
+  API_END
+}
+
+pasta_status pasta_coo_values(const pasta_coo *x, float **vals) {
+  API_BEGIN
+  require(x && vals, "x/vals is NULL");
+  *vals = x->val.p;
+  API_END
+}
+
+pasta_status pasta_coo_ts(const pasta_coo *x, uint32_t op, float s, pasta_coo **out) {
+  API_BEGIN
+  require(x && out, "x/out is NULL");
+  *out = nullptr;
+  require(op <= PASTA_OP_DIV, "op must be PASTA_OP_ADD/SUB/MUL/DIV");
+  check_device(x->device);
+  auto y = std::make_unique<pasta_coo>();
+  copy_pattern_device(x, y.get(), nullptr);  // pre-processing: output indices
+  launch_ts(op, x->val.p, s, y->val.p, x->nnz, nullptr);
+  PASTA_CUDA(cudaStreamSynchronize(nullptr));
+  *out = y.release();
+  API_END
+}
+
+pasta_status pasta_coo_tew(pasta_coo *x, pasta_coo *y, uint32_t op, pasta_coo **out) {
+  API_BEGIN
+  require(x && y && out, "x/y/out is NULL");
+  *out = nullptr;
+  require(op <= PASTA_OP_DIV, "op must be PASTA_OP_ADD/SUB/MUL/DIV");
+  require(x->order == y->order, "tew: tensors of different orders");
+  for (uint32_t k = 0; k < x->order; ++k) require(x->dims[k] == y->dims[k], "tew: tensors of different shapes");
+  check_device(x->device);
+  check_device(y->device);
+  auto z = std::make_unique<pasta_coo>();
+  if (same_pattern_device(x, y, nullptr)) {
+    copy_pattern_device(x, z.get(), nullptr);
+    launch_tew(op, x->val.p, y->val.p, z->val.p, x->nnz, nullptr);
+    PASTA_CUDA(cudaStreamSynchronize(nullptr));
+  } else {
+    {
+      std::lock_guard<std::mutex> lk(x->mu);
+      coo_prepare_mode(x, 0, nullptr);
+    }
+    if (y != x) {
+      std::lock_guard<std::mutex> lk(y->mu);
+      coo_prepare_mode(y, 0, nullptr);
+    }
+    tew_merge_device(x, y, op, z.get(), nullptr);
+  }
+  *out = z.release();
+  API_END
+}
+
 pasta_status pasta_coo_info(const pasta_coo *x, uint32_t *order, uint32_t *dims, uint64_t *nnz) {
   API_BEGIN
   require(x != nullptr, "x is NULL");
@@ -979,7 +1063,7 @@ pasta_status pasta_profile_enable(int on) {
 
 pasta_status pasta_profile_read(uint32_t which, double *total_ms, uint64_t *launches, int reset) {
   API_BEGIN
-  require(which < kProfKinds, "which must be 0 (COO), 1 (HiCOO) or 2 (zero-fill)");
+  require(which < kProfKinds, "which must be 0 (COO), 1 (HiCOO), 2 (zero-fill) or 3 (TEW/TS)");
   std::lock_guard<std::mutex> lk(g_prof_mu);
   double sum = 0.0;
   for (auto &r : g_prof[which]) {

@@ -2,6 +2,9 @@
 // (R#19-R#23).  Counter-based: draw d's randomness is a pure function of
 // (seed, d, level), so the result is independent of launch geometry and identical to any
 // other implementation of the same recipe (include/pasta.h documents it).
+#include <cmath>
+#include <vector>
+
 #include "internal.cuh"
 
 namespace pasta {
@@ -14,6 +17,9 @@ constexpr uint64_t kValueStream = 0xFFFF;
 __constant__ double c_cum[1 << kMaxOrder];
 
 struct GenArgs {
+  uint32_t kind;  // 1: Kronecker ball dropping (also kind 0 = uniform table), 2: slice power law
+  // kind 2 (R#30): per-mode cumulative weight tables (device) and their totals
+  const double *cumk[kMaxOrder];
   uint32_t order;
   uint32_t ncell;
   uint32_t last_pos;  // last cell with positive weight (rounding fallback)
@@ -39,6 +45,21 @@ __device__ inline double uniform01(uint64_t key, uint64_t d, uint64_t s) {
 }
 
 __device__ inline bool draw_coords(const GenArgs &a, uint64_t d, uint32_t *c) {
+  if (a.kind == 2) {
+    // slice power law (R#30): i_k = first i with u(d, k) * cum_k[I_k - 1] < cum_k[i]
+    for (uint32_t k = 0; k < a.order; ++k) {
+      const double *cum = a.cumk[k];
+      const uint32_t I = a.dims[k];
+      const double u = __dmul_rn(uniform01(a.key, d, k), cum[I - 1]);
+      uint32_t lo = 0, hi = I;
+      while (lo < hi) {
+        const uint32_t mid = lo + (hi - lo) / 2;
+        if (u < cum[mid]) hi = mid; else lo = mid + 1;
+      }
+      c[k] = lo < I ? lo : I - 1;
+    }
+    return true;
+  }
   for (uint32_t k = 0; k < a.order; ++k) c[k] = 0;
   for (uint32_t l = 0; l < a.Lmax; ++l) {
     double u = __dmul_rn(uniform01(a.key, d, l), a.total);
@@ -132,13 +153,32 @@ inline unsigned grid_for(uint64_t n) {
 
 // x->order, x->dims, x->nnz are set by the caller; fills x->inds / x->val.
 void gen_powerlaw_device(pasta_coo *x, uint64_t seed, const double *table, uint32_t ncell,
-                         float val_lo, float val_hi, cudaStream_t s) {
+                         float val_lo, float val_hi, cudaStream_t s, double alpha) {
   const uint32_t N = x->order;
   const uint64_t M = x->nnz;
   GenArgs a{};
   a.order = N;
+  a.kind = ncell == 0 ? 2 : 1;
+  DevArray<double> cumk[kMaxOrder];
+  if (a.kind == 2) {
+    // weights w_i = (i + 1)^-alpha, running fp64 sums in ascending i, computed on the host so
+    // that every implementation of the recipe reproduces the same table (include/pasta.h)
+    std::vector<double> h;
+    for (uint32_t k = 0; k < N; ++k) {
+      h.resize(x->dims[k]);
+      double run = 0.0;
+      for (uint32_t i = 0; i < x->dims[k]; ++i) {
+        run = run + std::pow(double(i) + 1.0, -alpha);
+        h[i] = run;
+      }
+      cumk[k].alloc(x->dims[k], s);
+      PASTA_CUDA(cudaMemcpyAsync(cumk[k].p, h.data(), sizeof(double) * x->dims[k], cudaMemcpyHostToDevice, s));
+      PASTA_CUDA(cudaStreamSynchronize(s));
+      a.cumk[k] = cumk[k].p;
+    }
+  }
   a.ncell = ncell;
-  double cum[1 << kMaxOrder];
+  double cum[1 << kMaxOrder] = {};
   double run = 0.0;
   for (uint32_t c = 0; c < ncell; ++c) {
     run = run + table[c];
@@ -146,7 +186,7 @@ void gen_powerlaw_device(pasta_coo *x, uint64_t seed, const double *table, uint3
     if (table[c] > 0.0) a.last_pos = c;
   }
   a.total = run;
-  PASTA_CUDA(cudaMemcpyToSymbolAsync(c_cum, cum, sizeof(double) * ncell, 0, cudaMemcpyHostToDevice, s));
+  if (ncell) PASTA_CUDA(cudaMemcpyToSymbolAsync(c_cum, cum, sizeof(double) * ncell, 0, cudaMemcpyHostToDevice, s));
   for (uint32_t k = 0; k < N; ++k) {
     a.dims[k] = x->dims[k];
     a.L[k] = ceil_log2(x->dims[k]);

@@ -239,8 +239,9 @@ uint64_t select_flagged(const uint8_t *flags, uint64_t M, DevArray<uint32_t> &id
 // ------------------------------------------------------------------------- operations
 void coo_prepare_mode(pasta_coo *x, uint32_t mode, cudaStream_t s);
 void hicoo_prepare_mode(pasta_hicoo *h, uint32_t mode, cudaStream_t s);
+// ncell = 0 selects the slice power-law generator (kind 2, exponent alpha; R#30)
 void gen_powerlaw_device(pasta_coo *x, uint64_t seed, const double *table, uint32_t ncell,
-                         float val_lo, float val_hi, cudaStream_t s);
+                         float val_lo, float val_hi, cudaStream_t s, double alpha = 1.0);
 void coo_to_hicoo_device(const pasta_coo *x, pasta_hicoo *h, cudaStream_t s);  // honours h->cmask
 // number of distinct block keys (i_k >> block_bits, k in cmask) of a COO tensor
 uint64_t count_blocks_device(const pasta_coo *x, uint32_t block_bits, uint32_t cmask, cudaStream_t s);
@@ -268,8 +269,15 @@ void row_counts_device(const uint32_t *rows, uint64_t nnz, uint32_t nrows, uint6
 uint64_t lower_bound_device(const uint32_t *a, uint64_t M, uint32_t v, cudaStream_t s);
 bool is_lex_sorted_device(const uint32_t *const *inds, uint32_t order, uint64_t M, cudaStream_t s);
 
+// TEW / TS (tew.cu)
+void launch_ts(uint32_t op, const float *x, float s, float *y, uint64_t n, cudaStream_t st);
+void launch_tew(uint32_t op, const float *a, const float *b, float *z, uint64_t n, cudaStream_t st);
+bool same_pattern_device(const pasta_coo *x, const pasta_coo *y, cudaStream_t s);
+void copy_pattern_device(const pasta_coo *x, pasta_coo *y, cudaStream_t s);
+void tew_merge_device(const pasta_coo *x, const pasta_coo *y, uint32_t op, pasta_coo *z, cudaStream_t s);
+
 // ------------------------------------------------------------------------- profiling
-enum ProfKind { kProfCoo = 0, kProfHicoo = 1, kProfZero = 2, kProfKinds = 3 };
+enum ProfKind { kProfCoo = 0, kProfHicoo = 1, kProfZero = 2, kProfEw = 3, kProfKinds = 4 };
 struct ProfScope {
   cudaEvent_t a = nullptr, b = nullptr;
   int kind;

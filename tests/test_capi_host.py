@@ -54,8 +54,14 @@ def test_validation_happens_before_side_effects(pasta, tmp_path):
                                 np.ones(2, np.float32))
     assert e.value.code == -4 and "dims[0]" in str(e.value)
     with pytest.raises(P.PastaError) as e:
-        P.pasta_gen_powerlaw([10, 10], 5, seed=1, kind=2)
-    assert e.value.code == -7
+        P.pasta_gen_powerlaw([10, 10], 5, seed=1, kind=2, alpha=9.0)
+    assert e.value.code == -1
+    with pytest.raises(P.PastaError) as e:
+        P.pasta_gen_powerlaw([10, 10], 5, seed=1, kind=3)
+    assert e.value.code == -1
+    with pytest.raises(P.PastaError) as e:
+        P.pasta_gen_powerlaw([10, (1 << 27) + 1], 5, seed=1, kind=2)
+    assert e.value.code == -4
     with pytest.raises(P.PastaError) as e:
         P.pasta_gen_powerlaw([2, 2], 5, seed=1)
     assert e.value.code == -1
