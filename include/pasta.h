@@ -218,6 +218,39 @@ pasta_status pasta_gram(const float *U, uint64_t rows, uint32_t R, double *G, vo
  * pivot Gauss-Jordan, tiny ridge if singular); colsq[r] += sum_i U(i, r)^2 (fp64). */
 pasta_status pasta_cpals_solve(const float *M, uint64_t rows, uint32_t R, const double *const *grams,
                                uint32_t ngrams, float *U, double *colsq, void *stream);
+/* Fused CP-ALS update algebra (one CTA, fp64): from GM = M^T M (R x R, e.g. pasta_gram of the
+ * MTTKRP output, all-reduced across row shards) and the other modes' grams G_k:
+ *   W = (Hadamard_k G_k)^{-1};  GU = W^T GM W (= U^T U for U = M W);
+ *   lambda_r = sqrt(GU_rr) (1 if GU_rr <= 0);  Wn = W diag(1/lambda) (fp32, row-major R x R);
+ *   Gn = GU ./ (lambda lambda^T)  (the gram of the normalised factor).
+ * The normalised factor is then U_n = M Wn (pasta_rows_times): the solve, the column
+ * normalisation and the gram of the factor without the two extra passes over U_n.  DEVICE
+ * pointers; R <= 64 (EUNSUPPORTED otherwise). */
+pasta_status pasta_cpals_prepare(const double *GM, const double *const *grams, uint32_t ngrams,
+                                 uint32_t R, float *Wn, double *Gn, double *lambda, void *stream);
+/* U = M Wn: rows x R (row-major, fp32) times R x R (fp32).  DEVICE pointers; R <= 64. */
+pasta_status pasta_rows_times(const float *M, uint64_t rows, uint32_t R, const float *Wn, float *U,
+                              void *stream);
+/* The factor update fused with its all-gather (a9): rows [row_lo, row_hi) of
+ * M Wn (M: DEVICE [rows][R], the rank's MTTKRP output rows at their global positions) are
+ * computed once and stored into each of the `ndst` (1..8) full-size replicas dsts[k]
+ * ([rows][R], row-major): the local factor and the peers' factors mapped with
+ * pasta_ipc_open (P2P stores over NVLink / NVSwitch).  The kernel ends with a system-scope
+ * fence; the caller orders the peers' next reads after it (a collective on the stream).
+ * R in {4, 8, 16, 32, 64} (EUNSUPPORTED otherwise). */
+pasta_status pasta_rows_times_bcast(const float *M, uint64_t row_lo, uint64_t row_hi, uint32_t R,
+                                    const float *Wn, float *const *dsts, uint32_t ndst, void *stream);
+
+/* Peer memory (CUDA IPC) for the fused exchange.  pasta_dev_alloc returns an exportable
+ * device allocation (cudaMalloc base pointer; free with pasta_dev_free);
+ * pasta_ipc_get_handle writes its PASTA_IPC_HANDLE_BYTES-byte handle; another process maps
+ * it with pasta_ipc_open (peer access enabled lazily) and unmaps with pasta_ipc_close. */
+#define PASTA_IPC_HANDLE_BYTES 64
+pasta_status pasta_dev_alloc(uint64_t bytes, void **ptr);
+pasta_status pasta_dev_free(void *ptr);
+pasta_status pasta_ipc_get_handle(void *base, void *handle);
+pasta_status pasta_ipc_open(const void *handle, void **ptr);
+pasta_status pasta_ipc_close(void *ptr);
 /* lambda[r] = sqrt(colsq[r]) (1 where zero); U(:, r) /= lambda[r].  lambda: DEVICE fp64 [R]. */
 pasta_status pasta_normalize_columns(float *U, uint64_t rows, uint32_t R, const double *colsq,
                                      double *lambda, void *stream);

@@ -26,7 +26,8 @@ __all__ = [
     "pasta_cpals_solve", "pasta_normalize_columns", "pasta_weighted_inner", "pasta_coo_norm2",
     "pasta_cpals_coo", "pasta_coo_fibers", "pasta_coo_fiber_export", "pasta_ttm_coo",
     "pasta_ttv_coo", "pasta_coo_to_ghicoo", "pasta_ghicoo_auto_mask", "pasta_ghicoo_export",
-    "pasta_ts", "pasta_tew", "pasta_coo_values_ptr", "pasta_coo_ts", "pasta_coo_tew", "OPS",
+    "pasta_cpals_prepare", "pasta_rows_times", "pasta_rows_times_bcast", "pasta_dev_alloc",
+    "pasta_dev_free", "pasta_ipc_get_handle", "pasta_ipc_open", "pasta_ipc_close", "pasta_ts", "pasta_tew", "pasta_coo_values_ptr", "pasta_coo_ts", "pasta_coo_tew", "OPS",
 ]
 
 _u32p = C.POINTER(C.c_uint32)
@@ -447,6 +448,34 @@ def pasta_cpals_solve(M, grams, U=None, colsq=None, stream=None):
     return U, colsq
 
 
+def pasta_cpals_prepare(GM, grams, Wn=None, Gn=None, lam=None, stream=None):
+    """Fused CP-ALS algebra (include/pasta.h): from GM = M^T M and the other grams ->
+    (Wn fp32 [R, R], Gn fp64 [R, R], lambda fp64 [R]); the factor is then M @ Wn."""
+    import torch
+    R = int(GM.shape[0])
+    dev = GM.device
+    if Wn is None:
+        Wn = torch.empty((R, R), dtype=torch.float32, device=dev)
+    if Gn is None:
+        Gn = torch.empty((R, R), dtype=torch.float64, device=dev)
+    if lam is None:
+        lam = torch.empty(R, dtype=torch.float64, device=dev)
+    gp = (C.c_void_p * max(len(grams), 1))(*[g.data_ptr() for g in grams])
+    check(lib().pasta_cpals_prepare(_dptr(GM), gp, len(grams), R, _dptr(Wn), _dptr(Gn), _dptr(lam),
+                                    _stream_ptr(stream)))
+    return Wn, Gn, lam
+
+
+def pasta_rows_times(M, Wn, U=None, stream=None):
+    """U = M Wn (rows x R times R x R, fp32) in a libpasta kernel."""
+    import torch
+    if U is None:
+        U = torch.empty_like(M)
+    check(lib().pasta_rows_times(_dptr(M), int(M.shape[0]), int(M.shape[1]), _dptr(Wn), _dptr(U),
+                                 _stream_ptr(stream)))
+    return U
+
+
 def pasta_normalize_columns(U, colsq, lam=None, stream=None):
     import torch
     R = int(U.shape[1])
@@ -585,3 +614,53 @@ def pasta_coo_tew(x: Coo, y: Coo, op) -> Coo:
     out = C.c_void_p()
     check(lib().pasta_coo_tew(x.ptr, y.ptr, _op(op), C.byref(out)))
     return Coo(out.value)
+
+
+# ----------------------------------------------------------------------------- peer memory
+def pasta_rows_times_bcast(M, row_lo: int, row_hi: int, Wn, dst_ptrs, stream=None) -> None:
+    """Rows [row_lo, row_hi) of M @ Wn stored into every replica in ``dst_ptrs`` (device
+    addresses: the local factor and peers' factors mapped with :func:`pasta_ipc_open`)."""
+    R = int(M.shape[1])
+    dp = (C.c_void_p * len(dst_ptrs))(*[int(p) for p in dst_ptrs])
+    check(lib().pasta_rows_times_bcast(_dptr(M), int(row_lo), int(row_hi), R, _dptr(Wn), dp,
+                                       len(dst_ptrs), _stream_ptr(stream)))
+
+
+class _CudaArray:
+    """Zero-copy view of a libpasta device allocation for torch.as_tensor."""
+
+    def __init__(self, ptr: int, shape, typestr="<f4"):
+        self.__cuda_array_interface__ = {"shape": tuple(shape), "typestr": typestr,
+                                         "data": (int(ptr), False), "version": 3, "strides": None}
+
+
+def pasta_dev_alloc(shape, dtype="float32"):
+    """An IPC-exportable device allocation wrapped as a torch tensor; returns (tensor, ptr).
+    Free with :func:`pasta_dev_free` after the last use of the tensor."""
+    import torch
+    n = int(np.prod(shape))
+    p = C.c_void_p()
+    check(lib().pasta_dev_alloc(max(n, 1) * 4, C.byref(p)))
+    t = torch.as_tensor(_CudaArray(p.value, shape), device="cuda")
+    return t, p.value
+
+
+def pasta_dev_free(ptr: int) -> None:
+    check(lib().pasta_dev_free(C.c_void_p(ptr)))
+
+
+def pasta_ipc_get_handle(ptr: int) -> bytes:
+    buf = (C.c_uint8 * 64)()
+    check(lib().pasta_ipc_get_handle(C.c_void_p(ptr), buf))
+    return bytes(buf)
+
+
+def pasta_ipc_open(handle: bytes) -> int:
+    buf = (C.c_uint8 * 64).from_buffer_copy(handle)
+    p = C.c_void_p()
+    check(lib().pasta_ipc_open(buf, C.byref(p)))
+    return p.value
+
+
+def pasta_ipc_close(ptr: int) -> None:
+    check(lib().pasta_ipc_close(C.c_void_p(ptr)))

@@ -84,6 +84,15 @@ SIGNATURES = {
     "pasta_hicoo_free": (None, [_vp]),
     "pasta_gram": (_st, [_vp, C.c_uint64, C.c_uint32, _vp, _vp]),
     "pasta_cpals_solve": (_st, [_vp, C.c_uint64, C.c_uint32, C.POINTER(_vp), C.c_uint32, _vp, _vp, _vp]),
+    "pasta_cpals_prepare": (_st, [_vp, C.POINTER(_vp), C.c_uint32, C.c_uint32, _vp, _vp, _vp, _vp]),
+    "pasta_rows_times": (_st, [_vp, C.c_uint64, C.c_uint32, _vp, _vp, _vp]),
+    "pasta_rows_times_bcast": (_st, [_vp, C.c_uint64, C.c_uint64, C.c_uint32, _vp, C.POINTER(_vp),
+                                     C.c_uint32, _vp]),
+    "pasta_dev_alloc": (_st, [C.c_uint64, C.POINTER(_vp)]),
+    "pasta_dev_free": (_st, [_vp]),
+    "pasta_ipc_get_handle": (_st, [_vp, _vp]),
+    "pasta_ipc_open": (_st, [_vp, C.POINTER(_vp)]),
+    "pasta_ipc_close": (_st, [_vp]),
     "pasta_normalize_columns": (_st, [_vp, C.c_uint64, C.c_uint32, _vp, _vp, _vp]),
     "pasta_weighted_inner": (_st, [_vp, _vp, C.c_uint64, C.c_uint32, _vp, _vp, _vp]),
     "pasta_coo_norm2": (_st, [_vp, C.POINTER(C.c_double)]),

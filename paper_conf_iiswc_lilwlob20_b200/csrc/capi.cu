@@ -722,6 +722,76 @@ pasta_status pasta_cpals_solve(const float *M, uint64_t rows, uint32_t R, const 
   API_END
 }
 
+pasta_status pasta_cpals_prepare(const double *GM, const double *const *grams, uint32_t ngrams, uint32_t R,
+                                 float *Wn, double *Gn, double *lambda, void *stream) {
+  API_BEGIN
+  require_R64(R);
+  require(GM && Wn && Gn && lambda && (grams || ngrams == 0), "NULL argument");
+  for (uint32_t k = 0; k < ngrams; ++k) require(grams[k] != nullptr, "grams[k] is NULL");
+  launch_cpals_prep(GM, grams, ngrams, R, Wn, Gn, lambda, as_stream(stream));
+  API_END
+}
+
+pasta_status pasta_rows_times(const float *M, uint64_t rows, uint32_t R, const float *Wn, float *U,
+                              void *stream) {
+  API_BEGIN
+  require_R64(R);
+  require((M && U && Wn) || rows == 0, "NULL argument");
+  if (rows) launch_apply(M, rows, R, Wn, U, as_stream(stream));
+  API_END
+}
+
+pasta_status pasta_rows_times_bcast(const float *M, uint64_t row_lo, uint64_t row_hi, uint32_t R,
+                                    const float *Wn, float *const *dsts, uint32_t ndst, void *stream) {
+  API_BEGIN
+  require(M && Wn && dsts, "NULL argument");
+  require(row_lo <= row_hi, "row_lo > row_hi");
+  for (uint32_t k = 0; k < ndst; ++k) require(dsts[k] != nullptr, "dsts[k] is NULL");
+  launch_apply_bcast(M, row_lo, row_hi, R, Wn, dsts, ndst, as_stream(stream));
+  API_END
+}
+
+// ---------------------------------------------------------------------------- peer memory
+pasta_status pasta_dev_alloc(uint64_t bytes, void **ptr) {
+  API_BEGIN
+  require(ptr != nullptr, "ptr is NULL");
+  *ptr = nullptr;
+  PASTA_CUDA(cudaMalloc(ptr, bytes ? bytes : 1));
+  API_END
+}
+
+pasta_status pasta_dev_free(void *ptr) {
+  API_BEGIN
+  if (ptr) PASTA_CUDA(cudaFree(ptr));
+  API_END
+}
+
+pasta_status pasta_ipc_get_handle(void *base, void *handle) {
+  API_BEGIN
+  require(base && handle, "NULL argument");
+  static_assert(sizeof(cudaIpcMemHandle_t) == PASTA_IPC_HANDLE_BYTES, "IPC handle size");
+  cudaIpcMemHandle_t h;
+  PASTA_CUDA(cudaIpcGetMemHandle(&h, base));
+  std::memcpy(handle, &h, sizeof(h));
+  API_END
+}
+
+pasta_status pasta_ipc_open(const void *handle, void **ptr) {
+  API_BEGIN
+  require(handle && ptr, "NULL argument");
+  *ptr = nullptr;
+  cudaIpcMemHandle_t h;
+  std::memcpy(&h, handle, sizeof(h));
+  PASTA_CUDA(cudaIpcOpenMemHandle(ptr, h, cudaIpcMemLazyEnablePeerAccess));
+  API_END
+}
+
+pasta_status pasta_ipc_close(void *ptr) {
+  API_BEGIN
+  if (ptr) PASTA_CUDA(cudaIpcCloseMemHandle(ptr));
+  API_END
+}
+
 pasta_status pasta_normalize_columns(float *U, uint64_t rows, uint32_t R, const double *colsq,
                                      double *lambda, void *stream) {
   API_BEGIN
@@ -769,7 +839,12 @@ pasta_status pasta_cpals_coo(pasta_coo *x, uint32_t R, uint32_t max_iters, doubl
   uint64_t maxd = 0;
   for (uint32_t k = 0; k < N; ++k) maxd = x->dims[k] > maxd ? x->dims[k] : maxd;
   DevArray<float> Mbuf(maxd * R, s);
-  DevArray<double> grams(uint64_t(N) * R * R, s), colsq(R, s), lam(R, s), scal(2, s);
+  DevArray<double> grams(uint64_t(N) * R * R, s), colsq(R, s), lam(R, s), scal(2, s), GM(uint64_t(R) * R, s);
+  DevArray<float> Wn(uint64_t(R) * R, s);
+  // fused epilogue (default): gram of M, R x R algebra, one pass U = M Wn; PASTA_CPALS_FUSED=0
+  // runs the unfused solve -> normalise -> gram sequence
+  const char *fz = getenv("PASTA_CPALS_FUSED");
+  const bool fused = !(fz && *fz == '0');
   auto G = [&](uint32_t k) { return grams.p + uint64_t(k) * R * R; };
   PASTA_CUDA(cudaMemsetAsync(grams.p, 0, grams.bytes(), s));
   for (uint32_t k = 0; k < N; ++k) launch_gram(factors[k], x->dims[k], R, G(k), s);
@@ -791,6 +866,13 @@ pasta_status pasta_cpals_coo(pasta_coo *x, uint32_t R, uint32_t max_iters, doubl
       uint32_t ng = 0;
       for (uint32_t k = 0; k < N; ++k)
         if (k != n) gl[ng++] = G(k);
+      if (fused) {
+        PASTA_CUDA(cudaMemsetAsync(GM.p, 0, GM.bytes(), s));
+        launch_gram(Mbuf.p, x->dims[n], R, GM.p, s);
+        launch_cpals_prep(GM.p, gl, ng, R, Wn.p, G(n), lam.p, s);
+        launch_apply(Mbuf.p, x->dims[n], R, Wn.p, factors[n], s);
+        continue;
+      }
       PASTA_CUDA(cudaMemsetAsync(colsq.p, 0, colsq.bytes(), s));
       launch_solve(Mbuf.p, x->dims[n], R, gl, ng, factors[n], colsq.p, s);
       launch_normalize(factors[n], x->dims[n], R, colsq.p, lam.p, s);

@@ -10,6 +10,7 @@
 // Building blocks are exported through the C ABI so the multi-GPU driver (parallel.py) can
 // all-reduce the R x R partials and all-gather the owned rows in between.
 #include <cmath>
+#include <cstdlib>
 
 #include "internal.cuh"
 
@@ -19,6 +20,17 @@ namespace {
 
 constexpr int kThreads = 256;
 constexpr int kMaxR = 64;
+
+int sm_count_cpals() {
+  static int sms = 0;
+  if (!sms) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    if (sms <= 0) sms = 148;
+  }
+  return sms;
+}
 
 unsigned grid_rows(uint64_t rows, int per_cta) {
   static int sms = 0;
@@ -73,6 +85,140 @@ __global__ void __launch_bounds__(kThreads) gram_kernel(const float *__restrict_
     atomicAdd(&G[a * R + b], acc[q]);
     if (a != b) atomicAdd(&G[b * R + a], acc[q]);
   }
+}
+
+// Tiled kernels for R in {4, 8, 16, 32, 64}: a CTA stages kTile rows of the I x R matrix in
+// shared memory with coalesced 128-bit loads, then
+//   gram_tile_kernel:  groups of (R/4)^2 threads own the 4 x 4 blocks of U^T U; group g sums
+//                      rows g, g + G, ... of the tile (two LDS.128 broadcasts + 16 FMAs per
+//                      row), fp32 over <= 64 rows, fp64 beyond; one fp64 atomic per entry per CTA.
+//   apply_tile_kernel: thread t owns output column c = t % R with W(:, c) in registers and
+//                      rows t / R + j * (256 / R) of the tile (LDS.128 broadcasts, R FMAs per
+//                      row); stores are coalesced (consecutive threads, consecutive columns).
+// Both are HBM-streaming passes over the factor-sized matrix (one read; apply also writes).
+constexpr int kTile = 256;
+// rows per staged tile: 256, fewer for R = 64 so that static shared memory stays <= 48 KB
+template <int R>
+constexpr int tile_rows() { return R <= 32 ? kTile : 64; }
+
+template <int R>
+__global__ void __launch_bounds__(kThreads) gram_tile_kernel(const float *__restrict__ U, uint64_t rows,
+                                                             double *__restrict__ G) {
+  constexpr int RB = R / 4, GS = RB * RB, NG = kThreads / GS, T = tile_rows<R>();
+  __shared__ __align__(16) float tile[T * R];
+  __shared__ double red[R * R];
+  const int t = threadIdx.x, g = t / GS, blk = t % GS, ba = blk / RB, bb = blk % RB;
+  float acc[4][4] = {};
+  double acc64[4][4] = {};
+  int since = 0;
+  for (uint32_t e = t; e < R * R; e += kThreads) red[e] = 0.0;
+  for (uint64_t r0 = uint64_t(blockIdx.x) * T; r0 < rows; r0 += uint64_t(gridDim.x) * T) {
+    const int nr = int(rows - r0 < T ? rows - r0 : T);
+    __syncthreads();
+    const float4 *src = reinterpret_cast<const float4 *>(U + r0 * R);
+    float4 *dst = reinterpret_cast<float4 *>(tile);
+    for (int e = t; e < nr * RB; e += kThreads) dst[e] = src[e];
+    __syncthreads();
+    for (int i = g; i < nr; i += NG) {
+      const float4 x = *reinterpret_cast<const float4 *>(tile + i * R + 4 * ba);
+      const float4 y = *reinterpret_cast<const float4 *>(tile + i * R + 4 * bb);
+      const float xa[4] = {x.x, x.y, x.z, x.w}, ya[4] = {y.x, y.y, y.z, y.w};
+#pragma unroll
+      for (int p = 0; p < 4; ++p)
+#pragma unroll
+        for (int q = 0; q < 4; ++q) acc[p][q] = fmaf(xa[p], ya[q], acc[p][q]);
+      if (++since == 64) {
+#pragma unroll
+        for (int p = 0; p < 4; ++p)
+#pragma unroll
+          for (int q = 0; q < 4; ++q) { acc64[p][q] += double(acc[p][q]); acc[p][q] = 0.f; }
+        since = 0;
+      }
+    }
+  }
+  __syncthreads();
+#pragma unroll
+  for (int p = 0; p < 4; ++p)
+#pragma unroll
+    for (int q = 0; q < 4; ++q) atomicAdd(&red[(4 * ba + p) * R + 4 * bb + q], acc64[p][q] + double(acc[p][q]));
+  __syncthreads();
+  for (uint32_t e = t; e < R * R; e += kThreads) atomicAdd(&G[e], red[e]);
+}
+
+template <int R>
+__global__ void __launch_bounds__(kThreads) apply_tile_kernel(const float *__restrict__ M, uint64_t rows,
+                                                              const float *__restrict__ W, float *__restrict__ U) {
+  constexpr int RB = R / 4, RPP = kThreads / R, T = tile_rows<R>();  // RPP: rows per pass
+  __shared__ __align__(16) float tile[T * R];
+  const int t = threadIdx.x, c = t % R, r = t / R;
+  float w[R];
+#pragma unroll
+  for (int a = 0; a < R; ++a) w[a] = W[a * R + c];
+  for (uint64_t r0 = uint64_t(blockIdx.x) * T; r0 < rows; r0 += uint64_t(gridDim.x) * T) {
+    const int nr = int(rows - r0 < T ? rows - r0 : T);
+    __syncthreads();
+    const float4 *src = reinterpret_cast<const float4 *>(M + r0 * R);
+    float4 *dst = reinterpret_cast<float4 *>(tile);
+    for (int e = t; e < nr * RB; e += kThreads) dst[e] = src[e];
+    __syncthreads();
+    for (int i = r; i < nr; i += RPP) {
+      float acc = 0.f;
+#pragma unroll
+      for (int a = 0; a < R; a += 4) {
+        const float4 m = *reinterpret_cast<const float4 *>(tile + i * R + a);
+        acc = fmaf(m.x, w[a], acc);
+        acc = fmaf(m.y, w[a + 1], acc);
+        acc = fmaf(m.z, w[a + 2], acc);
+        acc = fmaf(m.w, w[a + 3], acc);
+      }
+      U[(r0 + i) * R + c] = acc;
+    }
+  }
+}
+
+// Fused factor update + all-gather over peer memory (a9 / NEXT-1, B200-native exchange):
+// the rows [row_lo, row_hi) this rank owns are computed once (U = M Wn, as apply_tile_kernel)
+// and stored into every replica of U_n -- the local one and each peer's, mapped through CUDA
+// IPC (NVLink / NVSwitch P2P stores) -- so the all-gather overlaps the arithmetic tile by
+// tile instead of following it as a separate collective.
+struct DstList {
+  float *d[kMaxOrder];
+  uint32_t n;
+};
+
+template <int R>
+__global__ void __launch_bounds__(kThreads) apply_bcast_kernel(const float *__restrict__ M, uint64_t row_lo,
+                                                               uint64_t row_hi, const float *__restrict__ W,
+                                                               DstList dst) {
+  constexpr int RB = R / 4, RPP = kThreads / R, T = R <= 32 ? 256 : 64;
+  __shared__ __align__(16) float tile[T * R];
+  const int t = threadIdx.x, c = t % R, r = t / R;
+  float w[R];
+#pragma unroll
+  for (int a = 0; a < R; ++a) w[a] = W[a * R + c];
+  const uint64_t rows = row_hi - row_lo;
+  for (uint64_t r0 = uint64_t(blockIdx.x) * T; r0 < rows; r0 += uint64_t(gridDim.x) * T) {
+    const int nr = int(rows - r0 < T ? rows - r0 : T);
+    __syncthreads();
+    const float4 *src = reinterpret_cast<const float4 *>(M + (row_lo + r0) * R);
+    float4 *sd = reinterpret_cast<float4 *>(tile);
+    for (int e = t; e < nr * RB; e += kThreads) sd[e] = src[e];
+    __syncthreads();
+    for (int i = r; i < nr; i += RPP) {
+      float acc = 0.f;
+#pragma unroll
+      for (int a = 0; a < R; a += 4) {
+        const float4 m = *reinterpret_cast<const float4 *>(tile + i * R + a);
+        acc = fmaf(m.x, w[a], acc);
+        acc = fmaf(m.y, w[a + 1], acc);
+        acc = fmaf(m.z, w[a + 2], acc);
+        acc = fmaf(m.w, w[a + 3], acc);
+      }
+      const uint64_t off = (row_lo + r0 + i) * R + c;
+      for (uint32_t k = 0; k < dst.n; ++k) dst.d[k][off] = acc;
+    }
+  }
+  __threadfence_system();  // peer stores performed before the kernel is seen complete
 }
 
 struct GramList {
@@ -135,16 +281,19 @@ __device__ void hadamard_inverse(const GramList &gl, uint32_t R, double *V, doub
 // `width` lanes (next power of two >= R, at most 32) handles one row; lane l owns columns
 // l, l + width (R <= 64); M(i, a) is broadcast inside the sub-warp with shuffles and W is read
 // from shared memory (consecutive lanes, consecutive columns: conflict-free).
+// Wg != nullptr: the fp32 right-hand matrix is given (cpals_prep_kernel) and neither the
+// inverse nor colsq is computed (colsq may be NULL).
 __global__ void __launch_bounds__(kThreads) solve_kernel(const float *__restrict__ M, uint64_t rows,
                                                          uint32_t R, GramList gl, float *__restrict__ U,
-                                                         double *__restrict__ colsq) {
+                                                         double *__restrict__ colsq,
+                                                         const float *__restrict__ Wg) {
   extern __shared__ double solve_smem[];  // V[R*R], W[R*R], csq[R], Wf[R*R] (fp32)
   double *V = solve_smem, *W = solve_smem + R * R, *csq = solve_smem + 2 * R * R;
   float *Wf = reinterpret_cast<float *>(solve_smem + 2 * R * R + R);
-  if (threadIdx.x < 32) hadamard_inverse(gl, R, V, W);
+  if (Wg == nullptr && threadIdx.x < 32) hadamard_inverse(gl, R, V, W);
   for (uint32_t r = threadIdx.x; r < R; r += kThreads) csq[r] = 0.0;
   __syncthreads();
-  for (uint32_t e = threadIdx.x; e < R * R; e += kThreads) Wf[e] = float(W[e]);
+  for (uint32_t e = threadIdx.x; e < R * R; e += kThreads) Wf[e] = Wg ? Wg[e] : float(W[e]);
   __syncthreads();
   uint32_t width = 1, lw = 0;
   while (width < R && width < 32) { width <<= 1; ++lw; }
@@ -189,11 +338,12 @@ __global__ void __launch_bounds__(kThreads) solve_kernel(const float *__restrict
         const uint32_t c = l + width * q2;
         if (i < rows && c < R) {
           U[i * R + c] = x[b][q2];
-          mine[q2] = fmaf(x[b][q2], x[b][q2], mine[q2]);
+          if (colsq) mine[q2] = fmaf(x[b][q2], x[b][q2], mine[q2]);
         }
       }
     }
   }
+  if (colsq == nullptr) return;  // uniform across the grid
   // reduce over the sub-warps (lanes with equal l hold the same columns)
 #pragma unroll
   for (int q2 = 0; q2 < 2; ++q2) {
@@ -204,6 +354,48 @@ __global__ void __launch_bounds__(kThreads) solve_kernel(const float *__restrict
   }
   __syncthreads();
   for (uint32_t r = threadIdx.x; r < R; r += kThreads) atomicAdd(&colsq[r], csq[r]);
+}
+
+// Fused CP-ALS epilogue algebra for mode n (one CTA), so that the factor update needs a
+// single pass over M and none over U: with GM = M^T M (R x R, from gram_kernel on M),
+//   W = V^{-1}, V = Hadamard_{k != n} G_k          (hadamard_inverse, one warp, fp64)
+//   U = M W  =>  U^T U = W^T GM W =: GU,  lambda_r = sqrt(GU_rr)  (1 if GU_rr <= 0)
+//   normalised U_n = M Wn,  Wn = W diag(1 / lambda),  G_n = GU ./ (lambda lambda^T).
+// Same algebra as solve -> normalise -> gram (Kolda & Bader), without two of the
+// three passes over the I_n x R factor.
+__global__ void cpals_prep_kernel(const double *__restrict__ GM, GramList gl, uint32_t R,
+                                  float *__restrict__ Wn, double *__restrict__ Gn,
+                                  double *__restrict__ lambda) {
+  extern __shared__ double prep_smem[];  // V[R*R], W[R*R], T[R*R], lam[R]
+  double *V = prep_smem, *W = prep_smem + R * R, *T = prep_smem + 2 * R * R, *lam = prep_smem + 3 * R * R;
+  if (threadIdx.x < 32) hadamard_inverse(gl, R, V, W);
+  __syncthreads();
+  for (uint32_t e = threadIdx.x; e < R * R; e += blockDim.x) {  // T = GM W
+    const uint32_t a = e / R, c = e % R;
+    double t = 0.0;
+    for (uint32_t b = 0; b < R; ++b) t += GM[a * R + b] * W[b * R + c];
+    T[e] = t;
+  }
+  __syncthreads();
+  for (uint32_t e = threadIdx.x; e < R * R; e += blockDim.x) {  // GU = W^T T  (into V)
+    const uint32_t a = e / R, c = e % R;
+    double t = 0.0;
+    for (uint32_t b = 0; b < R; ++b) t += W[b * R + a] * T[b * R + c];
+    V[e] = t;
+  }
+  __syncthreads();
+  for (uint32_t r = threadIdx.x; r < R; r += blockDim.x) {
+    const double d = V[r * R + r];
+    const double l = d > 0.0 ? sqrt(d) : 1.0;
+    lam[r] = l;
+    lambda[r] = l;
+  }
+  __syncthreads();
+  for (uint32_t e = threadIdx.x; e < R * R; e += blockDim.x) {
+    const uint32_t a = e / R, c = e % R;
+    Gn[e] = V[e] / (lam[a] * lam[c]);
+    Wn[e] = float(W[e] / lam[c]);
+  }
 }
 
 // lambda_r = sqrt(colsq_r) (1 if zero); U(:, r) /= lambda_r.  VW = 4: float4 path (R % 4 == 0),
@@ -300,9 +492,52 @@ __global__ void sumsq_kernel(const float *__restrict__ v, uint64_t n, double *__
 
 }  // namespace
 
+bool tiled_ok(uint32_t R, const void *a, const void *b) {
+  const bool al = ((reinterpret_cast<uintptr_t>(a) | reinterpret_cast<uintptr_t>(b)) & 15u) == 0;
+  return al && (R == 4 || R == 8 || R == 16 || R == 32 || R == 64);
+}
+
+template <template <int> class K, class... Args>
+void launch_tiled(uint32_t R, uint64_t rows, cudaStream_t s, Args... args) {
+  // persistent-style grid: PASTA_TILE_CTAS_PER_SM (default 8) CTAs per SM walk the row tiles,
+  // so the per-CTA prologue / epilogue (W load, smem and global reductions) is amortised
+  static int per_sm = 0;
+  if (!per_sm) {
+    const char *e = getenv("PASTA_TILE_CTAS_PER_SM");
+    per_sm = (e && *e) ? atoi(e) : 8;
+    if (per_sm < 1) per_sm = 8;
+  }
+  unsigned grid = grid_rows(rows, kTile);
+  const unsigned cap = unsigned(sm_count_cpals()) * unsigned(per_sm);
+  if (grid > cap) grid = cap;
+  switch (R) {
+    case 4: K<4>::go(grid, s, args...); break;
+    case 8: K<8>::go(grid, s, args...); break;
+    case 16: K<16>::go(grid, s, args...); break;
+    case 32: K<32>::go(grid, s, args...); break;
+    default: K<64>::go(grid, s, args...); break;
+  }
+  PASTA_LAUNCHED();
+}
+
+template <int R>
+struct GramTile {
+  static void go(unsigned grid, cudaStream_t s, const float *U, uint64_t rows, double *G) {
+    gram_tile_kernel<R><<<grid, kThreads, 0, s>>>(U, rows, G);
+  }
+};
+
+template <int R>
+struct ApplyTile {
+  static void go(unsigned grid, cudaStream_t s, const float *M, uint64_t rows, const float *W, float *U) {
+    apply_tile_kernel<R><<<grid, kThreads, 0, s>>>(M, rows, W, U);
+  }
+};
+
 void launch_gram(const float *U, uint64_t rows, uint32_t R, double *G, cudaStream_t s) {
   if (R > kMaxR) fail(PASTA_EUNSUPPORTED, "CP-ALS building blocks support R <= 64");
   if (!rows) return;
+  if (tiled_ok(R, U, U)) return launch_tiled<GramTile>(R, rows, s, U, rows, G);
   gram_kernel<<<grid_rows(rows, 64 * 8), kThreads, 0, s>>>(U, rows, R, G);
   PASTA_LAUNCHED();
 }
@@ -318,10 +553,55 @@ void launch_solve(const float *M, uint64_t rows, uint32_t R, const double *const
   auto go = [&](auto kern) {
     if (smem > 48 * 1024)
       PASTA_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem)));
-    kern<<<grid_rows(rows ? rows : 1, kThreads * 4), kThreads, smem, s>>>(M, rows, R, gl, U, colsq);
+    kern<<<grid_rows(rows ? rows : 1, kThreads * 4), kThreads, smem, s>>>(M, rows, R, gl, U, colsq, nullptr);
     PASTA_LAUNCHED();
   };
   go(solve_kernel);
+}
+
+void launch_cpals_prep(const double *GM, const double *const *grams, uint32_t ngrams, uint32_t R,
+                       float *Wn, double *Gn, double *lambda, cudaStream_t s) {
+  if (R > kMaxR) fail(PASTA_EUNSUPPORTED, "CP-ALS building blocks support R <= 64");
+  if (ngrams > kMaxOrder) fail(PASTA_EINVAL, "too many gram matrices");
+  GramList gl{};
+  gl.n = ngrams;
+  for (uint32_t k = 0; k < ngrams; ++k) gl.g[k] = grams[k];
+  const size_t smem = (3 * size_t(R) * R + R) * sizeof(double);
+  if (smem > 48 * 1024)
+    PASTA_CUDA(cudaFuncSetAttribute(cpals_prep_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem)));
+  cpals_prep_kernel<<<1, kThreads, smem, s>>>(GM, gl, R, Wn, Gn, lambda);
+  PASTA_LAUNCHED();
+}
+
+void launch_apply(const float *M, uint64_t rows, uint32_t R, const float *Wn, float *U, cudaStream_t s) {
+  if (R > kMaxR) fail(PASTA_EUNSUPPORTED, "CP-ALS building blocks support R <= 64");
+  if (tiled_ok(R, M, U)) return launch_tiled<ApplyTile>(R, rows, s, M, rows, Wn, U);
+  GramList gl{};
+  const size_t smem = (2 * size_t(R) * R + R) * sizeof(double) + size_t(R) * R * sizeof(float);
+  if (smem > 48 * 1024)
+    PASTA_CUDA(cudaFuncSetAttribute(solve_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem)));
+  solve_kernel<<<grid_rows(rows ? rows : 1, kThreads * 4), kThreads, smem, s>>>(M, rows, R, gl, U, nullptr, Wn);
+  PASTA_LAUNCHED();
+}
+
+template <int R>
+struct ApplyBcast {
+  static void go(unsigned grid, cudaStream_t s, const float *M, uint64_t lo, uint64_t hi, const float *W,
+                 DstList d) {
+    apply_bcast_kernel<R><<<grid, kThreads, 0, s>>>(M, lo, hi, W, d);
+  }
+};
+
+void launch_apply_bcast(const float *M, uint64_t row_lo, uint64_t row_hi, uint32_t R, const float *Wn,
+                        float *const *dsts, uint32_t ndst, cudaStream_t s) {
+  if (!(R == 4 || R == 8 || R == 16 || R == 32 || R == 64))
+    fail(PASTA_EUNSUPPORTED, "pasta_rows_times_bcast: R must be 4, 8, 16, 32 or 64");
+  if (ndst < 1 || ndst > kMaxOrder) fail(PASTA_EINVAL, "pasta_rows_times_bcast: 1..8 destinations");
+  if (row_hi <= row_lo) return;
+  DstList d{};
+  d.n = ndst;
+  for (uint32_t k = 0; k < ndst; ++k) d.d[k] = dsts[k];
+  launch_tiled<ApplyBcast>(R, row_hi - row_lo, s, M, row_lo, row_hi, Wn, d);
 }
 
 void launch_normalize(float *U, uint64_t rows, uint32_t R, const double *colsq, double *lambda,

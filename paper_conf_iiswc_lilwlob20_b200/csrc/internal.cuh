@@ -256,6 +256,14 @@ void launch_solve(const float *M, uint64_t rows, uint32_t R, const double *const
                   float *U, double *colsq, cudaStream_t s);
 void launch_normalize(float *U, uint64_t rows, uint32_t R, const double *colsq, double *lambda,
                       cudaStream_t s);
+// fused CP-ALS epilogue: from GM = M^T M and the other grams -> Wn (fp32), G_n, lambda
+void launch_cpals_prep(const double *GM, const double *const *grams, uint32_t ngrams, uint32_t R,
+                       float *Wn, double *Gn, double *lambda, cudaStream_t s);
+// U = M Wn (rows x R times R x R)
+void launch_apply(const float *M, uint64_t rows, uint32_t R, const float *Wn, float *U, cudaStream_t s);
+// rows [row_lo, row_hi) of M Wn stored into each of `ndst` full-size replicas (local / peer)
+void launch_apply_bcast(const float *M, uint64_t row_lo, uint64_t row_hi, uint32_t R, const float *Wn,
+                        float *const *dsts, uint32_t ndst, cudaStream_t s);
 void launch_inner(const float *A, const float *B, uint64_t rows, uint32_t R, const double *lambda,
                   double *out, cudaStream_t s);
 void launch_sumsq(const float *v, uint64_t n, double *out, cudaStream_t s);

@@ -10,8 +10,8 @@
 //        intersection for mul/div), then the values are computed per merged coordinate.
 //
 // Design for HBM: 128-bit loads with an L2 evict_first hint (each byte is used once),
-// 128-bit stores, four vectors in flight per thread, a grid of 148 x 8 CTAs walking the
-// arrays in grid-stride order.  IEEE fp32 operations (correctly rounded, incl. division).
+// 128-bit stores (streaming .cs for TEW, plain for TS: measured), four vectors in flight per
+// thread, a grid of 148 x 8 CTAs walking the arrays in grid-stride order.  IEEE fp32 operations (correctly rounded, incl. division).
 #include <cub/cub.cuh>
 
 #include <cstdlib>
@@ -132,11 +132,15 @@ void launch_ew_op(bool vec, const float *a, const float *b, float s, float *out,
     PASTA_LAUNCHED();
   };
   if (!vec) return go(ew_scalar_kernel<OP, kScalar>);
-  switch (var) {  // PASTA_EW_VARIANT: tuning knob (1: 2 in flight, 2: 8 in flight, 3: plain stores)
+  // PASTA_EW_VARIANT: tuning knob (1: 2 in flight, 2: 8 in flight, 3: plain stores, 5:
+  // streaming stores).  Default (measured on B200, tools/ew_sweep.py): TS (1 read : 1 write)
+  // with plain stores 6.0 TB/s vs 5.66 with .cs; TEW (2 : 1) with .cs stores 6.4 vs 6.2.
+  switch (var) {
     case 1: go(ew_kernel<OP, kScalar, 2, true>); break;
     case 2: go(ew_kernel<OP, kScalar, 8, true>); break;
     case 3: go(ew_kernel<OP, kScalar, 4, false>); break;
-    default: go(ew_kernel<OP, kScalar, 4, true>); break;
+    case 5: go(ew_kernel<OP, kScalar, 4, true>); break;
+    default: go(ew_kernel<OP, kScalar, 4, !kScalar>); break;
   }
 }
 

@@ -73,6 +73,51 @@ class RowPartitionedMTTKRP:
         return self.out
 
 
+class PeerReplicas:
+    """Replicated factor matrices in IPC-exportable device memory, with every peer's replicas
+    mapped into this process (CUDA IPC over NVLink / NVSwitch).  ``tensors[k]`` is this rank's
+    [I_k, R] replica; ``dsts[k]`` the device addresses of all ranks' replicas (own first),
+    the destination list of :func:`pasta_rows_times_bcast`.  Handles are exchanged once over
+    the process group (``all_gather_object``)."""
+
+    def __init__(self, dims, R: int, group=None):
+        import torch.distributed as dist
+
+        from . import pasta_dev_alloc, pasta_ipc_get_handle, pasta_ipc_open
+        self.own, self.tensors, self.peers = [], [], []
+        world = dist.get_world_size(group) if dist.is_initialized() else 1
+        rank = dist.get_rank(group) if dist.is_initialized() else 0
+        for d in dims:
+            t, p = pasta_dev_alloc((int(d), R))
+            self.tensors.append(t)
+            self.own.append(p)
+        handles = [pasta_ipc_get_handle(p) for p in self.own]
+        allh = [None] * world
+        if world > 1:
+            dist.all_gather_object(allh, handles, group=group)
+        else:
+            allh = [handles]
+        self.dsts = []
+        for k in range(len(dims)):
+            lst = [self.own[k]]
+            for q in range(world):
+                if q == rank:
+                    continue
+                ptr = pasta_ipc_open(allh[q][k])
+                self.peers.append(ptr)
+                lst.append(ptr)
+            self.dsts.append(lst)
+
+    def close(self):
+        from . import pasta_dev_free, pasta_ipc_close
+        for p in self.peers:
+            pasta_ipc_close(p)
+        self.tensors = []
+        for p in self.own:
+            pasta_dev_free(p)
+        self.own, self.peers, self.dsts = [], [], []
+
+
 def _all_reduce(t):
     import torch.distributed as dist
     if dist.is_available() and dist.is_initialized() and dist.get_world_size() > 1:
@@ -82,17 +127,23 @@ def _all_reduce(t):
 
 class RowPartitionedCPALS(RowPartitionedMTTKRP):
     """CP-ALS over row-partitioned MTTKRP: per mode n, each rank computes the
-    MTTKRP rows it owns, solves its rows of U_n = M V^-1 (V from the replicated R x R grams),
-    all-reduces the column sums of squares (lambda) and its partial gram, and all-gathers the
-    owned rows of U_n -- the step that makes the output all-gather necessary.
-    Every arithmetic step runs in libpasta kernels; only R-sized vectors and R x R matrices
-    cross the process group besides the gathered rows."""
+    MTTKRP rows it owns and their R x R gram M_p^T M_p; one all-reduce gives M^T M, from which
+    every rank derives the same update matrix Wn, the normalised gram G_n and lambda
+    (pasta_cpals_prepare); each rank writes its rows U_n = M Wn, and the owned rows of U_n are
+    all-gathered -- the step that makes the output all-gather necessary.
+    Every arithmetic step runs in libpasta kernels; only R x R matrices cross the process
+    group besides the gathered rows.  fused=False runs the unfused solve / normalise / gram
+    sequence (two all-reduces per mode)."""
 
-    def run(self, factors, max_iters=20, tol=1e-5):
+    def run(self, factors, max_iters=20, tol=1e-5, fused=True, replicas=None):
+        """replicas: a :class:`PeerReplicas` whose ``tensors`` are ``factors`` -- the factor
+        update then stores every rank's rows straight into all replicas (fused P2P
+        all-gather, pasta_rows_times_bcast) instead of NCCL broadcasts."""
         import torch
 
-        from . import (pasta_coo_norm2, pasta_cpals_solve, pasta_gram, pasta_mttkrp_coo,
-                       pasta_normalize_columns, pasta_weighted_inner)
+        from . import (pasta_coo_norm2, pasta_cpals_prepare, pasta_cpals_solve, pasta_gram,
+                       pasta_mttkrp_coo, pasta_normalize_columns, pasta_rows_times,
+                       pasta_rows_times_bcast, pasta_weighted_inner)
         N, R = self.order, self.R
         dev = factors[0].device
         grams = [pasta_gram(u) for u in factors]  # factors are replicated: full grams locally
@@ -106,6 +157,19 @@ class RowPartitionedCPALS(RowPartitionedMTTKRP):
                 lo, hi = int(self.bounds[n][self.rank]), int(self.bounds[n][self.rank + 1])
                 M = pasta_mttkrp_coo(self.shards[n], n, factors, out=self.out[n])
                 others = [grams[k] for k in range(N) if k != n]
+                if fused:
+                    GM = _all_reduce(pasta_gram(M[lo:hi]))
+                    Wn, grams[n], lam = pasta_cpals_prepare(GM, others)
+                    if replicas is not None:
+                        # every rank finished reading U_n (its MTTKRPs precede the all-reduce
+                        # above); after the P2P stores, a collective orders the peers' reads
+                        pasta_rows_times_bcast(M, lo, hi, Wn, replicas.dsts[n])
+                        _all_reduce(torch.zeros(1, dtype=torch.float64, device=dev))
+                        continue
+                    pasta_rows_times(M[lo:hi], Wn, U=factors[n][lo:hi])
+                    if self.world > 1:
+                        gather_rows(factors[n], self.bounds[n])
+                    continue
                 colsq = torch.zeros(R, dtype=torch.float64, device=dev)
                 pasta_cpals_solve(M[lo:hi], others, U=factors[n][lo:hi], colsq=colsq)
                 _all_reduce(colsq)

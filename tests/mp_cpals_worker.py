@@ -1,5 +1,8 @@
 """Worker for tests/test_gpu_multirank.py: 2 ranks sharing cuda:0 (gloo) run the
-row-partitioned CP-ALS and must match the single-process CP-ALS oracle's fit."""
+row-partitioned CP-ALS and must match the single-process CP-ALS oracle's fit.
+PASTA_TEST_EXCHANGE=p2p: factors live in IPC-exportable replicas and the factor update
+stores every rank's rows into both replicas (pasta_rows_times_bcast through CUDA IPC);
+=unfused: the solve / normalise / gram sequence with NCCL-style broadcasts."""
 import os
 import sys
 
@@ -25,8 +28,32 @@ def main():
     U0 = si.factors(dims, R, seed=13)
     x = pasta.pasta_coo_from_arrays(dims, inds, vals)
     runner = RowPartitionedCPALS(x, rank, world, R, torch.device("cuda", 0))
-    Ud = [torch.from_numpy(u.copy()).cuda() for u in U0]
-    lam, fits = runner.run(Ud, max_iters=3, tol=0.0)
+    mode = os.environ.get("PASTA_TEST_EXCHANGE", "nccl")
+    reps = None
+    if mode == "p2p":
+        from paper_conf_iiswc_lilwlob20_b200.parallel import PeerReplicas
+        reps = PeerReplicas(dims, R)
+        for k in range(len(dims)):
+            reps.tensors[k].copy_(torch.from_numpy(U0[k]))
+        torch.cuda.synchronize()
+        dist.barrier()
+        Ud = reps.tensors
+    else:
+        Ud = [torch.from_numpy(u.copy()).cuda() for u in U0]
+    lam, fits = runner.run(Ud, max_iters=3, tol=0.0, fused=(mode != "unfused"), replicas=reps)
+    if reps is not None:
+        torch.cuda.synchronize()
+        dist.barrier()
+        # both replicas hold identical factors after the fused exchange
+        local = [t.cpu() for t in reps.tensors]
+        allf = [None] * world
+        dist.all_gather_object(allf, [t.numpy() for t in local])
+        same = all(np.array_equal(allf[0][k], allf[q][k]) for q in range(world) for k in range(len(dims)))
+        dist.barrier()
+        reps.close()
+        if not same:
+            print("replicas differ", flush=True)
+            sys.exit(4)
     _, lam_o, fits_o = cp_als(dims, inds, vals, U0, iters=3)
     ok = np.allclose(fits, fits_o, atol=2e-4) and np.allclose(lam, lam_o, rtol=2e-3)
     flag = torch.tensor([1 if ok else 0])

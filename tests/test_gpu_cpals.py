@@ -44,10 +44,33 @@ def test_building_blocks(env):
         assert np.allclose(np.linalg.norm(Uo.cpu().numpy().astype(np.float64), axis=0), 1.0, atol=1e-5)
 
 
+def test_fused_update_blocks(env):
+    """pasta_cpals_prepare + pasta_rows_times == solve -> normalise -> gram (numpy fp64)."""
+    pasta, oracle, torch = env
+    rng = np.random.default_rng(1)
+    for R in (1, 7, 16, 32, 64):
+        grams = [pasta.pasta_gram(torch.from_numpy(rng.uniform(0, 1, (400, R)).astype(np.float32)).cuda())
+                 for _ in range(2)]
+        M = rng.uniform(-1, 1, size=(3000, R)).astype(np.float32)
+        Md = torch.from_numpy(M).cuda()
+        GM = pasta.pasta_gram(Md)
+        Wn, Gn, lam = pasta.pasta_cpals_prepare(GM, grams)
+        U = pasta.pasta_rows_times(Md, Wn).cpu().numpy().astype(np.float64)
+        V = grams[0].cpu().numpy() * grams[1].cpu().numpy()
+        Uref = np.linalg.solve(V.T, M.astype(np.float64).T).T
+        lref = np.linalg.norm(Uref, axis=0)
+        assert np.allclose(lam.cpu().numpy(), lref, rtol=1e-4), R
+        Un = Uref / lref
+        assert np.allclose(U, Un, rtol=1e-3, atol=1e-4 * np.abs(Un).max()), R
+        assert np.allclose(Gn.cpu().numpy(), Un.T @ Un, atol=1e-4), R
+
+
+@pytest.mark.parametrize("fused", ["1", "0"])
 @pytest.mark.parametrize("dims,nnz,R,iters", [((60, 50, 40), 8000, 8, 1), ((60, 50, 40), 8000, 8, 3),
                                                ((40, 30, 20, 10), 6000, 16, 2)])
-def test_cpals_matches_oracle(env, dims, nnz, R, iters):
+def test_cpals_matches_oracle(env, dims, nnz, R, iters, fused, monkeypatch):
     pasta, oracle, torch = env
+    monkeypatch.setenv("PASTA_CPALS_FUSED", fused)
     from oracle.cpals import cp_als
     inds, vals = si.powerlaw_coo(dims, nnz, seed=nnz + R)
     U0 = si.factors(dims, R, seed=R)

@@ -52,6 +52,8 @@ def test_bench_two_ranks_shared_gpu():
     assert len(lines) == 1 and json.loads(lines[0])["impl"] == "reference"
 
 
-def test_row_partitioned_cpals_two_ranks_gloo():
-    r = _torchrun([os.path.join(ROOT, "tests", "mp_cpals_worker.py")])
+@pytest.mark.parametrize("exchange", ["nccl", "unfused", "p2p"])
+def test_row_partitioned_cpals_two_ranks_gloo(exchange):
+    """exchange = p2p: the fused factor update + all-gather over CUDA-IPC peer memory."""
+    r = _torchrun([os.path.join(ROOT, "tests", "mp_cpals_worker.py")], {"PASTA_TEST_EXCHANGE": exchange})
     assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-4000:]

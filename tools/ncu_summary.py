@@ -48,7 +48,7 @@ def launches(path, out):
     for k, (n, t) in agg.items():
         lines.append(f"| {n} | {t:.3f} | {t / n:.4f} | `{k}` |")
     # the last bench steps: mttkrp vs zero-fill share
-    mt = [t for n, t in seq if "mttkrp_kernel" in n and "CooSrc" in n]
+    mt = [t for n, t in seq if ("mttkrp_kernel" in n and "CooSrc" in n) or "coo_staged_kernel" in n]
     ht = [t for n, t in seq if "mttkrp_kernel" in n and "Hicoo" in n]
     zf = [t for n, t in seq if "zero_rows_kernel" in n]
     zc = zf[: len(mt)]  # bench order: every COO launch is preceded by its zero-fill
@@ -75,7 +75,7 @@ WANT = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum
         "smsp__inst_executed.sum"]
 
 
-def full(path, config, out):
+def full(path, config, out, family=None):
     txt = subprocess.check_output(["ncu", "-i", path, "--page", "raw", "--csv"], text=True)
     rows = list(csv.reader(io.StringIO(txt)))
     hdr, units, data = rows[0], rows[1], rows[2:]
@@ -103,7 +103,11 @@ def full(path, config, out):
     summ_path = os.path.join(ROOT, "profiles", "ncu_summary.json")
     summ = json.load(open(summ_path)) if os.path.exists(summ_path) else {}
     for kname, lst in per.items():
-        fam = "hicoo_mttkrp" if "Hicoo" in kname else ("coo_mttkrp" if "CooSrc" in kname else None)
+        fam = "hicoo_mttkrp" if "Hicoo" in kname else (
+            "coo_mttkrp" if ("CooSrc" in kname or "coo_staged" in kname) else (
+                "ew" if "ew_kernel" in kname else None))
+        if family:
+            fam = family
         if not fam:
             continue
         db = [to_bytes(v["dram__bytes_read.sum"]) + to_bytes(v["dram__bytes_write.sum"]) for v in lst]
@@ -119,4 +123,4 @@ if __name__ == "__main__":
     if sys.argv[1] == "launches":
         launches(sys.argv[2], sys.argv[3])
     else:
-        full(sys.argv[2], sys.argv[3], sys.argv[4])
+        full(sys.argv[2], sys.argv[3], sys.argv[4], sys.argv[5] if len(sys.argv) > 5 else None)
