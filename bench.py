@@ -358,6 +358,38 @@ def main():
                                                    ((elapsed_ms / args.steps + g_ms) * 1e-3) / 1e9, 3),
                      "how": "in-place uneven all-gather of owned output rows: one NCCL broadcast "
                             "per rank per mode (parallel.gather_rows)"}
+        # the same exchange by peer stores over NVLink (CUDA IPC replicas, pasta_bcast_f32)
+        try:
+            from paper_conf_iiswc_lilwlob20_b200.parallel import PeerReplicas, gather_rows_p2p
+            reps = PeerReplicas(dims, R)
+            flag = torch.zeros(1, device=dev)
+
+            def p2p_step():
+                for n in range(N):
+                    gather_rows_p2p(reps, n, part.bounds[n], rank)
+                dist.all_reduce(flag)  # orders the peers' reads after the stores
+
+            for _ in range(2):
+                p2p_step()
+            torch.cuda.synchronize()
+            dist.barrier()
+            g0.record(stream)
+            for _ in range(gsteps):
+                p2p_step()
+            g1.record(stream)
+            torch.cuda.synchronize()
+            dist.barrier()
+            t = torch.tensor([g0.elapsed_time(g1) / gsteps], device=dev)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            p_ms = float(t.item())
+            allgather["p2p"] = {"ms_per_step": round(p_ms, 4),
+                                "gbs_per_rank": round(recv / (p_ms * 1e-3) / 1e9, 1),
+                                "how": "owned rows stored into every peer's replica by one kernel "
+                                       "per mode (CUDA IPC P2P stores) + a 1-element all-reduce"}
+            dist.barrier()
+            reps.close()
+        except Exception as e:  # e.g. no IPC between the ranks' GPUs
+            allgather["p2p"] = {"unavailable": str(e)[:200]}
     if world > 1 and args.e2e_steps > 0:
         hf = [u.cpu().pin_memory() for u in U]
         own = [(int(part.bounds[n][rank]), int(part.bounds[n][rank + 1])) for n in range(N)]
@@ -460,6 +492,39 @@ def main():
                          "per-sweep fit read-back"}
         del Uc
 
+    # NEXT-3: semi-sparse TTM (R) and TTV along mode 0 (Table I: TTM 4MR + 4M_F R + 16M_F + 8M,
+    # TTV 12M + 12M_F bytes; 2MR / 2M flops); fibers are pre-processing
+    ttm = None
+    if world == 1 and args.ew_steps > 0:
+        t0 = time.perf_counter()
+        MF = pasta.pasta_coo_fibers(x, 0)
+        torch.cuda.synchronize()
+        t_fib = time.perf_counter() - t0
+        Ut = torch.rand((dims[0], R), device=dev)
+        vt = torch.rand(dims[0], device=dev)
+        yt = torch.empty((MF, R), device=dev)
+        yv = torch.empty(MF, device=dev)
+        peak_t, _ = load_peaks()
+        ttm = {"mode": 0, "fibers": MF, "preprocess_s": round(t_fib, 3)}
+        for name, fn, nbytes, flops in (
+                ("ttm", lambda: pasta.pasta_ttm_coo(x, 0, Ut, out=yt), 4 * M * R + 4 * MF * R + 16 * MF + 8 * M,
+                 2 * M * R),
+                ("ttv", lambda: pasta.pasta_ttv_coo(x, 0, vt, out=yv), 12 * M + 12 * MF, 2 * M)):
+            for _ in range(3):
+                fn()
+            torch.cuda.synchronize()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            for _ in range(args.ew_steps):
+                fn()
+            e1.record(stream)
+            torch.cuda.synchronize()
+            ms = e0.elapsed_time(e1) / args.ew_steps
+            gbs = nbytes / (ms * 1e-3) / 1e9
+            ttm[name] = {"ms": round(ms, 4), "GFLOP/s": round(flops / (ms * 1e-3) / 1e9, 1),
+                         "model_gbs": round(gbs, 1), "frac": round(gbs / peak_t, 4)}
+        del Ut, vt, yt, yv
+
     # NEXT-4: TS and same-pattern TEW on the tensor's value array (Table I: TS 8M bytes, TEW
     # 12M bytes, M flops) -- the streaming kernels that bound the HBM roofline
     ew = None
@@ -503,6 +568,17 @@ def main():
     launch_bytes = sum(model_bytes_coo(N, m, R) for m in my_launch_nnz) / N
     achieved = launch_bytes / (avg_launch_ms * 1e-3) / 1e9
     traffic = ncu_traffic(args.config) if world == 1 else None
+    # SURVEY 8(d) compulsory bytes per launch (the honest lower bound): the stream, every
+    # distinct gathered factor row once, the output rows once
+    compulsory = None
+    if world == 1:
+        touched = [int(np.count_nonzero(pasta.pasta_coo_row_counts(x, k))) for k in range(N)]
+        cb = sum(4 * (N + 1) * M + 4 * R * sum(touched[k] for k in range(N) if k != n) + 4 * R * dims[n]
+                 for n in range(N)) / N
+        cg = cb / (avg_launch_ms * 1e-3) / 1e9
+        compulsory = {"bytes_per_launch": round(cb), "gbs": round(cg, 1), "frac": round(cg / peak, 4),
+                      "touched_rows": touched,
+                      "def": "4(N+1)M + 4R sum_{k!=n} touched_k + 4R I_n, averaged over modes"}
 
     cpu = None
     if not args.no_cpu_baseline and world == 1:
@@ -536,6 +612,7 @@ def main():
                      if traffic else None,
                      "note": "frac uses the paper's byte model, which counts every factor gather as a "
                              "DRAM access (P:117); dram_* use the ncu-measured traffic"},
+        "compulsory": compulsory,
         "zero_fill_ms_per_step": round(zero_ms / args.steps, 4),
         "preprocess_s": {"generate": round(t_gen, 3), "mode_sort_all": round(t_prep, 3)},
         "clocks": clk,
@@ -545,6 +622,7 @@ def main():
         "ghicoo": ghicoo,
         "cpals": cpals,
         "ew": ew,
+        "ttm": ttm,
         "gpu_launches": launches,
         "cpu_baseline": cpu,
         "max_shard_nnz": per_launch_nnz,

@@ -246,6 +246,12 @@ pasta_status pasta_rows_times_bcast(const float *M, uint64_t row_lo, uint64_t ro
  * pasta_ipc_get_handle writes its PASTA_IPC_HANDLE_BYTES-byte handle; another process maps
  * it with pasta_ipc_open (peer access enabled lazily) and unmaps with pasta_ipc_close. */
 #define PASTA_IPC_HANDLE_BYTES 64
+/* The all-gather of owned rows by peer stores (a9): dsts[k][i] = src[i] for i < n and each of
+ * the `ndst` (1..8) destinations (local or pasta_ipc_open-mapped peer buffers, all 16-byte
+ * aligned; EINVAL otherwise).  Ends with a system-scope fence; the caller orders the peers'
+ * reads after it. */
+pasta_status pasta_bcast_f32(const float *src, uint64_t n, float *const *dsts, uint32_t ndst,
+                             void *stream);
 pasta_status pasta_dev_alloc(uint64_t bytes, void **ptr);
 pasta_status pasta_dev_free(void *ptr);
 pasta_status pasta_ipc_get_handle(void *base, void *handle);

@@ -26,7 +26,7 @@ __all__ = [
     "pasta_cpals_solve", "pasta_normalize_columns", "pasta_weighted_inner", "pasta_coo_norm2",
     "pasta_cpals_coo", "pasta_coo_fibers", "pasta_coo_fiber_export", "pasta_ttm_coo",
     "pasta_ttv_coo", "pasta_coo_to_ghicoo", "pasta_ghicoo_auto_mask", "pasta_ghicoo_export",
-    "pasta_cpals_prepare", "pasta_rows_times", "pasta_rows_times_bcast", "pasta_dev_alloc",
+    "pasta_cpals_prepare", "pasta_rows_times", "pasta_rows_times_bcast", "pasta_bcast_f32", "pasta_dev_alloc",
     "pasta_dev_free", "pasta_ipc_get_handle", "pasta_ipc_open", "pasta_ipc_close", "pasta_ts", "pasta_tew", "pasta_coo_values_ptr", "pasta_coo_ts", "pasta_coo_tew", "OPS",
 ]
 
@@ -624,6 +624,13 @@ def pasta_rows_times_bcast(M, row_lo: int, row_hi: int, Wn, dst_ptrs, stream=Non
     dp = (C.c_void_p * len(dst_ptrs))(*[int(p) for p in dst_ptrs])
     check(lib().pasta_rows_times_bcast(_dptr(M), int(row_lo), int(row_hi), R, _dptr(Wn), dp,
                                        len(dst_ptrs), _stream_ptr(stream)))
+
+
+def pasta_bcast_f32(src, dst_ptrs, stream=None) -> None:
+    """Copy the contiguous float32 tensor ``src`` to every device address in ``dst_ptrs``
+    (peer stores; the P2P all-gather of owned rows)."""
+    dp = (C.c_void_p * len(dst_ptrs))(*[int(p) for p in dst_ptrs])
+    check(lib().pasta_bcast_f32(_dptr(src), src.numel(), dp, len(dst_ptrs), _stream_ptr(stream)))
 
 
 class _CudaArray:

@@ -88,6 +88,7 @@ SIGNATURES = {
     "pasta_rows_times": (_st, [_vp, C.c_uint64, C.c_uint32, _vp, _vp, _vp]),
     "pasta_rows_times_bcast": (_st, [_vp, C.c_uint64, C.c_uint64, C.c_uint32, _vp, C.POINTER(_vp),
                                      C.c_uint32, _vp]),
+    "pasta_bcast_f32": (_st, [_vp, C.c_uint64, C.POINTER(_vp), C.c_uint32, _vp]),
     "pasta_dev_alloc": (_st, [C.c_uint64, C.POINTER(_vp)]),
     "pasta_dev_free": (_st, [_vp]),
     "pasta_ipc_get_handle": (_st, [_vp, _vp]),

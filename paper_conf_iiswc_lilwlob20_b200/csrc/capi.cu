@@ -752,6 +752,15 @@ pasta_status pasta_rows_times_bcast(const float *M, uint64_t row_lo, uint64_t ro
 }
 
 // ---------------------------------------------------------------------------- peer memory
+pasta_status pasta_bcast_f32(const float *src, uint64_t n, float *const *dsts, uint32_t ndst, void *stream) {
+  API_BEGIN
+  require((src && dsts) || n == 0, "NULL argument");
+  for (uint32_t k = 0; k < ndst && dsts; ++k) require(dsts[k] != nullptr, "dsts[k] is NULL");
+  launch_bcast(src, n, dsts, ndst, as_stream(stream));
+  API_END
+}
+
+
 pasta_status pasta_dev_alloc(uint64_t bytes, void **ptr) {
   API_BEGIN
   require(ptr != nullptr, "ptr is NULL");

@@ -281,6 +281,7 @@ bool is_lex_sorted_device(const uint32_t *const *inds, uint32_t order, uint64_t 
 void launch_ts(uint32_t op, const float *x, float s, float *y, uint64_t n, cudaStream_t st);
 void launch_tew(uint32_t op, const float *a, const float *b, float *z, uint64_t n, cudaStream_t st);
 bool same_pattern_device(const pasta_coo *x, const pasta_coo *y, cudaStream_t s);
+void launch_bcast(const float *src, uint64_t n, float *const *dsts, uint32_t ndst, cudaStream_t st);
 void copy_pattern_device(const pasta_coo *x, pasta_coo *y, cudaStream_t s);
 void tew_merge_device(const pasta_coo *x, const pasta_coo *y, uint32_t op, pasta_coo *z, cudaStream_t s);
 

@@ -926,7 +926,8 @@ void launch_coo_mttkrp(const pasta_coo *x, uint32_t mode, const float *const *fa
   const bool vec4 = vec4_ok(x->order, mode, factors, R, out);
   const int staged = env_int("PASTA_COO_STAGED", 1);
   const int no = int(x->order) - 1;
-  if (staged && vec4 && (R == 16 || R == 32) && (no == 2 || no == 3)) {
+  // no == 1: order-2 matrices, e.g. the fiberised (fiber, i_n) matrix of TTM (ttm.cu)
+  if (staged && vec4 && (R == 16 || R == 32) && (no >= 1 && no <= 3)) {
     // the hot-row cache pays only when the gathered factors do not fit in L2 already
     static int l2 = 0;
     if (!l2) {
@@ -999,7 +1000,9 @@ void launch_coo_mttkrp(const pasta_coo *x, uint32_t mode, const float *const *fa
     const int wa = env_int("PASTA_STAGED_WA", 1);
     auto pick = [&](auto tag) {
       constexpr int W = decltype(tag)::value;
-      if (no == 2 && lpn == 4) go(coo_staged_kernel<2, 4, W>);
+      if (no == 1 && lpn == 4) go(coo_staged_kernel<1, 4, 1>);  // one code path for order 2
+      else if (no == 1) go(coo_staged_kernel<1, 8, 1>);
+      else if (no == 2 && lpn == 4) go(coo_staged_kernel<2, 4, W>);
       else if (no == 2) go(coo_staged_kernel<2, 8, W>);
       else if (lpn == 4) go(coo_staged_kernel<3, 4, W>);
       else go(coo_staged_kernel<3, 8, W>);

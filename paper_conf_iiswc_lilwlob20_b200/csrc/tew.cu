@@ -236,6 +236,27 @@ __global__ void copy_u32_kernel(const uint32_t *__restrict__ a, uint32_t *__rest
     b[i] = a[i];
 }
 
+// All-gather by peer stores (a9): a contiguous float range copied into up to 8 replicas
+// (local and CUDA-IPC-mapped peers); 128-bit loads once, one 128-bit store per replica.
+struct Dst8 {
+  float *d[8];
+  uint32_t n;
+};
+
+__global__ void __launch_bounds__(kThreads) bcast_kernel(const float *__restrict__ src, uint64_t n, Dst8 dst) {
+  uint64_t pol;
+  asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+  const uint64_t n4 = n / 4, stride = uint64_t(gridDim.x) * kThreads;
+  const float4 *s4 = reinterpret_cast<const float4 *>(src);
+  for (uint64_t i = uint64_t(blockIdx.x) * kThreads + threadIdx.x; i < n4; i += stride) {
+    const float4 v = ld_stream(s4 + i, pol);
+    for (uint32_t k = 0; k < dst.n; ++k) reinterpret_cast<float4 *>(dst.d[k])[i] = v;
+  }
+  for (uint64_t e = n4 * 4 + uint64_t(blockIdx.x) * kThreads + threadIdx.x; e < n; e += stride)
+    for (uint32_t k = 0; k < dst.n; ++k) dst.d[k][e] = src[e];
+  __threadfence_system();
+}
+
 }  // namespace
 
 void launch_ts(uint32_t op, const float *x, float s, float *y, uint64_t n, cudaStream_t st) {
@@ -244,6 +265,21 @@ void launch_ts(uint32_t op, const float *x, float s, float *y, uint64_t n, cudaS
 
 void launch_tew(uint32_t op, const float *a, const float *b, float *z, uint64_t n, cudaStream_t st) {
   launch_ew<false>(op, a, b, 0.f, z, n, st);
+}
+
+void launch_bcast(const float *src, uint64_t n, float *const *dsts, uint32_t ndst, cudaStream_t st) {
+  if (ndst < 1 || ndst > 8) fail(PASTA_EINVAL, "pasta_bcast_f32: 1..8 destinations");
+  if (n == 0) return;
+  Dst8 d{};
+  d.n = ndst;
+  bool al = aligned16(src);
+  for (uint32_t k = 0; k < ndst; ++k) { d.d[k] = dsts[k]; al = al && aligned16(dsts[k]); }
+  if (!al) fail(PASTA_EINVAL, "pasta_bcast_f32: pointers must be 16-byte aligned");
+  uint64_t want = (n / 4 + kThreads - 1) / kThreads;
+  uint64_t grid = uint64_t(sms()) * 8;
+  if (want < grid) grid = want ? want : 1;
+  bcast_kernel<<<unsigned(grid), kThreads, 0, st>>>(src, n, d);
+  PASTA_LAUNCHED();
 }
 
 bool same_pattern_device(const pasta_coo *x, const pasta_coo *y, cudaStream_t s) {

@@ -73,6 +73,20 @@ class RowPartitionedMTTKRP:
         return self.out
 
 
+def gather_rows_p2p(replicas, k: int, bounds: Sequence[int], rank: int, stream=None) -> None:
+    """All-gather of this rank's owned rows [bounds[rank], bounds[rank+1]) of replica k by
+    peer stores (pasta_bcast_f32 into every rank's replica).  The caller orders the peers'
+    reads after it with a collective."""
+    from . import pasta_bcast_f32
+    lo, hi = int(bounds[rank]), int(bounds[rank + 1])
+    if hi <= lo or len(replicas.dsts[k]) < 2:
+        return
+    t = replicas.tensors[k]
+    R = int(t.shape[1])
+    off = lo * R * 4
+    pasta_bcast_f32(t[lo:hi], [p + off for p in replicas.dsts[k][1:]], stream=stream)
+
+
 class PeerReplicas:
     """Replicated factor matrices in IPC-exportable device memory, with every peer's replicas
     mapped into this process (CUDA IPC over NVLink / NVSwitch).  ``tensors[k]`` is this rank's

@@ -49,6 +49,19 @@ def main():
         allf = [None] * world
         dist.all_gather_object(allf, [t.numpy() for t in local])
         same = all(np.array_equal(allf[0][k], allf[q][k]) for q in range(world) for k in range(len(dims)))
+        # the plain P2P all-gather of owned rows: rank-tagged rows land in every replica
+        from paper_conf_iiswc_lilwlob20_b200.parallel import gather_rows_p2p
+        b = runner.bounds[0]
+        lo, hi = int(b[rank]), int(b[rank + 1])
+        reps.tensors[0][lo:hi] = float(rank + 1)
+        torch.cuda.synchronize()
+        dist.barrier()
+        gather_rows_p2p(reps, 0, b, rank)
+        torch.cuda.synchronize()
+        dist.barrier()
+        t0 = reps.tensors[0].cpu()
+        for q in range(world):
+            same = same and bool((t0[int(b[q]):int(b[q + 1])] == float(q + 1)).all())
         dist.barrier()
         reps.close()
         if not same:

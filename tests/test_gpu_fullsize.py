@@ -101,3 +101,80 @@ def test_fullsize_hicoo_conversion_and_mode_sort_bit_exact(env):
     gi, gv = pasta.pasta_coo_export_mode(x, 3)
     oi, ov = oracle.mode_sort(inds, vals, 3)
     assert np.array_equal(gi, oi) and np.array_equal(gv.view(np.uint32), ov.view(np.uint32))
+
+
+@pytest.mark.parametrize("key", ["h", "c3"])
+def test_fullsize_ghicoo_sampled_rows(env, key):
+    """gHiCOO (NEXT-2) with the storage-minimising mask, as bench.py times it, at full size."""
+    pasta, oracle, torch = env
+    cfg = si.CONFIGS[key]
+    dims, R, M = cfg["dims"], cfg["R"], cfg["nnz"]
+    inds, vals = si.powerlaw_coo(dims, M, seed=cfg["seed"] + 91, dedup=False)
+    g = torch.Generator(device="cuda")
+    g.manual_seed(7)
+    Ud = [torch.rand((d, R), generator=g, device="cuda") for d in dims]
+    U = [u.cpu().numpy() for u in Ud]
+    x = pasta.pasta_coo_from_arrays(dims, inds, vals)
+    gh = pasta.pasta_coo_to_ghicoo(x, 7, 0)
+    assert 0 < gh.cmask < (1 << len(dims))
+    rng = np.random.default_rng(2)
+    for n in range(len(dims)):
+        rows = _sample_rows(inds[n], dims[n], rng)
+        ref, ab = oracle.mttkrp_rows(dims, inds, vals, n, U, rows)
+        got = pasta.pasta_mttkrp_hicoo(gh, n, Ud)[torch.from_numpy(rows.astype(np.int64)).cuda()].cpu().numpy()
+        excess = np.abs(got.astype(np.float64) - ref) - (1e-4 * ab + 1e-6)
+        assert excess.max() <= 0, f"{key} ghicoo mask {gh.cmask:b} mode {n}: excess {excess.max():.3e}"
+        del ref, ab
+
+
+def test_fullsize_ghicoo_conversion_bit_exact(env):
+    pasta, oracle, torch = env
+    cfg = si.CONFIGS["c4"]
+    dims, M = cfg["dims"], cfg["nnz"]
+    inds, vals = si.powerlaw_coo(dims, M, seed=cfg["seed"] + 6, dedup=False)
+    x = pasta.pasta_coo_from_arrays(dims, inds, vals)
+    mask = 0b0101
+    gx = pasta.pasta_ghicoo_export(pasta.pasta_coo_to_ghicoo(x, 7, mask))
+    o = oracle.coo_to_ghicoo(inds, vals, 7, mask)
+    assert gx["nblocks"] == o["nblocks"]
+    assert np.array_equal(gx["bptr"], o["bptr"])
+    for k in range(4):
+        for key in ("binds", "einds", "uinds"):
+            if o[key][k] is not None:
+                assert np.array_equal(gx[key][k], o[key][k]), (key, k)
+    assert np.array_equal(gx["vals"].view(np.uint32), o["vals"].view(np.uint32))
+
+
+def test_fullsize_ts_tew_bit_exact(env):
+    """TEW / TS (NEXT-4) on the bench's 100M-element value arrays, every element."""
+    pasta, oracle, torch = env
+    M = si.CONFIGS["h"]["nnz"]
+    rng = np.random.default_rng(3)
+    a = rng.uniform(-1, 1, M).astype(np.float32)
+    b = rng.uniform(-1, 1, M).astype(np.float32)
+    ad, bd = torch.from_numpy(a).cuda(), torch.from_numpy(b).cuda()
+    for op in ("mul", "div"):
+        got = pasta.pasta_ts(ad, op, 0.5).cpu().numpy()
+        assert np.array_equal(got.view(np.uint32), oracle.ts(a, op, np.float32(0.5)).view(np.uint32)), op
+    for op in ("add", "sub"):
+        got = pasta.pasta_tew(ad, bd, op).cpu().numpy()
+        assert np.array_equal(got.view(np.uint32), oracle.tew_same(a, b, op).view(np.uint32)), op
+
+
+def test_fullsize_slice_powerlaw_contains_oracle_prefix(env):
+    """irrL-shaped (Table II s6: (4.2M)^2 x 168, 84M nonzeros) slice power-law tensor on the GPU
+    contains the oracle's independently generated first 200k distinct nonzeros, same values."""
+    pasta, oracle, torch = env
+    dims, M, seed = (4_200_000, 4_200_000, 168), 84_000_000, 1006
+    x = pasta.pasta_gen_powerlaw(dims, M, seed, kind=2)
+    gi, gv = pasta.pasta_coo_export(x)
+    assert gi.shape == (3, M)
+    oi, ov = oracle.gen_slice_powerlaw(dims, 200_000, seed)
+    key_g = (gi[0].astype(np.uint64) << np.uint64(40)) | (gi[1].astype(np.uint64) << np.uint64(8)) \
+        | gi[2].astype(np.uint64)
+    key_o = (oi[0].astype(np.uint64) << np.uint64(40)) | (oi[1].astype(np.uint64) << np.uint64(8)) \
+        | oi[2].astype(np.uint64)
+    assert np.all(key_g[1:] > key_g[:-1])  # lexicographic, distinct
+    pos = np.searchsorted(key_g, key_o)
+    assert np.all(pos < M) and np.array_equal(key_g[pos], key_o)
+    assert np.array_equal(gv[pos].view(np.uint32), ov.view(np.uint32))
