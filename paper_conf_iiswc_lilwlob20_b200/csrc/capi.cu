@@ -969,7 +969,30 @@ pasta_status pasta_ttm_coo(pasta_coo *x, uint32_t mode, const float *U, uint32_t
 }
 
 pasta_status pasta_ttv_coo(pasta_coo *x, uint32_t mode, const float *v, float *out, void *stream) {
-  return pasta_ttm_coo(x, mode, v, 1, out, stream);
+  API_BEGIN
+  require(x && v && out, "x/v/out is NULL");
+  require(mode < x->order, "mode >= order");
+  check_device(x->device);
+  cudaStream_t s = as_stream(stream);
+  if (!x->fib[mode]) {
+    std::lock_guard<std::mutex> lk(x->mu);
+    coo_build_fibers(x, mode, s);
+  }
+  FiberCopy &f = *x->fib[mode];
+  if (!f.mat.mc[0].ready) {
+    std::lock_guard<std::mutex> lk(f.mat.mu);
+    coo_prepare_mode(&f.mat, 0, s);
+  }
+  launch_zero_rows(out, 0, f.nf, 1, s);
+  // PASTA_TTV_SEGSUM=0: the R = 1 MTTKRP path of pasta_ttm_coo instead of the segmented sum
+  const char *e = getenv("PASTA_TTV_SEGSUM");
+  if (e && *e == '0') {
+    const float *fac[2] = {nullptr, v};
+    launch_coo_mttkrp(&f.mat, 0, fac, 1, out, s);
+  } else {
+    launch_ttv(f.mat, v, out, s);
+  }
+  API_END
 }
 
 // ---------------------------------------------------------------------------- introspection

@@ -269,6 +269,8 @@ void launch_inner(const float *A, const float *B, uint64_t rows, uint32_t R, con
 void launch_sumsq(const float *v, uint64_t n, double *out, cudaStream_t s);
 void coo_mark_hot(pasta_coo *x, uint32_t mode, uint32_t R, cudaStream_t s);
 void coo_build_fibers(pasta_coo *x, uint32_t mode, cudaStream_t s);
+// TTV on the fiberised matrix (warp-level segmented reduction); y zeroed by the caller
+void launch_ttv(const pasta_coo &mat, const float *v, float *y, cudaStream_t s);
 void launch_hot_fill(const CooModeCopy &mc, const float *const *factors, uint32_t order, uint32_t mode,
                      uint32_t R, cudaStream_t s);
 void row_counts_device(const uint32_t *rows, uint64_t nnz, uint32_t nrows, uint64_t *counts_host,

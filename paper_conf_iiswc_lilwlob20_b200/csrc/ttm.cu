@@ -49,6 +49,95 @@ __global__ void u32_to_u8_kernel(const uint32_t *__restrict__ in, uint64_t M, ui
     out[x] = uint8_t(in[x]);
 }
 
+// TTV (Eq. 1) on the fiberised matrix: y[f] = sum_{x in fiber f} val[x] * v[i_n[x]].
+// Warp-level segmented reduction (the north_star's "warp-level segmented reduction
+// (shuffles) over runs of equal output index, and atomics only at segment boundaries"): a warp
+// takes a tile of 128 consecutive nonzeros, lane l the 4 at 4l (128-bit loads of fiber ids,
+// i_n and values: fully coalesced); runs inside a lane are summed in registers; the lanes'
+// trailing runs are combined by a 5-step segmented Kogge-Stone scan with shuffles; a run is
+// written by the lane where it ends -- a plain store when it lies inside the tile (the fiber
+// is exclusively this warp's), an atomicAdd when it touches the tile's first or last entry
+// (it may continue in the neighbouring tile).  y must be zeroed.
+__global__ void __launch_bounds__(256) ttv_segsum_kernel(const uint32_t *__restrict__ fid,
+                                                         const uint32_t *__restrict__ in,
+                                                         const float *__restrict__ val,
+                                                         const float *__restrict__ v, uint64_t M,
+                                                         float *__restrict__ y) {
+  constexpr uint32_t kNone = 0xFFFFFFFFu;
+  const unsigned full = 0xFFFFFFFFu;
+  const int lane = threadIdx.x & 31;
+  const uint64_t warp = (uint64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5;
+  const uint64_t nwarps = (uint64_t(gridDim.x) * blockDim.x) >> 5;
+  for (uint64_t t0 = warp * 128; t0 < M; t0 += nwarps * 128) {
+    const uint64_t x = t0 + 4 * uint64_t(lane);
+    uint32_t f[4];
+    float p[4];
+    if (x + 3 < M) {
+      const uint4 a = __ldg(reinterpret_cast<const uint4 *>(fid + x));
+      const uint4 b = __ldg(reinterpret_cast<const uint4 *>(in + x));
+      const float4 c = __ldg(reinterpret_cast<const float4 *>(val + x));
+      f[0] = a.x; f[1] = a.y; f[2] = a.z; f[3] = a.w;
+      p[0] = c.x * __ldg(v + b.x); p[1] = c.y * __ldg(v + b.y);
+      p[2] = c.z * __ldg(v + b.z); p[3] = c.w * __ldg(v + b.w);
+    } else {
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        const bool ok = x + i < M;
+        f[i] = ok ? fid[x + i] : kNone;
+        p[i] = ok ? val[x + i] * __ldg(v + in[x + i]) : 0.f;
+      }
+    }
+    const uint32_t tile_first = __shfl_sync(full, f[0], 0);
+    // lane-local runs: first run, interior runs (complete, exclusive), trailing run
+    const uint32_t ff = f[0];
+    float first_sum = p[0];
+    int i = 1;
+    while (i < 4 && f[i] == ff) first_sum += p[i++];
+    const bool single = i == 4;
+    float last_sum = first_sum;
+    uint32_t lf = ff;
+    if (!single) {
+      lf = f[i];
+      last_sum = p[i];
+      for (int j = i + 1; j < 4; ++j) {
+        if (f[j] == lf) {
+          last_sum += p[j];
+        } else {
+          y[lf] = last_sum;  // interior run: the whole fiber
+          lf = f[j];
+          last_sum = p[j];
+        }
+      }
+    }
+    const uint32_t tile_last = __shfl_sync(full, lf, 31);
+    // segmented inclusive scan of the trailing runs across lanes
+    const uint32_t plf = __shfl_up_sync(full, lf, 1);
+    bool head = !single || lane == 0 || plf != ff;
+    float sv = last_sum;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+      const float ov = __shfl_up_sync(full, sv, d);
+      const bool oh = __shfl_up_sync(full, head, d);
+      if (lane >= d) {
+        if (!head) sv += ov;
+        head = head || oh;
+      }
+    }
+    const float carry_src = __shfl_up_sync(full, sv, 1);
+    const uint32_t nff = __shfl_down_sync(full, ff, 1);
+    auto emit = [&](uint32_t fb, float val_) {
+      if (fb == kNone) return;
+      if (fb == tile_first || fb == tile_last) atomicAdd(y + fb, val_);
+      else y[fb] = val_;
+    };
+    if (!single) {
+      const float carry = (lane > 0 && plf == ff) ? carry_src : 0.f;
+      emit(ff, first_sum + carry);  // the first run ends inside this lane
+    }
+    if (lane == 31 || nff != lf) emit(lf, sv);  // the trailing run ends here
+  }
+}
+
 }  // namespace
 
 void coo_build_fibers(pasta_coo *x, uint32_t mode, cudaStream_t s) {
@@ -118,6 +207,23 @@ void coo_build_fibers(pasta_coo *x, uint32_t mode, cudaStream_t s) {
     throw;
   }
   x->fib[mode] = fc;
+}
+
+void launch_ttv(const pasta_coo &mat, const float *v, float *y, cudaStream_t s) {
+  const uint64_t M = mat.nnz;
+  if (M == 0) return;
+  const CooModeCopy &mc = mat.mc[0];
+  const bool al = ((reinterpret_cast<uintptr_t>(mc.inds[0]) | reinterpret_cast<uintptr_t>(mc.inds[1]) |
+                    reinterpret_cast<uintptr_t>(mc.val)) & 15u) == 0;
+  if (!al) fail(PASTA_ECUDA, "ttv: fiber arrays not 16-byte aligned");
+  int dev = 0, sms = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  uint64_t want = (M + 128 * 8 - 1) / (128 * 8);
+  uint64_t grid = uint64_t(sms) * 8;
+  if (want < grid) grid = want;
+  ttv_segsum_kernel<<<unsigned(grid), 256, 0, s>>>(mc.inds[0], mc.inds[1], mc.val, v, M, y);
+  PASTA_LAUNCHED();
 }
 
 }  // namespace pasta

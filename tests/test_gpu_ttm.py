@@ -55,5 +55,38 @@ def test_ttm_hot_fiber_and_empty(env):
     fib, Y, Ya = oracle.ttm(dims, inds, vals, 1, U)
     got = pasta.pasta_ttm_coo(x, 1, torch.from_numpy(U).cuda()).cpu().numpy().astype(np.float64)
     assert np.all(np.abs(got - Y) <= 1e-4 * Ya + 1e-6)
+    # TTV's warp-segmented sum: the 3000-entry fiber spans many 128-entry tiles
+    v = U[:, 0].copy()
+    fv, yv, yva = oracle.ttv(dims, inds, vals, 1, v)
+    gv = pasta.pasta_ttv_coo(x, 1, torch.from_numpy(v).cuda()).cpu().numpy().astype(np.float64)
+    assert np.all(np.abs(gv - yv) <= 1e-4 * yva + 1e-6)
     e = pasta.pasta_coo_from_arrays(dims, np.zeros((3, 0), np.uint32), np.zeros(0, np.float32))
     assert pasta.pasta_coo_fibers(e, 0) == 0
+
+
+@pytest.mark.parametrize("M,maxlen,seed", [(1, 1, 0), (127, 3, 1), (129, 200, 2), (100_003, 9, 3),
+                                           (300_001, 700, 4), (65_536, 1, 5)])
+def test_ttv_segmented_sum_run_lengths(env, M, maxlen, seed):
+    """Order-2 tensors whose mode-0 fibers (rows of X^T) have lengths 1..maxlen: fibers start
+    and end at every position relative to lanes and 128-entry tiles."""
+    pasta, oracle, torch = env
+    rng = np.random.default_rng(seed)
+    lens = []
+    tot = 0
+    while tot < M:
+        l = int(min(rng.integers(1, maxlen + 1), M - tot))
+        lens.append(l)
+        tot += l
+    nf = len(lens)
+    J = max(maxlen, 1) + 5
+    i1 = np.repeat(np.arange(nf, dtype=np.uint32), lens)
+    i0 = np.concatenate([rng.choice(J, l, replace=False) for l in lens]).astype(np.uint32)
+    inds = np.ascontiguousarray(np.stack([i0, i1]))
+    vals = rng.uniform(-1, 1, M).astype(np.float32)
+    dims = (J, nf)
+    x = pasta.pasta_coo_from_arrays(dims, inds, vals)
+    v = rng.uniform(0, 1, J).astype(np.float32)
+    fv, yv, yva = oracle.ttv(dims, inds, vals, 0, v)
+    gv = pasta.pasta_ttv_coo(x, 0, torch.from_numpy(v).cuda()).cpu().numpy().astype(np.float64)
+    assert gv.shape == yv.shape
+    assert np.all(np.abs(gv - yv) <= 1e-4 * yva + 1e-6)
