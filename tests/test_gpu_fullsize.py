@@ -27,7 +27,7 @@ def _sample_rows(inds_n, dim, rng):
     return np.unique(np.concatenate([heavy, rnd]).astype(np.uint32))
 
 
-@pytest.mark.parametrize("key", ["h", "c4"])
+@pytest.mark.parametrize("key", ["h", "c4", "c2", "c3"])
 def test_fullsize_sampled_rows(env, key):
     pasta, oracle, torch = env
     cfg = si.CONFIGS[key]
@@ -178,3 +178,28 @@ def test_fullsize_slice_powerlaw_contains_oracle_prefix(env):
     pos = np.searchsorted(key_g, key_o)
     assert np.all(pos < M) and np.array_equal(key_g[pos], key_o)
     assert np.array_equal(gv[pos].view(np.uint32), ov.view(np.uint32))
+
+
+def test_fullsize_c5_one_billion_mode0(env):
+    """BASELINE config 5 (regL-shaped, 1B nonzeros, R = 32) as the GPU generates it: mode-0
+    MTTKRP on sampled rows against the oracle over the exported tensor.  Needs ~40 GB of host
+    memory; skipped when the host has less than 96 GB available."""
+    import psutil
+    if psutil.virtual_memory().available < 96 * (1 << 30):
+        pytest.skip("needs >= 96 GB of available host memory")
+    pasta, oracle, torch = env
+    cfg = si.CONFIGS["c5"]
+    dims, R, M = cfg["dims"], cfg["R"], cfg["nnz"]
+    x = pasta.pasta_gen_powerlaw(dims, M, cfg["seed"])
+    g = torch.Generator(device="cuda")
+    g.manual_seed(11)
+    Ud = [torch.rand((d, R), generator=g, device="cuda") for d in dims]
+    got_full = pasta.pasta_mttkrp_coo(x, 0, Ud)
+    inds, vals = pasta.pasta_coo_export(x)
+    del x
+    U = [u.cpu().numpy() for u in Ud]
+    rows = _sample_rows(inds[0], dims[0], np.random.default_rng(4))[:1024]
+    ref, ab = oracle.mttkrp_rows(dims, inds, vals, 0, U, rows)
+    got = got_full[torch.from_numpy(rows.astype(np.int64)).cuda()].cpu().numpy()
+    excess = np.abs(got.astype(np.float64) - ref) - (1e-4 * ab + 1e-6)
+    assert excess.max() <= 0, f"c5 mode 0: excess {excess.max():.3e}"
