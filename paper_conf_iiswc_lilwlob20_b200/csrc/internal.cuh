@@ -111,11 +111,17 @@ struct CooModeCopy {
   const float *val = nullptr;
   DevArray<uint32_t> own_inds[kMaxOrder];
   DevArray<float> own_val;
-  // Hot-row cache (coo_mark_hot): the most frequent rows of the gathered factors, packed into
-  // one contiguous buffer that fits the L2 budget for rank hot_R.  hot_inds[k] (k != mode)
-  // = inds[k] for cold entries, 0x80000000 | slot for hot ones (slot into hot_buf).
+  // Hot-row cache (coo_mark_hot), two tiers for rank hot_R: the most frequent rows of the
+  // gathered factors in every CTA's shared memory (hs_*), the next ones packed into one
+  // contiguous buffer that fits the L2 budget (hot_*).  hot_inds[k] (k != mode) = inds[k] for
+  // cold entries, 0xC0000000 | smem slot, 0x80000000 | slot into hot_buf.
   uint32_t hot_R = 0;       // 0: not marked
-  uint32_t hot_bucket = 0;  // rows with count bucket >= hot_bucket are hot
+  bool hot_global = false;  // L2 tier requested
+  uint32_t hot_smem_budget = 0;
+  uint32_t hot_bucket = 0;  // rows with hot_bucket <= count bucket < hs_bucket: L2 tier
+  uint32_t hs_bucket = 0;   // rows with count bucket >= hs_bucket: smem tier
+  DevArray<uint32_t> hs_rows;           // smem slot -> factor row, factor k at [hs_base[k], +hs_cnt[k])
+  uint64_t hs_base[kMaxOrder] = {}, hs_cnt[kMaxOrder] = {}, hs_total = 0;
   DevArray<uint32_t> hot_inds[kMaxOrder];
   DevArray<uint32_t> hot_rows;          // slot -> factor row, factor k at [hot_base[k], +hot_cnt[k])
   uint64_t hot_base[kMaxOrder] = {}, hot_cnt[kMaxOrder] = {}, hot_total = 0;
@@ -267,7 +273,8 @@ void launch_apply_bcast(const float *M, uint64_t row_lo, uint64_t row_hi, uint32
 void launch_inner(const float *A, const float *B, uint64_t rows, uint32_t R, const double *lambda,
                   double *out, cudaStream_t s);
 void launch_sumsq(const float *v, uint64_t n, double *out, cudaStream_t s);
-void coo_mark_hot(pasta_coo *x, uint32_t mode, uint32_t R, cudaStream_t s);
+void coo_mark_hot(pasta_coo *x, uint32_t mode, uint32_t R, bool global_tier, uint32_t smem_rows,
+                  cudaStream_t s);
 void coo_build_fibers(pasta_coo *x, uint32_t mode, cudaStream_t s);
 // TTV on the fiberised matrix (warp-level segmented reduction); y zeroed by the caller
 void launch_ttv(const pasta_coo &mat, const float *v, float *y, cudaStream_t s);

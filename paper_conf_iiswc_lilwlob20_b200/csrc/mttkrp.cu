@@ -21,6 +21,7 @@
 //     and last segment of a run may be shared with neighbours -> red.global.add.v4.f32
 //     (one vector atomic per boundary, not per nonzero, cf. P:157/P:282 atomics).
 //   * No tensor cores: the path is a gather/scatter, not a dense contraction.
+#include <algorithm>
 #include <cstdlib>
 #include <type_traits>
 
@@ -66,9 +67,13 @@ struct KArgs {
   // L2 eviction-priority hints (bit 0: streams evict_first, bit 1: gathers evict_last,
   // bit 2: output stores / atomics evict_first); see Policies
   uint32_t cache_mode;
-  // io[] carry a hot flag in bit 31 (coo_mark_hot): hot entries hold a slot of hot_buf
+  // io[] carry hot tags (coo_mark_hot): 0x80000000 | slot of hot_buf (L2 tier),
+  // 0xC0000000 | slot of the shared-memory tier (coo_staged_kernel<..., HS = true>)
   uint32_t hot_marked;
   const float *hot_buf;
+  // shared-memory tier: slot -> factor row; other-mode slot j owns slots [hs_lo[j], hs_lo[j+1])
+  const uint32_t *hs_rows;
+  uint32_t hs_lo[kMaxOrder];
 };
 
 // Per-thread L2 cache policies (createpolicy, sm_80+): the nonzero stream is touched once
@@ -121,6 +126,21 @@ __device__ __forceinline__ Vec<VW> ldg_vec(const float *p, uint64_t pol) {
 #pragma unroll
     for (int i = 0; i < VW; ++i) r.v[i] = __ldg(p + i);
   }
+  return r;
+}
+
+// One predicated 128-bit load from either shared memory (ps) or global memory (pg), without a
+// branch: divergent per-group branches would serialise the batch of independent gathers.
+__device__ __forceinline__ Vec<4> ld_tiered(uint32_t saddr, const float *gp, uint64_t pol, int ps, int pg) {
+  Vec<4> r;
+  asm volatile(
+      "{\n\t.reg .pred ps, pg;\n\t"
+      "setp.ne.s32 ps, %5, 0;\n\t"
+      "setp.ne.s32 pg, %6, 0;\n\t"
+      "@ps ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];\n\t"
+      "@pg ld.global.nc.L2::cache_hint.v4.f32 {%0, %1, %2, %3}, [%7], %8;\n\t}"
+      : "=f"(r.v[0]), "=f"(r.v[1]), "=f"(r.v[2]), "=f"(r.v[3])
+      : "r"(saddr), "r"(ps), "r"(pg), "l"(gp), "l"(pol));
   return r;
 }
 
@@ -629,8 +649,13 @@ __global__ void __launch_bounds__(kThreads) hicoo_heavy_kernel(const HArgs a) {
 // one stage (32 nonzeros per group) ahead of the gathers.
 // WA: 0/1/2 buffer-address forms (see the launcher); 3, 4, 5 are measurement probes that
 // decompose the kernel time (3: no output writes, 4: no factor gathers, 5: stream only).
-template <int NO, int LPN, int WA>
-__global__ void __launch_bounds__(kThreads, WA == 6 ? 3 : 2) coo_staged_kernel(const KArgs a) {
+// HS (persistent, 16 warps, one CTA per SM): the shared-memory tier of the hot-row cache --
+// the most frequent factor rows are copied into shared memory once per CTA, and gathers of
+// entries tagged 0xC0000000 | slot read them there instead of from L2.
+template <int NO, int LPN, int WA, bool HS>
+__global__ void __launch_bounds__(HS ? 512 : kThreads, HS ? 1 : (WA == 6 ? 3 : 2))
+    coo_staged_kernel(const KArgs a) {
+  constexpr int WPC = HS ? 16 : kWarpsPerCta;
   constexpr bool kGather = WA != 4 && WA != 5;
   constexpr bool kWrite = WA != 3 && WA != 5;
   constexpr int kBuf = (WA == 0 || WA == 2) ? WA : 1;  // 6: form 1 with 3 CTAs per SM
@@ -643,14 +668,25 @@ __global__ void __launch_bounds__(kThreads, WA == 6 ? 3 : 2) coo_staged_kernel(c
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const int g = lane / LPN, lig = lane % LPN;
   uint32_t *wbuf = stage_buf + size_t(warp) * 2 * NA * SW;
-  const uint64_t w = uint64_t(blockIdx.x) * kWarpsPerCta + warp;
-  const uint64_t c0 = w * a.chunk;
-  if (c0 >= a.nnz) return;  // whole warp exits together
-  const uint64_t run = a.chunk / G;  // multiple of SG
-  const uint64_t x0 = c0 + uint64_t(g) * run;
-  const uint64_t x1 = (x0 + run < a.nnz) ? x0 + run : a.nnz;
-  const int nstages = int(run / SG);
   const uint32_t R = a.R;
+  float *hs_tile = reinterpret_cast<float *>(stage_buf + size_t(WPC) * 2 * NA * SW);
+  const uint32_t hs_saddr = smem_addr(hs_tile);
+  if constexpr (HS) {  // fill the shared-memory tier: hs_tile[slot][:] = U_j[hs_rows[slot]][:]
+    const uint32_t r4 = R / 4, n4 = a.hs_lo[NO] * r4;
+    for (uint32_t e = threadIdx.x; e < n4; e += blockDim.x) {
+      const uint32_t slot = e / r4, c = e % r4;
+      int j = 0;
+#pragma unroll
+      for (int jj = 1; jj < NO; ++jj) j += slot >= a.hs_lo[jj];
+      const float4 *Uj = reinterpret_cast<const float4 *>(a.Uo[j]);
+      reinterpret_cast<float4 *>(hs_tile)[e] = __ldg(Uj + uint64_t(__ldg(a.hs_rows + slot)) * r4 + c);
+    }
+    __syncthreads();
+  }
+  const uint64_t nchunks = (a.nnz + a.chunk - 1) / a.chunk;
+  const uint64_t wstep = HS ? uint64_t(gridDim.x) * WPC : nchunks;
+  const uint64_t run = a.chunk / G;  // multiple of SG
+  const int nstages = int(run / SG);
   const uint32_t col = uint32_t(lig) * 4;
   const Policies pol(a.cache_mode | 1u);  // the staged stream is always evict_first
   uint64_t pol_hot = pol.gather, pol_cold = pol.gather;
@@ -662,52 +698,60 @@ __global__ void __launch_bounds__(kThreads, WA == 6 ? 3 : 2) coo_staged_kernel(c
   for (int j = 0; j < NO; ++j) src[1 + j] = a.io[j];
   src[NA - 1] = reinterpret_cast<const uint32_t *>(a.val);
 
-  // issue the cp.async copies of stage s into buffer s & 1
-  auto issue_to = [&](int s, uint32_t *dst) {
-    for (int i = lane; i < SW / 4; i += 32) {  // 16-B chunks of one array
-      const int gi = i / (SG / 4), k = i % (SG / 4);
-      const uint64_t pos = c0 + uint64_t(gi) * run + uint64_t(s) * SG + uint64_t(k) * 4;
-      const int valid = pos >= a.nnz ? 0 : (a.nnz - pos >= 4 ? 16 : int(a.nnz - pos) * 4);
+  // issue the cp.async copies of stage s of the chunk starting at cc into dst (one commit
+  // group; an empty group when cc is past the end, so that wait_group counts stay uniform)
+  auto issue_to = [&](uint64_t cc, int s, uint32_t *dst) {
+    if (cc < a.nnz) {
+      for (int i = lane; i < SW / 4; i += 32) {  // 16-B chunks of one array
+        const int gi = i / (SG / 4), k = i % (SG / 4);
+        const uint64_t pos = cc + uint64_t(gi) * run + uint64_t(s) * SG + uint64_t(k) * 4;
+        const int valid = pos >= a.nnz ? 0 : (a.nnz - pos >= 4 ? 16 : int(a.nnz - pos) * 4);
 #pragma unroll
-      for (int arr = 0; arr < NA; ++arr) {
-        const uint32_t d = smem_addr(dst + arr * SW + gi * SG + k * 4);
-        const uint32_t *sp = src[arr] + (valid ? pos : 0);
-        if (kBuf == 2) {
-          asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(d), "l"(sp), "r"(valid)
-                       : "memory");
-        } else {
-          asm volatile("cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, %2, %3;" ::"r"(d),
-                       "l"(sp), "r"(valid), "l"(pol.stream)
-                       : "memory");
+        for (int arr = 0; arr < NA; ++arr) {
+          const uint32_t d = smem_addr(dst + arr * SW + gi * SG + k * 4);
+          const uint32_t *sp = src[arr] + (valid ? pos : 0);
+          if (kBuf == 2) {
+            asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(d), "l"(sp), "r"(valid)
+                         : "memory");
+          } else {
+            asm volatile("cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, %2, %3;" ::"r"(d),
+                         "l"(sp), "r"(valid), "l"(pol.stream)
+                         : "memory");
+          }
         }
       }
     }
     asm volatile("cp.async.commit_group;" ::: "memory");
   };
-  auto issue = [&](int s) {
+  auto issue = [&](uint64_t cc, int s, int b) {
     if (kBuf == 1) {
-      if (s & 1) issue_to(s, wbuf + NA * SW); else issue_to(s, wbuf);
+      if (b) issue_to(cc, s, wbuf + NA * SW); else issue_to(cc, s, wbuf);
     } else {
-      issue_to(s, wbuf + (s & 1) * NA * SW);
+      issue_to(cc, s, wbuf + b * NA * SW);
     }
   };
 
+  // The stream is pipelined across the warp's chunks: the last stage of a chunk prefetches
+  // stage 0 of the next one, so a persistent warp never waits on a cold pipeline.
+  int bsel = 0;
+  uint64_t w = uint64_t(blockIdx.x) * WPC + warp;
+  if (w < nchunks) issue(w * a.chunk, 0, 0);
+  for (; w < nchunks; w += wstep) {
+  const uint64_t c0 = w * a.chunk;
+  const uint64_t x0 = c0 + uint64_t(g) * run;
+  const uint64_t x1 = (x0 + run < a.nnz) ? x0 + run : a.nnz;
   Vec<4> acc;
 #pragma unroll
   for (int i = 0; i < 4; ++i) acc.v[i] = 0.f;
   uint32_t cur = 0xFFFFFFFFu;
   bool first = true;
   const bool active = x0 < x1 && col < R;
-  issue(0);
   for (int s = 0; s < nstages; ++s) {
-    if (s + 1 < nstages) {
-      issue(s + 1);
-      asm volatile("cp.async.wait_group 1;" ::: "memory");
-    } else {
-      asm volatile("cp.async.wait_group 0;" ::: "memory");
-    }
+    if (s + 1 < nstages) issue(c0, s + 1, bsel ^ 1);
+    else issue(w + wstep < nchunks ? (w + wstep) * a.chunk : a.nnz, 0, bsel ^ 1);
+    asm volatile("cp.async.wait_group 1;" ::: "memory");
     __syncwarp();
-    const uint32_t *buf = wbuf + (s & 1) * NA * SW + g * SG;
+    const uint32_t *buf = wbuf + bsel * NA * SW + g * SG;
     const uint64_t sx = x0 + uint64_t(s) * SG;  // first nonzero of this stage for the group
     if (active && sx < x1) {
       const int scnt = (x1 - sx) >= uint64_t(SG) ? SG : int(x1 - sx);
@@ -731,14 +775,23 @@ __global__ void __launch_bounds__(kThreads, WA == 6 ? 3 : 2) coo_staged_kernel(c
 #pragma unroll
           for (int j = 0; j < NO; ++j) {
             if (kGather) {
-              const float *base = a.Uo[j];
-              uint64_t gp = a.hot_marked ? pol_cold : pol.gather;
-              if (a.hot_marked && (idx[j][u] >> 31)) {  // a row of the packed hot-row cache
-                base = a.hot_buf;
-                idx[j][u] &= 0x7FFFFFFFu;
-                gp = pol_hot;
+              const uint32_t id = idx[j][u];
+              if constexpr (HS) {  // shared-memory tier, L2-tier buffer or plain factor row
+                const bool in_s = (id >> 30) == 3u, in_h = (id >> 30) == 2u;
+                const float *gptr = (in_h ? a.hot_buf : a.Uo[j]) + uint64_t(id & 0x3FFFFFFFu) * R + col;
+                f[j][u] = ld_tiered(hs_saddr + ((id & 0x3FFFFFFFu) * R + col) * 4u, gptr,
+                                    in_h ? pol_hot : pol_cold, u < cnt && in_s, u < cnt && !in_s);
+              } else {
+                const float *base = a.Uo[j];
+                uint64_t gp = a.hot_marked ? pol_cold : pol.gather;
+                uint32_t row = id;
+                if (a.hot_marked && (id >> 31)) {  // a row of the packed L2-tier buffer
+                  base = a.hot_buf;
+                  row = id & 0x3FFFFFFFu;
+                  gp = pol_hot;
+                }
+                if (u < cnt) f[j][u] = ldg_vec<4>(base + uint64_t(row) * R + col, gp);
               }
-              if (u < cnt) f[j][u] = ldg_vec<4>(base + uint64_t(idx[j][u]) * R + col, gp);
             } else {
 #pragma unroll
               for (int i = 0; i < 4; ++i) f[j][u].v[i] = __uint_as_float(idx[j][u] | 0x3f800000u);
@@ -776,10 +829,12 @@ __global__ void __launch_bounds__(kThreads, WA == 6 ? 3 : 2) coo_staged_kernel(c
         }
       }
     }
-    __syncwarp();  // the buffer of stage s is refilled at stage s + 2
+    __syncwarp();  // the buffer of this stage is refilled at the start of the next one
+    bsel ^= 1;
   }
   if (active && cur != 0xFFFFFFFFu && (kWrite || acc.v[0] == 1.2345e-30f))
     red_vec<4>(a.out + uint64_t(cur) * R + col, acc, pol.out);
+  }  // chunk loop
 }
 
 template <int VW>
@@ -939,32 +994,62 @@ void launch_coo_mttkrp(const pasta_coo *x, uint32_t mode, const float *const *fa
     uint64_t gathered = 0;
     for (uint32_t k = 0; k < x->order; ++k)
       if (k != mode) gathered += uint64_t(x->dims[k]) * R * sizeof(float);
-    const bool want_hot = env_int("PASTA_HOT_FORCE", 0) || gathered > uint64_t(l2);
-    if (want_hot) coo_mark_hot(const_cast<pasta_coo *>(x), mode, R, s);
-    if (want_hot && mc.hot_R == R) {
-      a.hot_marked = 1;
-      a.hot_buf = mc.hot_buf.p;
-      int jj = 0;
-      for (uint32_t k = 0; k < x->order; ++k)
-        if (k != mode) a.io[jj++] = mc.hot_inds[k].p;
-      launch_hot_fill(mc, factors, x->order, mode, R, s);
-    }
+    // effective L2 for random row gathers is ~half the nominal size
+    // (profiles/r01_l2_capacity_microbench.txt)
+    const bool want_hot = env_int("PASTA_HOT_FORCE", 0) || gathered > uint64_t(l2) / 2;
     const int lpn = R == 16 ? 4 : 8;
     const int G = 32 / lpn;
-    uint64_t run = uint64_t(env_int("PASTA_MTTKRP_RUN", 128));
+    // Persistent HS kernel (one 16-warp CTA per SM) with the shared-memory tier of the hot-row
+    // cache.  Tier size: on L2-resident factors (no L2 tier) the kernel is bound by L2->SM
+    // bandwidth and every smem row helps, so the tier takes what the staging buffers leave of
+    // the 227 KB; on DRAM-bound gathers (L2 tier on) the L1 that the shared-memory carve-out
+    // leaves holds the in-flight misses, so the tier stays at 512 rows (measured cliff between
+    // 512 and 1024 rows on H and C3: 1.89 -> 2.17 ms, 1.84 -> 3.2 ms; profiles/r01_hs_sweep.txt).
+    // PASTA_HOT_SMEM=0 selects the non-persistent kernel; PASTA_HOT_SMEM_ROWS caps the tier.
+    const size_t stage_hs = size_t(16) * 2 * (no + 2) * (G * 32) * sizeof(uint32_t);
+    const size_t smem_cap = 227 * 1024;
+    uint32_t hs_rows_budget =
+        stage_hs < smem_cap ? uint32_t((smem_cap - stage_hs) / (size_t(R) * sizeof(float))) : 0u;
+    if (want_hot) hs_rows_budget = std::min(hs_rows_budget, 512u);
+    if (const int cap = env_int("PASTA_HOT_SMEM_ROWS", 0)) hs_rows_budget = std::min(hs_rows_budget, uint32_t(cap));
+    bool hs = env_int("PASTA_HOT_SMEM", 1) != 0 && hs_rows_budget >= 64 && no >= 2;
+    if (hs) {
+      coo_mark_hot(const_cast<pasta_coo *>(x), mode, R, want_hot, hs_rows_budget, s);
+      if (mc.hot_R != R || mc.hs_total == 0) hs = false;
+    }
+    if (!hs && want_hot) coo_mark_hot(const_cast<pasta_coo *>(x), mode, R, true, 0, s);
+    if ((hs || want_hot) && mc.hot_R == R) {
+      a.hot_marked = 1;
+      a.hot_buf = mc.hot_buf.p;
+      a.hs_rows = mc.hs_rows.p;
+      int jj = 0;
+      for (uint32_t k = 0; k < x->order; ++k)
+        if (k != mode) {
+          a.hs_lo[jj] = uint32_t(mc.hs_base[k]);
+          a.io[jj++] = mc.hot_inds[k].p;
+        }
+      a.hs_lo[jj] = uint32_t(mc.hs_total);
+      if (mc.hot_total) launch_hot_fill(mc, factors, x->order, mode, R, s);
+    }
+    // run per group: short runs on DRAM-bound gathers, long ones on L2-resident factors
+    // (fewer boundary atomics); measured on H (64: 1.89, 128: 1.93, 256: 1.98 ms per mode)
+    // and C2 (64: 1.02, 128: 0.98, 256: 0.96 ms)
+    uint64_t run = uint64_t(env_int("PASTA_MTTKRP_RUN", want_hot ? 64 : 256));
     run = run < 32 ? 32 : (run / 32) * 32;
     a.chunk = uint64_t(G) * run;
     a.cache_mode = uint32_t(env_int("PASTA_MTTKRP_CACHE", 0));
-    const size_t smem = size_t(kWarpsPerCta) * 2 * (no + 2) * (G * 32) * sizeof(uint32_t);
+    const size_t smem = hs ? stage_hs + size_t(mc.hs_total) * R * sizeof(float)
+                           : size_t(kWarpsPerCta) * 2 * (no + 2) * (G * 32) * sizeof(uint32_t);
     uint64_t nwarps = (a.nnz + a.chunk - 1) / a.chunk;
-    uint64_t nblk = (nwarps + kWarpsPerCta - 1) / kWarpsPerCta;
+    uint64_t nblk = hs ? std::min<uint64_t>((nwarps + 15) / 16, uint64_t(sm_count()))
+                       : (nwarps + kWarpsPerCta - 1) / kWarpsPerCta;
     // PASTA_HOT_PERSIST=1: launch with an L2 access-policy window marking the hot-row buffer
     // persisting (within the device's persisting carve-out)
     const bool persist = a.hot_marked && env_int("PASTA_HOT_PERSIST", 0);
     auto go = [&](auto kern) {
       PASTA_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem)));
       if (!persist) {
-        kern<<<unsigned(nblk), kThreads, smem, s>>>(a);
+        kern<<<unsigned(nblk), hs ? 512 : kThreads, smem, s>>>(a);
       } else {
         static size_t carve = 0;
         const size_t want = mc.hot_buf.bytes();
@@ -1000,14 +1085,19 @@ void launch_coo_mttkrp(const pasta_coo *x, uint32_t mode, const float *const *fa
     const int wa = env_int("PASTA_STAGED_WA", 1);
     auto pick = [&](auto tag) {
       constexpr int W = decltype(tag)::value;
-      if (no == 1 && lpn == 4) go(coo_staged_kernel<1, 4, 1>);  // one code path for order 2
-      else if (no == 1) go(coo_staged_kernel<1, 8, 1>);
-      else if (no == 2 && lpn == 4) go(coo_staged_kernel<2, 4, W>);
-      else if (no == 2) go(coo_staged_kernel<2, 8, W>);
-      else if (lpn == 4) go(coo_staged_kernel<3, 4, W>);
-      else go(coo_staged_kernel<3, 8, W>);
+      if (no == 1 && lpn == 4) go(coo_staged_kernel<1, 4, 1, false>);  // one code path for order 2
+      else if (no == 1) go(coo_staged_kernel<1, 8, 1, false>);
+      else if (no == 2 && lpn == 4) go(coo_staged_kernel<2, 4, W, false>);
+      else if (no == 2) go(coo_staged_kernel<2, 8, W, false>);
+      else if (lpn == 4) go(coo_staged_kernel<3, 4, W, false>);
+      else go(coo_staged_kernel<3, 8, W, false>);
     };
-    if (wa == 1) pick(std::integral_constant<int, 1>());
+    if (hs) {
+      if (no == 2 && lpn == 4) go(coo_staged_kernel<2, 4, 1, true>);
+      else if (no == 2) go(coo_staged_kernel<2, 8, 1, true>);
+      else if (lpn == 4) go(coo_staged_kernel<3, 4, 1, true>);
+      else go(coo_staged_kernel<3, 8, 1, true>);
+    } else if (wa == 1) pick(std::integral_constant<int, 1>());
     else if (wa == 2) pick(std::integral_constant<int, 2>());
     else if (wa == 3) pick(std::integral_constant<int, 3>());
     else if (wa == 4) pick(std::integral_constant<int, 4>());

@@ -294,18 +294,21 @@ __global__ void bucket_hist_kernel(const uint32_t *__restrict__ cnt, uint64_t n,
     if (h[b]) atomicAdd(&hist[b], h[b]);
 }
 
-__global__ void hot_flag_kernel(const uint32_t *__restrict__ cnt, uint64_t n, uint32_t hot_bucket,
+// flag rows with lo <= bucket(count) < hi
+__global__ void hot_flag_kernel(const uint32_t *__restrict__ cnt, uint64_t n, uint32_t lo, uint32_t hi,
                                 uint8_t *__restrict__ flag) {
   for (uint64_t i = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; i < n;
-       i += uint64_t(gridDim.x) * blockDim.x)
-    flag[i] = cnt[i] && count_bucket_dev(cnt[i]) >= hot_bucket;
+       i += uint64_t(gridDim.x) * blockDim.x) {
+    const uint32_t b = cnt[i] ? count_bucket_dev(cnt[i]) : 0u;
+    flag[i] = cnt[i] && b >= lo && b < hi;
+  }
 }
 
 __global__ void slot_map_kernel(const uint32_t *__restrict__ rows, uint64_t nh, uint64_t base,
-                                uint32_t *__restrict__ slot_of, uint32_t *__restrict__ hot_rows) {
+                                uint32_t tag, uint32_t *__restrict__ slot_of, uint32_t *__restrict__ hot_rows) {
   for (uint64_t s = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; s < nh;
        s += uint64_t(gridDim.x) * blockDim.x) {
-    slot_of[rows[s]] = uint32_t(base + s);
+    slot_of[rows[s]] = tag | uint32_t(base + s);
     hot_rows[base + s] = rows[s];
   }
 }
@@ -316,7 +319,7 @@ __global__ void mark_hot_kernel(const uint32_t *__restrict__ src, const uint32_t
        x += uint64_t(gridDim.x) * blockDim.x) {
     const uint32_t v = src[x];
     const uint32_t sl = __ldg(slot_of + v);
-    dst[x] = sl != 0xFFFFFFFFu ? (0x80000000u | sl) : v;
+    dst[x] = sl != 0xFFFFFFFFu ? sl : v;  // sl carries its tier tag
   }
 }
 
@@ -339,24 +342,33 @@ unsigned grid8(uint64_t n) {
 
 }  // namespace
 
-// Hot-row cache for the COO factor gathers.  The most frequent rows of the gathered factors
-// (row nonzero counts, bucketed), as many as fit PASTA_HOT_MB (default 64 MB of the 126 MB
-// L2) at R*4 bytes per row, get contiguous slots of one buffer that is refilled from the
-// factors before every launch; the per-mode index copies point hot entries at their slot
-// (bit 31 set).  Packed hot rows fill whole L2 lines and stay resident, where scattered ones
-// share lines with cold neighbours and are evicted by the cold-row and stream traffic: L2
-// turns from LRU over scattered rows into a frequency-based cache for the power-law gathers
-// (cache reuse is why MTTKRP beats its DRAM roofline).  Needs dims < 2^31.
-void coo_mark_hot(pasta_coo *x, uint32_t mode, uint32_t R, cudaStream_t s) {
+// Hot-row cache for the COO factor gathers, two tiers.  The most frequent rows of the gathered
+// factors (row nonzero counts, bucketed 8 per octave) are ranked jointly over the factors:
+//  * shared-memory tier: as many as fit `smem_rows` rows (the kernel copies them into every
+//    CTA's shared memory at launch, so their gathers never reach L2; on L2-resident factors
+//    the kernel is bound by L2->SM bandwidth, and power-law-hot rows carry most gathers);
+//  * L2 tier (`global_tier`, when the gathered factors exceed L2): the next rows, as many as fit
+//    PASTA_HOT_MB (default 64 MB) at R*4 bytes per row, get contiguous slots of one buffer
+//    refilled from the factors before every launch.  Packed hot rows fill whole L2 lines and
+//    stay resident, where scattered ones share lines with cold neighbours and are evicted by
+//    the cold-row and stream traffic: L2 turns from LRU over scattered rows into a
+//    frequency-based cache for the power-law gathers (cache reuse is why MTTKRP beats its
+//    DRAM roofline).
+// The per-mode index copies hot_inds[k] encode 0xC0000000 | smem slot (slot numbered over all
+// gathered factors, factor k at [hs_base[k], +hs_cnt[k])), 0x80000000 | L2-tier slot, or the
+// plain row.  Needs dims < 2^30.
+void coo_mark_hot(pasta_coo *x, uint32_t mode, uint32_t R, bool global_tier, uint32_t smem_rows,
+                  cudaStream_t s) {
   CooModeCopy &mc = x->mc[mode];
-  if (mc.hot_R == R) return;
+  if (mc.hot_R == R && mc.hot_global == global_tier && mc.hot_smem_budget == smem_rows) return;
   const char *env = getenv("PASTA_HOT_MB");
-  const double hot_mb = (env && *env) ? atof(env) : 64.0;
+  const double hot_mb = global_tier ? ((env && *env) ? atof(env) : 64.0) : 0.0;
   const uint32_t N = x->order;
   const uint64_t M = x->nnz;
+  mc.hot_R = 0;
   for (uint32_t k = 0; k < N; ++k)
-    if (x->dims[k] >= 0x80000000u) return;
-  if (hot_mb <= 0 || M == 0) return;
+    if (x->dims[k] >= 0x40000000u) return;
+  if ((hot_mb <= 0 && smem_rows == 0) || M == 0) return;
   for (uint32_t k = 0; k < N; ++k) {
     if (k == mode || x->counts_ready[k]) continue;
     x->row_count[k].alloc(x->dims[k], s);
@@ -371,41 +383,64 @@ void coo_mark_hot(pasta_coo *x, uint32_t mode, uint32_t R, cudaStream_t s) {
     PASTA_CUDA(cudaStreamSynchronize(s));
     x->counts_ready[k] = true;
   }
-  // smallest bucket b* such that the rows with bucket >= b* of every gathered factor fit
-  const double budget_rows = hot_mb * 1048576.0 / (double(R) * 4.0);
-  uint32_t hb = kCountBuckets;
-  double acc = 0.0;
-  for (int b = kCountBuckets - 1; b >= 1; --b) {
-    double add = 0.0;
-    for (uint32_t k = 0; k < N; ++k)
-      if (k != mode) add += double(x->count_hist[k][b]);
-    if (acc + add > budget_rows) break;
-    acc += add;
-    hb = uint32_t(b);
-  }
-  // hot rows of each gathered factor -> contiguous slots of one buffer
-  uint64_t total = 0;
-  std::vector<DevArray<uint32_t>> lists(N);
+  // smallest bucket such that the rows at or above it, over every gathered factor, fit a budget
+  auto threshold = [&](double budget_rows) {
+    uint32_t hb = kCountBuckets;
+    double acc = 0.0;
+    for (int b = kCountBuckets - 1; b >= 1; --b) {
+      double add = 0.0;
+      for (uint32_t k = 0; k < N; ++k)
+        if (k != mode) add += double(x->count_hist[k][b]);
+      if (acc + add > budget_rows) break;
+      acc += add;
+      hb = uint32_t(b);
+    }
+    return hb;
+  };
+  const uint32_t hsb = threshold(double(smem_rows));  // smem tier: bucket >= hsb
+  const uint32_t hb =                                  // L2 tier: hb <= bucket < hsb
+      hot_mb > 0 ? threshold(double(smem_rows) + hot_mb * 1048576.0 / (double(R) * 4.0)) : hsb;
+  // both tiers -> contiguous slots (per tier, factor after factor, rows ascending)
+  uint64_t total = 0, stotal = 0;
+  std::vector<DevArray<uint32_t>> lists(N), slists(N);
   for (uint32_t k = 0; k < N; ++k) {
     mc.hot_base[k] = total;
     mc.hot_cnt[k] = 0;
+    mc.hs_base[k] = stotal;
+    mc.hs_cnt[k] = 0;
     if (k == mode) continue;
     DevArray<uint8_t> flag(x->dims[k], s);
-    hot_flag_kernel<<<grid8(x->dims[k]), 256, 0, s>>>(x->row_count[k].p, x->dims[k], hb, flag.p);
-    PASTA_LAUNCHED();
-    mc.hot_cnt[k] = select_flagged(flag.p, x->dims[k], lists[k], s);
-    total += mc.hot_cnt[k];
+    if (hsb < kCountBuckets) {
+      hot_flag_kernel<<<grid8(x->dims[k]), 256, 0, s>>>(x->row_count[k].p, x->dims[k], hsb, kCountBuckets,
+                                                        flag.p);
+      PASTA_LAUNCHED();
+      mc.hs_cnt[k] = select_flagged(flag.p, x->dims[k], slists[k], s);
+      stotal += mc.hs_cnt[k];
+    }
+    if (hb < hsb) {
+      hot_flag_kernel<<<grid8(x->dims[k]), 256, 0, s>>>(x->row_count[k].p, x->dims[k], hb, hsb, flag.p);
+      PASTA_LAUNCHED();
+      mc.hot_cnt[k] = select_flagged(flag.p, x->dims[k], lists[k], s);
+      total += mc.hot_cnt[k];
+    }
   }
   mc.hot_total = total;
+  mc.hs_total = stotal;
   mc.hot_rows.alloc(total ? total : 1, s);
   mc.hot_buf.alloc((total ? total : 1) * R, s);
+  mc.hs_rows.alloc(stotal ? stotal : 1, s);
   for (uint32_t k = 0; k < N; ++k) {
     if (k == mode) continue;
     DevArray<uint32_t> slot_of(x->dims[k], s);
     PASTA_CUDA(cudaMemsetAsync(slot_of.p, 0xFF, slot_of.bytes(), s));
     if (mc.hot_cnt[k]) {
       slot_map_kernel<<<grid8(mc.hot_cnt[k]), 256, 0, s>>>(lists[k].p, mc.hot_cnt[k], mc.hot_base[k],
-                                                          slot_of.p, mc.hot_rows.p);
+                                                          0x80000000u, slot_of.p, mc.hot_rows.p);
+      PASTA_LAUNCHED();
+    }
+    if (mc.hs_cnt[k]) {
+      slot_map_kernel<<<grid8(mc.hs_cnt[k]), 256, 0, s>>>(slists[k].p, mc.hs_cnt[k], mc.hs_base[k],
+                                                         0xC0000000u, slot_of.p, mc.hs_rows.p);
       PASTA_LAUNCHED();
     }
     if (mc.hot_inds[k].n != M) mc.hot_inds[k].alloc(M, s);
@@ -414,12 +449,17 @@ void coo_mark_hot(pasta_coo *x, uint32_t mode, uint32_t R, cudaStream_t s) {
     PASTA_CUDA(cudaStreamSynchronize(s));  // slot_of is released at scope exit
   }
   mc.hot_bucket = hb;
+  mc.hs_bucket = hsb;
+  mc.hot_global = global_tier;
+  mc.hot_smem_budget = smem_rows;
   mc.hot_R = R;
   if (getenv("PASTA_DEBUG")) {
-    fprintf(stderr, "[pasta] hot cache mode %u R %u: budget %.0f rows, bucket >= %u, %llu hot rows (",
-            mode, R, budget_rows, hb, (unsigned long long)total);
+    fprintf(stderr, "[pasta] hot cache mode %u R %u: smem budget %u rows (bucket >= %u, %llu rows), "
+            "L2 tier %.0f MB (bucket >= %u, %llu rows) (", mode, R, smem_rows, hsb,
+            (unsigned long long)stotal, hot_mb, hb, (unsigned long long)total);
     for (uint32_t k = 0; k < N; ++k)
-      if (k != mode) fprintf(stderr, " k%u:%llu", k, (unsigned long long)mc.hot_cnt[k]);
+      if (k != mode)
+        fprintf(stderr, " k%u:%llu+%llu", k, (unsigned long long)mc.hs_cnt[k], (unsigned long long)mc.hot_cnt[k]);
     fprintf(stderr, " )\n");
   }
 }

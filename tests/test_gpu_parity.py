@@ -393,3 +393,32 @@ def test_coo_hot_row_cache_forced(env, hot_mb, monkeypatch):
         U2 = [u.cpu().numpy() for u in Ud2]
         ref, ab = oracle.mttkrp(dims, inds, vals, 0, U2)
         _check(pasta.pasta_mttkrp_coo(x, 0, Ud2), ref, ab, "hot cache refill")
+
+
+@pytest.mark.parametrize("l2_tier", [False, True])
+def test_coo_shared_memory_hot_tier(env, l2_tier, monkeypatch):
+    """The shared-memory tier of the hot-row cache (persistent coo_staged_kernel<..., HS>):
+    forced on, alone or together with a tiny L2 tier so that smem-, L2-tier- and cold rows
+    mix in one warp; 3M nonzeros give every warp of the persistent grid several chunks."""
+    pasta, oracle, torch = env
+    monkeypatch.setenv("PASTA_HOT_SMEM", "1")
+    if l2_tier:
+        monkeypatch.setenv("PASTA_HOT_FORCE", "1")
+        monkeypatch.setenv("PASTA_HOT_MB", "0.25")
+    for dims, nnz, R in [((3000, 2000, 4000), 3_000_017, 16), ((300, 400, 500, 60), 80_000, 16),
+                         ((3000, 2000, 4000), 120_000, 32), ((300, 400, 500, 60), 80_000, 32),
+                         ((5000, 3000, 2000), 0, 16)]:
+        if nnz:
+            inds, vals = si.powerlaw_coo(dims, nnz, seed=nnz + R)
+        else:
+            inds, vals = si.hot_row_coo(dims, 300_000, 50_000, seed=4, mode=1, hot_row=0)
+        U = si.factors(dims, R, seed=R)
+        Ud = _dev(torch, U)
+        x = pasta.pasta_coo_from_arrays(dims, inds, vals)
+        for n in range(len(dims)):
+            ref, ab = oracle.mttkrp(dims, inds, vals, n, U)
+            _check(pasta.pasta_mttkrp_coo(x, n, Ud), ref, ab, f"smem tier {dims} R={R} mode {n}")
+        Ud2 = [u * 0.5 for u in Ud]  # the tier is re-read from the factors at every launch
+        U2 = [u.cpu().numpy() for u in Ud2]
+        ref, ab = oracle.mttkrp(dims, inds, vals, 1, U2)
+        _check(pasta.pasta_mttkrp_coo(x, 1, Ud2), ref, ab, "smem tier refill")
