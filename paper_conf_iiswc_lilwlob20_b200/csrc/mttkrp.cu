@@ -652,15 +652,17 @@ __global__ void __launch_bounds__(kThreads) hicoo_heavy_kernel(const HArgs a) {
 // HS (persistent, 16 warps, one CTA per SM): the shared-memory tier of the hot-row cache --
 // the most frequent factor rows are copied into shared memory once per CTA, and gathers of
 // entries tagged 0xC0000000 | slot read them there instead of from L2.
-template <int NO, int LPN, int WA, bool HS>
-__global__ void __launch_bounds__(HS ? 512 : kThreads, HS ? 1 : (WA == 6 ? 3 : 2))
+template <int NO, int LPN, int WA, bool HS, int WPC_ = 16, int SG_ = 32>
+__global__ void __launch_bounds__(HS ? WPC_ * 32 : kThreads, HS ? 1 : (WA == 6 ? 3 : 2))
     coo_staged_kernel(const KArgs a) {
-  constexpr int WPC = HS ? 16 : kWarpsPerCta;
+  constexpr int WPC = HS ? WPC_ : kWarpsPerCta;
   constexpr bool kGather = WA != 4 && WA != 5;
   constexpr bool kWrite = WA != 3 && WA != 5;
   constexpr int kBuf = (WA == 0 || WA == 2) ? WA : 1;  // 6: form 1 with 3 CTAs per SM
   constexpr int G = 32 / LPN;
-  constexpr int SG = 32;          // nonzeros per group per stage
+  constexpr int SG = SG_;         // nonzeros per group per stage (32 or 16)
+  constexpr int CG = SG / 4;      // 16-B chunks per group and array
+  constexpr int GL = 8 / CG;      // groups per 128-B line
   constexpr int SW = G * SG;      // nonzeros per warp per stage
   constexpr int NA = NO + 2;      // arrays: i_n, i_k (k != n), val
   constexpr int U = 4;
@@ -668,7 +670,7 @@ __global__ void __launch_bounds__(HS ? 512 : kThreads, HS ? 1 : (WA == 6 ? 3 : 2
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const int g = lane / LPN, lig = lane % LPN;
   uint32_t *wbuf = stage_buf + size_t(warp) * 2 * NA * SW;
-  const uint32_t R = a.R;
+  constexpr uint32_t R = 4 * LPN;  // the launcher picks LPN = R / 4 (R = 16 or 32)
   float *hs_tile = reinterpret_cast<float *>(stage_buf + size_t(WPC) * 2 * NA * SW);
   const uint32_t hs_saddr = smem_addr(hs_tile);
   if constexpr (HS) {  // fill the shared-memory tier: hs_tile[slot][:] = U_j[hs_rows[slot]][:]
@@ -689,9 +691,8 @@ __global__ void __launch_bounds__(HS ? 512 : kThreads, HS ? 1 : (WA == 6 ? 3 : 2
   const int nstages = int(run / SG);
   const uint32_t col = uint32_t(lig) * 4;
   const Policies pol(a.cache_mode | 1u);  // the staged stream is always evict_first
-  uint64_t pol_hot = pol.gather, pol_cold = pol.gather;
-  if (a.cache_mode & 8) asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol_hot));
-  if (a.cache_mode & 16) asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol_cold));
+  // one L2 policy for every gather: a per-lane choice would force a predicated R2UR of the
+  // policy descriptor per load (separate hot/cold policies measured no gain, DESIGN 9b)
   const uint32_t *src[NA];
   src[0] = a.irow;
 #pragma unroll
@@ -708,7 +709,9 @@ __global__ void __launch_bounds__(HS ? 512 : kThreads, HS ? 1 : (WA == 6 ? 3 : 2
         const int valid = pos >= a.nnz ? 0 : (a.nnz - pos >= 4 ? 16 : int(a.nnz - pos) * 4);
 #pragma unroll
         for (int arr = 0; arr < NA; ++arr) {
-          const uint32_t d = smem_addr(dst + arr * SW + gi * SG + k * 4);
+          // 16-B chunk k of group gi lands at chunk k ^ ((gi / GL) % CG) of the group's region:
+          // the groups of a warp then read different bank quads at every step
+          const uint32_t d = smem_addr(dst + arr * SW + gi * SG + ((k ^ (gi / GL)) & (CG - 1)) * 4);
           const uint32_t *sp = src[arr] + (valid ? pos : 0);
           if (kBuf == 2) {
             asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(d), "l"(sp), "r"(valid)
@@ -758,15 +761,16 @@ __global__ void __launch_bounds__(HS ? 512 : kThreads, HS ? 1 : (WA == 6 ? 3 : 2
 #pragma unroll 1
       for (int q = 0; q < scnt; q += U) {
         const int cnt = (scnt - q) >= U ? U : scnt - q;
-        const uint4 r4 = *reinterpret_cast<const uint4 *>(buf + q);
-        const uint4 v4 = *reinterpret_cast<const uint4 *>(buf + (NA - 1) * SW + q);
+        const int qs = (((q / 4) ^ (g / GL)) & (CG - 1)) * 4;  // swizzled chunk (see issue_to)
+        const uint4 r4 = *reinterpret_cast<const uint4 *>(buf + qs);
+        const uint4 v4 = *reinterpret_cast<const uint4 *>(buf + (NA - 1) * SW + qs);
         uint32_t row[U] = {r4.x, r4.y, r4.z, r4.w};
         float v[U] = {__uint_as_float(v4.x), __uint_as_float(v4.y), __uint_as_float(v4.z),
                       __uint_as_float(v4.w)};
         uint32_t idx[NO][U];
 #pragma unroll
         for (int j = 0; j < NO; ++j) {
-          const uint4 i4 = *reinterpret_cast<const uint4 *>(buf + (1 + j) * SW + q);
+          const uint4 i4 = *reinterpret_cast<const uint4 *>(buf + (1 + j) * SW + qs);
           idx[j][0] = i4.x; idx[j][1] = i4.y; idx[j][2] = i4.z; idx[j][3] = i4.w;
         }
         Vec<4> f[NO][U];
@@ -780,17 +784,15 @@ __global__ void __launch_bounds__(HS ? 512 : kThreads, HS ? 1 : (WA == 6 ? 3 : 2
                 const bool in_s = (id >> 30) == 3u, in_h = (id >> 30) == 2u;
                 const float *gptr = (in_h ? a.hot_buf : a.Uo[j]) + uint64_t(id & 0x3FFFFFFFu) * R + col;
                 f[j][u] = ld_tiered(hs_saddr + ((id & 0x3FFFFFFFu) * R + col) * 4u, gptr,
-                                    in_h ? pol_hot : pol_cold, u < cnt && in_s, u < cnt && !in_s);
+                                    pol.gather, u < cnt && in_s, u < cnt && !in_s);
               } else {
                 const float *base = a.Uo[j];
-                uint64_t gp = a.hot_marked ? pol_cold : pol.gather;
                 uint32_t row = id;
                 if (a.hot_marked && (id >> 31)) {  // a row of the packed L2-tier buffer
                   base = a.hot_buf;
                   row = id & 0x3FFFFFFFu;
-                  gp = pol_hot;
                 }
-                if (u < cnt) f[j][u] = ldg_vec<4>(base + uint64_t(row) * R + col, gp);
+                if (u < cnt) f[j][u] = ldg_vec<4>(base + uint64_t(row) * R + col, pol.gather);
               }
             } else {
 #pragma unroll
@@ -1006,7 +1008,14 @@ void launch_coo_mttkrp(const pasta_coo *x, uint32_t mode, const float *const *fa
     // leaves holds the in-flight misses, so the tier stays at 512 rows (measured cliff between
     // 512 and 1024 rows on H and C3: 1.89 -> 2.17 ms, 1.84 -> 3.2 ms; profiles/r01_hs_sweep.txt).
     // PASTA_HOT_SMEM=0 selects the non-persistent kernel; PASTA_HOT_SMEM_ROWS caps the tier.
-    const size_t stage_hs = size_t(16) * 2 * (no + 2) * (G * 32) * sizeof(uint32_t);
+    // HS shape (warps per CTA, nonzeros per group per stage): PASTA_HS_CFG = 0 (16, 32) or
+    // 1 (24, 16).  More warps = more gathers in flight; 24 warps fit 80 registers for order 3
+    // (H 1.81 -> 1.64 ms, C2 0.83 -> 0.77, C3 1.78 -> 1.58) but spill for order 4 (C4 0.74 ->
+    // 0.80), so the default is 1 for order 3 and 0 above (32 warps spill for every order).
+    const int hs_cfg = env_int("PASTA_HS_CFG", no == 2 ? 1 : 0);
+    const int hs_wpc = hs_cfg == 1 ? 24 : 16;
+    const int hs_sg = hs_cfg == 1 ? 16 : 32;
+    const size_t stage_hs = size_t(hs_wpc) * 2 * (no + 2) * (G * hs_sg) * sizeof(uint32_t);
     const size_t smem_cap = 227 * 1024;
     uint32_t hs_rows_budget =
         stage_hs < smem_cap ? uint32_t((smem_cap - stage_hs) / (size_t(R) * sizeof(float))) : 0u;
@@ -1031,17 +1040,17 @@ void launch_coo_mttkrp(const pasta_coo *x, uint32_t mode, const float *const *fa
       a.hs_lo[jj] = uint32_t(mc.hs_total);
       if (mc.hot_total) launch_hot_fill(mc, factors, x->order, mode, R, s);
     }
-    // run per group: short runs on DRAM-bound gathers, long ones on L2-resident factors
-    // (fewer boundary atomics); measured on H (64: 1.89, 128: 1.93, 256: 1.98 ms per mode)
-    // and C2 (64: 1.02, 128: 0.98, 256: 0.96 ms)
-    uint64_t run = uint64_t(env_int("PASTA_MTTKRP_RUN", want_hot ? 64 : 256));
+    // run per group: short runs on DRAM-bound gathers, longer ones on L2-resident factors
+    // (fewer boundary atomics); measured on H (64: 1.82, 128: 1.87 ms per mode), C2 (128 and
+    // 256: 0.83 ms) and C4 (128: 0.74, 256: 0.76 ms); profiles/r01_hs_sweep.txt
+    uint64_t run = uint64_t(env_int("PASTA_MTTKRP_RUN", want_hot ? 64 : 128));
     run = run < 32 ? 32 : (run / 32) * 32;
     a.chunk = uint64_t(G) * run;
     a.cache_mode = uint32_t(env_int("PASTA_MTTKRP_CACHE", 0));
     const size_t smem = hs ? stage_hs + size_t(mc.hs_total) * R * sizeof(float)
                            : size_t(kWarpsPerCta) * 2 * (no + 2) * (G * 32) * sizeof(uint32_t);
     uint64_t nwarps = (a.nnz + a.chunk - 1) / a.chunk;
-    uint64_t nblk = hs ? std::min<uint64_t>((nwarps + 15) / 16, uint64_t(sm_count()))
+    uint64_t nblk = hs ? std::min<uint64_t>((nwarps + hs_wpc - 1) / hs_wpc, uint64_t(sm_count()))
                        : (nwarps + kWarpsPerCta - 1) / kWarpsPerCta;
     // PASTA_HOT_PERSIST=1: launch with an L2 access-policy window marking the hot-row buffer
     // persisting (within the device's persisting carve-out)
@@ -1049,7 +1058,7 @@ void launch_coo_mttkrp(const pasta_coo *x, uint32_t mode, const float *const *fa
     auto go = [&](auto kern) {
       PASTA_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem)));
       if (!persist) {
-        kern<<<unsigned(nblk), hs ? 512 : kThreads, smem, s>>>(a);
+        kern<<<unsigned(nblk), hs ? hs_wpc * 32 : kThreads, smem, s>>>(a);
       } else {
         static size_t carve = 0;
         const size_t want = mc.hot_buf.bytes();
@@ -1092,11 +1101,17 @@ void launch_coo_mttkrp(const pasta_coo *x, uint32_t mode, const float *const *fa
       else if (lpn == 4) go(coo_staged_kernel<3, 4, W, false>);
       else go(coo_staged_kernel<3, 8, W, false>);
     };
+    auto pick_hs = [&](auto wtag, auto stag) {
+      constexpr int W = decltype(wtag)::value, S = decltype(stag)::value;
+      if (no == 2 && lpn == 4) go(coo_staged_kernel<2, 4, 1, true, W, S>);
+      else if (no == 2) go(coo_staged_kernel<2, 8, 1, true, W, S>);
+      else if (lpn == 4) go(coo_staged_kernel<3, 4, 1, true, W, S>);
+      else go(coo_staged_kernel<3, 8, 1, true, W, S>);
+    };
+    using I16 = std::integral_constant<int, 16>;
     if (hs) {
-      if (no == 2 && lpn == 4) go(coo_staged_kernel<2, 4, 1, true>);
-      else if (no == 2) go(coo_staged_kernel<2, 8, 1, true>);
-      else if (lpn == 4) go(coo_staged_kernel<3, 4, 1, true>);
-      else go(coo_staged_kernel<3, 8, 1, true>);
+      if (hs_cfg == 1) pick_hs(std::integral_constant<int, 24>(), I16());
+      else pick_hs(I16(), std::integral_constant<int, 32>());
     } else if (wa == 1) pick(std::integral_constant<int, 1>());
     else if (wa == 2) pick(std::integral_constant<int, 2>());
     else if (wa == 3) pick(std::integral_constant<int, 3>());

@@ -51,7 +51,10 @@ def main():
             if True:
                 os.environ["PASTA_MTTKRP_CACHE"] = str(cache)
                 os.environ["PASTA_MTTKRP_VARIANT"] = str(var)
-                os.environ["PASTA_MTTKRP_RUN"] = str(run)
+                if run:
+                    os.environ["PASTA_MTTKRP_RUN"] = str(run)
+                else:  # 0: the library's default for the regime
+                    os.environ.pop("PASTA_MTTKRP_RUN", None)
                 per_mode = []
                 for n in range(len(dims)):
                     for _ in range(2):
