@@ -691,8 +691,9 @@ __global__ void __launch_bounds__(HS ? WPC_ * 32 : kThreads, HS ? 1 : (WA == 6 ?
   const int nstages = int(run / SG);
   const uint32_t col = uint32_t(lig) * 4;
   const Policies pol(a.cache_mode | 1u);  // the staged stream is always evict_first
-  // one L2 policy for every gather: a per-lane choice would force a predicated R2UR of the
-  // policy descriptor per load (separate hot/cold policies measured no gain, DESIGN 9b)
+  // one L2 policy for every gather: a per-lane choice forces a predicated R2UR of the policy
+  // descriptor per load, and separate predicated loads per policy (hot rows evict_last, cold
+  // ones evict_first) measured 2x slower on H (profiles/r01_hs_sweep.txt)
   const uint32_t *src[NA];
   src[0] = a.irow;
 #pragma unroll
@@ -782,9 +783,10 @@ __global__ void __launch_bounds__(HS ? WPC_ * 32 : kThreads, HS ? 1 : (WA == 6 ?
               const uint32_t id = idx[j][u];
               if constexpr (HS) {  // shared-memory tier, L2-tier buffer or plain factor row
                 const bool in_s = (id >> 30) == 3u, in_h = (id >> 30) == 2u;
-                const float *gptr = (in_h ? a.hot_buf : a.Uo[j]) + uint64_t(id & 0x3FFFFFFFu) * R + col;
-                f[j][u] = ld_tiered(hs_saddr + ((id & 0x3FFFFFFFu) * R + col) * 4u, gptr,
-                                    pol.gather, u < cnt && in_s, u < cnt && !in_s);
+                const uint64_t off = uint64_t(id & 0x3FFFFFFFu) * R + col;
+                const float *gptr = (in_h ? a.hot_buf : a.Uo[j]) + off;
+                f[j][u] = ld_tiered(hs_saddr + uint32_t(off) * 4u, gptr, pol.gather, u < cnt && in_s,
+                                    u < cnt && !in_s);
               } else {
                 const float *base = a.Uo[j];
                 uint32_t row = id;
