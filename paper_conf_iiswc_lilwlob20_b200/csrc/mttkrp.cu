@@ -652,7 +652,7 @@ __global__ void __launch_bounds__(kThreads) hicoo_heavy_kernel(const HArgs a) {
 // HS (persistent, 16 warps, one CTA per SM): the shared-memory tier of the hot-row cache --
 // the most frequent factor rows are copied into shared memory once per CTA, and gathers of
 // entries tagged 0xC0000000 | slot read them there instead of from L2.
-template <int NO, int LPN, int WA, bool HS, int WPC_ = 16, int SG_ = 32>
+template <int NO, int LPN, int WA, bool HS, int WPC_ = 16, int SG_ = 32, int U_ = 4>
 __global__ void __launch_bounds__(HS ? WPC_ * 32 : kThreads, HS ? 1 : (WA == 6 ? 3 : 2))
     coo_staged_kernel(const KArgs a) {
   constexpr int WPC = HS ? WPC_ : kWarpsPerCta;
@@ -665,7 +665,7 @@ __global__ void __launch_bounds__(HS ? WPC_ * 32 : kThreads, HS ? 1 : (WA == 6 ?
   constexpr int GL = 8 / CG;      // groups per 128-B line
   constexpr int SW = G * SG;      // nonzeros per warp per stage
   constexpr int NA = NO + 2;      // arrays: i_n, i_k (k != n), val
-  constexpr int U = 4;
+  constexpr int U = U_;           // nonzeros per group per step (4 or 8; divides SG)
   extern __shared__ __align__(16) uint32_t stage_buf[];  // [warp][2][NA][SW]
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const int g = lane / LPN, lig = lane % LPN;
@@ -762,17 +762,22 @@ __global__ void __launch_bounds__(HS ? WPC_ * 32 : kThreads, HS ? 1 : (WA == 6 ?
 #pragma unroll 1
       for (int q = 0; q < scnt; q += U) {
         const int cnt = (scnt - q) >= U ? U : scnt - q;
-        const int qs = (((q / 4) ^ (g / GL)) & (CG - 1)) * 4;  // swizzled chunk (see issue_to)
-        const uint4 r4 = *reinterpret_cast<const uint4 *>(buf + qs);
-        const uint4 v4 = *reinterpret_cast<const uint4 *>(buf + (NA - 1) * SW + qs);
-        uint32_t row[U] = {r4.x, r4.y, r4.z, r4.w};
-        float v[U] = {__uint_as_float(v4.x), __uint_as_float(v4.y), __uint_as_float(v4.z),
-                      __uint_as_float(v4.w)};
+        uint32_t row[U];
+        float v[U];
         uint32_t idx[NO][U];
 #pragma unroll
-        for (int j = 0; j < NO; ++j) {
-          const uint4 i4 = *reinterpret_cast<const uint4 *>(buf + (1 + j) * SW + qs);
-          idx[j][0] = i4.x; idx[j][1] = i4.y; idx[j][2] = i4.z; idx[j][3] = i4.w;
+        for (int p = 0; p < U / 4; ++p) {
+          const int qs = ((((q / 4) + p) ^ (g / GL)) & (CG - 1)) * 4;  // swizzled chunk (see issue_to)
+          const uint4 r4 = *reinterpret_cast<const uint4 *>(buf + qs);
+          const uint4 v4 = *reinterpret_cast<const uint4 *>(buf + (NA - 1) * SW + qs);
+          row[4 * p] = r4.x; row[4 * p + 1] = r4.y; row[4 * p + 2] = r4.z; row[4 * p + 3] = r4.w;
+          v[4 * p] = __uint_as_float(v4.x); v[4 * p + 1] = __uint_as_float(v4.y);
+          v[4 * p + 2] = __uint_as_float(v4.z); v[4 * p + 3] = __uint_as_float(v4.w);
+#pragma unroll
+          for (int j = 0; j < NO; ++j) {
+            const uint4 i4 = *reinterpret_cast<const uint4 *>(buf + (1 + j) * SW + qs);
+            idx[j][4 * p] = i4.x; idx[j][4 * p + 1] = i4.y; idx[j][4 * p + 2] = i4.z; idx[j][4 * p + 3] = i4.w;
+          }
         }
         Vec<4> f[NO][U];
 #pragma unroll
@@ -1010,11 +1015,14 @@ void launch_coo_mttkrp(const pasta_coo *x, uint32_t mode, const float *const *fa
     // leaves holds the in-flight misses, so the tier stays at 512 rows (measured cliff between
     // 512 and 1024 rows on H and C3: 1.89 -> 2.17 ms, 1.84 -> 3.2 ms; profiles/r01_hs_sweep.txt).
     // PASTA_HOT_SMEM=0 selects the non-persistent kernel; PASTA_HOT_SMEM_ROWS caps the tier.
-    // HS shape (warps per CTA, nonzeros per group per stage): PASTA_HS_CFG = 0 (16, 32) or
-    // 1 (24, 16).  More warps = more gathers in flight; 24 warps fit 80 registers for order 3
-    // (H 1.81 -> 1.64 ms, C2 0.83 -> 0.77, C3 1.78 -> 1.58) but spill for order 4 (C4 0.74 ->
-    // 0.80), so the default is 1 for order 3 and 0 above (32 warps spill for every order).
-    const int hs_cfg = env_int("PASTA_HS_CFG", no == 2 ? 1 : 0);
+    // HS shape (warps per CTA, nonzeros per group per stage, nonzeros per group step):
+    // PASTA_HS_CFG = 0 (16, 32, 4), 1 (24, 16, 4), 2 (16, 32, 8; order 3 only).  More gathers
+    // in flight is the lever: 24 warps fit 80 registers for order 3 (H 1.81 -> 1.64 ms, C2
+    // 0.83 -> 0.77, C3 1.78 -> 1.58) but spill for order 4 (C4 0.74 -> 0.80); 8-deep steps
+    // (126 registers, 16 warps) gain another 5-7 % where the gathers go to DRAM (H 1.69 ->
+    // 1.57, C5 27.2 -> 26.6) but lose on L2-resident factors, whose shared-memory tier shrinks
+    // (C2 0.80 -> 0.88).  32 warps spill for every order.
+    const int hs_cfg = env_int("PASTA_HS_CFG", no == 2 ? (want_hot ? 2 : 1) : 0);
     const int hs_wpc = hs_cfg == 1 ? 24 : 16;
     const int hs_sg = hs_cfg == 1 ? 16 : 32;
     const size_t stage_hs = size_t(hs_wpc) * 2 * (no + 2) * (G * hs_sg) * sizeof(uint32_t);
@@ -1113,7 +1121,10 @@ void launch_coo_mttkrp(const pasta_coo *x, uint32_t mode, const float *const *fa
     using I16 = std::integral_constant<int, 16>;
     if (hs) {
       if (hs_cfg == 1) pick_hs(std::integral_constant<int, 24>(), I16());
-      else pick_hs(I16(), std::integral_constant<int, 32>());
+      else if (hs_cfg == 2 && no == 2) {
+        if (lpn == 4) go(coo_staged_kernel<2, 4, 1, true, 16, 32, 8>);
+        else go(coo_staged_kernel<2, 8, 1, true, 16, 32, 8>);
+      } else pick_hs(I16(), std::integral_constant<int, 32>());
     } else if (wa == 1) pick(std::integral_constant<int, 1>());
     else if (wa == 2) pick(std::integral_constant<int, 2>());
     else if (wa == 3) pick(std::integral_constant<int, 3>());

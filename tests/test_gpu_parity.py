@@ -395,12 +395,13 @@ def test_coo_hot_row_cache_forced(env, hot_mb, monkeypatch):
         _check(pasta.pasta_mttkrp_coo(x, 0, Ud2), ref, ab, "hot cache refill")
 
 
-@pytest.mark.parametrize("l2_tier,hs_cfg", [(False, "0"), (True, "0"), (False, "1"), (True, "1")])
+@pytest.mark.parametrize("l2_tier,hs_cfg", [(False, "0"), (True, "0"), (False, "1"), (True, "1"), (True, "2")])
 def test_coo_shared_memory_hot_tier(env, l2_tier, hs_cfg, monkeypatch):
     """The shared-memory tier of the hot-row cache (persistent coo_staged_kernel<..., HS>):
     forced on, alone or together with a tiny L2 tier so that smem-, L2-tier- and cold rows
     mix in one warp; 3M nonzeros give every warp of the persistent grid several chunks.
-    Both kernel shapes (16 warps x 32-deep stages, 24 warps x 16-deep) for every order."""
+    Every kernel shape (16 warps x 32-deep stages, 24 warps x 16-deep, 8 nonzeros per group
+    step) for every order."""
     pasta, oracle, torch = env
     monkeypatch.setenv("PASTA_HOT_SMEM", "1")
     monkeypatch.setenv("PASTA_HS_CFG", hs_cfg)
