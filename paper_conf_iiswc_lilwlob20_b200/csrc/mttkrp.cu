@@ -1021,7 +1021,8 @@ void launch_coo_mttkrp(const pasta_coo *x, uint32_t mode, const float *const *fa
     // 0.83 -> 0.77, C3 1.78 -> 1.58) but spill for order 4 (C4 0.74 -> 0.80); 8-deep steps
     // (126 registers, 16 warps) gain another 5-7 % where the gathers go to DRAM (H 1.69 ->
     // 1.57, C5 27.2 -> 26.6) but lose on L2-resident factors, whose shared-memory tier shrinks
-    // (C2 0.80 -> 0.88).  32 warps spill for every order.
+    // (C2 0.80 -> 0.88).  32 warps spill for every order; 8 warps x 16-deep steps (220
+    // registers) and 12 warps x 8-deep steps are slower everywhere (H 1.80 / 1.73 ms).
     const int hs_cfg = env_int("PASTA_HS_CFG", no == 2 ? (want_hot ? 2 : 1) : 0);
     const int hs_wpc = hs_cfg == 1 ? 24 : 16;
     const int hs_sg = hs_cfg == 1 ? 16 : 32;
