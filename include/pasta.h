@@ -185,6 +185,15 @@ pasta_status pasta_mttkrp_hicoo(pasta_hicoo *h, uint32_t mode, const float *cons
  * buffers are cached in the handle. */
 pasta_status pasta_mttkrp_coo_allmodes_host(pasta_coo *x, const float *const *host_factors,
                                             uint32_t R, float *const *host_out, void *stream);
+/* `nsteps` independent all-modes steps in one call (a stream of factor sets, e.g. serving):
+ * step i reads host_factors[i*order + k] and writes host_out[i*order + m] (same shapes as
+ * above; the arrays hold nsteps*order pointers).  Two device staging slots: step i+1's
+ * uploads overlap step i's downloads, so the per-step cost approaches the larger of the two
+ * transfer totals instead of their sum.  Every step's copies still happen.  Returns after the
+ * last result is in host memory; nsteps = 0 is a no-op. */
+pasta_status pasta_mttkrp_coo_allmodes_host_batch(pasta_coo *x, uint32_t nsteps,
+                                                  const float *const *host_factors, uint32_t R,
+                                                  float *const *host_out, void *stream);
 
 /* --------------------------------------------------------------- multi-GPU (a9) ------ */
 

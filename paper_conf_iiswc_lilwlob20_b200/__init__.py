@@ -19,7 +19,8 @@ __all__ = [
     "PastaError", "Coo", "Hicoo", "pasta_version", "pasta_set_allocator", "use_torch_allocator",
     "pasta_load_coo", "pasta_save_coo", "pasta_coo_from_arrays", "pasta_gen_powerlaw",
     "pasta_coo_to_hicoo", "pasta_coo_prepare", "pasta_hicoo_prepare", "pasta_mttkrp_coo",
-    "pasta_mttkrp_hicoo", "pasta_mttkrp_coo_allmodes_host", "pasta_coo_row_counts",
+    "pasta_mttkrp_hicoo", "pasta_mttkrp_coo_allmodes_host", "pasta_mttkrp_coo_allmodes_host_batch",
+    "pasta_coo_row_counts",
     "pasta_row_partition", "pasta_coo_partition", "pasta_coo_shard", "pasta_coo_info",
     "pasta_coo_export", "pasta_coo_export_mode", "pasta_hicoo_info", "pasta_hicoo_export",
     "pasta_launch_count", "pasta_profile_enable", "pasta_profile_read", "pasta_gram",
@@ -299,6 +300,23 @@ def pasta_mttkrp_coo_allmodes_host(x: Coo, host_factors, host_out, stream=None) 
         fp[k] = f.data_ptr() if hasattr(f, "data_ptr") else f.ctypes.data
         op[k] = o.data_ptr() if hasattr(o, "data_ptr") else o.ctypes.data
     check(lib().pasta_mttkrp_coo_allmodes_host(x.ptr, fp, R, op, _stream_ptr(stream)))
+
+
+def pasta_mttkrp_coo_allmodes_host_batch(x: Coo, steps, stream=None) -> None:
+    """`steps` = list of (host_factors, host_out) pairs, each like pasta_mttkrp_coo_allmodes_host's;
+    one pipelined call (step i+1's uploads overlap step i's downloads)."""
+    n = len(steps)
+    if n == 0:
+        return
+    R = int(steps[0][0][0].shape[1])
+    fp = (C.c_void_p * (n * x.order))()
+    op = (C.c_void_p * (n * x.order))()
+    for i, (hf, ho) in enumerate(steps):
+        for k in range(x.order):
+            f, o = hf[k], ho[k]
+            fp[i * x.order + k] = f.data_ptr() if hasattr(f, "data_ptr") else f.ctypes.data
+            op[i * x.order + k] = o.data_ptr() if hasattr(o, "data_ptr") else o.ctypes.data
+    check(lib().pasta_mttkrp_coo_allmodes_host_batch(x.ptr, n, fp, R, op, _stream_ptr(stream)))
 
 
 # ----------------------------------------------------------------------------- multi-GPU

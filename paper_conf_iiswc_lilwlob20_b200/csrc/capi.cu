@@ -562,6 +562,64 @@ pasta_status pasta_mttkrp_hicoo(pasta_hicoo *h, uint32_t mode, const float *cons
   API_END
 }
 
+// nsteps independent all-modes steps from/to host buffers (step i: host_factors[i*N + k],
+// host_out[i*N + m]).  Pipelined: factors go up on a copy stream in the order the modes need
+// them (U1..U_{N-1}, then U0), mode m's kernel starts as soon as its factors have landed, its
+// result goes down on a second copy stream while later modes compute (PCIe/C2C is full
+// duplex), and with nsteps > 1 step i+1's uploads (slot (i+1) & 1) overlap step i's
+// downloads.  Returns after the last result is in host memory.
+static void allmodes_host_steps(pasta_coo *x, uint32_t nsteps, const float *const *host_factors,
+                                uint32_t R, float *const *host_out, cudaStream_t s) {
+  const uint32_t N = x->order;
+  for (uint32_t k = 0; k < N; ++k) coo_prepare_mode(x, k, s);
+  const int nslots = nsteps > 1 ? 2 : 1;
+  for (int b = 0; b < nslots; ++b) {
+    if (x->stage_R[b] == R) continue;
+    for (uint32_t k = 0; k < N; ++k) {
+      x->stage_f[b][k].alloc(uint64_t(x->dims[k]) * R, s);
+      x->stage_o[b][k].alloc(uint64_t(x->dims[k]) * R, s);
+    }
+    x->stage_R[b] = R;
+  }
+  E2EStreams &e = x->e2e;
+  e.init();
+  PASTA_CUDA(cudaEventRecord(e.start, s));
+  PASTA_CUDA(cudaStreamWaitEvent(e.h2d, e.start, 0));
+  PASTA_CUDA(cudaStreamWaitEvent(e.d2h, e.start, 0));
+  for (uint32_t i = 0; i < nsteps; ++i) {
+    const int b = int(i & 1u);
+    const float *const *hf = host_factors + size_t(i) * N;
+    float *const *ho = host_out + size_t(i) * N;
+    const float *dfac[kMaxOrder];
+    if (i >= 2) PASTA_CUDA(cudaStreamWaitEvent(e.h2d, e.kd[b], 0));  // step i-2 done reading
+    for (uint32_t j = 0; j < N; ++j) {
+      const uint32_t k = (j + 1) % N;  // 1, 2, ..., N-1, 0
+      PASTA_CUDA(cudaMemcpyAsync(x->stage_f[b][k].p, hf[k], uint64_t(x->dims[k]) * R * sizeof(float),
+                                 cudaMemcpyHostToDevice, e.h2d));
+      PASTA_CUDA(cudaEventRecord(e.f[b][k], e.h2d));
+      dfac[k] = x->stage_f[b][k].p;
+    }
+    for (uint32_t m = 0; m < N; ++m) {
+      for (uint32_t k = 0; k < N; ++k)
+        if (k != m) PASTA_CUDA(cudaStreamWaitEvent(s, e.f[b][k], 0));
+      if (i >= 2) PASTA_CUDA(cudaStreamWaitEvent(s, e.od[b][m], 0));  // step i-2's result is out
+      uint64_t lo = 0, hi = x->dims[m];
+      if (x->shard_mode == int(m)) { lo = x->row_lo; hi = x->row_hi; }
+      launch_zero_rows(x->stage_o[b][m].p, lo, hi, R, s);
+      launch_coo_mttkrp(x, m, dfac, R, x->stage_o[b][m].p, s);
+      PASTA_CUDA(cudaEventRecord(e.o[b][m], s));
+      PASTA_CUDA(cudaStreamWaitEvent(e.d2h, e.o[b][m], 0));
+      PASTA_CUDA(cudaMemcpyAsync(ho[m], x->stage_o[b][m].p, uint64_t(x->dims[m]) * R * sizeof(float),
+                                 cudaMemcpyDeviceToHost, e.d2h));
+      PASTA_CUDA(cudaEventRecord(e.od[b][m], e.d2h));
+    }
+    PASTA_CUDA(cudaEventRecord(e.kd[b], s));
+  }
+  PASTA_CUDA(cudaStreamSynchronize(e.d2h));
+  PASTA_CUDA(cudaStreamSynchronize(e.h2d));
+  PASTA_CUDA(cudaStreamSynchronize(s));
+}
+
 pasta_status pasta_mttkrp_coo_allmodes_host(pasta_coo *x, const float *const *host_factors, uint32_t R,
                                             float *const *host_out, void *stream) {
   API_BEGIN
@@ -572,45 +630,21 @@ pasta_status pasta_mttkrp_coo_allmodes_host(pasta_coo *x, const float *const *ho
   check_device(x->device);
   cudaStream_t s = as_stream(stream);
   std::lock_guard<std::mutex> lk(x->mu);
-  for (uint32_t k = 0; k < x->order; ++k) coo_prepare_mode(x, k, s);
-  if (x->stage_R != R) {
-    for (uint32_t k = 0; k < x->order; ++k) {
-      x->stage_f[k].alloc(uint64_t(x->dims[k]) * R, s);
-      x->stage_o[k].alloc(uint64_t(x->dims[k]) * R, s);
-    }
-    x->stage_R = R;
-  }
-  // Pipelined: factors go up on a copy stream in the order the modes need them
-  // (U1..U_{N-1}, then U0), mode m's kernel starts as soon as its factors have landed,
-  // and its result goes down on a second copy stream while later modes compute
-  // (PCIe/C2C is full duplex).
-  E2EStreams &e = x->e2e;
-  e.init();
-  const uint32_t N = x->order;
-  const float *dfac[kMaxOrder];
-  PASTA_CUDA(cudaEventRecord(e.start, s));
-  PASTA_CUDA(cudaStreamWaitEvent(e.h2d, e.start, 0));
-  for (uint32_t j = 0; j < N; ++j) {
-    uint32_t k = (j + 1) % N;  // 1, 2, ..., N-1, 0
-    PASTA_CUDA(cudaMemcpyAsync(x->stage_f[k].p, host_factors[k], uint64_t(x->dims[k]) * R * sizeof(float),
-                               cudaMemcpyHostToDevice, e.h2d));
-    PASTA_CUDA(cudaEventRecord(e.f[k], e.h2d));
-    dfac[k] = x->stage_f[k].p;
-  }
-  for (uint32_t m = 0; m < N; ++m) {
-    for (uint32_t k = 0; k < N; ++k)
-      if (k != m) PASTA_CUDA(cudaStreamWaitEvent(s, e.f[k], 0));
-    uint64_t lo = 0, hi = x->dims[m];
-    if (x->shard_mode == int(m)) { lo = x->row_lo; hi = x->row_hi; }
-    launch_zero_rows(x->stage_o[m].p, lo, hi, R, s);
-    launch_coo_mttkrp(x, m, dfac, R, x->stage_o[m].p, s);
-    PASTA_CUDA(cudaEventRecord(e.o[m], s));
-    PASTA_CUDA(cudaStreamWaitEvent(e.d2h, e.o[m], 0));
-    PASTA_CUDA(cudaMemcpyAsync(host_out[m], x->stage_o[m].p, uint64_t(x->dims[m]) * R * sizeof(float),
-                               cudaMemcpyDeviceToHost, e.d2h));
-  }
-  PASTA_CUDA(cudaStreamSynchronize(e.d2h));
-  PASTA_CUDA(cudaStreamSynchronize(s));
+  allmodes_host_steps(x, 1, host_factors, R, host_out, s);
+  API_END
+}
+
+pasta_status pasta_mttkrp_coo_allmodes_host_batch(pasta_coo *x, uint32_t nsteps, const float *const *host_factors,
+                                                  uint32_t R, float *const *host_out, void *stream) {
+  API_BEGIN
+  require(x && host_factors && host_out, "x/host_factors/host_out is NULL");
+  require(R >= 1, "R must be >= 1");
+  for (uint64_t k = 0; k < uint64_t(nsteps) * x->order; ++k)
+    require(host_factors[k] && host_out[k], "host_factors[i*order+k]/host_out[i*order+k] is NULL");
+  check_device(x->device);
+  cudaStream_t s = as_stream(stream);
+  std::lock_guard<std::mutex> lk(x->mu);
+  if (nsteps) allmodes_host_steps(x, nsteps, host_factors, R, host_out, s);
   API_END
 }
 

@@ -77,26 +77,38 @@ struct DevArray {
 };
 
 // Copy streams and events of the end-to-end host path (created on first use).
+// Two staging slots: step i of a batch uses slot i & 1, so that step i+1's uploads overlap
+// step i's downloads.  f: factor k of a slot landed; o: output m of a slot computed; od:
+// output m of a slot downloaded (slot reusable); kd: every kernel of a slot done.
 struct E2EStreams {
   cudaStream_t h2d = nullptr, d2h = nullptr;
-  cudaEvent_t f[kMaxOrder] = {}, o[kMaxOrder] = {}, start = nullptr;
+  cudaEvent_t f[2][kMaxOrder] = {}, o[2][kMaxOrder] = {}, od[2][kMaxOrder] = {}, kd[2] = {};
+  cudaEvent_t start = nullptr;
   bool ready = false;
   void init() {
     if (ready) return;
     cudaStreamCreateWithFlags(&h2d, cudaStreamNonBlocking);
     cudaStreamCreateWithFlags(&d2h, cudaStreamNonBlocking);
-    for (int k = 0; k < kMaxOrder; ++k) {
-      cudaEventCreateWithFlags(&f[k], cudaEventDisableTiming);
-      cudaEventCreateWithFlags(&o[k], cudaEventDisableTiming);
+    for (int b = 0; b < 2; ++b) {
+      for (int k = 0; k < kMaxOrder; ++k) {
+        cudaEventCreateWithFlags(&f[b][k], cudaEventDisableTiming);
+        cudaEventCreateWithFlags(&o[b][k], cudaEventDisableTiming);
+        cudaEventCreateWithFlags(&od[b][k], cudaEventDisableTiming);
+      }
+      cudaEventCreateWithFlags(&kd[b], cudaEventDisableTiming);
     }
     cudaEventCreateWithFlags(&start, cudaEventDisableTiming);
     ready = true;
   }
   ~E2EStreams() {
     if (!ready) return;
-    for (int k = 0; k < kMaxOrder; ++k) {
-      cudaEventDestroy(f[k]);
-      cudaEventDestroy(o[k]);
+    for (int b = 0; b < 2; ++b) {
+      for (int k = 0; k < kMaxOrder; ++k) {
+        cudaEventDestroy(f[b][k]);
+        cudaEventDestroy(o[b][k]);
+        cudaEventDestroy(od[b][k]);
+      }
+      cudaEventDestroy(kd[b]);
     }
     cudaEventDestroy(start);
     cudaStreamDestroy(h2d);
@@ -177,9 +189,9 @@ struct pasta_coo {
   int shard_mode = -1;  // >= 0: this handle is the [row_lo, row_hi) shard of that mode
   uint32_t row_lo = 0, row_hi = 0;
   // e2e staging (pasta_mttkrp_coo_allmodes_host)
-  uint32_t stage_R = 0;
-  pasta::DevArray<float> stage_f[pasta::kMaxOrder];
-  pasta::DevArray<float> stage_o[pasta::kMaxOrder];
+  uint32_t stage_R[2] = {};
+  pasta::DevArray<float> stage_f[2][pasta::kMaxOrder];
+  pasta::DevArray<float> stage_o[2][pasta::kMaxOrder];
   pasta::E2EStreams e2e;
   // per-mode row nonzero counts (device u32) and their bucket histogram (host)
   bool counts_ready[pasta::kMaxOrder] = {};

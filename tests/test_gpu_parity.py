@@ -226,6 +226,29 @@ def test_allmodes_host_e2e_matches_device(env):
         _check(ho[n].numpy().astype(np.float64), ref, ab, f"e2e mode {n}")
 
 
+def test_allmodes_host_batch_pipelined_steps(env):
+    """pasta_mttkrp_coo_allmodes_host_batch: independent steps with different factors share two
+    device staging slots (step i+1 uploads while step i downloads); every step's result must
+    match the oracle for that step's factors (a slot reused too early would mix steps)."""
+    pasta, oracle, torch = env
+    dims = (700, 500, 900)
+    inds, vals = si.powerlaw_coo(dims, 80_000, seed=21)
+    x = pasta.pasta_coo_from_arrays(dims, inds, vals)
+    steps, Us = [], []
+    for i in range(5):
+        U = si.factors(dims, 16, seed=100 + i)
+        Us.append(U)
+        hf = [torch.from_numpy(u).pin_memory() for u in U]
+        ho = [torch.full((d, 16), float("nan"), dtype=torch.float32).pin_memory() for d in dims]
+        steps.append((hf, ho))
+    pasta.pasta_mttkrp_coo_allmodes_host_batch(x, steps)
+    for i, (hf, ho) in enumerate(steps):
+        for n in range(3):
+            ref, ab = oracle.mttkrp(dims, inds, vals, n, Us[i])
+            _check(ho[n].numpy().astype(np.float64), ref, ab, f"batch step {i} mode {n}")
+    pasta.pasta_mttkrp_coo_allmodes_host_batch(x, [])  # no-op
+
+
 def test_tns_roundtrip(env, tmp_path):
     pasta, oracle, torch = env
     dims = (50, 60, 70)
