@@ -1016,14 +1016,14 @@ void launch_coo_mttkrp(const pasta_coo *x, uint32_t mode, const float *const *fa
     // 512 and 1024 rows on H and C3: 1.89 -> 2.17 ms, 1.84 -> 3.2 ms; profiles/r01_hs_sweep.txt).
     // PASTA_HOT_SMEM=0 selects the non-persistent kernel; PASTA_HOT_SMEM_ROWS caps the tier.
     // HS shape (warps per CTA, nonzeros per group per stage, nonzeros per group step):
-    // PASTA_HS_CFG = 0 (16, 32, 4), 1 (24, 16, 4), 2 (16, 32, 8; order 3 only).  More gathers
+    // PASTA_HS_CFG = 0 (16, 32, 4), 1 (24, 16, 4), 2 (16, 32, 8; orders 2 and 3).  More gathers
     // in flight is the lever: 24 warps fit 80 registers for order 3 (H 1.81 -> 1.64 ms, C2
     // 0.83 -> 0.77, C3 1.78 -> 1.58) but spill for order 4 (C4 0.74 -> 0.80); 8-deep steps
     // (126 registers, 16 warps) gain another 5-7 % where the gathers go to DRAM (H 1.69 ->
     // 1.57, C5 27.2 -> 26.6) but lose on L2-resident factors, whose shared-memory tier shrinks
     // (C2 0.80 -> 0.88).  32 warps spill for every order; 8 warps x 16-deep steps (220
     // registers) and 12 warps x 8-deep steps are slower everywhere (H 1.80 / 1.73 ms).
-    const int hs_cfg = env_int("PASTA_HS_CFG", no == 2 ? (want_hot ? 2 : 1) : 0);
+    const int hs_cfg = env_int("PASTA_HS_CFG", no <= 2 ? (want_hot ? 2 : 1) : 0);
     const int hs_wpc = hs_cfg == 1 ? 24 : 16;
     const int hs_sg = hs_cfg == 1 ? 16 : 32;
     const size_t stage_hs = size_t(hs_wpc) * 2 * (no + 2) * (G * hs_sg) * sizeof(uint32_t);
@@ -1032,7 +1032,7 @@ void launch_coo_mttkrp(const pasta_coo *x, uint32_t mode, const float *const *fa
         stage_hs < smem_cap ? uint32_t((smem_cap - stage_hs) / (size_t(R) * sizeof(float))) : 0u;
     if (want_hot) hs_rows_budget = std::min(hs_rows_budget, 512u);
     if (const int cap = env_int("PASTA_HOT_SMEM_ROWS", 0)) hs_rows_budget = std::min(hs_rows_budget, uint32_t(cap));
-    bool hs = env_int("PASTA_HOT_SMEM", 1) != 0 && hs_rows_budget >= 64 && no >= 2;
+    bool hs = env_int("PASTA_HOT_SMEM", 1) != 0 && hs_rows_budget >= 64;
     if (hs) {
       coo_mark_hot(const_cast<pasta_coo *>(x), mode, R, want_hot, hs_rows_budget, s);
       if (mc.hot_R != R || mc.hs_total == 0) hs = false;
@@ -1114,7 +1114,9 @@ void launch_coo_mttkrp(const pasta_coo *x, uint32_t mode, const float *const *fa
     };
     auto pick_hs = [&](auto wtag, auto stag) {
       constexpr int W = decltype(wtag)::value, S = decltype(stag)::value;
-      if (no == 2 && lpn == 4) go(coo_staged_kernel<2, 4, 1, true, W, S>);
+      if (no == 1 && lpn == 4) go(coo_staged_kernel<1, 4, 1, true, W, S>);
+      else if (no == 1) go(coo_staged_kernel<1, 8, 1, true, W, S>);
+      else if (no == 2 && lpn == 4) go(coo_staged_kernel<2, 4, 1, true, W, S>);
       else if (no == 2) go(coo_staged_kernel<2, 8, 1, true, W, S>);
       else if (lpn == 4) go(coo_staged_kernel<3, 4, 1, true, W, S>);
       else go(coo_staged_kernel<3, 8, 1, true, W, S>);
@@ -1122,7 +1124,10 @@ void launch_coo_mttkrp(const pasta_coo *x, uint32_t mode, const float *const *fa
     using I16 = std::integral_constant<int, 16>;
     if (hs) {
       if (hs_cfg == 1) pick_hs(std::integral_constant<int, 24>(), I16());
-      else if (hs_cfg == 2 && no == 2) {
+      else if (hs_cfg == 2 && no == 1) {
+        if (lpn == 4) go(coo_staged_kernel<1, 4, 1, true, 16, 32, 8>);
+        else go(coo_staged_kernel<1, 8, 1, true, 16, 32, 8>);
+      } else if (hs_cfg == 2 && no == 2) {
         if (lpn == 4) go(coo_staged_kernel<2, 4, 1, true, 16, 32, 8>);
         else go(coo_staged_kernel<2, 8, 1, true, 16, 32, 8>);
       } else pick_hs(I16(), std::integral_constant<int, 32>());
