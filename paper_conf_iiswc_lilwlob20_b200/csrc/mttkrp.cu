@@ -296,30 +296,16 @@ struct HicooRowSrc {
   static constexpr bool kSortedRows = true;
   static constexpr int kMinBlocks = 2;  // cap registers at 128: >= 16 resident warps per SM
   static constexpr int NOA = NO > 0 ? NO : kMaxOrder - 1;
-  // current slice and the next one, loaded one slice ahead so that advancing through
-  // short slices does not wait on a dependent load
-  uint64_t sb, sbend, nend;
-  uint32_t srow, nrow;
-  uint32_t base[NOA], nbase[NOA];
+  // current slice (the one holding the next entry).  A step of U entries spans at most U
+  // slices, so each step loads the metadata of slices sb+1 .. sb+U-1 at once (independent
+  // loads, one latency per step) instead of walking slice after slice with a dependent load
+  // each -- at ~1 entry per slice (hypersparse tensors) the walk was the kernel's critical path.
+  uint64_t sb, sbend;
+  uint32_t srow;
+  uint32_t base[NOA];
   int no;
   uint32_t wide;
   uint64_t pol;
-  __device__ __forceinline__ void load_next(const KArgs &a) {
-    const uint64_t n1 = sb + 1 < a.nsb ? sb + 1 : sb;  // clamp: never read past the end
-    nend = __ldg(a.sbptr + n1 + 1);
-    nrow = __ldg(a.sbrow + n1);
-#pragma unroll
-    for (int j = 0; j < NOA; ++j)
-      if (j < no) nbase[j] = ((wide >> j) & 1u) ? 0u : __ldg(a.sbbase[j] + n1);
-  }
-  __device__ __forceinline__ void advance(const KArgs &a) {
-    ++sb;
-    sbend = nend;
-    srow = nrow;
-#pragma unroll
-    for (int j = 0; j < NOA; ++j) base[j] = nbase[j];
-    load_next(a);
-  }
   __device__ __forceinline__ void init(const KArgs &a, uint64_t x0, uint64_t p) {
     pol = p;
     no = int(a.order) - 1;
@@ -335,10 +321,25 @@ struct HicooRowSrc {
 #pragma unroll
     for (int j = 0; j < NOA; ++j)
       if (j < no) base[j] = ((wide >> j) & 1u) ? 0u : __ldg(a.sbbase[j] + sb);
-    load_next(a);
   }
   __device__ __forceinline__ void load(const KArgs &a, uint64_t x, int cnt, uint32_t (&row)[U],
                                        uint32_t (&idx)[NOA][U], float (&v)[U], int) {
+    // slice window: slot 0 = current slice, slots 1 .. U-1 = the next ones (clamped)
+    uint64_t wend[U];
+    uint32_t wrow[U], wbase[NOA][U];
+    wend[0] = sbend;
+    wrow[0] = srow;
+#pragma unroll
+    for (int j = 0; j < NOA; ++j) wbase[j][0] = base[j];
+#pragma unroll
+    for (int t = 1; t < U; ++t) {
+      const uint64_t st = sb + t < a.nsb ? sb + t : a.nsb - 1;
+      wend[t] = __ldg(a.sbptr + st + 1);
+      wrow[t] = __ldg(a.sbrow + st);
+#pragma unroll
+      for (int j = 0; j < NOA; ++j)
+        if (j < no) wbase[j][t] = ((wide >> j) & 1u) ? 0u : __ldg(a.sbbase[j] + st);
+    }
     uint32_t ej[NOA][U];
     if (cnt == U && (x & 3) == 0) {
 #pragma unroll
@@ -371,15 +372,55 @@ struct HicooRowSrc {
         }
       }
     }
+    // entry u lies in window slot c_u = #{t : wend[t] <= x + u} (ends ascend); selects are
+    // unrolled compares so the window stays in registers
+    int clast = 0;
 #pragma unroll
     for (int u = 0; u < U; ++u) {
       if (u < cnt) {
-        while (x + u >= sbend) advance(a);  // walk to the entry's slice
-        row[u] = srow;
+        int c = 0;
+#pragma unroll
+        for (int t = 0; t < U - 1; ++t) c += (x + u >= wend[t]) ? 1 : 0;
+        uint32_t r = wrow[0];
+        uint32_t bsel[NOA];
+#pragma unroll
+        for (int j = 0; j < NOA; ++j) bsel[j] = wbase[j][0];
+#pragma unroll
+        for (int t = 1; t < U; ++t) {
+          if (c == t) {
+            r = wrow[t];
+#pragma unroll
+            for (int j = 0; j < NOA; ++j) bsel[j] = wbase[j][t];
+          }
+        }
+        row[u] = r;
 #pragma unroll
         for (int j = 0; j < NOA; ++j)
-          if (j < no) idx[j][u] = base[j] + ej[j][u];
+          if (j < no) idx[j][u] = bsel[j] + ej[j][u];
+        clast = c;
       }
+    }
+    // the slice of the last entry becomes the current one
+#pragma unroll
+    for (int t = 1; t < U; ++t) {
+      if (clast == t) {
+        sbend = wend[t];
+        srow = wrow[t];
+#pragma unroll
+        for (int j = 0; j < NOA; ++j) base[j] = wbase[j][t];
+      }
+    }
+    sb += uint64_t(clast);
+    // the next entry may start the following slice: advance once more if so (slot clast + 1
+    // is loaded when clast + 1 < U; otherwise the next step's window starts from here)
+    if (x + cnt >= sbend) {
+      const uint64_t st = sb + 1 < a.nsb ? sb + 1 : a.nsb - 1;
+      sb = st;
+      sbend = __ldg(a.sbptr + st + 1);
+      srow = __ldg(a.sbrow + st);
+#pragma unroll
+      for (int j = 0; j < NOA; ++j)
+        if (j < no) base[j] = ((wide >> j) & 1u) ? 0u : __ldg(a.sbbase[j] + st);
     }
   }
 };
