@@ -697,6 +697,9 @@ template <int NO, int LPN, int WA, bool HS, int WPC_ = 16, int SG_ = 32, int U_ 
 __global__ void __launch_bounds__(HS ? WPC_ * 32 : kThreads, HS ? 1 : (WA == 6 ? 3 : 2))
     coo_staged_kernel(const KArgs a) {
   constexpr int WPC = HS ? WPC_ : kWarpsPerCta;
+  // 7: HS kernel without the L2 tier (no hot_buf rows) whose gathered factors are < 4 GB each:
+  // no base-pointer select, 32-bit byte offsets
+  constexpr bool kL2T = WA != 7;
   constexpr bool kGather = WA != 4 && WA != 5;
   constexpr bool kWrite = WA != 3 && WA != 5;
   constexpr int kBuf = (WA == 0 || WA == 2) ? WA : 1;  // 6: form 1 with 3 CTAs per SM
@@ -828,11 +831,19 @@ __global__ void __launch_bounds__(HS ? WPC_ * 32 : kThreads, HS ? 1 : (WA == 6 ?
             if (kGather) {
               const uint32_t id = idx[j][u];
               if constexpr (HS) {  // shared-memory tier, L2-tier buffer or plain factor row
-                const bool in_s = (id >> 30) == 3u, in_h = (id >> 30) == 2u;
-                const uint64_t off = uint64_t(id & 0x3FFFFFFFu) * R + col;
-                const float *gptr = (in_h ? a.hot_buf : a.Uo[j]) + off;
-                f[j][u] = ld_tiered(hs_saddr + uint32_t(off) * 4u, gptr, pol.gather, u < cnt && in_s,
-                                    u < cnt && !in_s);
+                const bool in_s = (id >> 30) == 3u;
+                if constexpr (kL2T) {
+                  const bool in_h = (id >> 30) == 2u;
+                  const uint64_t off = uint64_t(id & 0x3FFFFFFFu) * R + col;
+                  const float *gptr = (in_h ? a.hot_buf : a.Uo[j]) + off;
+                  f[j][u] = ld_tiered(hs_saddr + uint32_t(off) * 4u, gptr, pol.gather, u < cnt && in_s,
+                                      u < cnt && !in_s);
+                } else {
+                  const uint32_t boff = ((id & 0x3FFFFFFFu) * R + col) * 4u;  // < 4 GB
+                  const float *gptr = reinterpret_cast<const float *>(
+                      reinterpret_cast<const char *>(a.Uo[j]) + boff);
+                  f[j][u] = ld_tiered(hs_saddr + boff, gptr, pol.gather, u < cnt && in_s, u < cnt && !in_s);
+                }
               } else {
                 const float *base = a.Uo[j];
                 uint32_t row = id;
@@ -1153,14 +1164,23 @@ void launch_coo_mttkrp(const pasta_coo *x, uint32_t mode, const float *const *fa
       else if (lpn == 4) go(coo_staged_kernel<3, 4, W, false>);
       else go(coo_staged_kernel<3, 8, W, false>);
     };
+    // WA 7 = the HS kernel without the L2 tier (no tag-2 entries): no base-pointer select
+    uint64_t max_factor = 0;
+    for (uint32_t k = 0; k < x->order; ++k)
+      if (k != mode) max_factor = std::max<uint64_t>(max_factor, uint64_t(x->dims[k]) * R * sizeof(float));
+    const bool l2t = mc.hot_total > 0 || max_factor >= (uint64_t(1) << 32);
+    auto pick_hs3 = [&](auto wtag, auto stag, auto atag) {
+      constexpr int W = decltype(wtag)::value, S = decltype(stag)::value, A = decltype(atag)::value;
+      if (no == 1 && lpn == 4) go(coo_staged_kernel<1, 4, A, true, W, S>);
+      else if (no == 1) go(coo_staged_kernel<1, 8, A, true, W, S>);
+      else if (no == 2 && lpn == 4) go(coo_staged_kernel<2, 4, A, true, W, S>);
+      else if (no == 2) go(coo_staged_kernel<2, 8, A, true, W, S>);
+      else if (lpn == 4) go(coo_staged_kernel<3, 4, A, true, W, S>);
+      else go(coo_staged_kernel<3, 8, A, true, W, S>);
+    };
     auto pick_hs = [&](auto wtag, auto stag) {
-      constexpr int W = decltype(wtag)::value, S = decltype(stag)::value;
-      if (no == 1 && lpn == 4) go(coo_staged_kernel<1, 4, 1, true, W, S>);
-      else if (no == 1) go(coo_staged_kernel<1, 8, 1, true, W, S>);
-      else if (no == 2 && lpn == 4) go(coo_staged_kernel<2, 4, 1, true, W, S>);
-      else if (no == 2) go(coo_staged_kernel<2, 8, 1, true, W, S>);
-      else if (lpn == 4) go(coo_staged_kernel<3, 4, 1, true, W, S>);
-      else go(coo_staged_kernel<3, 8, 1, true, W, S>);
+      if (l2t) pick_hs3(wtag, stag, std::integral_constant<int, 1>());
+      else pick_hs3(wtag, stag, std::integral_constant<int, 7>());
     };
     using I16 = std::integral_constant<int, 16>;
     if (hs) {
