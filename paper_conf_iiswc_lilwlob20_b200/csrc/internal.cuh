@@ -166,6 +166,9 @@ struct HicooModeCopy {
   DevArray<uint32_t> sbrow;              // nsb: output row of the slice
   DevArray<uint32_t> sbbase[kMaxOrder];  // nsb each (k != mode, k compressed): binds_k << block_bits
   DevArray<uint32_t> uinds[kMaxOrder];   // gHiCOO: nnz each (k != mode, k uncompressed): i_k
+  // staged decode (launch_hicoo_mttkrp): slice holding the first entry of every group run
+  DevArray<uint64_t> run_sb;
+  uint64_t run_sb_run = 0;
 };
 
 }  // namespace pasta

@@ -74,6 +74,9 @@ struct KArgs {
   // shared-memory tier: slot -> factor row; other-mode slot j owns slots [hs_lo[j], hs_lo[j+1])
   const uint32_t *hs_rows;
   uint32_t hs_lo[kMaxOrder];
+  // HiCOO row slices decoded into the staged kernel (WA 9): run_sb[r] = slice holding entry
+  // r * (chunk / G), the first entry of group run r
+  const uint64_t *run_sb;
 };
 
 // Per-thread L2 cache policies (createpolicy, sm_80+): the nonzero stream is touched once
@@ -698,8 +701,10 @@ __global__ void __launch_bounds__(HS ? WPC_ * 32 : kThreads, HS ? 1 : (WA == 6 ?
     coo_staged_kernel(const KArgs a) {
   constexpr int WPC = HS ? WPC_ : kWarpsPerCta;
   // 7: HS kernel without the L2 tier (no hot_buf rows) whose gathered factors are < 4 GB each:
-  // no base-pointer select, 32-bit byte offsets
-  constexpr bool kL2T = WA != 7;
+  // no base-pointer select, 32-bit byte offsets.  9: HiCOO row slices decoded warp-wide into
+  // the stage buffer (no hot tiers, 64-bit offsets)
+  constexpr bool kHic = WA == 9;
+  constexpr bool kL2T = WA != 7 && !kHic;
   constexpr bool kGather = WA != 4 && WA != 5;
   constexpr bool kWrite = WA != 3 && WA != 5;
   constexpr int kBuf = (WA == 0 || WA == 2) ? WA : 1;  // 6: form 1 with 3 CTAs per SM
@@ -771,7 +776,61 @@ __global__ void __launch_bounds__(HS ? WPC_ * 32 : kThreads, HS ? 1 : (WA == 6 ?
     }
     asm volatile("cp.async.commit_group;" ::: "memory");
   };
+  // HiCOO decode (WA 9, SG == 32): for each group window of 32 entries, lane l takes entry
+  // p + l and slice slot sb + l (the window's entries lie in at most 32 consecutive slices);
+  // an entry's slot = #{slots whose end <= entry} by a 5-step shuffle search over the sorted
+  // slot ends; row and block bases come from the owning lane by shuffle; i_k = base + e_k
+  // (Alg. 3's rebased pointers).  gsb[g] = current slice of group g (warp-uniform).
+  uint64_t gsb[G];
+  auto decode_to = [&](uint64_t cc, int s, uint32_t *dst) {
+    if (cc >= a.nnz) return;
+    const uint64_t r0 = cc / run;
+#pragma unroll
+    for (int gi = 0; gi < G; ++gi) {
+      const uint64_t p = cc + uint64_t(gi) * run + uint64_t(s) * SG;
+      if (p >= a.nnz) continue;  // warp-uniform
+      if (s == 0) gsb[gi] = __ldg(a.run_sb + r0 + gi);
+      const uint64_t sb0 = gsb[gi];
+      const uint64_t st = sb0 + lane < a.nsb ? sb0 + lane : a.nsb - 1;
+      const uint64_t eabs = __ldg(a.sbptr + st + 1);
+      const uint32_t erel = eabs - p > 64 ? 64u : uint32_t(eabs - p);
+      const uint32_t srow = __ldg(a.sbrow + st);
+      uint32_t sbase[NO];
+#pragma unroll
+      for (int j = 0; j < NO; ++j) sbase[j] = ((a.wide >> j) & 1u) ? 0u : __ldg(a.sbbase[j] + st);
+      const uint64_t x = p + lane;
+      const bool ok = x < a.nnz;
+      const float v = ok ? __ldg(a.val + x) : 0.f;
+      uint32_t e[NO];
+#pragma unroll
+      for (int j = 0; j < NO; ++j)
+        e[j] = !ok ? 0u : ((a.wide >> j) & 1u) ? __ldg(a.io[j] + x) : uint32_t(__ldg(a.eo[j] + x));
+      int c = 0;  // <= 31: slot 0 holds entry p, so 32 entries span at most 32 slots
+#pragma unroll
+      for (int k = 16; k >= 1; k >>= 1) {
+        const uint32_t et = __shfl_sync(0xFFFFFFFFu, erel, c + k - 1);
+        if (et <= uint32_t(lane)) c += k;
+      }
+      const uint32_t row = __shfl_sync(0xFFFFFFFFu, srow, c);
+      const int d = gi * SG + (((lane / 4) ^ (gi / GL)) & (CG - 1)) * 4 + (lane & 3);
+      dst[d] = row;
+#pragma unroll
+      for (int j = 0; j < NO; ++j) dst[(1 + j) * SW + d] = __shfl_sync(0xFFFFFFFFu, sbase[j], c) + e[j];
+      dst[(NA - 1) * SW + d] = __float_as_uint(v);
+      // the next window starts at the slice holding entry p + SG: the last entry's slice, or
+      // the one after it when that slice ends inside this window
+      const uint64_t nleft = a.nnz - p;
+      const int last = nleft >= uint64_t(SG) ? SG - 1 : int(nleft) - 1;
+      const int clast = __shfl_sync(0xFFFFFFFFu, c, last);
+      const uint32_t elast = __shfl_sync(0xFFFFFFFFu, erel, clast);
+      gsb[gi] = sb0 + uint64_t(clast) + (elast <= uint32_t(SG) ? 1u : 0u);
+    }
+  };
   auto issue = [&](uint64_t cc, int s, int b) {
+    if constexpr (kHic) {
+      decode_to(cc, s, wbuf + b * NA * SW);
+      return;
+    }
     if (kBuf == 1) {
       if (b) issue_to(cc, s, wbuf + NA * SW); else issue_to(cc, s, wbuf);
     } else {
@@ -830,7 +889,9 @@ __global__ void __launch_bounds__(HS ? WPC_ * 32 : kThreads, HS ? 1 : (WA == 6 ?
           for (int j = 0; j < NO; ++j) {
             if (kGather) {
               const uint32_t id = idx[j][u];
-              if constexpr (HS) {  // shared-memory tier, L2-tier buffer or plain factor row
+              if constexpr (kHic) {  // decoded HiCOO coordinate: plain factor row
+                if (u < cnt) f[j][u] = ldg_vec<4>(a.Uo[j] + uint64_t(id) * R + col, pol.gather);
+              } else if constexpr (HS) {  // shared-memory tier, L2-tier buffer or plain factor row
                 const bool in_s = (id >> 30) == 3u;
                 if constexpr (kL2T) {
                   const bool in_h = (id >> 30) == 2u;
@@ -1222,9 +1283,91 @@ void launch_heavy_lpn(const HArgs &h, int lpn, uint64_t n_pieces, size_t smem, c
   }
 }
 
+namespace {
+// run_sb[r] = last slice s with sbptr[s] <= r * run (the slice holding entry r * run)
+__global__ void run_slice_kernel(const uint64_t *__restrict__ sbptr, uint64_t nsb, uint64_t run,
+                                 uint64_t nruns, uint64_t *__restrict__ run_sb) {
+  for (uint64_t r = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; r < nruns;
+       r += uint64_t(gridDim.x) * blockDim.x) {
+    const uint64_t x = r * run;
+    uint64_t lo = 0, hi = nsb;
+    while (hi - lo > 1) {
+      const uint64_t mid = (lo + hi) / 2;
+      if (sbptr[mid] <= x) lo = mid; else hi = mid;
+    }
+    run_sb[r] = lo;
+  }
+}
+}  // namespace
+
 void launch_hicoo_mttkrp(const pasta_hicoo *h, uint32_t mode, const float *const *factors,
                          uint32_t R, float *out, cudaStream_t s) {
   const HicooModeCopy &mc = h->mc[mode];
+  const int hno = int(h->order) - 1;
+  if (mc.layout == 0 && env_int("PASTA_HICOO_STAGED", 1) && (R == 16 || R == 32) && hno >= 1 &&
+      hno <= 3 && h->nnz > 0 && vec4_ok(h->order, mode, factors, R, out)) {
+    // Row slices decoded warp-wide into the persistent staged COO kernel (WA 9)
+    KArgs a{};
+    a.nnz = h->nnz;
+    a.order = h->order;
+    a.R = R;
+    a.sbptr = mc.sbptr.p;
+    a.nsb = mc.nsb;
+    a.sbrow = mc.sbrow.p;
+    a.val = mc.val.p;
+    int j = 0;
+    for (uint32_t k = 0; k < h->order; ++k) {
+      if (k == mode) continue;
+      if ((h->cmask >> k) & 1u) {
+        a.sbbase[j] = mc.sbbase[k].p;
+        a.eo[j] = mc.einds[k].p;
+      } else {
+        a.io[j] = mc.uinds[k].p;
+        a.wide |= 1u << j;
+      }
+      a.Uo[j] = factors[k];
+      ++j;
+    }
+    a.out = out;
+    const int lpn = R == 16 ? 4 : 8;
+    const int G = 32 / lpn;
+    uint64_t run = uint64_t(env_int("PASTA_MTTKRP_RUN", 128));
+    run = run < 32 ? 32 : (run / 32) * 32;
+    a.chunk = uint64_t(G) * run;
+    HicooModeCopy &mcw = const_cast<HicooModeCopy &>(mc);
+    const uint64_t nruns = (a.nnz + run - 1) / run;
+    if (mcw.run_sb_run != run || mcw.run_sb.n != nruns) {
+      mcw.run_sb.alloc(nruns, s);
+      uint64_t g = (nruns + 255) / 256;
+      if (g > 148 * 32) g = 148 * 32;
+      run_slice_kernel<<<unsigned(g), 256, 0, s>>>(mc.sbptr.p, mc.nsb, run, nruns, mcw.run_sb.p);
+      PASTA_LAUNCHED();
+      mcw.run_sb_run = run;
+    }
+    a.run_sb = mcw.run_sb.p;
+    ProfScope prof(kProfHicoo, s);
+    const int cfg = env_int("PASTA_HS_CFG", 0);  // 2 (8-deep steps) spills here
+    const size_t smem = size_t(16) * 2 * (hno + 2) * (G * 32) * sizeof(uint32_t);
+    const uint64_t nwarps = (a.nnz + a.chunk - 1) / a.chunk;
+    const uint64_t nblk = std::min<uint64_t>((nwarps + 15) / 16, uint64_t(sm_count()));
+    auto go = [&](auto kern) {
+      PASTA_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem)));
+      kern<<<unsigned(nblk), 512, smem, s>>>(a);
+      PASTA_LAUNCHED();
+    };
+    if (cfg == 2 && hno == 1) {
+      if (lpn == 4) go(coo_staged_kernel<1, 4, 9, true, 16, 32, 8>); else go(coo_staged_kernel<1, 8, 9, true, 16, 32, 8>);
+    } else if (cfg == 2 && hno == 2) {
+      if (lpn == 4) go(coo_staged_kernel<2, 4, 9, true, 16, 32, 8>); else go(coo_staged_kernel<2, 8, 9, true, 16, 32, 8>);
+    } else if (hno == 1) {
+      if (lpn == 4) go(coo_staged_kernel<1, 4, 9, true, 16, 32, 4>); else go(coo_staged_kernel<1, 8, 9, true, 16, 32, 4>);
+    } else if (hno == 2) {
+      if (lpn == 4) go(coo_staged_kernel<2, 4, 9, true, 16, 32, 4>); else go(coo_staged_kernel<2, 8, 9, true, 16, 32, 4>);
+    } else {
+      if (lpn == 4) go(coo_staged_kernel<3, 4, 9, true, 16, 32, 4>); else go(coo_staged_kernel<3, 8, 9, true, 16, 32, 4>);
+    }
+    return;
+  }
   if (mc.layout == 0) {
     KArgs a{};
     a.nnz = h->nnz;

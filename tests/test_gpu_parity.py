@@ -448,3 +448,36 @@ def test_coo_shared_memory_hot_tier(env, l2_tier, hs_cfg, monkeypatch):
         U2 = [u.cpu().numpy() for u in Ud2]
         ref, ab = oracle.mttkrp(dims, inds, vals, 1, U2)
         _check(pasta.pasta_mttkrp_coo(x, 1, Ud2), ref, ab, "smem tier refill")
+
+
+@pytest.mark.parametrize("staged", ["1", "0"])
+def test_hicoo_row_slices_staged_decode(env, staged, monkeypatch):
+    """HiCOO / gHiCOO row-slice MTTKRP with the slices decoded warp-wide into the staged kernel
+    (default) and with the per-group slice walk (PASTA_HICOO_STAGED=0): hypersparse blocks
+    (~1 entry per slice, a window spans 32 slices), dense blocks (long slices), a 300K-entry
+    hot row (slices longer than any window), R = 16 / 32, orders 2-4, gHiCOO masks with
+    uncompressed (32-bit) modes, and enough nonzeros for several chunks per persistent warp."""
+    pasta, oracle, torch = env
+    monkeypatch.setenv("PASTA_HICOO_STAGED", staged)
+    cases = [((1 << 20, 1 << 20, 1 << 20), 400_000, 16, "powerlaw", 7, None),
+             ((300, 200, 500), 2_500_000, 16, "uniform", 7, None),
+             ((600, 500, 400), 200_000, 32, "uniform", 5, None),
+             ((2000, 1500), 150_000, 16, "powerlaw", 6, None),
+             ((60, 70, 80, 90), 300_000, 16, "powerlaw", 4, None),
+             ((3000, 2000, 4000), 300_000, 16, "powerlaw", 7, 0b101),
+             ((3000, 2000, 4000), 300_000, 32, "powerlaw", 7, 0b010),
+             ((5000, 3000, 2000), 0, 16, "hot", 7, None)]
+    for dims, nnz, R, gen, bb, mask in cases:
+        if gen == "hot":
+            inds, vals = si.hot_row_coo(dims, 300_000, 50_000, seed=8, mode=0, hot_row=7)
+        else:
+            mk = si.powerlaw_coo if gen == "powerlaw" else si.uniform_coo
+            inds, vals = mk(dims, nnz, seed=nnz + R + bb)
+        U = si.factors(dims, R, seed=R + 1)
+        Ud = _dev(torch, U)
+        x = pasta.pasta_coo_from_arrays(dims, inds, vals)
+        h = pasta.pasta_coo_to_ghicoo(x, bb, mask) if mask else pasta.pasta_coo_to_hicoo(x, bb)
+        for n in range(len(dims)):
+            ref, ab = oracle.mttkrp(dims, inds, vals, n, U)
+            _check(pasta.pasta_mttkrp_hicoo(h, n, Ud), ref, ab,
+                   f"hicoo staged={staged} {dims} R={R} mask={mask} mode {n}")
