@@ -172,7 +172,11 @@ pasta_status pasta_hicoo_prepare(pasta_hicoo *h, uint32_t mode, void *stream);
  * made for this mode.  fp32 arithmetic; partial sums combined with fp32 atomics at segment
  * boundaries (R#24).  Asynchronous on `stream`.  Prepares the mode on first use
  * (synchronising once).  R >= 1 (any value; R % 4 == 0 and 16-byte aligned pointers take
- * the 128-bit vector path). */
+ * the 128-bit vector path).  For R = 16 / 32 the first call per (mode, R) also ranks the
+ * gathered factors' rows by nonzero count (hot-row cache, synchronising once); the L2-tier
+ * buffer is per handle and refilled from `factors` at every launch, so launches of the same
+ * handle must be ordered on one stream (concurrent launches on different streams with
+ * different factors are not supported). */
 pasta_status pasta_mttkrp_coo(pasta_coo *x, uint32_t mode, const float *const *factors,
                               uint32_t R, float *out, void *stream);
 pasta_status pasta_mttkrp_hicoo(pasta_hicoo *h, uint32_t mode, const float *const *factors,
