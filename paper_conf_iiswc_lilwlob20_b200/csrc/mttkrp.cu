@@ -1195,7 +1195,7 @@ void launch_coo_mttkrp(const pasta_coo *x, uint32_t mode, const float *const *fa
         }
         cudaLaunchConfig_t cfg = {};
         cfg.gridDim = dim3(unsigned(nblk));
-        cfg.blockDim = dim3(kThreads);
+        cfg.blockDim = dim3(hs ? hs_wpc * 32 : kThreads);
         cfg.dynamicSmemBytes = smem;
         cfg.stream = s;
         cudaLaunchAttribute attr[1];

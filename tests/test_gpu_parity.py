@@ -392,13 +392,15 @@ def test_torch_caching_allocator_hook(env):
         pasta.pasta_set_allocator(None)
 
 
-@pytest.mark.parametrize("hot_mb", ["0.05", "1"])
-def test_coo_hot_row_cache_forced(env, hot_mb, monkeypatch):
+@pytest.mark.parametrize("hot_mb,persist", [("0.05", "0"), ("1", "0"), ("1", "1")])
+def test_coo_hot_row_cache_forced(env, hot_mb, persist, monkeypatch):
     """The packed hot-row cache (coo_mark_hot) is enabled automatically only when the gathered
-    factors exceed L2; force it on small tensors (tiny budgets so that hot and cold rows mix)."""
+    factors exceed L2; force it on small tensors (tiny budgets so that hot and cold rows mix),
+    with and without the persisting-L2 access-policy window (a separate launch path)."""
     pasta, oracle, torch = env
     monkeypatch.setenv("PASTA_HOT_FORCE", "1")
     monkeypatch.setenv("PASTA_HOT_MB", hot_mb)
+    monkeypatch.setenv("PASTA_HOT_PERSIST", persist)
     for dims, nnz, R in [((3000, 2000, 4000), 120_000, 16), ((300, 400, 500, 60), 80_000, 32),
                          ((5000, 3000, 2000), 0, 16)]:
         if nnz:
