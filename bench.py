@@ -475,7 +475,8 @@ def main():
                "roofline": {"bound": "hbm", "achieved": round(ach, 1), "peak": peak_h,
                             "unit": "GB/s", "frac": round(ach / peak_h, 4),
                             "traffic": ncu_traffic(args.config, label + "_mttkrp"),
-                            "kernel": f"mttkrp_kernel<HicooRowSrc> ({label}, row-slice layout)",
+                            "kernel": f"coo_staged_kernel<..., WA 9> ({label} row slices decoded "
+                                      "warp-wide into the staged kernel)",
                             "bytes_model": bm,
                             "avg_launch_ms": round(hk_ms / max(hk_n, 1), 4)},
                "preprocess_s": {"convert": round(t_conv, 3), "mode_copies_all": round(t_hprep, 3)}}

@@ -19,3 +19,10 @@ for CFG in h c2; do
 done
 cp profiles/ncu_summary.json $OUT/ncu_summary.json
 ls -la $OUT
+# HiCOO / gHiCOO row slices through the staged kernel (WA 9) on H
+for FMT in hicoo ghicoo; do
+  timeout 900 $NCU -k regex:coo_staged_kernel -s 3 -c 1 -o /tmp/${TAG}_${FMT}_h \
+    python tools/sweep.py --config h --variants 0 --runs 0 --formats $FMT --reps 1 > $OUT/${FMT}_h.log 2>&1
+  python tools/ncu_summary.py full /tmp/${TAG}_${FMT}_h.ncu-rep h $OUT/${TAG}_ncu_full_${FMT}_h.md ${FMT}_mttkrp > /dev/null
+done
+cp profiles/ncu_summary.json $OUT/ncu_summary.json
