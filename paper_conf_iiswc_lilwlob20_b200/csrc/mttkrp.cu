@@ -1073,6 +1073,27 @@ void launch_zero_rows(float *out, uint64_t row_lo, uint64_t row_hi, uint32_t R, 
   PASTA_LAUNCHED();
 }
 
+// Runtime (order - 1, lanes per nonzero) -> compile-time tags for the staged kernels
+// (R = 4 * LPN in {8, 16, 32, 64}).
+template <class F>
+static void with_lpn(int lpn, F &&f) {
+  switch (lpn) {
+    case 2: f(std::integral_constant<int, 2>()); break;
+    case 4: f(std::integral_constant<int, 4>()); break;
+    case 8: f(std::integral_constant<int, 8>()); break;
+    default: f(std::integral_constant<int, 16>()); break;
+  }
+}
+template <int MAXNO, class F>
+static void with_no_lpn(int no, int lpn, F &&f) {
+  with_lpn(lpn, [&](auto L) {
+    if (no == 1) f(std::integral_constant<int, 1>(), L);
+    else if (no == 2 || MAXNO == 2) f(std::integral_constant<int, 2>(), L);
+    else f(std::integral_constant<int, 3>(), L);
+  });
+}
+static bool staged_rank(uint32_t R) { return R == 8 || R == 16 || R == 32 || R == 64; }
+
 static bool vec4_ok(uint32_t order, uint32_t mode, const float *const *factors, uint32_t R,
                     const float *out) {
   if (R % 4 != 0 || !aligned16(out)) return false;
@@ -1104,7 +1125,7 @@ void launch_coo_mttkrp(const pasta_coo *x, uint32_t mode, const float *const *fa
   const int staged = env_int("PASTA_COO_STAGED", 1);
   const int no = int(x->order) - 1;
   // no == 1: order-2 matrices, e.g. the fiberised (fiber, i_n) matrix of TTM (ttm.cu)
-  if (staged && vec4 && (R == 16 || R == 32) && (no >= 1 && no <= 3)) {
+  if (staged && vec4 && staged_rank(R) && (no >= 1 && no <= 3)) {
     // the hot-row cache pays only when the gathered factors do not fit in L2 already
     static int l2 = 0;
     if (!l2) {
@@ -1119,7 +1140,7 @@ void launch_coo_mttkrp(const pasta_coo *x, uint32_t mode, const float *const *fa
     // effective L2 for random row gathers is ~half the nominal size
     // (profiles/r01_l2_capacity_microbench.txt)
     const bool want_hot = env_int("PASTA_HOT_FORCE", 0) || gathered > uint64_t(l2) / 2;
-    const int lpn = R == 16 ? 4 : 8;
+    const int lpn = int(R / 4);  // 2, 4, 8 or 16 lanes per nonzero, 16 B of each factor row per lane
     const int G = 32 / lpn;
     // Persistent HS kernel (one 16-warp CTA per SM) with the shared-memory tier of the hot-row
     // cache.  Tier size: on L2-resident factors (no L2 tier) the kernel is bound by L2->SM
@@ -1218,7 +1239,9 @@ void launch_coo_mttkrp(const pasta_coo *x, uint32_t mode, const float *const *fa
     const int wa = env_int("PASTA_STAGED_WA", 1);
     auto pick = [&](auto tag) {
       constexpr int W = decltype(tag)::value;
-      if (no == 1 && lpn == 4) go(coo_staged_kernel<1, 4, 1, false>);  // one code path for order 2
+      if (lpn != 4 && lpn != 8) {  // R = 8 / 64: the default code path only
+        with_no_lpn<3>(no, lpn, [&](auto NOt, auto Lt) { go(coo_staged_kernel<NOt.value, Lt.value, 1, false>); });
+      } else if (no == 1 && lpn == 4) go(coo_staged_kernel<1, 4, 1, false>);  // one code path for order 2
       else if (no == 1) go(coo_staged_kernel<1, 8, 1, false>);
       else if (no == 2 && lpn == 4) go(coo_staged_kernel<2, 4, W, false>);
       else if (no == 2) go(coo_staged_kernel<2, 8, W, false>);
@@ -1230,29 +1253,19 @@ void launch_coo_mttkrp(const pasta_coo *x, uint32_t mode, const float *const *fa
     for (uint32_t k = 0; k < x->order; ++k)
       if (k != mode) max_factor = std::max<uint64_t>(max_factor, uint64_t(x->dims[k]) * R * sizeof(float));
     const bool l2t = mc.hot_total > 0 || max_factor >= (uint64_t(1) << 32);
-    auto pick_hs3 = [&](auto wtag, auto stag, auto atag) {
-      constexpr int W = decltype(wtag)::value, S = decltype(stag)::value, A = decltype(atag)::value;
-      if (no == 1 && lpn == 4) go(coo_staged_kernel<1, 4, A, true, W, S>);
-      else if (no == 1) go(coo_staged_kernel<1, 8, A, true, W, S>);
-      else if (no == 2 && lpn == 4) go(coo_staged_kernel<2, 4, A, true, W, S>);
-      else if (no == 2) go(coo_staged_kernel<2, 8, A, true, W, S>);
-      else if (lpn == 4) go(coo_staged_kernel<3, 4, A, true, W, S>);
-      else go(coo_staged_kernel<3, 8, A, true, W, S>);
-    };
     auto pick_hs = [&](auto wtag, auto stag) {
-      if (l2t) pick_hs3(wtag, stag, std::integral_constant<int, 1>());
-      else pick_hs3(wtag, stag, std::integral_constant<int, 7>());
+      constexpr int W = decltype(wtag)::value, S = decltype(stag)::value;
+      with_no_lpn<3>(no, lpn, [&](auto NOt, auto Lt) {
+        if (l2t) go(coo_staged_kernel<NOt.value, Lt.value, 1, true, W, S>);
+        else go(coo_staged_kernel<NOt.value, Lt.value, 7, true, W, S>);
+      });
     };
     using I16 = std::integral_constant<int, 16>;
     if (hs) {
       if (hs_cfg == 1) pick_hs(std::integral_constant<int, 24>(), I16());
-      else if (hs_cfg == 2 && no == 1) {
-        if (lpn == 4) go(coo_staged_kernel<1, 4, 1, true, 16, 32, 8>);
-        else go(coo_staged_kernel<1, 8, 1, true, 16, 32, 8>);
-      } else if (hs_cfg == 2 && no == 2) {
-        if (lpn == 4) go(coo_staged_kernel<2, 4, 1, true, 16, 32, 8>);
-        else go(coo_staged_kernel<2, 8, 1, true, 16, 32, 8>);
-      } else pick_hs(I16(), std::integral_constant<int, 32>());
+      else if (hs_cfg == 2 && no <= 2)
+        with_no_lpn<2>(no, lpn, [&](auto NOt, auto Lt) { go(coo_staged_kernel<NOt.value, Lt.value, 1, true, 16, 32, 8>); });
+      else pick_hs(I16(), std::integral_constant<int, 32>());
     } else if (wa == 1) pick(std::integral_constant<int, 1>());
     else if (wa == 2) pick(std::integral_constant<int, 2>());
     else if (wa == 3) pick(std::integral_constant<int, 3>());
@@ -1304,8 +1317,11 @@ void launch_hicoo_mttkrp(const pasta_hicoo *h, uint32_t mode, const float *const
                          uint32_t R, float *out, cudaStream_t s) {
   const HicooModeCopy &mc = h->mc[mode];
   const int hno = int(h->order) - 1;
-  if (mc.layout == 0 && env_int("PASTA_HICOO_STAGED", 1) && (R == 16 || R == 32) && hno >= 1 &&
-      hno <= 3 && h->nnz > 0 && vec4_ok(h->order, mode, factors, R, out)) {
+  // staging of 16 warps x 2 buffers x (N+1) arrays x 32 entries per group (R = 8: 16 groups
+  // per warp -> 256 KB at N = 3, too large: the slice walk below takes it)
+  const size_t hic_smem = size_t(16) * 2 * (hno + 2) * (size_t(32) / std::max<uint32_t>(R / 4, 1u) * 32) * 4;
+  if (mc.layout == 0 && env_int("PASTA_HICOO_STAGED", 1) && staged_rank(R) && hno >= 1 &&
+      hno <= 3 && h->nnz > 0 && hic_smem <= 227 * 1024 && vec4_ok(h->order, mode, factors, R, out)) {
     // Row slices decoded warp-wide into the persistent staged COO kernel (WA 9)
     KArgs a{};
     a.nnz = h->nnz;
@@ -1329,7 +1345,7 @@ void launch_hicoo_mttkrp(const pasta_hicoo *h, uint32_t mode, const float *const
       ++j;
     }
     a.out = out;
-    const int lpn = R == 16 ? 4 : 8;
+    const int lpn = int(R / 4);
     const int G = 32 / lpn;
     uint64_t run = uint64_t(env_int("PASTA_MTTKRP_RUN", 128));
     run = run < 32 ? 32 : (run / 32) * 32;
@@ -1355,17 +1371,10 @@ void launch_hicoo_mttkrp(const pasta_hicoo *h, uint32_t mode, const float *const
       kern<<<unsigned(nblk), 512, smem, s>>>(a);
       PASTA_LAUNCHED();
     };
-    if (cfg == 2 && hno == 1) {
-      if (lpn == 4) go(coo_staged_kernel<1, 4, 9, true, 16, 32, 8>); else go(coo_staged_kernel<1, 8, 9, true, 16, 32, 8>);
-    } else if (cfg == 2 && hno == 2) {
-      if (lpn == 4) go(coo_staged_kernel<2, 4, 9, true, 16, 32, 8>); else go(coo_staged_kernel<2, 8, 9, true, 16, 32, 8>);
-    } else if (hno == 1) {
-      if (lpn == 4) go(coo_staged_kernel<1, 4, 9, true, 16, 32, 4>); else go(coo_staged_kernel<1, 8, 9, true, 16, 32, 4>);
-    } else if (hno == 2) {
-      if (lpn == 4) go(coo_staged_kernel<2, 4, 9, true, 16, 32, 4>); else go(coo_staged_kernel<2, 8, 9, true, 16, 32, 4>);
-    } else {
-      if (lpn == 4) go(coo_staged_kernel<3, 4, 9, true, 16, 32, 4>); else go(coo_staged_kernel<3, 8, 9, true, 16, 32, 4>);
-    }
+    if (cfg == 2 && hno <= 2)
+      with_no_lpn<2>(hno, lpn, [&](auto NOt, auto Lt) { go(coo_staged_kernel<NOt.value, Lt.value, 9, true, 16, 32, 8>); });
+    else
+      with_no_lpn<3>(hno, lpn, [&](auto NOt, auto Lt) { go(coo_staged_kernel<NOt.value, Lt.value, 9, true, 16, 32, 4>); });
     return;
   }
   if (mc.layout == 0) {

@@ -65,6 +65,10 @@ CASES = [
     ((400, 300, 200), 12_345, 160, "powerlaw", 8),     # R > 128: column loop
     ((1, 500, 300), 20_000, 16, "uniform", 7),         # a dimension of 1
     ((4096, 4096, 4096), 200_000, 16, "powerlaw", 7),  # several tiles, hypersparse blocks
+    ((3000, 2000, 4000), 300_000, 8, "powerlaw", 7),   # R = 8: 2 lanes per nonzero
+    ((3000, 2000, 4000), 200_000, 64, "powerlaw", 7),  # R = 64: 16 lanes per nonzero
+    ((60, 70, 80, 90), 100_000, 64, "powerlaw", 4),    # N = 4, R = 64
+    ((2000, 1500), 100_000, 8, "uniform", 6),          # N = 2, R = 8
 ]
 
 
@@ -435,6 +439,7 @@ def test_coo_shared_memory_hot_tier(env, l2_tier, hs_cfg, monkeypatch):
         monkeypatch.setenv("PASTA_HOT_MB", "0.25")
     for dims, nnz, R in [((3000, 2000, 4000), 3_000_017, 16), ((300, 400, 500, 60), 80_000, 16),
                          ((3000, 2000, 4000), 120_000, 32), ((300, 400, 500, 60), 80_000, 32),
+                         ((3000, 2000, 4000), 200_000, 8), ((3000, 2000, 4000), 200_000, 64),
                          ((5000, 3000, 2000), 0, 16)]:
         if nnz:
             inds, vals = si.powerlaw_coo(dims, nnz, seed=nnz + R)
@@ -468,6 +473,9 @@ def test_hicoo_row_slices_staged_decode(env, staged, monkeypatch):
              ((60, 70, 80, 90), 300_000, 16, "powerlaw", 4, None),
              ((3000, 2000, 4000), 300_000, 16, "powerlaw", 7, 0b101),
              ((3000, 2000, 4000), 300_000, 32, "powerlaw", 7, 0b010),
+             ((3000, 2000, 4000), 200_000, 8, "powerlaw", 7, None),
+             ((3000, 2000, 4000), 200_000, 64, "powerlaw", 7, None),
+             ((60, 70, 80, 90), 100_000, 64, "powerlaw", 4, 0b1011),
              ((5000, 3000, 2000), 0, 16, "hot", 7, None)]
     for dims, nnz, R, gen, bb, mask in cases:
         if gen == "hot":
