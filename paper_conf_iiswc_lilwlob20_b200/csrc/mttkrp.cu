@@ -1157,6 +1157,8 @@ void launch_coo_mttkrp(const pasta_coo *x, uint32_t mode, const float *const *fa
     // 1.57, C5 27.2 -> 26.6) but lose on L2-resident factors, whose shared-memory tier shrinks
     // (C2 0.80 -> 0.88).  32 warps spill for every order; 8 warps x 16-deep steps (220
     // registers) and 12 warps x 8-deep steps are slower everywhere (H 1.80 / 1.73 ms).
+    // (R = 8 with DRAM-bound gathers: the 32-deep shape does not fit -> non-persistent kernel,
+    // which measured faster there than forcing the 16-deep shape: H 1.80 vs 2.01 ms)
     const int hs_cfg = env_int("PASTA_HS_CFG", no <= 2 ? (want_hot ? 2 : 1) : 0);
     const int hs_wpc = hs_cfg == 1 ? 24 : 16;
     const int hs_sg = hs_cfg == 1 ? 16 : 32;

@@ -24,9 +24,11 @@ def main():
     ap.add_argument("--reps", type=int, default=10)
     ap.add_argument("--caches", default="0")
     ap.add_argument("--cmask", type=int, default=0, help="gHiCOO mask (0 = auto)")
+    ap.add_argument("--R", type=int, default=0, help="override the config's rank")
     args = ap.parse_args()
     cfg = si.CONFIGS[args.config]
     dims, R, M = cfg["dims"], cfg["R"], cfg["nnz"]
+    R = args.R or R
     x = pasta.pasta_gen_powerlaw(dims, M, cfg["seed"], kind=0 if cfg["kind"] == "uniform" else 1)
     fmts = args.formats.split(",")
     h = pasta.pasta_coo_to_hicoo(x, 7) if "hicoo" in fmts else None
