@@ -570,6 +570,13 @@ def main():
                                      "bytes_model": "TS 8M / TEW 12M per launch (Table I, P:117)"}}
         del vals, other, dst
 
+    balance = None
+    if world > 1:  # max / mean nonzeros per rank, per mode (every rank joins)
+        allsh = [None] * world
+        dist.all_gather_object(allsh, [int(v) for v in shard_nnz])
+        balance = [round(max(r[n] for r in allsh) / (sum(r[n] for r in allsh) / world), 4)
+                   for n in range(N)]
+
     if rank != 0:
         if world > 1:
             dist.destroy_process_group()
@@ -640,6 +647,7 @@ def main():
         "gpu_launches": launches,
         "cpu_baseline": cpu,
         "max_shard_nnz": per_launch_nnz,
+        "shard_max_over_mean": balance,
     }
     print(json.dumps(line), flush=True)
     if world > 1:

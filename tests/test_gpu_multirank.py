@@ -45,6 +45,8 @@ def test_bench_two_ranks_shared_gpu():
     assert d["config"]["nnz"] == 2 * 54_000_000  # the tensor grows with the GPU count
     assert d["allgather"]["ms_per_step"] > 0 and d["allgather"]["bytes_received_per_rank"] > 0
     assert d["e2e"]["value"] > 0 and d["gpu_launches"] > 0
+    bal = d["shard_max_over_mean"]  # nnz-balanced row ranges: max / mean nonzeros per rank
+    assert len(bal) == 4 and all(1.0 <= b < 1.05 for b in bal), bal
     r2 = _torchrun(["bench.py", "--impl", "reference", "--gpus", "2", "--config", "c1",
                     "--steps", "2", "--warmup", "3", "--ref-sample", "2000"])
     assert r2.returncode == 0, r2.stderr[-4000:]
