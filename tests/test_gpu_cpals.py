@@ -44,6 +44,19 @@ def test_building_blocks(env):
         assert np.allclose(np.linalg.norm(Uo.cpu().numpy().astype(np.float64), axis=0), 1.0, atol=1e-5)
 
 
+def test_gram_many_tiles_per_cta(env):
+    """The gram kernel's persistent CTAs walk several double-buffered (cp.async) row tiles each
+    (rows well above 148 x 8 tiles) and a ragged last tile, for every tiled rank."""
+    pasta, oracle, torch = env
+    rng = np.random.default_rng(3)
+    for R, rows in ((4, 5_000_011), (8, 2_500_007), (16, 700_001), (32, 400_003), (64, 200_009)):
+        U = rng.uniform(-1, 1, size=(rows, R)).astype(np.float32)
+        G = pasta.pasta_gram(torch.from_numpy(U).cuda()).cpu().numpy()
+        U64 = U.astype(np.float64)
+        ref = U64.T @ U64
+        assert np.allclose(G, ref, rtol=1e-5, atol=1e-6 * np.abs(ref).max()), R
+
+
 def test_fused_update_blocks(env):
     """pasta_cpals_prepare + pasta_rows_times == solve -> normalise -> gram (numpy fp64)."""
     pasta, oracle, torch = env
