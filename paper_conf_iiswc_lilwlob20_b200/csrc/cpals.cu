@@ -168,24 +168,38 @@ __global__ void __launch_bounds__(kThreads) gram_tile_kernel(const float *__rest
 template <int R>
 __global__ void __launch_bounds__(kThreads) apply_tile_kernel(const float *__restrict__ M, uint64_t rows,
                                                               const float *__restrict__ W, float *__restrict__ U) {
-  constexpr int RB = R / 4, RPP = kThreads / R, T = tile_rows<R>();  // RPP: rows per pass
-  __shared__ __align__(16) float tile[T * R];
+  // row tiles double-buffered with cp.async (as in gram_tile_kernel): 16 KB per buffer
+  constexpr int RB = R / 4, RPP = kThreads / R, T = gram_rows<R>();  // RPP: rows per pass
+  __shared__ __align__(16) float tile[2][T * R];
   const int t = threadIdx.x, c = t % R, r = t / R;
   float w[R];
 #pragma unroll
   for (int a = 0; a < R; ++a) w[a] = W[a * R + c];
-  for (uint64_t r0 = uint64_t(blockIdx.x) * T; r0 < rows; r0 += uint64_t(gridDim.x) * T) {
+  const uint64_t step = uint64_t(gridDim.x) * T;
+  auto issue = [&](uint64_t r0, int b) {
+    if (r0 < rows) {
+      const int nr = int(rows - r0 < T ? rows - r0 : T);
+      const float4 *src = reinterpret_cast<const float4 *>(M + r0 * R);
+      for (int e = t; e < nr * RB; e += kThreads) {
+        const uint32_t d = uint32_t(__cvta_generic_to_shared(reinterpret_cast<float4 *>(tile[b]) + e));
+        asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(d), "l"(src + e) : "memory");
+      }
+    }
+    asm volatile("cp.async.commit_group;" ::: "memory");
+  };
+  int b = 0;
+  issue(uint64_t(blockIdx.x) * T, 0);
+  for (uint64_t r0 = uint64_t(blockIdx.x) * T; r0 < rows; r0 += step, b ^= 1) {
     const int nr = int(rows - r0 < T ? rows - r0 : T);
+    issue(r0 + step, b ^ 1);
+    asm volatile("cp.async.wait_group 1;" ::: "memory");
     __syncthreads();
-    const float4 *src = reinterpret_cast<const float4 *>(M + r0 * R);
-    float4 *dst = reinterpret_cast<float4 *>(tile);
-    for (int e = t; e < nr * RB; e += kThreads) dst[e] = src[e];
-    __syncthreads();
+    const float *tb = tile[b];
     for (int i = r; i < nr; i += RPP) {
       float acc = 0.f;
 #pragma unroll
       for (int a = 0; a < R; a += 4) {
-        const float4 m = *reinterpret_cast<const float4 *>(tile + i * R + a);
+        const float4 m = *reinterpret_cast<const float4 *>(tb + i * R + a);
         acc = fmaf(m.x, w[a], acc);
         acc = fmaf(m.y, w[a + 1], acc);
         acc = fmaf(m.z, w[a + 2], acc);
@@ -193,7 +207,9 @@ __global__ void __launch_bounds__(kThreads) apply_tile_kernel(const float *__res
       }
       U[(r0 + i) * R + c] = acc;
     }
+    __syncthreads();  // tile[b] is refilled by the next iteration's issue
   }
+  asm volatile("cp.async.wait_group 0;" ::: "memory");
 }
 
 // Fused factor update + all-gather over peer memory (a9 / NEXT-1, B200-native exchange):

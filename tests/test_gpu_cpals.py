@@ -45,8 +45,9 @@ def test_building_blocks(env):
 
 
 def test_gram_many_tiles_per_cta(env):
-    """The gram kernel's persistent CTAs walk several double-buffered (cp.async) row tiles each
-    (rows well above 148 x 8 tiles) and a ragged last tile, for every tiled rank."""
+    """The gram and factor-update kernels' persistent CTAs walk several double-buffered
+    (cp.async) row tiles each (rows well above 148 x 8 tiles) and a ragged last tile, for every
+    tiled rank."""
     pasta, oracle, torch = env
     rng = np.random.default_rng(3)
     for R, rows in ((4, 5_000_011), (8, 2_500_007), (16, 700_001), (32, 400_003), (64, 200_009)):
@@ -55,6 +56,11 @@ def test_gram_many_tiles_per_cta(env):
         U64 = U.astype(np.float64)
         ref = U64.T @ U64
         assert np.allclose(G, ref, rtol=1e-5, atol=1e-6 * np.abs(ref).max()), R
+        # the factor update U = M Wn walks the same double-buffered tiles
+        W = rng.uniform(-1, 1, size=(R, R)).astype(np.float32)
+        got = pasta.pasta_rows_times(torch.from_numpy(U).cuda(), torch.from_numpy(W).cuda()).cpu().numpy()
+        want = U64 @ W.astype(np.float64)
+        assert np.allclose(got, want, rtol=1e-5, atol=1e-5 * R), R
 
 
 def test_fused_update_blocks(env):
