@@ -110,12 +110,16 @@ template <int R>
 __global__ void __launch_bounds__(kThreads) gram_tile_kernel(const float *__restrict__ U, uint64_t rows,
                                                              double *__restrict__ G) {
   constexpr int RB = R / 4, GS = RB * RB, NG = kThreads / GS, T = gram_rows<R>();
+  // a group reduces RPG rows of a full tile; the fp32 partials go to fp64 every FLUSH tiles
+  // (<= 64 rows in fp32, as before), so the row loop of a full tile has no flush test
+  constexpr int RPG = T / NG, FLUSH = 64 / RPG;
+  static_assert(T % NG == 0 && RPG <= 64, "gram tile shape");
   __shared__ __align__(16) float tile[2][T * R];
   __shared__ double red[R * R];
   const int t = threadIdx.x, g = t / GS, blk = t % GS, ba = blk / RB, bb = blk % RB;
   float acc[4][4] = {};
   double acc64[4][4] = {};
-  int since = 0;
+  int tiles = 0;
   for (uint32_t e = t; e < R * R; e += kThreads) red[e] = 0.0;
   const uint64_t step = uint64_t(gridDim.x) * T;
   auto issue = [&](uint64_t r0, int b) {
@@ -129,6 +133,15 @@ __global__ void __launch_bounds__(kThreads) gram_tile_kernel(const float *__rest
     }
     asm volatile("cp.async.commit_group;" ::: "memory");
   };
+  auto row = [&](const float *tb, int i) {
+    const float4 x = *reinterpret_cast<const float4 *>(tb + i * R + 4 * ba);
+    const float4 y = *reinterpret_cast<const float4 *>(tb + i * R + 4 * bb);
+    const float xa[4] = {x.x, x.y, x.z, x.w}, ya[4] = {y.x, y.y, y.z, y.w};
+#pragma unroll
+    for (int p = 0; p < 4; ++p)
+#pragma unroll
+      for (int q = 0; q < 4; ++q) acc[p][q] = fmaf(xa[p], ya[q], acc[p][q]);
+  };
   int b = 0;
   issue(uint64_t(blockIdx.x) * T, 0);
   for (uint64_t r0 = uint64_t(blockIdx.x) * T; r0 < rows; r0 += step, b ^= 1) {
@@ -137,21 +150,18 @@ __global__ void __launch_bounds__(kThreads) gram_tile_kernel(const float *__rest
     asm volatile("cp.async.wait_group 1;" ::: "memory");
     __syncthreads();
     const float *tb = tile[b];
-    for (int i = g; i < nr; i += NG) {
-      const float4 x = *reinterpret_cast<const float4 *>(tb + i * R + 4 * ba);
-      const float4 y = *reinterpret_cast<const float4 *>(tb + i * R + 4 * bb);
-      const float xa[4] = {x.x, x.y, x.z, x.w}, ya[4] = {y.x, y.y, y.z, y.w};
+    if (nr == T) {
+#pragma unroll 4
+      for (int j = 0; j < RPG; ++j) row(tb, g + j * NG);
+    } else {
+      for (int i = g; i < nr; i += NG) row(tb, i);
+    }
+    if (++tiles == FLUSH) {
 #pragma unroll
       for (int p = 0; p < 4; ++p)
 #pragma unroll
-        for (int q = 0; q < 4; ++q) acc[p][q] = fmaf(xa[p], ya[q], acc[p][q]);
-      if (++since == 64) {
-#pragma unroll
-        for (int p = 0; p < 4; ++p)
-#pragma unroll
-          for (int q = 0; q < 4; ++q) { acc64[p][q] += double(acc[p][q]); acc[p][q] = 0.f; }
-        since = 0;
-      }
+        for (int q = 0; q < 4; ++q) { acc64[p][q] += double(acc[p][q]); acc[p][q] = 0.f; }
+      tiles = 0;
     }
     __syncthreads();  // tile[b] is refilled by the next iteration's issue
   }
