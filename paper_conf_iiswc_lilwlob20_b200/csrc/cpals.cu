@@ -151,7 +151,7 @@ __global__ void __launch_bounds__(kThreads) gram_tile_kernel(const float *__rest
     __syncthreads();
     const float *tb = tile[b];
     if (nr == T) {
-#pragma unroll 4
+#pragma unroll
       for (int j = 0; j < RPG; ++j) row(tb, g + j * NG);
     } else {
       for (int i = g; i < nr; i += NG) row(tb, i);
