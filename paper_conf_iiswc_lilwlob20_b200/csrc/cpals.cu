@@ -205,7 +205,7 @@ __global__ void __launch_bounds__(kThreads) apply_tile_kernel(const float *__res
     asm volatile("cp.async.wait_group 1;" ::: "memory");
     __syncthreads();
     const float *tb = tile[b];
-    for (int i = r; i < nr; i += RPP) {
+    auto row = [&](int i) {
       float acc = 0.f;
 #pragma unroll
       for (int a = 0; a < R; a += 4) {
@@ -216,6 +216,12 @@ __global__ void __launch_bounds__(kThreads) apply_tile_kernel(const float *__res
         acc = fmaf(m.w, w[a + 3], acc);
       }
       U[(r0 + i) * R + c] = acc;
+    };
+    if (nr == T) {  // full tile: T / RPP rows per thread, unrolled (as in gram_tile_kernel)
+#pragma unroll
+      for (int j = 0; j < T / RPP; ++j) row(r + j * RPP);
+    } else {
+      for (int i = r; i < nr; i += RPP) row(i);
     }
     __syncthreads();  // tile[b] is refilled by the next iteration's issue
   }
