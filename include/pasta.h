@@ -172,11 +172,13 @@ pasta_status pasta_hicoo_prepare(pasta_hicoo *h, uint32_t mode, void *stream);
  * made for this mode.  fp32 arithmetic; partial sums combined with fp32 atomics at segment
  * boundaries (R#24).  Asynchronous on `stream`.  Prepares the mode on first use
  * (synchronising once).  R >= 1 (any value; R % 4 == 0 and 16-byte aligned pointers take
- * the 128-bit vector path).  For R = 16 / 32 the first call per (mode, R) also ranks the
- * gathered factors' rows by nonzero count (hot-row cache, synchronising once); the L2-tier
- * buffer is per handle and refilled from `factors` at every launch, so launches of the same
- * handle must be ordered on one stream (concurrent launches on different streams with
- * different factors are not supported). */
+ * the 128-bit vector path).  For R in {8, 16, 32, 64} the first call per (mode, R) also
+ * ranks the gathered factors' rows by nonzero count (hot-row cache, synchronising once; one
+ * cached ranking per mode: alternating R on one handle re-ranks at every change).  The
+ * L2-tier buffer is per handle and refilled from `factors` at every launch; the library
+ * orders same-handle launches that use it (a launch on another stream waits for the previous
+ * one through an event), so concurrent calls are safe but do not overlap.  Thread-safe: the
+ * handle's caches are built and the launches enqueued under the handle's lock. */
 pasta_status pasta_mttkrp_coo(pasta_coo *x, uint32_t mode, const float *const *factors,
                               uint32_t R, float *out, void *stream);
 pasta_status pasta_mttkrp_hicoo(pasta_hicoo *h, uint32_t mode, const float *const *factors,
@@ -185,8 +187,10 @@ pasta_status pasta_mttkrp_hicoo(pasta_hicoo *h, uint32_t mode, const float *cons
 /* End-to-end variant over ALL modes with HOST buffers (the e2e path): copies the `order`
  * factor matrices host->device (pinned host memory gives full PCIe/C2C bandwidth), computes
  * MTTKRP for every mode into library-owned device buffers, copies the `order` results back
- * to host_out[k] ([dims[k]][R] row-major) and synchronises `stream`.  Device staging
- * buffers are cached in the handle. */
+ * to host_out[k] ([dims[k]][R] row-major; for a shard handle only its rows [row_lo, row_hi)
+ * of the shard mode are written, the other host rows are left as they were) and synchronises
+ * `stream`.  Device staging buffers (2 slots x order x (factor + output)) are cached in the
+ * handle until pasta_coo_release_staging or pasta_coo_free. */
 pasta_status pasta_mttkrp_coo_allmodes_host(pasta_coo *x, const float *const *host_factors,
                                             uint32_t R, float *const *host_out, void *stream);
 /* `nsteps` independent all-modes steps in one call (a stream of factor sets, e.g. serving):
@@ -198,6 +202,10 @@ pasta_status pasta_mttkrp_coo_allmodes_host(pasta_coo *x, const float *const *ho
 pasta_status pasta_mttkrp_coo_allmodes_host_batch(pasta_coo *x, uint32_t nsteps,
                                                   const float *const *host_factors, uint32_t R,
                                                   float *const *host_out, void *stream);
+
+/* Free the e2e staging buffers of `x` (after the copies in flight have finished); the next
+ * host-buffer call allocates them again. */
+pasta_status pasta_coo_release_staging(pasta_coo *x);
 
 /* --------------------------------------------------------------- multi-GPU (a9) ------ */
 

@@ -26,9 +26,13 @@ import numpy as np
 from . import mttkrp
 
 
-def cp_als(dims, inds, vals, U0, iters, tol=0.0, record=None):
+def cp_als(dims, inds, vals, U0, iters, tol=0.0, record=None, perturb=None):
     """Run `iters` sweeps (or stop when |fit - previous| < tol after the first sweep).
-    U0: list of float32 [I_k, R] initial factors.  Returns (U list fp32, lambda fp64, fits)."""
+    U0: list of float32 [I_k, R] initial factors.  Returns (U list fp32, lambda fp64, fits).
+    perturb (test hook, default None = the plain algorithm): perturb(stage, n, array) -> array
+    applied to M ("M", with the oracle's sum|terms| as array.A), to each gram U_k^T U_k ("G")
+    and to the solved factor before normalisation ("U"); used to measure the algorithm's
+    sensitivity to the rounding of an fp32 implementation (R#33)."""
     N = len(dims)
     U = [np.ascontiguousarray(u, dtype=np.float32) for u in U0]
     R = U[0].shape[1]
@@ -38,13 +42,18 @@ def cp_als(dims, inds, vals, U0, iters, tol=0.0, record=None):
     M = None
     for it in range(iters):
         for n in range(N):
-            M, _ = mttkrp(dims, inds, vals, n, U, R=R)
+            M, A = mttkrp(dims, inds, vals, n, U, R=R)
+            if perturb is not None:
+                M = perturb("M", n, (M, A))
             V = np.ones((R, R))
             for k in range(N):
                 if k != n:
                     Uk = U[k].astype(np.float64)
-                    V *= Uk.T @ Uk
+                    Gk = Uk.T @ Uk
+                    V *= perturb("G", k, (Gk, np.abs(Uk).T @ np.abs(Uk))) if perturb is not None else Gk
             Un = np.linalg.solve(V.T, M.T).T  # U_n V = M
+            if perturb is not None:
+                Un = perturb("U", n, (Un, None))
             if record is not None:
                 record.append((n, M.copy(), V.copy(), Un.copy()))
             lam = np.sqrt(np.sum(Un * Un, axis=0))

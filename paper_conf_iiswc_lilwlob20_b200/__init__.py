@@ -224,9 +224,14 @@ def pasta_hicoo_prepare(h: Hicoo, mode: int, stream=None) -> None:
 
 
 # ----------------------------------------------------------------------------- MTTKRP
-def _factor_ptrs(order, mode, factors, R):
+def _factor_ptrs(order, mode, factors, R, dims=None, device=None):
+    """Device pointers of the factor list; every non-target factor must be a contiguous
+    float32 CUDA tensor [dims[k], R] (all on one device) -- the library reads dims[k] * R
+    floats from it (and CP-ALS writes as many), so a short or mistyped factor is rejected here."""
     import torch
     ptrs = (C.c_void_p * order)()
+    if len(factors) < order:
+        raise PastaError(-1, f"{len(factors)} factors given for an order-{order} tensor")
     for k in range(order):
         f = factors[k] if k < len(factors) else None
         if k == mode:
@@ -236,6 +241,10 @@ def _factor_ptrs(order, mode, factors, R):
             raise PastaError(-1, f"factors[{k}] must be a CUDA tensor")
         if f.dtype != torch.float32 or not f.is_contiguous() or f.dim() != 2 or f.shape[1] != R:
             raise PastaError(-1, f"factors[{k}] must be a contiguous float32 [I_k, R] tensor")
+        if dims is not None and f.shape[0] != dims[k]:
+            raise PastaError(-1, f"factors[{k}] has {f.shape[0]} rows, the tensor's dims[{k}] is {dims[k]}")
+        if device is not None and f.device != device:
+            raise PastaError(-1, f"factors[{k}] is on {f.device}, expected {device}")
         ptrs[k] = f.data_ptr()
     return ptrs
 
@@ -267,7 +276,7 @@ def pasta_mttkrp_coo(x: Coo, mode: int, factors, out=None, stream=None, R=None):
                    torch.device("cuda", torch.cuda.current_device()))
         out = torch.empty((x.dims[mode], R), dtype=torch.float32, device=dev)
     _check_out(out, x.dims[mode], R)
-    ptrs = _factor_ptrs(x.order, mode, factors, R)
+    ptrs = _factor_ptrs(x.order, mode, factors, R, x.dims, out.device)
     check(lib().pasta_mttkrp_coo(x.ptr, mode, ptrs, R, C.c_void_p(out.data_ptr()),
                                  _stream_ptr(stream)))
     return out
@@ -284,7 +293,7 @@ def pasta_mttkrp_hicoo(h: Hicoo, mode: int, factors, out=None, stream=None, R=No
                    torch.device("cuda", torch.cuda.current_device()))
         out = torch.empty((h.dims[mode], R), dtype=torch.float32, device=dev)
     _check_out(out, h.dims[mode], R)
-    ptrs = _factor_ptrs(h.order, mode, factors, R)
+    ptrs = _factor_ptrs(h.order, mode, factors, R, h.dims, out.device)
     check(lib().pasta_mttkrp_hicoo(h.ptr, mode, ptrs, R, C.c_void_p(out.data_ptr()),
                                    _stream_ptr(stream)))
     return out
@@ -300,6 +309,11 @@ def pasta_mttkrp_coo_allmodes_host(x: Coo, host_factors, host_out, stream=None) 
         fp[k] = f.data_ptr() if hasattr(f, "data_ptr") else f.ctypes.data
         op[k] = o.data_ptr() if hasattr(o, "data_ptr") else o.ctypes.data
     check(lib().pasta_mttkrp_coo_allmodes_host(x.ptr, fp, R, op, _stream_ptr(stream)))
+
+
+def pasta_coo_release_staging(x: Coo) -> None:
+    """Free the e2e staging buffers cached in the handle (re-allocated on next use)."""
+    check(lib().pasta_coo_release_staging(x.ptr))
 
 
 def pasta_mttkrp_coo_allmodes_host_batch(x: Coo, steps, stream=None) -> None:
@@ -523,7 +537,8 @@ def pasta_cpals_coo(x: Coo, factors, max_iters: int = 20, tol: float = 1e-5, str
     """Single-GPU CP-ALS; `factors` (CUDA float32 [I_k, R], the initial guess) are updated in
     place.  Returns (lambda float64[R], fit per sweep list, sweeps run)."""
     R = int(factors[0].shape[1])
-    fp = (C.c_void_p * x.order)(*[f.data_ptr() for f in factors])
+    # CP-ALS overwrites every factor with dims[k] * R floats: validate all of them (mode = -1)
+    fp = _factor_ptrs(x.order, -1, factors, R, x.dims, factors[0].device)
     lam = np.zeros(R, np.float64)
     fits = np.zeros(max(max_iters, 1), np.float64)
     it = C.c_uint32()

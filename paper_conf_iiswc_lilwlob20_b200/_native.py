@@ -68,6 +68,7 @@ SIGNATURES = {
     "pasta_mttkrp_coo_allmodes_host": (_st, [_vp, C.POINTER(_vp), C.c_uint32, C.POINTER(_vp), _vp]),
     "pasta_mttkrp_coo_allmodes_host_batch": (_st, [_vp, C.c_uint32, C.POINTER(_vp), C.c_uint32,
                                                    C.POINTER(_vp), _vp]),
+    "pasta_coo_release_staging": (_st, [_vp]),
     "pasta_coo_row_counts": (_st, [_vp, C.c_uint32, _u64p]),
     "pasta_row_partition": (_st, [C.c_uint32, _u64p, C.c_uint32, _u32p]),
     "pasta_coo_partition": (_st, [_vp, C.c_uint32, C.c_uint32, _u32p]),

@@ -535,10 +535,10 @@ pasta_status pasta_mttkrp_coo(pasta_coo *x, uint32_t mode, const float *const *f
   validate_mttkrp(x->order, mode, factors, R, out);
   check_device(x->device);
   cudaStream_t s = as_stream(stream);
-  if (!x->mc[mode].ready) {
-    std::lock_guard<std::mutex> lk(x->mu);
-    coo_prepare_mode(x, mode, s);
-  }
+  // the handle's per-mode caches (sorted copy, hot-row tiers) are built / refilled under the
+  // handle's lock; the launches are only enqueued while it is held
+  std::lock_guard<std::mutex> lk(x->mu);
+  if (!x->mc[mode].ready) coo_prepare_mode(x, mode, s);
   uint64_t lo = 0, hi = x->dims[mode];
   if (x->shard_mode == int(mode)) { lo = x->row_lo; hi = x->row_hi; }
   launch_zero_rows(out, lo, hi, R, s);
@@ -553,10 +553,8 @@ pasta_status pasta_mttkrp_hicoo(pasta_hicoo *h, uint32_t mode, const float *cons
   validate_mttkrp(h->order, mode, factors, R, out);
   check_device(h->device);
   cudaStream_t s = as_stream(stream);
-  if (!h->mc[mode].ready) {
-    std::lock_guard<std::mutex> lk(h->mu);
-    hicoo_prepare_mode(h, mode, s);
-  }
+  std::lock_guard<std::mutex> lk(h->mu);
+  if (!h->mc[mode].ready) hicoo_prepare_mode(h, mode, s);
   launch_zero_rows(out, 0, h->dims[mode], R, s);
   launch_hicoo_mttkrp(h, mode, factors, R, out, s);
   API_END
@@ -609,7 +607,8 @@ static void allmodes_host_steps(pasta_coo *x, uint32_t nsteps, const float *cons
       launch_coo_mttkrp(x, m, dfac, R, x->stage_o[b][m].p, s);
       PASTA_CUDA(cudaEventRecord(e.o[b][m], s));
       PASTA_CUDA(cudaStreamWaitEvent(e.d2h, e.o[b][m], 0));
-      PASTA_CUDA(cudaMemcpyAsync(ho[m], x->stage_o[b][m].p, uint64_t(x->dims[m]) * R * sizeof(float),
+      // only the rows this handle owns go down (a shard leaves the host's other rows alone)
+      PASTA_CUDA(cudaMemcpyAsync(ho[m] + lo * R, x->stage_o[b][m].p + lo * R, (hi - lo) * R * sizeof(float),
                                  cudaMemcpyDeviceToHost, e.d2h));
       PASTA_CUDA(cudaEventRecord(e.od[b][m], e.d2h));
     }
@@ -645,6 +644,25 @@ pasta_status pasta_mttkrp_coo_allmodes_host_batch(pasta_coo *x, uint32_t nsteps,
   cudaStream_t s = as_stream(stream);
   std::lock_guard<std::mutex> lk(x->mu);
   if (nsteps) allmodes_host_steps(x, nsteps, host_factors, R, host_out, s);
+  API_END
+}
+
+pasta_status pasta_coo_release_staging(pasta_coo *x) {
+  API_BEGIN
+  require(x != nullptr, "x is NULL");
+  check_device(x->device);
+  std::lock_guard<std::mutex> lk(x->mu);
+  if (x->e2e.ready) {
+    for (int b = 0; b < 2; ++b)
+      for (uint32_t m = 0; m < x->order; ++m) PASTA_CUDA(cudaEventSynchronize(x->e2e.od[b][m]));
+  }
+  for (int b = 0; b < 2; ++b) {
+    for (uint32_t k = 0; k < pasta::kMaxOrder; ++k) {
+      x->stage_f[b][k].reset();
+      x->stage_o[b][k].reset();
+    }
+    x->stage_R[b] = 0;
+  }
   API_END
 }
 
@@ -875,10 +893,8 @@ pasta_status pasta_cpals_coo(pasta_coo *x, uint32_t R, uint32_t max_iters, doubl
   require(N >= 2, "CP-ALS needs order >= 2");
   check_device(x->device);
   cudaStream_t s = as_stream(stream);
-  {
-    std::lock_guard<std::mutex> lk(x->mu);
-    for (uint32_t k = 0; k < N; ++k) coo_prepare_mode(x, k, s);
-  }
+  std::lock_guard<std::mutex> lk(x->mu);  // the MTTKRPs below use the handle's caches
+  for (uint32_t k = 0; k < N; ++k) coo_prepare_mode(x, k, s);
   uint64_t maxd = 0;
   for (uint32_t k = 0; k < N; ++k) maxd = x->dims[k] > maxd ? x->dims[k] : maxd;
   DevArray<float> Mbuf(maxd * R, s);

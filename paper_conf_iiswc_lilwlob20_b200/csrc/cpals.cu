@@ -650,6 +650,10 @@ void launch_apply_bcast(const float *M, uint64_t row_lo, uint64_t row_hi, uint32
     fail(PASTA_EUNSUPPORTED, "pasta_rows_times_bcast: R must be 4, 8, 16, 32 or 64");
   if (ndst < 1 || ndst > kMaxOrder) fail(PASTA_EINVAL, "pasta_rows_times_bcast: 1..8 destinations");
   if (row_hi <= row_lo) return;
+  // the kernel reads M and writes the replicas with 128-bit accesses
+  bool al = (reinterpret_cast<uintptr_t>(M) & 15) == 0;
+  for (uint32_t k = 0; k < ndst; ++k) al = al && (reinterpret_cast<uintptr_t>(dsts[k]) & 15) == 0;
+  if (!al) fail(PASTA_EINVAL, "pasta_rows_times_bcast: M and every destination must be 16-byte aligned");
   DstList d{};
   d.n = ndst;
   for (uint32_t k = 0; k < ndst; ++k) d.d[k] = dsts[k];

@@ -76,6 +76,22 @@ struct DevArray {
   size_t bytes() const { return n * sizeof(T); }
 };
 
+// Completion of the last launch that used a handle's per-mode mutable state (the hot-row
+// buffer, refilled from the factors before every launch): a launch on another stream waits
+// for it, so same-handle MTTKRPs on two streams are ordered instead of racing on the buffer.
+struct LaunchFence {
+  cudaEvent_t e = nullptr;
+  LaunchFence() = default;
+  LaunchFence(const LaunchFence &) = delete;
+  LaunchFence &operator=(const LaunchFence &) = delete;
+  ~LaunchFence() { if (e) cudaEventDestroy(e); }
+  void wait(cudaStream_t s) { if (e) cudaStreamWaitEvent(s, e, 0); }
+  void record(cudaStream_t s) {
+    if (!e) cudaEventCreateWithFlags(&e, cudaEventDisableTiming);
+    cudaEventRecord(e, s);
+  }
+};
+
 // Copy streams and events of the end-to-end host path (created on first use).
 // Two staging slots: step i of a batch uses slot i & 1, so that step i+1's uploads overlap
 // step i's downloads.  f: factor k of a slot landed; o: output m of a slot computed; od:
@@ -138,6 +154,7 @@ struct CooModeCopy {
   DevArray<uint32_t> hot_rows;          // slot -> factor row, factor k at [hot_base[k], +hot_cnt[k])
   uint64_t hot_base[kMaxOrder] = {}, hot_cnt[kMaxOrder] = {}, hot_total = 0;
   DevArray<float> hot_buf;              // hot_total x R, refilled from the factors every launch
+  LaunchFence fence;                    // last launch that read hot_buf
 };
 
 constexpr int kCountBuckets = 256;  // 8 sub-buckets per octave of a row's nonzero count

@@ -1185,6 +1185,8 @@ void launch_coo_mttkrp(const pasta_coo *x, uint32_t mode, const float *const *fa
           a.io[jj++] = mc.hot_inds[k].p;
         }
       a.hs_lo[jj] = uint32_t(mc.hs_total);
+      // hot_buf is shared by every launch on this handle and mode: wait for the previous one
+      const_cast<CooModeCopy &>(mc).fence.wait(s);
       if (mc.hot_total) launch_hot_fill(mc, factors, x->order, mode, R, s);
     }
     // run per group: short runs on DRAM-bound gathers, longer ones on L2-resident factors
@@ -1207,13 +1209,16 @@ void launch_coo_mttkrp(const pasta_coo *x, uint32_t mode, const float *const *fa
       if (!persist) {
         kern<<<unsigned(nblk), hs ? hs_wpc * 32 : kThreads, smem, s>>>(a);
       } else {
-        static size_t carve = 0;
+        // the device-wide persisting carve-out is set for this launch only and restored
+        // right after it (it would otherwise shrink the normal L2 of every later kernel)
+        size_t prev_carve = 0, carve = 0;
         const size_t want = mc.hot_buf.bytes();
-        if (carve == 0) {
+        {
           int dev = 0, maxp = 0;
           cudaGetDevice(&dev);
           cudaDeviceGetAttribute(&maxp, cudaDevAttrMaxPersistingL2CacheSize, dev);
           carve = size_t(maxp);
+          PASTA_CUDA(cudaDeviceGetLimit(&prev_carve, cudaLimitPersistingL2CacheSize));
           PASTA_CUDA(cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, carve));
         }
         cudaLaunchConfig_t cfg = {};
@@ -1231,8 +1236,10 @@ void launch_coo_mttkrp(const pasta_coo *x, uint32_t mode, const float *const *fa
         cfg.attrs = attr;
         cfg.numAttrs = 1;
         PASTA_CUDA(cudaLaunchKernelEx(&cfg, kern, a));
+        PASTA_CUDA(cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, prev_carve));
       }
       PASTA_LAUNCHED();
+      if (a.hot_marked) const_cast<CooModeCopy &>(mc).fence.record(s);
     };
     // WA 1 (default): one code path per buffer.  ptxas 12.9 turns the computed buffer
     // offset into an [R+UR] LDGSTS operand that, combined with the L2 cache-policy

@@ -90,6 +90,29 @@ def powerlaw_coo(dims, nnz, seed, q=0.75, shuffle=True, dedup=True):
     return np.ascontiguousarray(got.T), vals
 
 
+def powerlaw_coo_lean(dims, nnz, seed, chunk=1 << 24):
+    """powerlaw_coo(dedup=False, shuffle=False) for BASELINE-size inputs (C5: 1B nonzeros) in
+    bounded memory: every mode must be a power of two (no rejection step); arrays are filled
+    chunk by chunk (u32 [N, M] + f32 [M], nothing else of that size).  Bits of mode k are
+    1 with probability 1/4 (AND of two uniform words), the q = 0.75 product-form law."""
+    dims = [int(d) for d in dims]
+    for d in dims:
+        if d & (d - 1) or d > (1 << 32):
+            raise ValueError("powerlaw_coo_lean needs power-of-two dims")
+    rng = _rng(seed)
+    inds = np.empty((len(dims), nnz), np.uint32)
+    vals = np.empty(nnz, np.float32)
+    for lo in range(0, nnz, chunk):
+        n = min(chunk, nnz - lo)
+        for k, d in enumerate(dims):
+            a = rng.integers(0, 1 << 32, size=n, dtype=np.uint32)
+            a &= rng.integers(0, 1 << 32, size=n, dtype=np.uint32)
+            a &= np.uint32(d - 1)
+            inds[k, lo:lo + n] = a
+        vals[lo:lo + n] = rng.uniform(-1.0, 1.0, size=n)
+    return inds, vals
+
+
 def factors(dims, R, seed, lo=0.0, hi=1.0):
     """Dense factor matrices U^(k) in R^{I_k x R}, row-major float32, entries U[lo, hi)."""
     rng = _rng(seed + 7919)

@@ -78,9 +78,8 @@ def test_tensor_level_same_and_merged_patterns(env, op):
     np.testing.assert_array_equal(ti, xi)
     _bits_equal(tv, oracle.ts(xv, op, np.float32(1.5)))
     # same pattern: elementwise in X's order
-    x2 = pasta.pasta_coo_from_arrays(dims, xi, yv[: xi.shape[1]] if yv.shape[0] >= xi.shape[1]
-                                     else np.resize(yv, xi.shape[1]))
-    x2v = pasta.pasta_coo_export(x2)[1]
+    x2v = yv[: xi.shape[1]] if yv.shape[0] >= xi.shape[1] else np.resize(yv, xi.shape[1])
+    x2 = pasta.pasta_coo_from_arrays(dims, xi, x2v)
     z = pasta.pasta_coo_tew(x, x2, op)
     zi, zv = pasta.pasta_coo_export(z)
     np.testing.assert_array_equal(zi, xi)

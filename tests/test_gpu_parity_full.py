@@ -1,0 +1,103 @@
+"""Parity at the edges of the north_star tolerance and at full size (SURVEY 8(c) "GPU tolerance"
+row; P:157 / P:282 atomics; P:181 / P:205-207 HiCOO).
+
+* A single output row holding 10^7 nonzeros, in each mode in turn, every mode of COO and HiCOO
+  MTTKRP checked element by element: the case where a flat sequential fp32 sum would fail
+  (~1.1e-4 relative over 10^7 terms) and only hierarchical summation
+  (register runs + vector atomics at run ends) stays within 1e-4 * sum|terms| + 1e-6.
+* The headline workload H (regL-shaped (2^23)^3, 100M nonzeros, R = 16, the launch
+  configuration bench.py times): EVERY output row of every mode, COO and HiCOO, against the full
+  oracle.
+* COO -> HiCOO (B = 128) bit-exact (memcmp of bptr / binds / einds / vals) at the full sizes of
+  H, C2 and C3 (C4 is in test_gpu_fullsize.py).
+Inputs come from synth_inputs only, never from the CUDA path.
+"""
+import numpy as np
+import pytest
+
+import synth_inputs as si
+
+pytestmark = pytest.mark.gpu
+
+TOL_REL, TOL_ABS = 1e-4, 1e-6
+
+
+@pytest.fixture(scope="module")
+def env(oracle_mod):
+    import torch
+
+    import paper_conf_iiswc_lilwlob20_b200 as pasta
+    assert torch.cuda.is_available()
+    torch.cuda.set_device(0)
+    return pasta, oracle_mod, torch
+
+
+def _excess(got, ref, ab):
+    g = got.detach().cpu().numpy().astype(np.float64)
+    return np.abs(g - ref) - (TOL_REL * ab + TOL_ABS)
+
+
+@pytest.mark.parametrize("force_hot", ["0", "1"])
+@pytest.mark.parametrize("hot_mode", [0, 1, 2])
+def test_hot_row_ten_million(env, hot_mode, force_hot, monkeypatch):
+    """10^7 nonzeros in row 1234 of mode `hot_mode` (+ 10^6 uniform elsewhere), R = 16.  With
+    force_hot = 1 the hot-row cache tiers are on, so when the hot mode is a gathered mode its
+    row is served from the shared-memory tier."""
+    pasta, oracle, torch = env
+    monkeypatch.setenv("PASTA_HOT_FORCE", force_hot)
+    dims = (4096, 4096, 4096)
+    inds, vals = si.hot_row_coo(dims, 10_000_000, 1_000_000, seed=31 + hot_mode, mode=hot_mode, hot_row=1234)
+    assert np.count_nonzero(inds[hot_mode] == 1234) == 10_000_000
+    U = si.factors(dims, 16, seed=7)
+    Ud = [torch.from_numpy(u).cuda() for u in U]
+    x = pasta.pasta_coo_from_arrays(dims, inds, vals)
+    h = pasta.pasta_coo_to_hicoo(x, 7)
+    for n in range(3):
+        ref, ab = oracle.mttkrp(dims, inds, vals, n, U)
+        for name, got in (("coo", pasta.pasta_mttkrp_coo(x, n, Ud)), ("hicoo", pasta.pasta_mttkrp_hicoo(h, n, Ud))):
+            ex = _excess(got, ref, ab)
+            assert ex.max() <= 0, f"{name} hot mode {hot_mode} mode {n}: excess {ex.max():.3e}"
+            if n == hot_mode:  # the 10^7-term row itself: report how far inside the bound it is
+                g = got[1234].cpu().numpy().astype(np.float64)
+                rel = np.max(np.abs(g - ref[1234]) / ab[1234])
+                assert rel < TOL_REL, (name, rel)
+
+
+def test_fullsize_h_every_row(env):
+    """H at full size: every row of every mode, COO and HiCOO, vs the full fp64 oracle."""
+    pasta, oracle, torch = env
+    cfg = si.CONFIGS["h"]
+    dims, R, M = cfg["dims"], cfg["R"], cfg["nnz"]
+    inds, vals = si.powerlaw_coo_lean(dims, M, seed=cfg["seed"] + 101)
+    g = torch.Generator(device="cuda")
+    g.manual_seed(13)
+    Ud = [torch.rand((d, R), generator=g, device="cuda") for d in dims]
+    U = [u.cpu().numpy() for u in Ud]
+    x = pasta.pasta_coo_from_arrays(dims, inds, vals)
+    h = pasta.pasta_coo_to_hicoo(x, 7)
+    for n in range(3):
+        ref, ab = oracle.mttkrp(dims, inds, vals, n, U)
+        for name, fn, t in (("coo", pasta.pasta_mttkrp_coo, x), ("hicoo", pasta.pasta_mttkrp_hicoo, h)):
+            ex = _excess(fn(t, n, Ud), ref, ab)
+            assert ex.max() <= 0, f"h {name} mode {n}: excess {ex.max():.3e} at row {np.argmax(ex) // R}"
+            del ex
+        del ref, ab
+
+
+@pytest.mark.parametrize("key", ["h", "c2", "c3"])
+def test_fullsize_hicoo_conversion_bit_exact(env, key):
+    pasta, oracle, torch = env
+    cfg = si.CONFIGS[key]
+    dims, M = cfg["dims"], cfg["nnz"]
+    if key == "h":
+        inds, vals = si.powerlaw_coo_lean(dims, M, seed=cfg["seed"] + 5)
+    else:
+        inds, vals = si.powerlaw_coo(dims, M, seed=cfg["seed"] + 5, dedup=False)
+    x = pasta.pasta_coo_from_arrays(dims, inds, vals)
+    hx = pasta.pasta_hicoo_export(pasta.pasta_coo_to_hicoo(x, 7))
+    del x
+    o = oracle.coo_to_hicoo(inds, vals, 7)
+    assert hx["nblocks"] == o["nblocks"]
+    for k in ("bptr", "binds", "einds"):
+        assert np.array_equal(hx[k], o[k]), k
+    assert np.array_equal(hx["vals"].view(np.uint32), o["vals"].view(np.uint32))

@@ -40,13 +40,40 @@ def test_recovers_exact_low_rank_tensor(oracle_mod):
     assert np.linalg.norm(X - Xhat) / np.linalg.norm(X) < 2e-3
 
 
-def test_normal_equations_hold_after_each_update(oracle_mod):
+def _unfold(X, n):
+    """Mode-n unfolding, columns with the earliest remaining mode fastest (Kolda-Bader, R#3)."""
+    return np.reshape(np.moveaxis(X, n, 0), (X.shape[n], -1), order="F")
+
+
+def _krp(mats):
+    """Khatri-Rao product (Eq. 4): column r = kron(mats[0][:, r], mats[1][:, r], ...)."""
+    out = mats[0]
+    for m in mats[1:]:
+        out = np.einsum("ir,jr->ijr", out, m).reshape(-1, out.shape[1])
+    return out
+
+
+def test_each_update_is_the_dense_least_squares_solution(oracle_mod):
+    """Every ALS update U_n = argmin ||X_(n) - U_n KRP^T||_F (Kolda-Bader), solved here by
+    np.linalg.lstsq on the dense unfolding and the explicit Khatri-Rao product -- a formulation
+    that shares neither the MTTKRP nor the normal equations with the oracle."""
     dims, R = (15, 12, 9, 7), 4
     inds, vals = si.uniform_coo(dims, 600, seed=2)
+    X = np.zeros(dims)
+    X[tuple(inds)] = vals
     rec = []
-    cp_als(dims, inds, vals, si.factors(dims, R, seed=4), iters=2, record=rec)
+    U0 = si.factors(dims, R, seed=4)
+    cp_als(dims, inds, vals, U0, iters=2, record=rec)
+    # replay: the factors the oracle held before each update (fp32 storage, as the oracle)
+    cur = [u.astype(np.float32) for u in U0]
     for n, M, V, Un in rec:
-        assert np.allclose(Un @ V, M, rtol=1e-9, atol=1e-9 * np.abs(M).max())
+        others = [cur[k].astype(np.float64) for k in reversed(range(len(dims))) if k != n]
+        K = _krp(others)  # rows ordered with the earliest remaining mode fastest
+        ls = np.linalg.lstsq(K, _unfold(X, n).T, rcond=None)[0].T
+        assert np.allclose(Un, ls, rtol=1e-7, atol=1e-9 * np.abs(ls).max()), n
+        lam = np.sqrt(np.sum(Un * Un, axis=0))
+        lam[lam == 0] = 1.0
+        cur[n] = (Un / lam).astype(np.float32)
 
 
 def test_fit_formula_matches_dense_reconstruction(oracle_mod):
