@@ -8,8 +8,8 @@ Per target mode n:
   2. every rank keeps the mode-n sorted shard of its rows (``pasta_coo_shard``) and the
      replicated, read-only factors; MTTKRP on the shard writes only rows [lo, hi) of the
      full-size output (no cross-GPU atomics: rows are exclusively owned);
-  3. ``gather_rows``: rank p broadcasts its contiguous row block out[lo_p:hi_p] into every
-     replica (an uneven all-gather done in place, no packing copies).
+  3. ``gather_rows``: one padded all-gather per mode of the owned row blocks (NCCL
+     all_gather_into_tensor), then each peer block is copied into place.
 """
 from __future__ import annotations
 
@@ -18,11 +18,60 @@ from typing import List, Sequence
 import numpy as np
 
 
-def gather_rows(out, bounds: Sequence[int], group=None, async_op: bool = False):
-    """In-place all-gather(v) of contiguous row blocks: after the call every rank holds
-    out[bounds[p]:bounds[p+1]] of every rank p.  Works with NCCL (CUDA tensors) and gloo
-    (CPU tensors).  Returns the list of work handles when async_op."""
+_GATHER_BUFS = {}
+
+
+class _RowGather:
+    """One padded all-gather of the owned row blocks: rank p's rows [bounds[p], bounds[p+1])
+    travel in slot p of a [P, max_rows, R] buffer (all_gather_into_tensor, a single NCCL
+    collective -- NVLS-capable on NVSwitch -- instead of P broadcasts); wait() copies the
+    peers' slots into place."""
+
+    def __init__(self, out, bounds, group, async_op):
+        import torch.distributed as dist
+        self.out, self.bounds = out, [int(b) for b in bounds]
+        P = len(self.bounds) - 1
+        self.rank = dist.get_rank(group)
+        rows = [self.bounds[p + 1] - self.bounds[p] for p in range(P)]
+        m = max(max(rows), 1)
+        key = (P, m, tuple(out.shape[1:]), out.dtype, str(out.device))
+        buf = _GATHER_BUFS.get(key)
+        if buf is None:
+            buf = out.new_empty((P, m) + tuple(out.shape[1:]))
+            _GATHER_BUFS.clear()  # one cached buffer: the shapes of one workload
+            _GATHER_BUFS[key] = buf
+        self.buf, self.rows = buf, rows
+        lo, hi = self.bounds[self.rank], self.bounds[self.rank + 1]
+        send = buf[self.rank]
+        if hi > lo:
+            send[: hi - lo].copy_(out[lo:hi])
+        # in place: the input is this rank's slot of the output buffer
+        self.work = dist.all_gather_into_tensor(buf.view(-1), send.reshape(-1), group=group,
+                                                async_op=async_op)
+        if not async_op:
+            self._scatter()
+
+    def _scatter(self):
+        for p, r in enumerate(self.rows):
+            if p != self.rank and r > 0:
+                self.out[self.bounds[p]:self.bounds[p + 1]].copy_(self.buf[p, :r])
+
+    def wait(self):
+        if self.work is not None:
+            self.work.wait()
+            self.work = None
+            self._scatter()
+
+
+def gather_rows(out, bounds: Sequence[int], group=None, async_op: bool = False, method: str = "allgather"):
+    """All-gather(v) of contiguous row blocks: after the call every rank holds
+    out[bounds[p]:bounds[p+1]] of every rank p.  Works with NCCL (CUDA tensors) and gloo (CPU
+    tensors).  method "allgather": one padded all_gather_into_tensor (default); "broadcast":
+    P in-place broadcasts, no staging buffer.  Returns the list of work handles when async_op."""
     import torch.distributed as dist
+    if method == "allgather":
+        g = _RowGather(out, bounds, group, async_op)
+        return [g] if async_op else []
     works = []
     for p in range(len(bounds) - 1):
         lo, hi = int(bounds[p]), int(bounds[p + 1])

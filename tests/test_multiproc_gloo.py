@@ -25,7 +25,7 @@ def _free_port():
     return port
 
 
-def _worker(rank, world, port, result_q):
+def _worker(rank, world, port, result_q, method):
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
     dist.init_process_group("gloo", rank=rank, world_size=world)
@@ -47,7 +47,7 @@ def _worker(rank, world, port, result_q):
             part, _ = oracle.mttkrp(dims, np.ascontiguousarray(inds[:, mine]), vals[mine], n, U)
             out = torch.full((dims[n], R), float("nan"), dtype=torch.float32)
             out[lo:hi] = torch.from_numpy(part[lo:hi].astype(np.float32))
-            gather_rows(out, bounds[n])
+            gather_rows(out, bounds[n], method=method)
             full, _ = oracle.mttkrp(dims, inds, vals, n, U)
             ok &= bool(np.allclose(out.numpy(), full.astype(np.float32), rtol=0, atol=0))
             # the shards are disjoint and cover every nonzero
@@ -59,12 +59,13 @@ def _worker(rank, world, port, result_q):
         dist.destroy_process_group()
 
 
-def test_row_partitioned_allgather_world2():
+@pytest.mark.parametrize("method", ["allgather", "broadcast"])
+def test_row_partitioned_allgather_world2(method):
     world = 2
     port = _free_port()
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
-    procs = [ctx.Process(target=_worker, args=(r, world, port, q)) for r in range(world)]
+    procs = [ctx.Process(target=_worker, args=(r, world, port, q, method)) for r in range(world)]
     for p in procs:
         p.start()
     res = [q.get(timeout=300) for _ in range(world)]

@@ -34,25 +34,28 @@ __global__ void init_chase(uint32_t *buf, uint64_t nchunks) {
     buf[i * 32] = uint32_t(((i + 1) % 16) * 32);
 }
 
-// dependent chase of `len` coherent loads through the lines of chunk c: cycles per load
-__device__ __forceinline__ uint32_t chase(const uint32_t *chunk, int len) {
+// dependent chase of `len` coherent loads through the lines of chunk c: cycles per load.  The
+// chain's result is stored to shared memory (a side effect waiting on the last load) before
+// the second clock read, which ptxas otherwise hoists above the loads.
+__device__ __forceinline__ uint32_t chase(const uint32_t *chunk, int len, volatile uint32_t *sink) {
   uint32_t off = 0;
   const long long t0 = clock64();
+#pragma unroll 1
   for (int i = 0; i < len; ++i) off = ld_cv(chunk + off);
-  const long long t1 = clock64();  // at most one load latency early: the chain serialises
-  return uint32_t((t1 - t0) / len) + (off == 0xFFFFFFFFu);
+  *sink = off;
+  __syncwarp();
+  const long long t1 = clock64();
+  return uint32_t((t1 - t0) / len);
 }
 
 // one CTA per SM (forced by shared memory); thread 0 times NC chunks (64-load chase, min of 2)
 __global__ void sm_pattern(const uint32_t *buf, int nc, uint32_t *lat, uint32_t *sm_of_cta) {
   extern __shared__ uint32_t pad[];
   if (threadIdx.x != 0) return;
-  pad[0] = 0;
   sm_of_cta[blockIdx.x] = smid();
   for (int c = 0; c < nc; ++c) {
     const uint32_t *ch = buf + size_t(c) * 512;
-    const uint32_t a = chase(ch, 64), b = chase(ch, 64);
-    lat[size_t(blockIdx.x) * nc + c] = a < b ? a : b;
+    lat[size_t(blockIdx.x) * nc + c] = chase(ch, 64, pad);
   }
 }
 
@@ -60,8 +63,8 @@ __global__ void sm_pattern(const uint32_t *buf, int nc, uint32_t *lat, uint32_t 
 __global__ void chunk_home(const uint32_t *buf, uint64_t nchunks, uint32_t want_sm, uint32_t *lat, int *ran) {
   extern __shared__ uint32_t pad[];
   if (smid() != want_sm) return;
-  if (threadIdx.x == 0) { pad[0] = 1; *ran = 1; }
-  for (uint64_t c = threadIdx.x; c < nchunks; c += blockDim.x) lat[c] = chase(buf + c * 512, 16);
+  if (threadIdx.x == 0) *ran = 1;
+  for (uint64_t c = threadIdx.x; c < nchunks; c += blockDim.x) lat[c] = chase(buf + c * 512, 16, pad + threadIdx.x);
 }
 
 __device__ __forceinline__ uint32_t hash32(uint64_t z) {
