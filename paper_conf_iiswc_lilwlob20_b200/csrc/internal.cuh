@@ -186,6 +186,26 @@ struct HicooModeCopy {
   // staged decode (launch_hicoo_mttkrp): slice holding the first entry of every group run
   DevArray<uint64_t> run_sb;
   uint64_t run_sb_run = 0;
+  // Hot-BLOCK tiers (hicoo_mark_hot, R#34): the row-slice copy has no per-entry coordinate
+  // to retag (entries carry 8-bit offsets from a per-slice block base), so the tiers of the
+  // COO hot-row cache are built at block granularity: the most frequent block rows [b B,
+  // b B + B) of each gathered (compressed) factor go whole into the shared-memory tier or
+  // the packed L2-tier buffer, and the slice bases sbbase[k] of those blocks are retagged in
+  // place to 0xC0000000 | smem row slot / 0x80000000 | L2 row slot (slot = tier block x B,
+  // so base + einds stays inside the block's slots).  Same slot lists and fill kernel as the
+  // COO tiers; tier_block[k] lists the original block of every (smem, then L2) slot block so
+  // the retagging can be undone when R or the budgets change.
+  uint32_t hot_R = 0;
+  bool hot_global = false;
+  uint32_t hot_smem_budget = 0;
+  DevArray<uint32_t> hs_rows;
+  uint64_t hs_base[kMaxOrder] = {}, hs_cnt[kMaxOrder] = {}, hs_total = 0;
+  DevArray<uint32_t> hot_rows;
+  uint64_t hot_base[kMaxOrder] = {}, hot_cnt[kMaxOrder] = {}, hot_total = 0;
+  DevArray<float> hot_buf;
+  DevArray<uint32_t> tier_block[kMaxOrder];
+  bool tagged = false;
+  LaunchFence fence;
 };
 
 }  // namespace pasta
@@ -312,6 +332,12 @@ void coo_build_fibers(pasta_coo *x, uint32_t mode, cudaStream_t s);
 void launch_ttv(const pasta_coo &mat, const float *v, float *y, cudaStream_t s);
 void launch_hot_fill(const CooModeCopy &mc, const float *const *factors, uint32_t order, uint32_t mode,
                      uint32_t R, cudaStream_t s);
+void launch_hot_fill(const HicooModeCopy &mc, const float *const *factors, uint32_t order, uint32_t mode,
+                     uint32_t R, cudaStream_t s);
+// hot-block tiers of the HiCOO row-slice copy of `mode` (R#34); no-op when already marked for
+// (R, global_tier, smem_rows) or when the copy is not the row-slice layout
+void hicoo_mark_hot(pasta_hicoo *h, uint32_t mode, uint32_t R, bool global_tier, uint32_t smem_rows,
+                    cudaStream_t s);
 void row_counts_device(const uint32_t *rows, uint64_t nnz, uint32_t nrows, uint64_t *counts_host,
                        cudaStream_t s);
 // first position x in the sorted array a[0..M) with a[x] >= v (device binary search).

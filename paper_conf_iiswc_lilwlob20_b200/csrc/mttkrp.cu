@@ -702,9 +702,10 @@ __global__ void __launch_bounds__(HS ? WPC_ * 32 : kThreads, HS ? 1 : (WA == 6 ?
   constexpr int WPC = HS ? WPC_ : kWarpsPerCta;
   // 7: HS kernel without the L2 tier (no hot_buf rows) whose gathered factors are < 4 GB each:
   // no base-pointer select, 32-bit byte offsets.  9: HiCOO row slices decoded warp-wide into
-  // the stage buffer (no hot tiers, 64-bit offsets)
-  constexpr bool kHic = WA == 9;
-  constexpr bool kL2T = WA != 7 && !kHic;
+  // the stage buffer (no hot tiers, 64-bit offsets).  10: the same decode with the hot-block
+  // tiers (R#34): decoded coordinates carry the tier tags of their retagged slice bases
+  constexpr bool kHic = WA == 9 || WA == 10;
+  constexpr bool kL2T = WA != 7 && WA != 9;
   constexpr bool kGather = WA != 4 && WA != 5;
   constexpr bool kWrite = WA != 3 && WA != 5;
   constexpr int kBuf = (WA == 0 || WA == 2) ? WA : 1;  // 6: form 1 with 3 CTAs per SM
@@ -889,7 +890,7 @@ __global__ void __launch_bounds__(HS ? WPC_ * 32 : kThreads, HS ? 1 : (WA == 6 ?
           for (int j = 0; j < NO; ++j) {
             if (kGather) {
               const uint32_t id = idx[j][u];
-              if constexpr (kHic) {  // decoded HiCOO coordinate: plain factor row
+              if constexpr (WA == 9) {  // decoded HiCOO coordinate: plain factor row
                 if (u < cnt) f[j][u] = ldg_vec<4>(a.Uo[j] + uint64_t(id) * R + col, pol.gather);
               } else if constexpr (HS) {  // shared-memory tier, L2-tier buffer or plain factor row
                 const bool in_s = (id >> 30) == 3u;
@@ -1370,17 +1371,54 @@ void launch_hicoo_mttkrp(const pasta_hicoo *h, uint32_t mode, const float *const
       mcw.run_sb_run = run;
     }
     a.run_sb = mcw.run_sb.p;
+    // hot-block tiers (R#34), with the COO cache's policy: an L2 tier when the gathered factors
+    // exceed half the L2, a shared-memory tier of what the stage buffers leave (512 rows when
+    // the gathers go to DRAM); PASTA_HICOO_HOT=0 disables both
+    const size_t stage = size_t(16) * 2 * (hno + 2) * (G * 32) * sizeof(uint32_t);
+    bool tiers = false;
+    if (env_int("PASTA_HICOO_HOT", 1) && env_int("PASTA_HOT_SMEM", 1)) {
+      static int l2 = 0;
+      if (!l2) {
+        int dev = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, dev);
+        if (l2 <= 0) l2 = 126 << 20;
+      }
+      uint64_t gathered = 0;
+      for (uint32_t k = 0; k < h->order; ++k)
+        if (k != mode) gathered += uint64_t(h->dims[k]) * R * sizeof(float);
+      const bool want_hot = env_int("PASTA_HOT_FORCE", 0) || gathered > uint64_t(l2) / 2;
+      uint32_t budget = stage < 227 * 1024 ? uint32_t((227 * 1024 - stage) / (size_t(R) * sizeof(float))) : 0u;
+      if (want_hot) budget = std::min(budget, 512u);
+      if (const int cap = env_int("PASTA_HOT_SMEM_ROWS", 0)) budget = std::min(budget, uint32_t(cap));
+      hicoo_mark_hot(const_cast<pasta_hicoo *>(h), mode, R, want_hot, budget, s);
+      tiers = mc.hot_R == R && (mc.hs_total + mc.hot_total) > 0;
+    }
+    if (tiers) {
+      a.hot_marked = 1;
+      a.hot_buf = mc.hot_buf.p;
+      a.hs_rows = mc.hs_rows.p;
+      int jj = 0;
+      for (uint32_t k = 0; k < h->order; ++k)
+        if (k != mode) a.hs_lo[jj++] = uint32_t(mc.hs_base[k]);
+      a.hs_lo[jj] = uint32_t(mc.hs_total);
+      mcw.fence.wait(s);
+      if (mc.hot_total) launch_hot_fill(mc, factors, h->order, mode, R, s);
+    }
     ProfScope prof(kProfHicoo, s);
     const int cfg = env_int("PASTA_HS_CFG", 0);  // 2 (8-deep steps) spills here
-    const size_t smem = size_t(16) * 2 * (hno + 2) * (G * 32) * sizeof(uint32_t);
+    const size_t smem = stage + (tiers ? size_t(mc.hs_total) * R * sizeof(float) : 0);
     const uint64_t nwarps = (a.nnz + a.chunk - 1) / a.chunk;
     const uint64_t nblk = std::min<uint64_t>((nwarps + 15) / 16, uint64_t(sm_count()));
     auto go = [&](auto kern) {
       PASTA_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem)));
       kern<<<unsigned(nblk), 512, smem, s>>>(a);
       PASTA_LAUNCHED();
+      if (tiers) mcw.fence.record(s);
     };
-    if (cfg == 2 && hno <= 2)
+    if (tiers)
+      with_no_lpn<3>(hno, lpn, [&](auto NOt, auto Lt) { go(coo_staged_kernel<NOt.value, Lt.value, 10, true, 16, 32, 4>); });
+    else if (cfg == 2 && hno <= 2)
       with_no_lpn<2>(hno, lpn, [&](auto NOt, auto Lt) { go(coo_staged_kernel<NOt.value, Lt.value, 9, true, 16, 32, 8>); });
     else
       with_no_lpn<3>(hno, lpn, [&](auto NOt, auto Lt) { go(coo_staged_kernel<NOt.value, Lt.value, 9, true, 16, 32, 4>); });

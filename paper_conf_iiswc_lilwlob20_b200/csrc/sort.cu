@@ -3,6 +3,7 @@
 // gathers, compaction, histograms.  Pre-processing trades for kernel time.
 #include <cub/cub.cuh>
 
+#include <algorithm>
 #include <cstdio>
 #include <cstdlib>
 #include <vector>
@@ -464,8 +465,9 @@ void coo_mark_hot(pasta_coo *x, uint32_t mode, uint32_t R, bool global_tier, uin
   }
 }
 
-void launch_hot_fill(const CooModeCopy &mc, const float *const *factors, uint32_t order, uint32_t mode,
-                     uint32_t R, cudaStream_t s) {
+template <class MC>
+static void hot_fill_t(const MC &mc, const float *const *factors, uint32_t order, uint32_t mode,
+                       uint32_t R, cudaStream_t s) {
   for (uint32_t k = 0; k < order; ++k) {
     if (k == mode || mc.hot_cnt[k] == 0) continue;
     const uint64_t n = mc.hot_cnt[k] * (R / 4);
@@ -476,6 +478,153 @@ void launch_hot_fill(const CooModeCopy &mc, const float *const *factors, uint32_
                                                 reinterpret_cast<float4 *>(mc.hot_buf.p));
     PASTA_LAUNCHED();
   }
+}
+
+}  // namespace pasta
+
+namespace pasta {
+
+void launch_hot_fill(const CooModeCopy &mc, const float *const *factors, uint32_t order, uint32_t mode,
+                     uint32_t R, cudaStream_t s) {
+  hot_fill_t(mc, factors, order, mode, R, s);
+}
+void launch_hot_fill(const HicooModeCopy &mc, const float *const *factors, uint32_t order, uint32_t mode,
+                     uint32_t R, cudaStream_t s) {
+  hot_fill_t(mc, factors, order, mode, R, s);
+}
+
+namespace {
+
+// cnt[binds_k[b]] += entries of canonical block b: nonzeros per mode-k block row
+__global__ void block_row_count_kernel(const uint64_t *__restrict__ bptr, const uint32_t *__restrict__ binds,
+                                       uint64_t nb, unsigned long long *__restrict__ cnt) {
+  for (uint64_t b = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; b < nb; b += uint64_t(gridDim.x) * blockDim.x)
+    atomicAdd(&cnt[binds[b]], (unsigned long long)(bptr[b + 1] - bptr[b]));
+}
+
+// slice base (untagged: block << bb) -> tier tag | slot row, from the per-block-row map
+__global__ void retag_base_kernel(uint32_t *__restrict__ base, uint64_t n, uint32_t bb,
+                                  const uint32_t *__restrict__ map) {
+  for (uint64_t i = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; i < n; i += uint64_t(gridDim.x) * blockDim.x) {
+    const uint32_t v = base[i];
+    if ((v >> 30) == 0u) {
+      const uint32_t t = map[v >> bb];
+      if (t != 0xFFFFFFFFu) base[i] = t;
+    }
+  }
+}
+
+// undo retag_base_kernel: tagged slot row -> original block << bb (tier_block: smem slot
+// blocks of this factor, then its L2 slot blocks)
+__global__ void untag_base_kernel(uint32_t *__restrict__ base, uint64_t n, uint32_t bb, uint32_t hs_base,
+                                  uint32_t hot_base, uint32_t nsm, const uint32_t *__restrict__ tier_block) {
+  for (uint64_t i = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; i < n; i += uint64_t(gridDim.x) * blockDim.x) {
+    const uint32_t v = base[i], tag = v >> 30, slot = v & 0x3FFFFFFFu;
+    if (tag == 3u) base[i] = tier_block[(slot - hs_base) >> bb] << bb;
+    else if (tag == 2u) base[i] = tier_block[nsm + ((slot - hot_base) >> bb)] << bb;
+  }
+}
+
+}  // namespace
+
+// Hot-block tiers of the HiCOO row-slice copy (R#34): block rows of the gathered compressed
+// factors ranked jointly by their nonzero count; the top ones fill the shared-memory tier
+// (`smem_rows` rows = smem_rows / B blocks), the next ones the L2 tier (PASTA_HOT_MB, default
+// 64 MB, when `global_tier`); the slices' bases of those blocks are retagged in place.
+void hicoo_mark_hot(pasta_hicoo *h, uint32_t mode, uint32_t R, bool global_tier, uint32_t smem_rows,
+                    cudaStream_t s) {
+  HicooModeCopy &mc = h->mc[mode];
+  if (mc.layout != 0) return;
+  if (mc.hot_R == R && mc.hot_global == global_tier && mc.hot_smem_budget == smem_rows) return;
+  const uint32_t N = h->order, bb = h->block_bits, B = 1u << bb;
+  auto blocked = [&](uint32_t k) { return k != mode && ((h->cmask >> k) & 1u) != 0; };
+  if (mc.tagged) {  // undo the previous tiers before re-ranking
+    for (uint32_t k = 0; k < N; ++k) {
+      if (!blocked(k) || (mc.hs_cnt[k] + mc.hot_cnt[k]) == 0) continue;
+      untag_base_kernel<<<grid8(mc.nsb), 256, 0, s>>>(mc.sbbase[k].p, mc.nsb, bb, uint32_t(mc.hs_base[k]),
+                                                       uint32_t(mc.hot_base[k]), uint32_t(mc.hs_cnt[k] >> bb),
+                                                       mc.tier_block[k].p);
+      PASTA_LAUNCHED();
+    }
+    mc.tagged = false;
+  }
+  // the ranking is cached per (R, budgets), also when it yields no tiers
+  mc.hot_R = R;
+  mc.hot_global = global_tier;
+  mc.hot_smem_budget = smem_rows;
+  mc.hs_total = mc.hot_total = 0;
+  for (uint32_t k = 0; k < N; ++k) mc.hs_base[k] = mc.hs_cnt[k] = mc.hot_base[k] = mc.hot_cnt[k] = 0;
+  for (uint32_t k = 0; k < N; ++k)
+    if (h->dims[k] >= 0x40000000u) return;  // untagged bases must stay below 2^30
+  const char *env = getenv("PASTA_HOT_MB");
+  const double hot_mb = global_tier ? ((env && *env) ? atof(env) : 64.0) : 0.0;
+  const uint64_t sm_blocks = smem_rows / B;
+  const uint64_t l2_blocks = uint64_t(hot_mb * 1048576.0 / (double(B) * R * sizeof(float)));
+  if ((sm_blocks == 0 && l2_blocks == 0) || h->nnz == 0 || mc.nsb == 0) return;
+  struct Cand { unsigned long long cnt; uint32_t k, blk; };
+  std::vector<Cand> cand;
+  for (uint32_t k = 0; k < N; ++k) {
+    if (!blocked(k)) continue;
+    const uint64_t nbr = (uint64_t(h->dims[k]) + B - 1) >> bb;
+    DevArray<unsigned long long> c(nbr, s);
+    PASTA_CUDA(cudaMemsetAsync(c.p, 0, c.bytes(), s));
+    block_row_count_kernel<<<grid8(h->nblocks), 256, 0, s>>>(h->bptr.p, h->binds[k].p, h->nblocks, c.p);
+    PASTA_LAUNCHED();
+    std::vector<unsigned long long> hc(nbr);
+    PASTA_CUDA(cudaMemcpyAsync(hc.data(), c.p, c.bytes(), cudaMemcpyDeviceToHost, s));
+    PASTA_CUDA(cudaStreamSynchronize(s));
+    for (uint64_t b = 0; b < nbr; ++b)
+      if (hc[b]) cand.push_back({hc[b], k, uint32_t(b)});
+  }
+  std::stable_sort(cand.begin(), cand.end(), [](const Cand &a, const Cand &b) { return a.cnt > b.cnt; });
+  std::vector<std::vector<uint32_t>> smb(N), l2b(N);
+  for (uint64_t i = 0; i < cand.size() && i < sm_blocks + l2_blocks; ++i)
+    (i < sm_blocks ? smb : l2b)[cand[i].k].push_back(cand[i].blk);
+  std::vector<uint32_t> hs_rows, hot_rows;
+  for (uint32_t k = 0; k < N; ++k) {
+    mc.hs_base[k] = hs_rows.size();
+    for (uint32_t blk : smb[k])
+      for (uint32_t e = 0; e < B; ++e) hs_rows.push_back(std::min<uint64_t>(uint64_t(blk) * B + e, h->dims[k] - 1));
+    mc.hs_cnt[k] = hs_rows.size() - mc.hs_base[k];
+    mc.hot_base[k] = hot_rows.size();
+    for (uint32_t blk : l2b[k])
+      for (uint32_t e = 0; e < B; ++e) hot_rows.push_back(std::min<uint64_t>(uint64_t(blk) * B + e, h->dims[k] - 1));
+    mc.hot_cnt[k] = hot_rows.size() - mc.hot_base[k];
+  }
+  mc.hs_total = hs_rows.size();
+  mc.hot_total = hot_rows.size();
+  mc.hs_rows.alloc(std::max<size_t>(hs_rows.size(), 1), s);
+  mc.hot_rows.alloc(std::max<size_t>(hot_rows.size(), 1), s);
+  mc.hot_buf.alloc(std::max<uint64_t>(mc.hot_total, 1) * R, s);
+  if (!hs_rows.empty())
+    PASTA_CUDA(cudaMemcpyAsync(mc.hs_rows.p, hs_rows.data(), hs_rows.size() * 4, cudaMemcpyHostToDevice, s));
+  if (!hot_rows.empty())
+    PASTA_CUDA(cudaMemcpyAsync(mc.hot_rows.p, hot_rows.data(), hot_rows.size() * 4, cudaMemcpyHostToDevice, s));
+  for (uint32_t k = 0; k < N; ++k) {
+    if (!blocked(k) || (smb[k].empty() && l2b[k].empty())) continue;
+    const uint64_t nbr = (uint64_t(h->dims[k]) + B - 1) >> bb;
+    std::vector<uint32_t> map(nbr, 0xFFFFFFFFu), tb;
+    for (size_t i = 0; i < smb[k].size(); ++i) {
+      map[smb[k][i]] = 0xC0000000u | uint32_t(mc.hs_base[k] + i * B);
+      tb.push_back(smb[k][i]);
+    }
+    for (size_t i = 0; i < l2b[k].size(); ++i) {
+      map[l2b[k][i]] = 0x80000000u | uint32_t(mc.hot_base[k] + i * B);
+      tb.push_back(l2b[k][i]);
+    }
+    DevArray<uint32_t> dmap(nbr, s);
+    PASTA_CUDA(cudaMemcpyAsync(dmap.p, map.data(), nbr * 4, cudaMemcpyHostToDevice, s));
+    mc.tier_block[k].alloc(tb.size(), s);
+    PASTA_CUDA(cudaMemcpyAsync(mc.tier_block[k].p, tb.data(), tb.size() * 4, cudaMemcpyHostToDevice, s));
+    retag_base_kernel<<<grid8(mc.nsb), 256, 0, s>>>(mc.sbbase[k].p, mc.nsb, bb, dmap.p);
+    PASTA_LAUNCHED();
+    PASTA_CUDA(cudaStreamSynchronize(s));  // dmap and the host vectors are released at scope exit
+  }
+  PASTA_CUDA(cudaStreamSynchronize(s));
+  mc.tagged = mc.hs_total + mc.hot_total > 0;
+  if (getenv("PASTA_DEBUG"))
+    fprintf(stderr, "[pasta] hicoo hot blocks mode %u R %u: smem %llu rows, L2 %llu rows\n", mode, R,
+            (unsigned long long)mc.hs_total, (unsigned long long)mc.hot_total);
 }
 
 }  // namespace pasta

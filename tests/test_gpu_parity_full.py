@@ -101,3 +101,27 @@ def test_fullsize_hicoo_conversion_bit_exact(env, key):
     for k in ("bptr", "binds", "einds"):
         assert np.array_equal(hx[k], o[k]), k
     assert np.array_equal(hx["vals"].view(np.uint32), o["vals"].view(np.uint32))
+
+
+@pytest.mark.parametrize("hot_mb", ["0.05", "64"])
+def test_hicoo_hot_block_tiers_retag(env, hot_mb, monkeypatch):
+    """HiCOO hot-block tiers (R#34): shared-memory and L2 tiers forced on, ragged dims (partial
+    last blocks), and the rank changed on the same handle (R = 16 -> 32 -> 8 -> 16) so the
+    retagged slice bases are untagged and retagged between launches; every result against the
+    oracle.  hot_mb = 0.05 leaves most blocks cold (mixed tags inside a warp's window)."""
+    pasta, oracle, torch = env
+    monkeypatch.setenv("PASTA_HOT_FORCE", "1")
+    monkeypatch.setenv("PASTA_HOT_MB", hot_mb)
+    dims = (1000, 777, 1300)
+    inds, vals = si.powerlaw_coo(dims, 300_000, seed=77)
+    x = pasta.pasta_coo_from_arrays(dims, inds, vals)
+    h = pasta.pasta_coo_to_hicoo(x, 7)
+    gh = pasta.pasta_coo_to_ghicoo(x, 7, 0b101)  # mode 1 uncompressed: tiers on modes 0 and 2 only
+    for R in (16, 32, 8, 16):
+        U = si.factors(dims, R, seed=R)
+        Ud = [torch.from_numpy(u).cuda() for u in U]
+        for n in range(3):
+            ref, ab = oracle.mttkrp(dims, inds, vals, n, U)
+            for name, t in (("hicoo", h), ("ghicoo", gh)):
+                ex = _excess(pasta.pasta_mttkrp_hicoo(t, n, Ud), ref, ab)
+                assert ex.max() <= 0, f"{name} R={R} mode {n}: excess {ex.max():.3e}"
