@@ -368,6 +368,12 @@ void pasta_hicoo_free(pasta_hicoo *h);
 
 /* Number of kernels this library has launched in this process (all kinds). */
 uint64_t pasta_launch_count(void);
+/* The current device's SM -> die map used by the die-split COO MTTKRP (R#35; measured once
+ * per device and process, see csrc/die.cu): *nsms = number of SMs (0 when no plausible two-die
+ * map was found or PASTA_DIE_SPLIT=0), die_of_sm[s] (HOST buffer of >= *nsms entries, may be
+ * NULL) = 0 or 1 for SM id s, n_die[2] (may be NULL) = SMs per die.  Launches a calibration
+ * kernel on first use (synchronises the device). */
+pasta_status pasta_die_map(uint32_t *nsms, int8_t *die_of_sm, uint32_t *n_die);
 /* When enabled, every MTTKRP main-kernel launch is bracketed by CUDA events recorded on
  * its own stream.  pasta_profile_read synchronises those events and returns the summed
  * device time (ms) and the launch count of kernel family `which` (0 = COO MTTKRP,

@@ -23,7 +23,7 @@ __all__ = [
     "pasta_coo_row_counts",
     "pasta_row_partition", "pasta_coo_partition", "pasta_coo_shard", "pasta_coo_info",
     "pasta_coo_export", "pasta_coo_export_mode", "pasta_hicoo_info", "pasta_hicoo_export",
-    "pasta_launch_count", "pasta_profile_enable", "pasta_profile_read", "pasta_gram",
+    "pasta_launch_count", "pasta_die_map", "pasta_profile_enable", "pasta_profile_read", "pasta_gram",
     "pasta_cpals_solve", "pasta_normalize_columns", "pasta_weighted_inner", "pasta_coo_norm2",
     "pasta_cpals_coo", "pasta_coo_fibers", "pasta_coo_fiber_export", "pasta_ttm_coo",
     "pasta_ttv_coo", "pasta_coo_to_ghicoo", "pasta_ghicoo_auto_mask", "pasta_ghicoo_export",
@@ -437,6 +437,18 @@ def pasta_ghicoo_export(h: Hicoo) -> dict:
 # ----------------------------------------------------------------------------- measurement
 def pasta_launch_count() -> int:
     return int(lib().pasta_launch_count())
+
+
+def pasta_die_map():
+    """(die of every SM as an int8 array, SMs per die) of the current device, or (None, (0, 0))
+    when no two-die map was measured (the die-split COO MTTKRP is then off)."""
+    n = C.c_uint32()
+    die = (C.c_int8 * 1024)()
+    nd = (C.c_uint32 * 2)()
+    check(lib().pasta_die_map(C.byref(n), die, nd))
+    if n.value == 0:
+        return None, (0, 0)
+    return np.array(die[: n.value], np.int8), (nd[0], nd[1])
 
 
 def pasta_profile_enable(on: bool = True) -> None:

@@ -107,6 +107,7 @@ SIGNATURES = {
     "pasta_ttm_coo": (_st, [_vp, C.c_uint32, _vp, C.c_uint32, _vp, _vp]),
     "pasta_ttv_coo": (_st, [_vp, C.c_uint32, _vp, _vp, _vp]),
     "pasta_launch_count": (C.c_uint64, []),
+    "pasta_die_map": (_st, [_u32p, C.POINTER(C.c_int8), _u32p]),
     "pasta_profile_enable": (_st, [C.c_int]),
     "pasta_profile_read": (_st, [C.c_uint32, C.POINTER(C.c_double), _u64p, C.c_int]),
 }

@@ -1219,6 +1219,19 @@ void pasta_hicoo_free(pasta_hicoo *h) { delete h; }
 // ---------------------------------------------------------------------------- measurement
 uint64_t pasta_launch_count(void) { return g_launches.load(); }
 
+pasta_status pasta_die_map(uint32_t *nsms, int8_t *die_of_sm, uint32_t *n_die) {
+  API_BEGIN
+  require(nsms != nullptr, "nsms is NULL");
+  const DieMap &m = die_map();
+  *nsms = m.ok ? uint32_t(m.sms) : 0u;
+  if (m.ok && die_of_sm) memcpy(die_of_sm, m.die, size_t(m.sms));
+  if (n_die) {
+    n_die[0] = m.ok ? uint32_t(m.n[0]) : 0u;
+    n_die[1] = m.ok ? uint32_t(m.n[1]) : 0u;
+  }
+  API_END
+}
+
 pasta_status pasta_profile_enable(int on) {
   API_BEGIN
   g_prof_on.store(on != 0);

@@ -76,6 +76,31 @@ struct DevArray {
   size_t bytes() const { return n * sizeof(T); }
 };
 
+// SM -> die map of the current device (die.cu): measured once per device; ok = two
+// plausible groups found (else no die split is used).  d_die: device copy, die of %smid.
+constexpr int kMaxSms = 1024;
+struct DieMap {
+  bool ok = false;
+  int sms = 0;
+  int n[2] = {0, 0};
+  int8_t die[kMaxSms] = {};
+  int8_t *d_die = nullptr;
+};
+const DieMap &die_map();
+
+// Which half of factor k's rows a row belongs to in the die split (R#35): a fixed hash of
+// (row, k) compared with the die-0 share t (of 2^32).  Host (slot order of the L2 tier) and
+// device (nonzero classes) use the same function.
+__host__ __device__ inline uint32_t die_half(uint32_t row, uint32_t k, uint32_t t) {
+  uint32_t x = row * 0x9E3779B1u ^ (k * 0x85EBCA77u + 0x165667B1u);
+  x ^= x >> 16;
+  x *= 0x7FEB352Du;
+  x ^= x >> 15;
+  x *= 0x846CA68Bu;
+  x ^= x >> 16;
+  return x < t ? 0u : 1u;
+}
+
 // Completion of the last launch that used a handle's per-mode mutable state (the hot-row
 // buffer, refilled from the factors before every launch): a launch on another stream waits
 // for it, so same-handle MTTKRPs on two streams are ordered instead of racing on the buffer.
@@ -155,6 +180,18 @@ struct CooModeCopy {
   uint64_t hot_base[kMaxOrder] = {}, hot_cnt[kMaxOrder] = {}, hot_total = 0;
   DevArray<float> hot_buf;              // hot_total x R, refilled from the factors every launch
   LaunchFence fence;                    // last launch that read hot_buf
+  // Die split (R#35, order 3 with an L2 tier): each gathered factor's rows are split into two
+  // halves (die_half); nonzeros are reordered into 4 row-sorted segments by (half of the first
+  // gathered row, half of the second): die 0 walks [0, split_x) = (0,0) then (0,1), die 1 walks
+  // [split_x, nnz) = (1,1) then (1,0), so at any time the two dies gather disjoint halves of
+  // both factors and each die's L2 holds only its half of the hot rows.  The L2-tier slots of
+  // each factor are ordered half 0 first.  split_irow / split_val / hot_inds hold that order.
+  bool split = false;
+  uint64_t split_x = 0;
+  uint32_t split_t[2] = {};             // die-0 shares of the two gathered factors (of 2^32)
+  DevArray<uint32_t> split_irow;
+  DevArray<float> split_val;
+  DevArray<unsigned long long> claim;   // per-die chunk counters, zeroed before each launch
 };
 
 constexpr int kCountBuckets = 256;  // 8 sub-buckets per octave of a row's nonzero count
@@ -326,7 +363,7 @@ void launch_inner(const float *A, const float *B, uint64_t rows, uint32_t R, con
                   double *out, cudaStream_t s);
 void launch_sumsq(const float *v, uint64_t n, double *out, cudaStream_t s);
 void coo_mark_hot(pasta_coo *x, uint32_t mode, uint32_t R, bool global_tier, uint32_t smem_rows,
-                  cudaStream_t s);
+                  cudaStream_t s, bool die_split = false);
 void coo_build_fibers(pasta_coo *x, uint32_t mode, cudaStream_t s);
 // TTV on the fiberised matrix (warp-level segmented reduction); y zeroed by the caller
 void launch_ttv(const pasta_coo &mat, const float *v, float *y, cudaStream_t s);

@@ -77,6 +77,13 @@ struct KArgs {
   // HiCOO row slices decoded into the staged kernel (WA 9): run_sb[r] = slice holding entry
   // r * (chunk / G), the first entry of group run r
   const uint64_t *run_sb;
+  // die split (R#35, HS kernels): die 0's CTAs take the chunks of [0, split_x), die 1's those
+  // of [split_x, nnz), claimed dynamically (claim[die], zeroed per launch); every segment
+  // flush is an atomic (a row appears in up to four segments)
+  uint32_t split;
+  uint64_t split_x;
+  unsigned long long *claim;
+  const int8_t *die_of;
 };
 
 // Per-thread L2 cache policies (createpolicy, sm_80+): the nonzero stream is touched once
@@ -735,7 +742,18 @@ __global__ void __launch_bounds__(HS ? WPC_ * 32 : kThreads, HS ? 1 : (WA == 6 ?
     }
     __syncthreads();
   }
-  const uint64_t nchunks = (a.nnz + a.chunk - 1) / a.chunk;
+  // the nonzero range this CTA works on: all of them, or its die's half (die split)
+  uint64_t xbeg = 0, xend = a.nnz;
+  int die = 0;
+  const bool dyn = HS && !kHic && a.split;
+  if (dyn) {
+    uint32_t sm;
+    asm volatile("mov.u32 %0, %%smid;" : "=r"(sm));
+    die = a.die_of[sm];
+    xbeg = die ? a.split_x : 0;
+    xend = die ? a.nnz : a.split_x;
+  }
+  const uint64_t nchunks = (xend - xbeg + a.chunk - 1) / a.chunk;
   const uint64_t wstep = HS ? uint64_t(gridDim.x) * WPC : nchunks;
   const uint64_t run = a.chunk / G;  // multiple of SG
   const int nstages = int(run / SG);
@@ -753,11 +771,11 @@ __global__ void __launch_bounds__(HS ? WPC_ * 32 : kThreads, HS ? 1 : (WA == 6 ?
   // issue the cp.async copies of stage s of the chunk starting at cc into dst (one commit
   // group; an empty group when cc is past the end, so that wait_group counts stay uniform)
   auto issue_to = [&](uint64_t cc, int s, uint32_t *dst) {
-    if (cc < a.nnz) {
+    if (cc < xend) {
       for (int i = lane; i < SW / 4; i += 32) {  // 16-B chunks of one array
         const int gi = i / (SG / 4), k = i % (SG / 4);
         const uint64_t pos = cc + uint64_t(gi) * run + uint64_t(s) * SG + uint64_t(k) * 4;
-        const int valid = pos >= a.nnz ? 0 : (a.nnz - pos >= 4 ? 16 : int(a.nnz - pos) * 4);
+        const int valid = pos >= xend ? 0 : (xend - pos >= 4 ? 16 : int(xend - pos) * 4);
 #pragma unroll
         for (int arr = 0; arr < NA; ++arr) {
           // 16-B chunk k of group gi lands at chunk k ^ ((gi / GL) % CG) of the group's region:
@@ -841,13 +859,25 @@ __global__ void __launch_bounds__(HS ? WPC_ * 32 : kThreads, HS ? 1 : (WA == 6 ?
 
   // The stream is pipelined across the warp's chunks: the last stage of a chunk prefetches
   // stage 0 of the next one, so a persistent warp never waits on a cold pipeline.
+  // Chunk schedule: static round robin, or (die split) chunks of the die's range claimed with
+  // one atomic per chunk -- the CTA -> SM placement is not known in advance, so a static
+  // split by die rank could skip or repeat chunks.  The claim of the chunk after next is
+  // issued at the start of a chunk and consumed at its end (its latency hides behind it).
+  auto claim_issue = [&]() -> unsigned long long {
+    unsigned long long v = 0;
+    if (lane == 0) v = atomicAdd(a.claim + die, 1ull);
+    return v;
+  };
+  auto claim_get = [&](unsigned long long v) { return uint64_t(__shfl_sync(0xFFFFFFFFu, v, 0)); };
   int bsel = 0;
-  uint64_t w = uint64_t(blockIdx.x) * WPC + warp;
-  if (w < nchunks) issue(w * a.chunk, 0, 0);
-  for (; w < nchunks; w += wstep) {
-  const uint64_t c0 = w * a.chunk;
+  uint64_t w = dyn ? claim_get(claim_issue()) : uint64_t(blockIdx.x) * WPC + warp;
+  uint64_t wn = dyn ? (w < nchunks ? claim_get(claim_issue()) : nchunks) : w + wstep;
+  if (w < nchunks) issue(xbeg + w * a.chunk, 0, 0);
+  while (w < nchunks) {
+  const unsigned long long wnn_v = (dyn && wn < nchunks) ? claim_issue() : 0ull;
+  const uint64_t c0 = xbeg + w * a.chunk;
   const uint64_t x0 = c0 + uint64_t(g) * run;
-  const uint64_t x1 = (x0 + run < a.nnz) ? x0 + run : a.nnz;
+  const uint64_t x1 = (x0 + run < xend) ? x0 + run : xend;
   Vec<4> acc;
 #pragma unroll
   for (int i = 0; i < 4; ++i) acc.v[i] = 0.f;
@@ -856,7 +886,7 @@ __global__ void __launch_bounds__(HS ? WPC_ * 32 : kThreads, HS ? 1 : (WA == 6 ?
   const bool active = x0 < x1 && col < R;
   for (int s = 0; s < nstages; ++s) {
     if (s + 1 < nstages) issue(c0, s + 1, bsel ^ 1);
-    else issue(w + wstep < nchunks ? (w + wstep) * a.chunk : a.nnz, 0, bsel ^ 1);
+    else issue(wn < nchunks ? xbeg + wn * a.chunk : xend, 0, bsel ^ 1);
     asm volatile("cp.async.wait_group 1;" ::: "memory");
     __syncwarp();
     const uint32_t *buf = wbuf + bsel * NA * SW + g * SG;
@@ -939,7 +969,7 @@ __global__ void __launch_bounds__(HS ? WPC_ * 32 : kThreads, HS ? 1 : (WA == 6 ?
               if (cur != 0xFFFFFFFFu) {
                 float *dst = a.out + uint64_t(cur) * R + col;
                 if (kWrite) {
-                  if (first) red_vec<4>(dst, acc, pol.out); else st_vec<4>(dst, acc, pol.out);
+                  if (first || dyn) red_vec<4>(dst, acc, pol.out); else st_vec<4>(dst, acc, pol.out);
                 } else if (acc.v[0] == 1.2345e-30f) {
                   st_vec<4>(dst, acc, pol.out);  // keeps the arithmetic live in probes
                 }
@@ -957,6 +987,8 @@ __global__ void __launch_bounds__(HS ? WPC_ * 32 : kThreads, HS ? 1 : (WA == 6 ?
   }
   if (active && cur != 0xFFFFFFFFu && (kWrite || acc.v[0] == 1.2345e-30f))
     red_vec<4>(a.out + uint64_t(cur) * R + col, acc, pol.out);
+  w = wn;
+  wn = dyn ? (w < nchunks ? claim_get(wnn_v) : nchunks) : w + wstep;
   }  // chunk loop
 }
 
@@ -1170,8 +1202,12 @@ void launch_coo_mttkrp(const pasta_coo *x, uint32_t mode, const float *const *fa
     if (want_hot) hs_rows_budget = std::min(hs_rows_budget, 512u);
     if (const int cap = env_int("PASTA_HOT_SMEM_ROWS", 0)) hs_rows_budget = std::min(hs_rows_budget, uint32_t(cap));
     bool hs = env_int("PASTA_HOT_SMEM", 1) != 0 && hs_rows_budget >= 64;
+    // die split (R#35): order 3 with DRAM-bound gathers (an L2 tier), persistent kernel only
+    const bool split_want = env_int("PASTA_DIE_SPLIT", 1) != 0 && no == 2 && want_hot;
     if (hs) {
-      coo_mark_hot(const_cast<pasta_coo *>(x), mode, R, want_hot, hs_rows_budget, s);
+      // the nonzero order changes with the die split: wait for launches still reading the copy
+      const_cast<CooModeCopy &>(mc).fence.wait(s);
+      coo_mark_hot(const_cast<pasta_coo *>(x), mode, R, want_hot, hs_rows_budget, s, split_want);
       if (mc.hot_R != R || mc.hs_total == 0) hs = false;
     }
     if (!hs && want_hot) coo_mark_hot(const_cast<pasta_coo *>(x), mode, R, true, 0, s);
@@ -1189,6 +1225,15 @@ void launch_coo_mttkrp(const pasta_coo *x, uint32_t mode, const float *const *fa
       // hot_buf is shared by every launch on this handle and mode: wait for the previous one
       const_cast<CooModeCopy &>(mc).fence.wait(s);
       if (mc.hot_total) launch_hot_fill(mc, factors, x->order, mode, R, s);
+      if (hs && mc.split) {
+        a.irow = mc.split_irow.p;
+        a.val = mc.split_val.p;
+        a.split = 1;
+        a.split_x = mc.split_x;
+        a.claim = mc.claim.p;
+        a.die_of = die_map().d_die;
+        PASTA_CUDA(cudaMemsetAsync(mc.claim.p, 0, 2 * sizeof(unsigned long long), s));
+      }
     }
     // run per group: short runs on DRAM-bound gathers, longer ones on L2-resident factors
     // (fewer boundary atomics); measured on H (64: 1.82, 128: 1.87 ms per mode), C2 (128 and
@@ -1376,7 +1421,11 @@ void launch_hicoo_mttkrp(const pasta_hicoo *h, uint32_t mode, const float *const
     // the gathers go to DRAM); PASTA_HICOO_HOT=0 disables both
     const size_t stage = size_t(16) * 2 * (hno + 2) * (G * 32) * sizeof(uint32_t);
     bool tiers = false;
-    if (env_int("PASTA_HICOO_HOT", 1) && env_int("PASTA_HOT_SMEM", 1)) {
+    // every launch on this copy reads sbbase: a retag waits for the previous launch
+    mcw.fence.wait(s);
+    if (!(env_int("PASTA_HICOO_HOT", 1) && env_int("PASTA_HOT_SMEM", 1))) {
+      if (mc.tagged) hicoo_mark_hot(const_cast<pasta_hicoo *>(h), mode, R, false, 0, s);  // untag
+    } else {
       static int l2 = 0;
       if (!l2) {
         int dev = 0;
@@ -1402,7 +1451,6 @@ void launch_hicoo_mttkrp(const pasta_hicoo *h, uint32_t mode, const float *const
       for (uint32_t k = 0; k < h->order; ++k)
         if (k != mode) a.hs_lo[jj++] = uint32_t(mc.hs_base[k]);
       a.hs_lo[jj] = uint32_t(mc.hs_total);
-      mcw.fence.wait(s);
       if (mc.hot_total) launch_hot_fill(mc, factors, h->order, mode, R, s);
     }
     ProfScope prof(kProfHicoo, s);
@@ -1414,7 +1462,7 @@ void launch_hicoo_mttkrp(const pasta_hicoo *h, uint32_t mode, const float *const
       PASTA_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem)));
       kern<<<unsigned(nblk), 512, smem, s>>>(a);
       PASTA_LAUNCHED();
-      if (tiers) mcw.fence.record(s);
+      mcw.fence.record(s);
     };
     if (tiers)
       with_no_lpn<3>(hno, lpn, [&](auto NOt, auto Lt) { go(coo_staged_kernel<NOt.value, Lt.value, 10, true, 16, 32, 4>); });
@@ -1425,6 +1473,12 @@ void launch_hicoo_mttkrp(const pasta_hicoo *h, uint32_t mode, const float *const
     return;
   }
   if (mc.layout == 0) {
+    // the generic row-slice kernel reads plain block bases: undo any hot-block tagging
+    HicooModeCopy &mcw = const_cast<HicooModeCopy &>(mc);
+    if (mc.tagged) {
+      mcw.fence.wait(s);
+      hicoo_mark_hot(const_cast<pasta_hicoo *>(h), mode, R, false, 0, s);
+    }
     KArgs a{};
     a.nnz = h->nnz;
     a.order = h->order;

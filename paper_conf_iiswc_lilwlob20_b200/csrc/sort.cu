@@ -334,6 +334,20 @@ __global__ void hot_fill_kernel(const float4 *__restrict__ U, const uint32_t *__
   }
 }
 
+// die-split segment of each nonzero (R#35); n01 counts the die-0 segments (half of ia == 0)
+__global__ void split_seg_kernel(const uint32_t *__restrict__ ia, const uint32_t *__restrict__ ib, uint64_t M,
+                                 uint32_t ka, uint32_t kb, uint32_t ta, uint32_t tb, uint32_t *__restrict__ seg,
+                                 unsigned long long *__restrict__ n01) {
+  unsigned long long c = 0;
+  for (uint64_t x = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; x < M; x += uint64_t(gridDim.x) * blockDim.x) {
+    const uint32_t ha = die_half(ia[x], ka, ta), hb = die_half(ib[x], kb, tb);
+    seg[x] = ha ? (hb ? 2u : 3u) : (hb ? 1u : 0u);
+    c += ha == 0;
+  }
+  for (int o = 16; o; o >>= 1) c += __shfl_xor_sync(0xFFFFFFFFu, c, o);
+  if ((threadIdx.x & 31) == 0 && c) atomicAdd(n01, c);
+}
+
 unsigned grid8(uint64_t n) {
   uint64_t b = (n + 256 * 8 - 1) / (256 * 8);
   if (b < 1) b = 1;
@@ -359,13 +373,31 @@ unsigned grid8(uint64_t n) {
 // gathered factors, factor k at [hs_base[k], +hs_cnt[k])), 0x80000000 | L2-tier slot, or the
 // plain row.  Needs dims < 2^30.
 void coo_mark_hot(pasta_coo *x, uint32_t mode, uint32_t R, bool global_tier, uint32_t smem_rows,
-                  cudaStream_t s) {
+                  cudaStream_t s, bool die_split) {
   CooModeCopy &mc = x->mc[mode];
-  if (mc.hot_R == R && mc.hot_global == global_tier && mc.hot_smem_budget == smem_rows) return;
+  if (mc.hot_R == R && mc.hot_global == global_tier && mc.hot_smem_budget == smem_rows &&
+      mc.split == die_split)
+    return;
+  // die split (R#35): two gathered factors, an L2 tier and a measured SM -> die map
+  const DieMap &dm = die_map();
+  die_split = die_split && global_tier && x->order == 3 && dm.ok;
+  mc.split = false;
   const char *env = getenv("PASTA_HOT_MB");
-  const double hot_mb = global_tier ? ((env && *env) ? atof(env) : 64.0) : 0.0;
+  // the die split holds half of each factor's tier per die, so the tier can be larger
+  const double hot_mb = global_tier ? ((env && *env) ? atof(env) : (die_split ? 96.0 : 64.0)) : 0.0;
   const uint32_t N = x->order;
   const uint64_t M = x->nnz;
+  // die-0 shares: the first gathered factor in proportion to the dies' SM counts, the second
+  // half and half, so both phases of both dies get work in proportion to their SMs
+  uint32_t tsplit[kMaxOrder] = {};
+  if (die_split) {
+    int j = 0;
+    for (uint32_t k = 0; k < N; ++k) {
+      if (k == mode) continue;
+      tsplit[k] = j == 0 ? uint32_t(4294967296.0 * dm.n[0] / double(dm.n[0] + dm.n[1])) : 0x80000000u;
+      ++j;
+    }
+  }
   mc.hot_R = 0;
   for (uint32_t k = 0; k < N; ++k)
     if (x->dims[k] >= 0x40000000u) return;
@@ -423,6 +455,16 @@ void coo_mark_hot(pasta_coo *x, uint32_t mode, uint32_t R, bool global_tier, uin
       PASTA_LAUNCHED();
       mc.hot_cnt[k] = select_flagged(flag.p, x->dims[k], lists[k], s);
       total += mc.hot_cnt[k];
+      if (die_split && mc.hot_cnt[k]) {  // L2-tier slots: this factor's half-0 rows first
+        std::vector<uint32_t> hl(mc.hot_cnt[k]), part;
+        part.reserve(hl.size());
+        PASTA_CUDA(cudaMemcpyAsync(hl.data(), lists[k].p, hl.size() * 4, cudaMemcpyDeviceToHost, s));
+        PASTA_CUDA(cudaStreamSynchronize(s));
+        for (uint32_t r : hl) if (die_half(r, k, tsplit[k]) == 0) part.push_back(r);
+        for (uint32_t r : hl) if (die_half(r, k, tsplit[k]) == 1) part.push_back(r);
+        PASTA_CUDA(cudaMemcpyAsync(lists[k].p, part.data(), part.size() * 4, cudaMemcpyHostToDevice, s));
+        PASTA_CUDA(cudaStreamSynchronize(s));
+      }
     }
   }
   mc.hot_total = total;
@@ -448,6 +490,45 @@ void coo_mark_hot(pasta_coo *x, uint32_t mode, uint32_t R, bool global_tier, uin
     mark_hot_kernel<<<grid8(M), 256, 0, s>>>(mc.inds[k], slot_of.p, M, mc.hot_inds[k].p);
     PASTA_LAUNCHED();
     PASTA_CUDA(cudaStreamSynchronize(s));  // slot_of is released at scope exit
+  }
+  if (die_split) {
+    // nonzero segments (R#35): 0 = (0,0), 1 = (0,1) [die 0], 2 = (1,1), 3 = (1,0) [die 1]
+    uint32_t ka = 0, kb = 0, j = 0;
+    for (uint32_t k = 0; k < N; ++k) {
+      if (k == mode) continue;
+      (j++ == 0 ? ka : kb) = k;
+    }
+    DevArray<uint32_t> seg(M, s), perm(M, s);
+    DevArray<unsigned long long> n01(1, s);
+    PASTA_CUDA(cudaMemsetAsync(n01.p, 0, sizeof(unsigned long long), s));
+    split_seg_kernel<<<grid8(M), 256, 0, s>>>(mc.inds[ka], mc.inds[kb], M, ka, kb, tsplit[ka], tsplit[kb], seg.p,
+                                              n01.p);
+    PASTA_LAUNCHED();
+    iota_u32(perm.p, M, s);
+    const uint32_t *comps[1] = {seg.p};
+    const uint32_t bits[1] = {2};
+    lexsort(comps, bits, 1, perm, M, s);  // stable: rows stay sorted inside each segment
+    seg.reset();
+    mc.split_irow.alloc(M, s);
+    mc.split_val.alloc(M, s);
+    gather_u32(mc.inds[mode], perm.p, mc.split_irow.p, M, s);
+    gather_f32(mc.val, perm.p, mc.split_val.p, M, s);
+    DevArray<uint32_t> tmp(M, s);
+    for (uint32_t k : {ka, kb}) {
+      gather_u32(mc.hot_inds[k].p, perm.p, tmp.p, M, s);
+      std::swap(mc.hot_inds[k], tmp);
+    }
+    unsigned long long h01 = 0;
+    PASTA_CUDA(cudaMemcpyAsync(&h01, n01.p, sizeof(h01), cudaMemcpyDeviceToHost, s));
+    PASTA_CUDA(cudaStreamSynchronize(s));
+    mc.split_x = h01;
+    mc.split_t[0] = tsplit[ka];
+    mc.split_t[1] = tsplit[kb];
+    mc.claim.alloc(2, s);
+    mc.split = true;
+  } else {
+    mc.split_irow.reset();
+    mc.split_val.reset();
   }
   mc.hot_bucket = hb;
   mc.hs_bucket = hsb;

@@ -491,3 +491,34 @@ def test_hicoo_row_slices_staged_decode(env, staged, monkeypatch):
             ref, ab = oracle.mttkrp(dims, inds, vals, n, U)
             _check(pasta.pasta_mttkrp_hicoo(h, n, Ud), ref, ab,
                    f"hicoo staged={staged} {dims} R={R} mask={mask} mode {n}")
+
+
+@pytest.mark.parametrize("split", ["1", "0"])
+def test_coo_die_split(env, split, monkeypatch):
+    """Die-split COO MTTKRP (R#35): with the L2 tier forced on, order-3 nonzeros are reordered
+    into four row-sorted segments by the die halves of their two gathered rows and the
+    persistent kernel's CTAs claim chunks of their die's range; every flush is an atomic.
+    Checked against the oracle for both settings on the same handle (the ranking is redone
+    when the split changes), with a 1M-nonzero hot row crossing all four segments."""
+    pasta, oracle, torch = env
+    die, nd = pasta.pasta_die_map()
+    assert die is not None and min(nd) >= 148 // 3, nd  # a plausible two-die B200 split
+    assert np.count_nonzero(die == 0) == nd[0] and np.count_nonzero(die == 1) == nd[1]
+    monkeypatch.setenv("PASTA_HOT_FORCE", "1")
+    monkeypatch.setenv("PASTA_HOT_MB", "0.5")
+    monkeypatch.setenv("PASTA_DIE_SPLIT", split)
+    for dims, nnz, R in [((3000, 2000, 4000), 2_000_003, 16), ((4000, 900, 2500), 0, 32)]:
+        if nnz:
+            inds, vals = si.powerlaw_coo(dims, nnz, seed=nnz + R)
+        else:
+            inds, vals = si.hot_row_coo(dims, 1_000_000, 200_000, seed=8, mode=0, hot_row=17)
+        U = si.factors(dims, R, seed=R)
+        Ud = _dev(torch, U)
+        x = pasta.pasta_coo_from_arrays(dims, inds, vals)
+        for n in range(3):
+            ref, ab = oracle.mttkrp(dims, inds, vals, n, U)
+            _check(pasta.pasta_mttkrp_coo(x, n, Ud), ref, ab, f"die split {split} {dims} R={R} mode {n}")
+        monkeypatch.setenv("PASTA_DIE_SPLIT", "1" if split == "0" else "0")  # flip on the same handle
+        ref, ab = oracle.mttkrp(dims, inds, vals, 2, U)
+        _check(pasta.pasta_mttkrp_coo(x, 2, Ud), ref, ab, f"die split flipped {dims} R={R}")
+        monkeypatch.setenv("PASTA_DIE_SPLIT", split)
