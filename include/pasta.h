@@ -70,12 +70,17 @@ pasta_status pasta_set_allocator(const pasta_allocator *alloc);
  * whitespace-separated 1-based indices followed by the value; '#' lines are comments.
  * The order is the token count of the first data line minus one; dims are the per-mode
  * maximum index.  Repeated coordinates are kept as separate nonzeros (MTTKRP is linear in
- * them, R#15).  Errors: EIO (open/read), EFORMAT (ragged line, index 0, bad number),
- * ERANGE (index > 2^32-1 or > 2^32-1 nonzeros). */
+ * them, R#15).  A file that starts with the 8 bytes "PASTAB01" is read as the binary cache
+ * instead (.pbin, written by pasta_save_coo): little-endian u32 order, u32 0, u64 nnz,
+ * u32 dims[order], then the 0-based u32 indices of mode 0, 1, ..., order-1 (nnz each) and
+ * the nnz f32 values; its dims are the stored ones, and its size must match the header.
+ * Errors: EIO (open/read), EFORMAT (ragged line, index 0, bad number; bad .pbin header or
+ * size), ERANGE (index > 2^32-1, index >= a stored dim, or > 2^32-2 nonzeros). */
 pasta_status pasta_load_coo(const char *path, pasta_coo **out);
 
-/* Write `x` (canonical order) as a 1-based text file readable by pasta_load_coo.
- * Values are printed with 9 significant digits (exact fp32 round trip).  EIO on failure. */
+/* Write `x` (canonical order): as the binary cache when `path` ends in ".pbin" (format
+ * above; bit-exact round trip including dims), else as a 1-based text file readable by
+ * pasta_load_coo (values with 9 significant digits: exact fp32 round trip).  EIO on failure. */
 pasta_status pasta_save_coo(const pasta_coo *x, const char *path);
 
 /* Create a COO tensor from HOST arrays (copied; the caller keeps ownership).
@@ -92,7 +97,8 @@ typedef struct {
     const double *initiator;  /* 2^order non-negative cell weights, cell c sets bit k of mode
                                  k's index to (c >> k) & 1; NULL -> product form from q     */
     double q;                 /* product-form P(bit = 0) per mode per level; 0 -> 0.75      */
-    uint32_t permute;         /* must be 0 (random relabelling: EUNSUPPORTED)                */
+    uint32_t permute;         /* 1: relabel every mode by pi_k after the draws (R#22), see  */
+                              /* below; 0 keeps the generator's fractal locality (default)  */
     float val_lo, val_hi;     /* values uniform in [val_lo, val_hi); both 0 -> [-1, 1)       */
     double alpha;             /* kind 2: power-law exponent in (0, 8]; 0 -> 1.0              */
 } pasta_gen_params;
@@ -114,8 +120,14 @@ typedef struct {
  * i_k = the first i with u < cum_i, else I_k - 1.  No draw is stripped; the tensor is the
  * first `nnz` distinct coordinates in draw order with the values of kind 1, lexicographic.
  * dims <= 2^27 per mode (ERANGE otherwise).
- * Errors: EINVAL (order, dims, nnz > prod dims, bad initiator, alpha), ERANGE (more than
- * 2^32-2 draws would be needed), EUNSUPPORTED (permute). */
+ * permute = 1 (R#22): afterwards mode k's indices are relabelled by the bijection pi_k of
+ * [0, I_k): with L = ceil(log2 I_k), m = 2^L - 1, K = mix64(seed ^ 0xA0761D6478BD642F ^ k),
+ * f(v) = three rounds r = 0, 1, 2 of { v = v * (((K >> 16r) & 0xFFFF) | 1) & m;
+ * v ^= v >> ceil(L/2) (L >= 2); v = (v + ((K >> (32 + 8r)) & 0xFFFFFF)) & m } and
+ * pi_k(v) = the first f^j(v), j >= 1, below I_k (cycle walking); the nonzeros are then
+ * re-sorted lexicographically (values travel with their coordinates).
+ * Errors: EINVAL (order, dims, nnz > prod dims, bad initiator, alpha, permute > 1), ERANGE
+ * (more than 2^32-2 draws would be needed). */
 pasta_status pasta_gen_powerlaw(uint32_t order, const uint32_t *dims, uint64_t nnz,
                                 uint64_t seed, const pasta_gen_params *params,
                                 pasta_coo **out);
@@ -247,6 +259,13 @@ pasta_status pasta_cpals_solve(const float *M, uint64_t rows, uint32_t R, const 
  * The normalised factor is then U_n = M Wn (pasta_rows_times): the solve, the column
  * normalisation and the gram of the factor without the two extra passes over U_n.  DEVICE
  * pointers; R <= 64 (EUNSUPPORTED otherwise). */
+/* CP-ALS fit (P:93 via Kolda-Bader, one CTA, fp64): ||Xhat||^2 = lambda^T (Hadamard of the
+ * `ngrams` R x R grams, every mode's) lambda, resid^2 = normx2 + ||Xhat||^2 - 2 inner[0],
+ * *fit (HOST) = 1 - sqrt(max(resid^2, 0)) / sqrt(normx2) (0 when normx2 = 0).  grams, lambda
+ * (R doubles) and inner (<X, Xhat>, 1 double, e.g. all-reduced pasta_weighted_inner) are
+ * DEVICE pointers; synchronises `stream`.  R <= 64. */
+pasta_status pasta_cpals_fit(const double *const *grams, uint32_t ngrams, uint32_t R, const double *lambda,
+                             const double *inner, double normx2, double *fit, void *stream);
 pasta_status pasta_cpals_prepare(const double *GM, const double *const *grams, uint32_t ngrams,
                                  uint32_t R, float *Wn, double *Gn, double *lambda, void *stream);
 /* U = M Wn: rows x R (row-major, fp32) times R x R (fp32).  DEVICE pointers; R <= 64. */

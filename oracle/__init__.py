@@ -86,6 +86,10 @@ def _L():
         lib.oracle_ttm.restype = C.c_int64
         lib.oracle_ttm.argtypes = [C.c_uint32, _u32p, C.c_uint64, C.POINTER(_u32p), _f32p, C.c_uint32,
                                    _f32p, C.c_uint32, C.POINTER(_u32p), _f64p, _f64p]
+        lib.oracle_relabel.restype = C.c_int
+        lib.oracle_relabel.argtypes = [C.c_uint32, _u32p, C.c_uint64, C.c_uint64, C.POINTER(_u32p)]
+        lib.oracle_relabel_index.restype = C.c_uint32
+        lib.oracle_relabel_index.argtypes = [C.c_uint32, C.c_uint32, C.c_uint64, C.c_uint32]
         lib.oracle_gen_powerlaw.restype = C.c_int
         lib.oracle_gen_powerlaw.argtypes = [C.c_uint32, _u32p, C.c_uint64, C.c_uint64, _f64p,
                                             C.c_double, C.c_float, C.c_float, C.POINTER(_u32p),
@@ -284,9 +288,28 @@ def mttkrp_ghicoo(dims, g, mode, factors, R=None):
     return Mref, Aref
 
 
-def gen_powerlaw(dims, nnz, seed, initiator=None, q=0.75, val_lo=-1.0, val_hi=1.0):
+def relabel_index(v, dim, seed, k):
+    """pi_k(v): the label permutation of mode k (R#22, oracle.c)."""
+    return int(_L().oracle_relabel_index(int(v), int(dim), int(seed), int(k)))
+
+
+def relabel(dims, inds, vals, seed):
+    """permute = 1 (R#22): every mode relabelled by pi_k, then the nonzeros re-sorted
+    lexicographically (numpy lexsort; coordinates stay distinct, so the order is unique)."""
+    dims = np.ascontiguousarray(dims, dtype=np.uint32)
+    out = np.ascontiguousarray(inds, dtype=np.uint32).copy()
+    rows = [out[k] for k in range(out.shape[0])]
+    rc = _L().oracle_relabel(out.shape[0], _ptr(dims, _u32p), out.shape[1], seed, _ptr_list(rows, _u32p))
+    if rc != 0:
+        raise ValueError("oracle_relabel failed")
+    order = np.lexsort(out[::-1])
+    return np.ascontiguousarray(out[:, order]), np.ascontiguousarray(vals[order])
+
+
+def gen_powerlaw(dims, nnz, seed, initiator=None, q=0.75, val_lo=-1.0, val_hi=1.0, permute=False):
     """Stochastic Kronecker generator (R#19-R#23), counter-based.
-    Returns (inds u32[N][M] lexicographically sorted, vals f32[M])."""
+    Returns (inds u32[N][M] lexicographically sorted, vals f32[M]).  permute: the labels of
+    every mode relabelled by pi_k after the draws (R#22), then re-sorted."""
     dims = np.ascontiguousarray(dims, dtype=np.uint32)
     order = dims.shape[0]
     outs = [np.zeros(max(nnz, 1), np.uint32) for _ in range(order)]
@@ -300,7 +323,10 @@ def gen_powerlaw(dims, nnz, seed, initiator=None, q=0.75, val_lo=-1.0, val_hi=1.
                                   _ptr_list(outs, _u32p), _ptr(ov, _f32p))
     if rc != 0:
         raise ValueError(f"oracle_gen_powerlaw failed rc={rc}")
-    return np.stack([o[:nnz] for o in outs]), ov[:nnz].copy()
+    inds, vals = np.stack([o[:nnz] for o in outs]), ov[:nnz].copy()
+    if permute:
+        return relabel(dims, inds, vals, seed)
+    return inds, vals
 
 
 def gen_slice_powerlaw(dims, nnz, seed, alpha=1.0, val_lo=-1.0, val_hi=1.0):

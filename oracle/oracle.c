@@ -713,3 +713,45 @@ int64_t oracle_tew_merge(uint32_t order, uint64_t Mx, const uint32_t *const *ix,
     free(r);
     return nz;
 }
+
+/* ------------------------------------------------------------------------------ */
+/* Label permutation of the synthetic generators (R#22, permute = 1): mode k's      */
+/* indices are relabelled by a bijection pi_k of [0, I_k) derived from the seed:     */
+/*   L = ceil(log2 I_k), m = 2^L - 1, K = mix64(seed ^ 0xA0761D6478BD642F ^ k);      */
+/*   f(v): three rounds r of  v = (v * (((K >> 16r) & 0xFFFF) | 1)) & m;              */
+/*                            v ^= v >> ceil(L / 2)  (L >= 2);                         */
+/*                            v = (v + ((K >> (32 + 8r)) & 0xFFFFFF)) & m;           */
+/*   pi_k(v) = first f^j(v), j >= 1, below I_k (cycle walking: a bijection of [0, I_k) */
+/*   because f permutes [0, 2^L)).  Each step is written out below.                   */
+/* ------------------------------------------------------------------------------ */
+static uint64_t relabel_round(uint64_t v, uint64_t key, uint32_t L, uint64_t m)
+{
+    for (int r = 0; r < 3; ++r) {
+        uint64_t mul = ((key >> (16 * r)) & 0xFFFFull) | 1ull;  /* odd: a bijection mod 2^L */
+        v = (v * mul) & m;
+        if (L >= 2) v ^= v >> ((L + 1) / 2);                    /* xor-shift: a bijection */
+        uint64_t add = (key >> (32 + 8 * r)) & 0xFFFFFFull;
+        v = (v + add) & m;                                       /* translation mod 2^L */
+    }
+    return v;
+}
+
+uint32_t oracle_relabel_index(uint32_t v, uint32_t dim, uint64_t seed, uint32_t k)
+{
+    uint32_t L = 0;
+    while (L < 32 && (1ull << L) < (uint64_t)dim) ++L;
+    uint64_t m = (L >= 64) ? ~0ull : ((1ull << L) - 1ull);
+    uint64_t key = mix64(seed ^ 0xA0761D6478BD642Full ^ (uint64_t)k);
+    uint64_t y = v;
+    do { y = relabel_round(y, key, L, m); } while (y >= dim);
+    return (uint32_t)y;
+}
+
+/* in place: inds[k][x] = pi_k(inds[k][x]) for every mode and nonzero */
+int oracle_relabel(uint32_t order, const uint32_t *dims, uint64_t nnz, uint64_t seed, uint32_t *const *inds)
+{
+    if (order < 1 || order > ORACLE_MAX_ORDER) return -1;
+    for (uint32_t k = 0; k < order; ++k)
+        for (uint64_t x = 0; x < nnz; ++x) inds[k][x] = oracle_relabel_index(inds[k][x], dims[k], seed, k);
+    return 0;
+}

@@ -27,7 +27,7 @@ __all__ = [
     "pasta_cpals_solve", "pasta_normalize_columns", "pasta_weighted_inner", "pasta_coo_norm2",
     "pasta_cpals_coo", "pasta_coo_fibers", "pasta_coo_fiber_export", "pasta_ttm_coo",
     "pasta_ttv_coo", "pasta_coo_to_ghicoo", "pasta_ghicoo_auto_mask", "pasta_ghicoo_export",
-    "pasta_cpals_prepare", "pasta_rows_times", "pasta_rows_times_bcast", "pasta_bcast_f32", "pasta_dev_alloc",
+    "pasta_cpals_prepare", "pasta_cpals_fit", "pasta_rows_times", "pasta_rows_times_bcast", "pasta_bcast_f32", "pasta_dev_alloc",
     "pasta_dev_free", "pasta_ipc_get_handle", "pasta_ipc_open", "pasta_ipc_close", "pasta_ts", "pasta_tew", "pasta_coo_values_ptr", "pasta_coo_ts", "pasta_coo_tew", "OPS",
 ]
 
@@ -508,6 +508,16 @@ def pasta_cpals_prepare(GM, grams, Wn=None, Gn=None, lam=None, stream=None):
     check(lib().pasta_cpals_prepare(_dptr(GM), gp, len(grams), R, _dptr(Wn), _dptr(Gn), _dptr(lam),
                                     _stream_ptr(stream)))
     return Wn, Gn, lam
+
+
+def pasta_cpals_fit(grams, lam, inner, normx2: float, stream=None) -> float:
+    """CP-ALS fit in a libpasta kernel from the (all modes') grams, lambda and <X, Xhat>
+    (CUDA fp64 tensors; inner has one element)."""
+    gp = (C.c_void_p * len(grams))(*[g.data_ptr() for g in grams])
+    fit = C.c_double()
+    check(lib().pasta_cpals_fit(gp, len(grams), int(lam.shape[0]), _dptr(lam), _dptr(inner), float(normx2),
+                                C.byref(fit), _stream_ptr(stream)))
+    return fit.value
 
 
 def pasta_rows_times(M, Wn, U=None, stream=None):

@@ -89,6 +89,8 @@ SIGNATURES = {
     "pasta_cpals_solve": (_st, [_vp, C.c_uint64, C.c_uint32, C.POINTER(_vp), C.c_uint32, _vp, _vp, _vp]),
     "pasta_cpals_prepare": (_st, [_vp, C.POINTER(_vp), C.c_uint32, C.c_uint32, _vp, _vp, _vp, _vp]),
     "pasta_rows_times": (_st, [_vp, C.c_uint64, C.c_uint32, _vp, _vp, _vp]),
+    "pasta_cpals_fit": (_st, [C.POINTER(_vp), C.c_uint32, C.c_uint32, _vp, _vp, C.c_double,
+                              C.POINTER(C.c_double), _vp]),
     "pasta_rows_times_bcast": (_st, [_vp, C.c_uint64, C.c_uint64, C.c_uint32, _vp, C.POINTER(_vp),
                                      C.c_uint32, _vp]),
     "pasta_bcast_f32": (_st, [_vp, C.c_uint64, C.POINTER(_vp), C.c_uint32, _vp]),

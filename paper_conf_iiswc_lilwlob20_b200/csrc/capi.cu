@@ -225,12 +225,58 @@ pasta_status pasta_set_allocator(const pasta_allocator *alloc) {
 }
 
 // ---------------------------------------------------------------------------- ingest
+// Binary tensor cache (.pbin, R#17): little-endian "PASTAB01", u32 order, u32 0, u64 nnz,
+// u32 dims[order], then order x nnz u32 indices (0-based, mode after mode), nnz f32 values.
+static const char kPbinMagic[8] = {'P', 'A', 'S', 'T', 'A', 'B', '0', '1'};
+
+static std::unique_ptr<pasta_coo> load_pbin(FILE *f, const char *path) {
+  struct Closer { FILE *f; ~Closer() { std::fclose(f); } } closer{f};
+  uint32_t head[2];
+  uint64_t nnz = 0;
+  if (std::fread(head, 4, 2, f) != 2 || std::fread(&nnz, 8, 1, f) != 1)
+    fail(PASTA_EFORMAT, std::string("truncated .pbin header in ") + path);
+  const uint32_t order = head[0];
+  if (order < 1 || order > kMaxOrder || head[1] != 0) fail(PASTA_EFORMAT, "bad .pbin header (order / flags)");
+  if (nnz > 0xFFFFFFFEull) fail(PASTA_ERANGE, "more than 2^32-2 nonzeros");
+  uint32_t dims[kMaxOrder];
+  if (std::fread(dims, 4, order, f) != order) fail(PASTA_EFORMAT, "truncated .pbin dims");
+  validate_dims(order, dims);
+  // the file must hold exactly the arrays the header announces
+  const long here = std::ftell(f);
+  std::fseek(f, 0, SEEK_END);
+  const uint64_t size = uint64_t(std::ftell(f));
+  std::fseek(f, here, SEEK_SET);
+  if (size != uint64_t(here) + (uint64_t(order) + 1) * 4 * nnz)
+    fail(PASTA_EFORMAT, std::string(".pbin size does not match its header: ") + path);
+  std::vector<std::vector<uint32_t>> inds(order, std::vector<uint32_t>(nnz));
+  std::vector<float> vals(nnz);
+  for (uint32_t k = 0; k < order; ++k) {
+    if (std::fread(inds[k].data(), 4, nnz, f) != nnz) fail(PASTA_EIO, std::string("read error on ") + path);
+    for (uint64_t i = 0; i < nnz; ++i)
+      if (inds[k][i] >= dims[k])
+        fail(PASTA_ERANGE, "index " + std::to_string(inds[k][i]) + " >= dims[" + std::to_string(k) + "]");
+  }
+  if (std::fread(vals.data(), 4, nnz, f) != nnz) fail(PASTA_EIO, std::string("read error on ") + path);
+  const uint32_t *ip[kMaxOrder];
+  for (uint32_t k = 0; k < order; ++k) ip[k] = inds[k].data();
+  return coo_upload(order, dims, nnz, ip, vals.data(), nullptr);
+}
+
 pasta_status pasta_load_coo(const char *path, pasta_coo **out) {
   API_BEGIN
   require(path && out, "path/out is NULL");
   *out = nullptr;
   FILE *f = std::fopen(path, "rb");
   if (!f) fail(PASTA_EIO, std::string("cannot open ") + path);
+  {
+    char magic[8] = {};
+    const size_t got = std::fread(magic, 1, 8, f);
+    if (got == 8 && std::memcmp(magic, kPbinMagic, 8) == 0) {
+      *out = load_pbin(f, path).release();
+      return PASTA_OK;
+    }
+    std::rewind(f);
+  }
   std::string text;
   {
     char buf[1 << 16];
@@ -308,6 +354,18 @@ pasta_status pasta_save_coo(const pasta_coo *x, const char *path) {
   if (x->nnz) PASTA_CUDA(cudaMemcpy(v.data(), x->val.p, x->nnz * 4, cudaMemcpyDeviceToHost));
   FILE *f = std::fopen(path, "wb");
   if (!f) fail(PASTA_EIO, std::string("cannot create ") + path);
+  const size_t plen = std::strlen(path);
+  if (plen >= 5 && std::strcmp(path + plen - 5, ".pbin") == 0) {  // binary cache
+    const uint32_t head[2] = {x->order, 0};
+    const uint64_t nnz = x->nnz;
+    bool ok = std::fwrite(kPbinMagic, 1, 8, f) == 8 && std::fwrite(head, 4, 2, f) == 2 &&
+              std::fwrite(&nnz, 8, 1, f) == 1 && std::fwrite(x->dims, 4, x->order, f) == x->order;
+    for (uint32_t k = 0; k < x->order && ok; ++k) ok = std::fwrite(h[k].data(), 4, nnz, f) == nnz;
+    ok = ok && std::fwrite(v.data(), 4, nnz, f) == nnz;
+    ok = (std::fclose(f) == 0) && ok;
+    if (!ok) fail(PASTA_EIO, std::string("write error on ") + path);
+    return PASTA_OK;
+  }
   bool ok = true;
   for (uint64_t i = 0; i < x->nnz && ok; ++i) {
     for (uint32_t k = 0; k < x->order; ++k) ok &= std::fprintf(f, "%u ", h[k][i] + 1) > 0;
@@ -346,7 +404,7 @@ pasta_status pasta_gen_powerlaw(uint32_t order, const uint32_t *dims, uint64_t n
   pasta_gen_params p{1, nullptr, 0.0, 0, 0.f, 0.f, 0.0};
   if (params) p = *params;
   require(p.kind <= 2, "unknown generator kind");
-  if (p.permute) fail(PASTA_EUNSUPPORTED, "label permutation is not implemented");
+  require(p.permute <= 1, "permute must be 0 or 1");
   double cells = 1.0;
   for (uint32_t k = 0; k < order; ++k) cells *= double(dims[k]);
   require(double(nnz) <= cells, "nnz exceeds the number of cells");
@@ -365,6 +423,7 @@ pasta_status pasta_gen_powerlaw(uint32_t order, const uint32_t *dims, uint64_t n
     x->nnz = nnz;
     x->device = current_device();
     gen_powerlaw_device(x.get(), seed, nullptr, 0, lo, hi, nullptr, alpha);
+    if (p.permute) relabel_device(x.get(), seed, nullptr);
     x->lex_sorted = true;
     *out = x.release();
     return PASTA_OK;
@@ -403,6 +462,7 @@ pasta_status pasta_gen_powerlaw(uint32_t order, const uint32_t *dims, uint64_t n
   x->nnz = nnz;
   x->device = current_device();
   gen_powerlaw_device(x.get(), seed, table, ncell, lo, hi, nullptr);
+  if (p.permute) relabel_device(x.get(), seed, nullptr);
   x->lex_sorted = true;
   *out = x.release();
   API_END
@@ -784,6 +844,20 @@ pasta_status pasta_cpals_prepare(const double *GM, const double *const *grams, u
   API_END
 }
 
+pasta_status pasta_cpals_fit(const double *const *grams, uint32_t ngrams, uint32_t R, const double *lambda,
+                             const double *inner, double normx2, double *fit, void *stream) {
+  API_BEGIN
+  require_R64(R);
+  require(grams && lambda && inner && fit, "NULL argument");
+  for (uint32_t k = 0; k < ngrams; ++k) require(grams[k] != nullptr, "grams[k] is NULL");
+  cudaStream_t s = as_stream(stream);
+  DevArray<double> out(2, s);
+  launch_cpals_fit(grams, ngrams, R, lambda, inner, normx2, out.p, s);
+  PASTA_CUDA(cudaMemcpyAsync(fit, out.p, sizeof(double), cudaMemcpyDeviceToHost, s));
+  PASTA_CUDA(cudaStreamSynchronize(s));
+  API_END
+}
+
 pasta_status pasta_rows_times(const float *M, uint64_t rows, uint32_t R, const float *Wn, float *U,
                               void *stream) {
   API_BEGIN
@@ -900,6 +974,7 @@ pasta_status pasta_cpals_coo(pasta_coo *x, uint32_t R, uint32_t max_iters, doubl
   DevArray<float> Mbuf(maxd * R, s);
   DevArray<double> grams(uint64_t(N) * R * R, s), colsq(R, s), lam(R, s), scal(2, s), GM(uint64_t(R) * R, s);
   DevArray<float> Wn(uint64_t(R) * R, s);
+  DevArray<double> fitbuf(2, s);
   // fused epilogue (default): gram of M, R x R algebra, one pass U = M Wn; PASTA_CPALS_FUSED=0
   // runs the unfused solve -> normalise -> gram sequence
   const char *fz = getenv("PASTA_CPALS_FUSED");
@@ -912,7 +987,6 @@ pasta_status pasta_cpals_coo(pasta_coo *x, uint32_t R, uint32_t max_iters, doubl
   double normx2 = 0.0;
   PASTA_CUDA(cudaMemcpyAsync(&normx2, scal.p, sizeof(double), cudaMemcpyDeviceToHost, s));
   PASTA_CUDA(cudaStreamSynchronize(s));
-  std::vector<double> hg(uint64_t(N) * R * R), hl(R, 1.0);
   double prev = 0.0;
   uint32_t it = 0;
   const float *cf[kMaxOrder];
@@ -938,29 +1012,22 @@ pasta_status pasta_cpals_coo(pasta_coo *x, uint32_t R, uint32_t max_iters, doubl
       PASTA_CUDA(cudaMemsetAsync(G(n), 0, sizeof(double) * R * R, s));
       launch_gram(factors[n], x->dims[n], R, G(n), s);
     }
-    // fit from the last mode's MTTKRP (still in Mbuf) and the normalised factors
+    // fit from the last mode's MTTKRP (still in Mbuf) and the normalised factors, in a kernel
     PASTA_CUDA(cudaMemsetAsync(scal.p + 1, 0, sizeof(double), s));
     launch_inner(Mbuf.p, factors[N - 1], x->dims[N - 1], R, lam.p, scal.p + 1, s);
-    double inner = 0.0;
-    PASTA_CUDA(cudaMemcpyAsync(&inner, scal.p + 1, sizeof(double), cudaMemcpyDeviceToHost, s));
-    PASTA_CUDA(cudaMemcpyAsync(hg.data(), grams.p, grams.bytes(), cudaMemcpyDeviceToHost, s));
-    PASTA_CUDA(cudaMemcpyAsync(hl.data(), lam.p, lam.bytes(), cudaMemcpyDeviceToHost, s));
+    const double *gall[kMaxOrder];
+    for (uint32_t k = 0; k < N; ++k) gall[k] = G(k);
+    launch_cpals_fit(gall, N, R, lam.p, scal.p + 1, normx2, fitbuf.p, s);
+    double fit = 0.0;
+    PASTA_CUDA(cudaMemcpyAsync(&fit, fitbuf.p, sizeof(double), cudaMemcpyDeviceToHost, s));
     PASTA_CUDA(cudaStreamSynchronize(s));
-    double nxhat2 = 0.0;  // lambda^T (Hadamard_k G_k) lambda
-    for (uint32_t a = 0; a < R; ++a)
-      for (uint32_t b = 0; b < R; ++b) {
-        double v = hl[a] * hl[b];
-        for (uint32_t k = 0; k < N; ++k) v *= hg[uint64_t(k) * R * R + a * R + b];
-        nxhat2 += v;
-      }
-    const double resid2 = normx2 + nxhat2 - 2.0 * inner;
-    const double fit = normx2 > 0 ? 1.0 - std::sqrt(resid2 > 0 ? resid2 : 0.0) / std::sqrt(normx2) : 0.0;
     fit_history[it] = fit;
     const bool done = it > 0 && std::fabs(fit - prev) < tol;
     prev = fit;
     if (done) { ++it; break; }
   }
-  for (uint32_t r = 0; r < R; ++r) lambda[r] = hl[r];
+  PASTA_CUDA(cudaMemcpyAsync(lambda, lam.p, R * sizeof(double), cudaMemcpyDeviceToHost, s));
+  PASTA_CUDA(cudaStreamSynchronize(s));
   *iters = it;
   API_END
 }

@@ -690,4 +690,41 @@ void launch_sumsq(const float *v, uint64_t n, double *out, cudaStream_t s) {
   PASTA_LAUNCHED();
 }
 
+namespace {
+// CP-ALS fit (one CTA, fp64): ||Xhat||^2 = lambda^T (Hadamard_k G_k) lambda, resid^2 =
+// ||X||^2 + ||Xhat||^2 - 2 <X, Xhat>, fit = 1 - sqrt(max(resid^2, 0)) / ||X||.
+__global__ void cpals_fit_kernel(GramList gl, uint32_t R, const double *__restrict__ lambda,
+                                 const double *__restrict__ inner, double normx2, double *__restrict__ out) {
+  __shared__ double red[kThreads / 32];
+  double acc = 0.0;
+  for (uint32_t e = threadIdx.x; e < R * R; e += blockDim.x) {
+    const uint32_t a = e / R, b = e % R;
+    double v = lambda[a] * lambda[b];
+    for (uint32_t k = 0; k < gl.n; ++k) v *= gl.g[k][e];
+    acc += v;
+  }
+  for (int o = 16; o; o >>= 1) acc += __shfl_xor_sync(0xFFFFFFFFu, acc, o);
+  if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = acc;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    double nx = 0.0;
+    for (int w = 0; w < int(blockDim.x >> 5); ++w) nx += red[w];
+    const double resid2 = normx2 + nx - 2.0 * inner[0];
+    out[0] = normx2 > 0 ? 1.0 - sqrt(resid2 > 0 ? resid2 : 0.0) / sqrt(normx2) : 0.0;
+    out[1] = nx;
+  }
+}
+}  // namespace
+
+void launch_cpals_fit(const double *const *grams, uint32_t ngrams, uint32_t R, const double *lambda,
+                      const double *inner, double normx2, double *out, cudaStream_t s) {
+  if (R > kMaxR) fail(PASTA_EUNSUPPORTED, "CP-ALS building blocks support R <= 64");
+  if (ngrams > kMaxOrder) fail(PASTA_EINVAL, "at most 8 grams");
+  GramList gl{};
+  gl.n = ngrams;
+  for (uint32_t k = 0; k < ngrams; ++k) gl.g[k] = grams[k];
+  cpals_fit_kernel<<<1, kThreads, 0, s>>>(gl, R, lambda, inner, normx2, out);
+  PASTA_LAUNCHED();
+}
+
 }  // namespace pasta

@@ -278,4 +278,59 @@ void gen_powerlaw_device(pasta_coo *x, uint64_t seed, const double *table, uint3
   }
 }
 
+namespace {
+
+// Label permutation pi_k of [0, I_k) (R#22, include/pasta.h): cycle walking over a keyed
+// bijection f of [0, 2^L) made of three rounds of (odd multiply, xor-shift, add) mod 2^L.
+__host__ __device__ inline uint32_t relabel_index(uint32_t v, uint32_t dim, uint64_t key, uint32_t L) {
+  const uint64_t m = (uint64_t(1) << L) - 1;
+  uint64_t y = v;
+  do {
+    for (int r = 0; r < 3; ++r) {
+      y = (y * (((key >> (16 * r)) & 0xFFFFull) | 1ull)) & m;
+      if (L >= 2) y ^= y >> ((L + 1) / 2);
+      y = (y + ((key >> (32 + 8 * r)) & 0xFFFFFFull)) & m;
+    }
+  } while (y >= dim);
+  return uint32_t(y);
+}
+
+__global__ void relabel_kernel(uint32_t *inds, uint64_t M, uint32_t dim, uint64_t key, uint32_t L) {
+  for (uint64_t x = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; x < M; x += uint64_t(gridDim.x) * blockDim.x)
+    inds[x] = relabel_index(inds[x], dim, key, L);
+}
+
+}  // namespace
+
+// permute = 1 (R#22): relabel every mode by pi_k, then restore the lexicographic order
+void relabel_device(pasta_coo *x, uint64_t seed, cudaStream_t s) {
+  const uint32_t N = x->order;
+  const uint64_t M = x->nnz;
+  if (M == 0) return;
+  for (uint32_t k = 0; k < N; ++k) {
+    relabel_kernel<<<grid_for(M), kThreads, 0, s>>>(x->inds[k].p, M, x->dims[k],
+                                                    mix64(seed ^ 0xA0761D6478BD642Full ^ uint64_t(k)),
+                                                    ceil_log2(x->dims[k]));
+    PASTA_LAUNCHED();
+  }
+  DevArray<uint32_t> perm(M, s);
+  iota_u32(perm.p, M, s);
+  const uint32_t *comps[kMaxOrder];
+  uint32_t bits[kMaxOrder];
+  for (uint32_t k = 0; k < N; ++k) {
+    comps[k] = x->inds[k].p;
+    bits[k] = ceil_log2(x->dims[k]);
+  }
+  lexsort(comps, bits, int(N), perm, M, s);
+  for (uint32_t k = 0; k < N; ++k) {
+    DevArray<uint32_t> t(M, s);
+    gather_u32(x->inds[k].p, perm.p, t.p, M, s);
+    std::swap(x->inds[k], t);
+  }
+  DevArray<float> v(M, s);
+  gather_f32(x->val.p, perm.p, v.p, M, s);
+  std::swap(x->val, v);
+  PASTA_CUDA(cudaStreamSynchronize(s));
+}
+
 }  // namespace pasta

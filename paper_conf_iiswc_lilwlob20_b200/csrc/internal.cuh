@@ -183,11 +183,12 @@ struct CooModeCopy {
   // Die split (R#35, order 3 with an L2 tier): each gathered factor's rows are split into two
   // halves (die_half); nonzeros are reordered into 4 row-sorted segments by (half of the first
   // gathered row, half of the second): die 0 walks [0, split_x) = (0,0) then (0,1), die 1 walks
-  // [split_x, nnz) = (1,1) then (1,0), so at any time the two dies gather disjoint halves of
+  // [split_x, split_n) = (1,1) then (1,0), so at any time the two dies gather disjoint halves of
   // both factors and each die's L2 holds only its half of the hot rows.  The L2-tier slots of
   // each factor are ordered half 0 first.  split_irow / split_val / hot_inds hold that order.
   bool split = false;
-  uint64_t split_x = 0;
+  uint64_t split_x = 0;                 // die 1's first position (16-byte aligned)
+  uint64_t split_n = 0;                 // length of the split arrays (nnz + alignment gap)
   uint32_t split_t[2] = {};             // die-0 shares of the two gathered factors (of 2^32)
   DevArray<uint32_t> split_irow;
   DevArray<float> split_val;
@@ -338,6 +339,8 @@ void hicoo_prepare_mode(pasta_hicoo *h, uint32_t mode, cudaStream_t s);
 void gen_powerlaw_device(pasta_coo *x, uint64_t seed, const double *table, uint32_t ncell,
                          float val_lo, float val_hi, cudaStream_t s, double alpha = 1.0);
 void coo_to_hicoo_device(const pasta_coo *x, pasta_hicoo *h, cudaStream_t s);  // honours h->cmask
+// generator label permutation (permute = 1, R#22): relabel every mode, re-sort lexicographically
+void relabel_device(pasta_coo *x, uint64_t seed, cudaStream_t s);
 // number of distinct block keys (i_k >> block_bits, k in cmask) of a COO tensor
 uint64_t count_blocks_device(const pasta_coo *x, uint32_t block_bits, uint32_t cmask, cudaStream_t s);
 
@@ -362,6 +365,9 @@ void launch_apply_bcast(const float *M, uint64_t row_lo, uint64_t row_hi, uint32
 void launch_inner(const float *A, const float *B, uint64_t rows, uint32_t R, const double *lambda,
                   double *out, cudaStream_t s);
 void launch_sumsq(const float *v, uint64_t n, double *out, cudaStream_t s);
+// out[0] = CP-ALS fit, out[1] = ||Xhat||^2 (device), from the grams, lambda and <X, Xhat>
+void launch_cpals_fit(const double *const *grams, uint32_t ngrams, uint32_t R, const double *lambda,
+                      const double *inner, double normx2, double *out, cudaStream_t s);
 void coo_mark_hot(pasta_coo *x, uint32_t mode, uint32_t R, bool global_tier, uint32_t smem_rows,
                   cudaStream_t s, bool die_split = false);
 void coo_build_fibers(pasta_coo *x, uint32_t mode, cudaStream_t s);

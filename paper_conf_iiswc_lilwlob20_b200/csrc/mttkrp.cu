@@ -1226,6 +1226,7 @@ void launch_coo_mttkrp(const pasta_coo *x, uint32_t mode, const float *const *fa
       const_cast<CooModeCopy &>(mc).fence.wait(s);
       if (mc.hot_total) launch_hot_fill(mc, factors, x->order, mode, R, s);
       if (hs && mc.split) {
+        a.nnz = mc.split_n;
         a.irow = mc.split_irow.p;
         a.val = mc.split_val.p;
         a.split = 1;
@@ -1423,7 +1424,7 @@ void launch_hicoo_mttkrp(const pasta_hicoo *h, uint32_t mode, const float *const
     bool tiers = false;
     // every launch on this copy reads sbbase: a retag waits for the previous launch
     mcw.fence.wait(s);
-    if (!(env_int("PASTA_HICOO_HOT", 1) && env_int("PASTA_HOT_SMEM", 1))) {
+    if (!(env_int("PASTA_HICOO_HOT", 0) && env_int("PASTA_HOT_SMEM", 1))) {
       if (mc.tagged) hicoo_mark_hot(const_cast<pasta_hicoo *>(h), mode, R, false, 0, s);  // untag
     } else {
       static int l2 = 0;

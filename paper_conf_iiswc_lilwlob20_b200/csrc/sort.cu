@@ -334,6 +334,13 @@ __global__ void hot_fill_kernel(const float4 *__restrict__ U, const uint32_t *__
   }
 }
 
+void gather_any(const uint32_t *in, const uint32_t *perm, uint32_t *out, uint64_t n, cudaStream_t s) {
+  if (n) gather_u32(in, perm, out, n, s);
+}
+void gather_any(const float *in, const uint32_t *perm, float *out, uint64_t n, cudaStream_t s) {
+  if (n) gather_f32(in, perm, out, n, s);
+}
+
 // die-split segment of each nonzero (R#35); n01 counts the die-0 segments (half of ia == 0)
 __global__ void split_seg_kernel(const uint32_t *__restrict__ ia, const uint32_t *__restrict__ ib, uint64_t M,
                                  uint32_t ka, uint32_t kb, uint32_t ta, uint32_t tb, uint32_t *__restrict__ seg,
@@ -509,19 +516,29 @@ void coo_mark_hot(pasta_coo *x, uint32_t mode, uint32_t R, bool global_tier, uin
     const uint32_t bits[1] = {2};
     lexsort(comps, bits, 1, perm, M, s);  // stable: rows stay sorted inside each segment
     seg.reset();
-    mc.split_irow.alloc(M, s);
-    mc.split_val.alloc(M, s);
-    gather_u32(mc.inds[mode], perm.p, mc.split_irow.p, M, s);
-    gather_f32(mc.val, perm.p, mc.split_val.p, M, s);
-    DevArray<uint32_t> tmp(M, s);
-    for (uint32_t k : {ka, kb}) {
-      gather_u32(mc.hot_inds[k].p, perm.p, tmp.p, M, s);
-      std::swap(mc.hot_inds[k], tmp);
-    }
     unsigned long long h01 = 0;
     PASTA_CUDA(cudaMemcpyAsync(&h01, n01.p, sizeof(h01), cudaMemcpyDeviceToHost, s));
     PASTA_CUDA(cudaStreamSynchronize(s));
-    mc.split_x = h01;
+    // die 1's part starts 16-byte aligned (the kernel streams 4 nonzeros per cp.async); the
+    // gap holds zero-valued nonzeros of row 0 (die 0 walks them; they add nothing)
+    const uint64_t n0 = h01, x1 = (n0 + 3) & ~uint64_t(3), Mt = x1 + (M - n0);
+    auto split_gather = [&](auto *in, auto *out) {
+      gather_any(in, perm.p, out, n0, s);
+      if (x1 > n0) PASTA_CUDA(cudaMemsetAsync(out + n0, 0, (x1 - n0) * 4, s));
+      gather_any(in, perm.p + n0, out + x1, M - n0, s);
+    };
+    mc.split_irow.alloc(Mt, s);
+    mc.split_val.alloc(Mt, s);
+    split_gather(mc.inds[mode], mc.split_irow.p);
+    split_gather(mc.val, mc.split_val.p);
+    for (uint32_t k : {ka, kb}) {
+      DevArray<uint32_t> tmp(Mt, s);
+      split_gather(mc.hot_inds[k].p, tmp.p);
+      std::swap(mc.hot_inds[k], tmp);
+    }
+    PASTA_CUDA(cudaStreamSynchronize(s));
+    mc.split_x = x1;
+    mc.split_n = Mt;
     mc.split_t[0] = tsplit[ka];
     mc.split_t[1] = tsplit[kb];
     mc.claim.alloc(2, s);

@@ -204,7 +204,7 @@ class RowPartitionedCPALS(RowPartitionedMTTKRP):
         all-gather, pasta_rows_times_bcast) instead of NCCL broadcasts."""
         import torch
 
-        from . import (pasta_coo_norm2, pasta_cpals_prepare, pasta_cpals_solve, pasta_gram,
+        from . import (pasta_coo_norm2, pasta_cpals_fit, pasta_cpals_prepare, pasta_cpals_solve, pasta_gram,
                        pasta_mttkrp_coo, pasta_normalize_columns, pasta_rows_times,
                        pasta_rows_times_bcast, pasta_weighted_inner)
         N, R = self.order, self.R
@@ -244,13 +244,7 @@ class RowPartitionedCPALS(RowPartitionedMTTKRP):
             lo, hi = int(self.bounds[N - 1][self.rank]), int(self.bounds[N - 1][self.rank + 1])
             inner = _all_reduce(pasta_weighted_inner(self.out[N - 1][lo:hi],
                                                      factors[N - 1][lo:hi], lam))
-            G = np.ones((R, R))  # R x R host arithmetic: lambda^T (Hadamard_k G_k) lambda
-            for g in grams:
-                G *= g.cpu().numpy()
-            lh = lam.cpu().numpy()
-            nxhat2 = float(lh @ G @ lh)
-            resid2 = max(normx2 + nxhat2 - 2.0 * float(inner.item()), 0.0)
-            fits.append(1.0 - (resid2 ** 0.5) / (normx2 ** 0.5) if normx2 > 0 else 0.0)
+            fits.append(pasta_cpals_fit(grams, lam, inner, normx2))  # fit algebra in a kernel
             if it > 0 and abs(fits[-1] - fits[-2]) < tol:
                 break
         return lam.cpu().numpy(), fits

@@ -66,8 +66,8 @@ def test_validation_happens_before_side_effects(pasta, tmp_path):
         P.pasta_gen_powerlaw([2, 2], 5, seed=1)
     assert e.value.code == -1
     with pytest.raises(P.PastaError) as e:
-        P.pasta_gen_powerlaw([10, 10], 5, seed=1, permute=1)
-    assert e.value.code == -7
+        P.pasta_gen_powerlaw([10, 10], 5, seed=1, permute=2)
+    assert e.value.code == -1
     with pytest.raises(P.PastaError) as e:
         P.pasta_load_coo(str(tmp_path / "missing.tns"))
     assert e.value.code == -2
@@ -125,3 +125,31 @@ def test_row_partition_edge_cases(pasta):
     assert list(b) == [0, 0, 0, 5]
     with pytest.raises(pasta.PastaError):
         pasta.pasta_row_partition(np.ones(3, np.uint64), 0)
+
+
+def _pbin(order, nnz, dims, inds, vals, flags=0, extra=b""):
+    import struct
+    b = b"PASTAB01" + struct.pack("<IIQ", order, flags, nnz) + struct.pack(f"<{order}I", *dims)
+    for k in range(order):
+        b += np.asarray(inds[k], np.uint32).tobytes()
+    return b + np.asarray(vals, np.float32).tobytes() + extra
+
+
+def test_pbin_header_and_range_errors(pasta, tmp_path):
+    """.pbin binary cache (R#17): malformed files are rejected before any upload."""
+    P = pasta
+    p = tmp_path / "x.pbin"
+    inds = [[0, 1], [2, 0]]
+    cases = [
+        (_pbin(2, 2, (3, 3), inds, [1, 2], extra=b"\0"), -3),   # size != header
+        (_pbin(2, 2, (3, 3), inds, [1, 2])[:-3], -3),            # truncated
+        (_pbin(9, 2, (3,) * 9, [[0, 0]] * 9, [1, 2]), -3),       # order > 8
+        (_pbin(2, 2, (3, 3), inds, [1, 2], flags=1), -3),        # unknown flags
+        (_pbin(2, 2, (3, 2), inds, [1, 2]), -4),                 # index 2 >= dims[1]
+        (_pbin(2, 2, (0, 3), inds, [1, 2]), -1),                 # a zero dim
+    ]
+    for blob, code in cases:
+        p.write_bytes(blob)
+        with pytest.raises(P.PastaError) as e:
+            P.pasta_load_coo(str(p))
+        assert e.value.code == code, (code, str(e.value))

@@ -152,14 +152,17 @@ def test_generator_bit_exact_with_oracle(env):
         dict(dims=(64, 64, 64), nnz=20_000, seed=7),  # many repeated draws
         dict(dims=(1 << 16, 1 << 16), nnz=5000, seed=3, initiator=[0.57, 0.19, 0.19, 0.05]),
         dict(dims=(100, 100, 100), nnz=10_000, seed=1001, kind=0),
+        # permute = 1 (R#22): labels relabelled by pi_k, then re-sorted; odd and 2^k dims
+        dict(dims=(12092, 9184, 28818), nnz=100_000, seed=1002, permute=1),
+        dict(dims=(1 << 12, 1 << 12, 1 << 12), nnz=50_000, seed=9, permute=1),
     ]
     for c in cases:
         kind = c.get("kind", 1)
         x = pasta.pasta_gen_powerlaw(c["dims"], c["nnz"], c["seed"], kind=kind,
-                                     initiator=c.get("initiator"))
+                                     initiator=c.get("initiator"), permute=c.get("permute", 0))
         gi, gv = pasta.pasta_coo_export(x)
         oi, ov = oracle.gen_powerlaw(c["dims"], c["nnz"], c["seed"], initiator=c.get("initiator"),
-                                     q=0.5 if kind == 0 else 0.75)
+                                     q=0.5 if kind == 0 else 0.75, permute=bool(c.get("permute", 0)))
         np.testing.assert_array_equal(gi, oi)
         np.testing.assert_array_equal(gv.view(np.uint32), ov.view(np.uint32))
 
@@ -274,6 +277,17 @@ def test_tns_roundtrip(env, tmp_path):
     gi2, gv2 = pasta.pasta_coo_export(t2)
     np.testing.assert_array_equal(gi2, inds)
     np.testing.assert_array_equal(gv2, vals)
+    # binary cache (.pbin): bit-exact round trip, stored dims kept (larger than the max index)
+    big = pasta.pasta_coo_from_arrays((70, 80, 90), inds, vals)
+    b = tmp_path / "t.pbin"
+    pasta.pasta_save_coo(big, str(b))
+    assert b.read_bytes()[:8] == b"PASTAB01"
+    assert b.stat().st_size == 8 + 16 + 12 + 4 * 4 * 2000
+    t3 = pasta.pasta_load_coo(str(b))
+    assert t3.dims == (70, 80, 90) and t3.nnz == 2000
+    gi3, gv3 = pasta.pasta_coo_export(t3)
+    np.testing.assert_array_equal(gi3, inds)
+    np.testing.assert_array_equal(gv3.view(np.uint32), vals.view(np.uint32))
 
 
 def test_misaligned_factor_takes_scalar_path(env):

@@ -110,6 +110,7 @@ def test_hicoo_hot_block_tiers_retag(env, hot_mb, monkeypatch):
     retagged slice bases are untagged and retagged between launches; every result against the
     oracle.  hot_mb = 0.05 leaves most blocks cold (mixed tags inside a warp's window)."""
     pasta, oracle, torch = env
+    monkeypatch.setenv("PASTA_HICOO_HOT", "1")
     monkeypatch.setenv("PASTA_HOT_FORCE", "1")
     monkeypatch.setenv("PASTA_HOT_MB", hot_mb)
     dims = (1000, 777, 1300)

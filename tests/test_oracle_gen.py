@@ -101,3 +101,32 @@ def test_degenerate_initiators(oracle_mod):
     # the full box: every cell exactly once
     inds4, _ = oracle_mod.gen_powerlaw((3, 5), 15, seed=2)
     assert sorted(map(tuple, inds4.T)) == [(i, j) for i in range(3) for j in range(5)]
+
+
+def test_label_permutation_is_a_bijection_per_mode(oracle_mod):
+    """R#22 (permute = 1): pi_k is a bijection of [0, I_k) for powers of two, their
+    neighbours and odd sizes; different modes / seeds give different permutations."""
+    for dim in (1, 2, 3, 7, 64, 127, 128, 129, 1000, 4097):
+        img = [oracle_mod.relabel_index(v, dim, 11, 2) for v in range(dim)]
+        assert sorted(img) == list(range(dim)), dim
+    a = [oracle_mod.relabel_index(v, 1000, 11, 0) for v in range(1000)]
+    b = [oracle_mod.relabel_index(v, 1000, 11, 1) for v in range(1000)]
+    c = [oracle_mod.relabel_index(v, 1000, 12, 0) for v in range(1000)]
+    assert a != b and a != c and a != list(range(1000))
+
+
+def test_permuted_generator_keeps_the_row_count_multiset(oracle_mod):
+    """Relabelling moves rows but keeps every row's nonzeros: the sorted row counts of every
+    mode, the multiset of values and uniqueness are those of the unpermuted tensor, and the
+    permuted tensor is lexicographically sorted."""
+    dims, M, seed = (300, 200, 500), 20_000, 9
+    i0, v0 = oracle_mod.gen_powerlaw(dims, M, seed)
+    i1, v1 = oracle_mod.gen_powerlaw(dims, M, seed, permute=True)
+    for k, d in enumerate(dims):
+        assert np.array_equal(np.sort(np.bincount(i0[k], minlength=d)), np.sort(np.bincount(i1[k], minlength=d)))
+        # pi_k applied to the unpermuted coordinates gives exactly the permuted ones
+        mapped = np.array([oracle_mod.relabel_index(v, d, seed, k) for v in range(d)], np.uint32)[i0[k]]
+        assert np.array_equal(np.sort(mapped), np.sort(i1[k]))
+    assert np.array_equal(np.sort(v0.view(np.uint32)), np.sort(v1.view(np.uint32)))
+    key = (i1[0].astype(np.int64) * dims[1] + i1[1]) * dims[2] + i1[2]
+    assert np.all(np.diff(key) > 0)
