@@ -236,6 +236,13 @@ pasta_status pasta_coo_partition(const pasta_coo *x, uint32_t mode, uint32_t npa
  * rows [row_lo, row_hi) of `out`. */
 pasta_status pasta_coo_shard(pasta_coo *x, uint32_t mode, uint32_t row_lo, uint32_t row_hi,
                              pasta_coo **out);
+/* HiCOO (or gHiCOO) shard: a new handle of the same shape,
+ * block size and mask holding the entries with row_lo <= i_mode < row_hi, in the canonical
+ * order restricted to them, with blocks re-cut where a compressed mode's block index changes:
+ * bit-exact with the conversion of that sub-tensor.  MTTKRP of that mode on the shard writes
+ * only rows [row_lo, row_hi) of `out`.  Row bounds: pasta_row_partition / pasta_coo_partition. */
+pasta_status pasta_hicoo_shard(const pasta_hicoo *h, uint32_t mode, uint32_t row_lo, uint32_t row_hi,
+                               pasta_hicoo **out);
 
 /* ------------------------------------------------------- CP-ALS -------- */
 /* CANDECOMP/PARAFAC by alternating least squares around the MTTKRP: the paper's motivation

@@ -21,7 +21,7 @@ __all__ = [
     "pasta_coo_to_hicoo", "pasta_coo_prepare", "pasta_hicoo_prepare", "pasta_mttkrp_coo",
     "pasta_mttkrp_hicoo", "pasta_mttkrp_coo_allmodes_host", "pasta_mttkrp_coo_allmodes_host_batch",
     "pasta_coo_row_counts",
-    "pasta_row_partition", "pasta_coo_partition", "pasta_coo_shard", "pasta_coo_info",
+    "pasta_row_partition", "pasta_coo_partition", "pasta_coo_shard", "pasta_hicoo_shard", "pasta_coo_info",
     "pasta_coo_export", "pasta_coo_export_mode", "pasta_hicoo_info", "pasta_hicoo_export",
     "pasta_launch_count", "pasta_die_map", "pasta_profile_enable", "pasta_profile_read", "pasta_gram",
     "pasta_cpals_solve", "pasta_normalize_columns", "pasta_weighted_inner", "pasta_coo_norm2",
@@ -359,6 +359,13 @@ def pasta_coo_shard(x: Coo, mode: int, row_lo: int, row_hi: int) -> Coo:
     out = C.c_void_p()
     check(lib().pasta_coo_shard(x.ptr, mode, row_lo, row_hi, C.byref(out)))
     return Coo(out.value)
+
+
+def pasta_hicoo_shard(h: "Hicoo", mode: int, row_lo: int, row_hi: int) -> "Hicoo":
+    """The entries of `h` with row_lo <= i_mode < row_hi as a HiCOO handle (include/pasta.h)."""
+    out = C.c_void_p()
+    check(lib().pasta_hicoo_shard(h.ptr, mode, row_lo, row_hi, C.byref(out)))
+    return Hicoo(out.value)
 
 
 # ----------------------------------------------------------------------------- introspection

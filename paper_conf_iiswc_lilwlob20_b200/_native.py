@@ -73,6 +73,7 @@ SIGNATURES = {
     "pasta_row_partition": (_st, [C.c_uint32, _u64p, C.c_uint32, _u32p]),
     "pasta_coo_partition": (_st, [_vp, C.c_uint32, C.c_uint32, _u32p]),
     "pasta_coo_shard": (_st, [_vp, C.c_uint32, C.c_uint32, C.c_uint32, C.POINTER(_vp)]),
+    "pasta_hicoo_shard": (_st, [_vp, C.c_uint32, C.c_uint32, C.c_uint32, C.POINTER(_vp)]),
     "pasta_ts": (_st, [_vp, C.c_uint64, C.c_uint32, C.c_float, _vp, _vp]),
     "pasta_tew": (_st, [_vp, _vp, C.c_uint64, C.c_uint32, _vp, _vp]),
     "pasta_coo_values": (_st, [_vp, C.POINTER(_vp)]),

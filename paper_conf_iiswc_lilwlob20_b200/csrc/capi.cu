@@ -615,7 +615,9 @@ pasta_status pasta_mttkrp_hicoo(pasta_hicoo *h, uint32_t mode, const float *cons
   cudaStream_t s = as_stream(stream);
   std::lock_guard<std::mutex> lk(h->mu);
   if (!h->mc[mode].ready) hicoo_prepare_mode(h, mode, s);
-  launch_zero_rows(out, 0, h->dims[mode], R, s);
+  uint64_t lo = 0, hi = h->dims[mode];
+  if (h->shard_mode == int(mode)) { lo = h->row_lo; hi = h->row_hi; }
+  launch_zero_rows(out, lo, hi, R, s);
   launch_hicoo_mttkrp(h, mode, factors, R, out, s);
   API_END
 }
@@ -765,6 +767,20 @@ pasta_status pasta_coo_partition(const pasta_coo *x, uint32_t mode, uint32_t npa
   if (st != PASTA_OK) fail(st, t_last_error);
   st = pasta_row_partition(x->dims[mode], counts.data(), nparts, bounds);
   if (st != PASTA_OK) fail(st, t_last_error);
+  API_END
+}
+
+pasta_status pasta_hicoo_shard(const pasta_hicoo *h, uint32_t mode, uint32_t row_lo, uint32_t row_hi,
+                              pasta_hicoo **out) {
+  API_BEGIN
+  require(h && out, "h/out is NULL");
+  *out = nullptr;
+  require(mode < h->order, "mode >= order");
+  require(row_lo <= row_hi && row_hi <= h->dims[mode], "need row_lo <= row_hi <= dims[mode]");
+  check_device(h->device);
+  auto y = std::make_unique<pasta_hicoo>();
+  hicoo_shard_device(h, mode, row_lo, row_hi, y.get(), nullptr);
+  *out = y.release();
   API_END
 }
 

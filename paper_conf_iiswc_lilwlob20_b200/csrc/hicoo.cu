@@ -459,4 +459,106 @@ void hicoo_prepare_mode(pasta_hicoo *h, uint32_t mode, cudaStream_t s) {
   mc.ready = true;
 }
 
+namespace {
+// full coordinate of every entry (canonical gHiCOO order): binds_k[blk] << b | einds_k, or uinds_k
+__global__ void decode_coord_kernel(const uint32_t *__restrict__ blk, const uint32_t *__restrict__ binds,
+                                    const uint8_t *__restrict__ einds, const uint32_t *__restrict__ uinds,
+                                    uint32_t bb, uint64_t M, uint32_t *__restrict__ out) {
+  for (uint64_t x = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; x < M; x += uint64_t(gridDim.x) * blockDim.x)
+    out[x] = uinds ? uinds[x] : ((binds[blk[x]] << bb) | einds[x]);
+}
+__global__ void range_flag_kernel(const uint32_t *__restrict__ c, uint64_t M, uint32_t lo, uint32_t hi,
+                                  uint8_t *__restrict__ flag) {
+  for (uint64_t x = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; x < M; x += uint64_t(gridDim.x) * blockDim.x)
+    flag[x] = c[x] >= lo && c[x] < hi;
+}
+}  // namespace
+
+// The entries of `h` with row_lo <= i_mode < row_hi, as a HiCOO handle of the same shape,
+// block size and mask: the canonical order restricted to the
+// subset (a Morton / gHiCOO order restricted to a subset is that subset's order), blocks
+// re-cut where a compressed mode's block index changes -- the conversion of the sub-tensor.
+void hicoo_shard_device(const pasta_hicoo *h, uint32_t mode, uint32_t row_lo, uint32_t row_hi, pasta_hicoo *y,
+                        cudaStream_t s) {
+  const uint32_t N = h->order, bb = h->block_bits, cmask = h->cmask;
+  const uint64_t M = h->nnz;
+  y->order = N;
+  for (uint32_t k = 0; k < N; ++k) y->dims[k] = h->dims[k];
+  y->block_bits = bb;
+  y->cmask = cmask;
+  y->device = h->device;
+  DevArray<uint32_t> blk(M, s);
+  if (M) {
+    entry_block_kernel<<<grid_for(M), kThreads, 0, s>>>(h->bptr.p, h->nblocks, M, blk.p);
+    PASTA_LAUNCHED();
+  }
+  auto decode = [&](uint32_t k, uint32_t *out) {
+    const bool comp = (cmask >> k) & 1u;
+    decode_coord_kernel<<<grid_for(M), kThreads, 0, s>>>(blk.p, comp ? h->binds[k].p : nullptr,
+                                                         comp ? h->einds[k].p : nullptr,
+                                                         comp ? nullptr : h->uinds[k].p, bb, M, out);
+    PASTA_LAUNCHED();
+  };
+  DevArray<uint32_t> idx;
+  uint64_t Ms = 0;
+  if (M) {
+    DevArray<uint32_t> rows(M, s);
+    decode(mode, rows.p);
+    DevArray<uint8_t> flag(M, s);
+    range_flag_kernel<<<grid_for(M), kThreads, 0, s>>>(rows.p, M, row_lo, row_hi, flag.p);
+    PASTA_LAUNCHED();
+    Ms = select_flagged(flag.p, M, idx, s);
+  }
+  DevArray<uint32_t> sc[kMaxOrder];
+  Coords co{};
+  co.order = 0;
+  for (uint32_t k = 0; k < N; ++k) {
+    sc[k].alloc(Ms, s);
+    if (Ms) {
+      DevArray<uint32_t> full(M, s);
+      decode(k, full.p);
+      gather_u32(full.p, idx.p, sc[k].p, Ms, s);
+    }
+    if ((cmask >> k) & 1u) co.c[co.order++] = sc[k].p;
+  }
+  uint64_t nb = 0;
+  DevArray<uint32_t> starts;
+  if (Ms) {
+    DevArray<uint8_t> flag(Ms, s);
+    block_flag_kernel<<<grid_for(Ms), kThreads, 0, s>>>(co, bb, Ms, flag.p);
+    PASTA_LAUNCHED();
+    nb = select_flagged(flag.p, Ms, starts, s);
+  }
+  y->nblocks = nb;
+  y->nnz = Ms;
+  y->bptr.alloc(nb + 1, s);
+  if (!Ms) {
+    uint64_t zero = 0;
+    PASTA_CUDA(cudaMemcpyAsync(y->bptr.p, &zero, sizeof(zero), cudaMemcpyHostToDevice, s));
+  }
+  bool bptr_written = false;
+  for (uint32_t k = 0; k < N; ++k) {
+    if (!((cmask >> k) & 1u)) {
+      y->uinds[k] = std::move(sc[k]);
+      continue;
+    }
+    y->binds[k].alloc(nb, s);
+    y->einds[k].alloc(Ms, s);
+    if (Ms) {
+      emit_blocks_kernel<<<grid_for(nb + 1), kThreads, 0, s>>>(starts.p, nb, Ms, sc[k].p, bb, y->bptr.p,
+                                                             y->binds[k].p, !bptr_written);
+      PASTA_LAUNCHED();
+      bptr_written = true;
+      emit_einds_kernel<<<grid_for(Ms), kThreads, 0, s>>>(sc[k].p, Ms, (1u << bb) - 1u, y->einds[k].p);
+      PASTA_LAUNCHED();
+    }
+  }
+  y->val.alloc(Ms, s);
+  if (Ms) gather_f32(h->val.p, idx.p, y->val.p, Ms, s);
+  y->shard_mode = int(mode);
+  y->row_lo = row_lo;
+  y->row_hi = row_hi;
+  PASTA_CUDA(cudaStreamSynchronize(s));
+}
+
 }  // namespace pasta

@@ -296,6 +296,8 @@ struct pasta_hicoo {
   pasta::DevArray<uint32_t> uinds[pasta::kMaxOrder];
   pasta::DevArray<float> val;
   pasta::HicooModeCopy mc[pasta::kMaxOrder];
+  int shard_mode = -1;  // >= 0: the [row_lo, row_hi) shard of that mode (pasta_hicoo_shard)
+  uint32_t row_lo = 0, row_hi = 0;
   std::mutex mu;
 };
 
@@ -339,6 +341,8 @@ void hicoo_prepare_mode(pasta_hicoo *h, uint32_t mode, cudaStream_t s);
 void gen_powerlaw_device(pasta_coo *x, uint64_t seed, const double *table, uint32_t ncell,
                          float val_lo, float val_hi, cudaStream_t s, double alpha = 1.0);
 void coo_to_hicoo_device(const pasta_coo *x, pasta_hicoo *h, cudaStream_t s);  // honours h->cmask
+void hicoo_shard_device(const pasta_hicoo *h, uint32_t mode, uint32_t row_lo, uint32_t row_hi, pasta_hicoo *y,
+                        cudaStream_t s);
 // generator label permutation (permute = 1, R#22): relabel every mode, re-sort lexicographically
 void relabel_device(pasta_coo *x, uint64_t seed, cudaStream_t s);
 // number of distinct block keys (i_k >> block_bits, k in cmask) of a COO tensor

@@ -90,19 +90,26 @@ def partition_bounds(counts_per_mode: Sequence[np.ndarray], world: int) -> List[
 
 
 class RowPartitionedMTTKRP:
-    """Holds this rank's per-mode shards of a COO tensor and runs all-mode MTTKRP steps."""
+    """Holds this rank's per-mode shards of a COO tensor and runs all-mode MTTKRP steps.
+    fmt="hicoo": the shards are HiCOO (pasta_hicoo_shard of the tensor's HiCOO form with
+    block_bits, or of `hicoo` when given) and the step runs the HiCOO MTTKRP."""
 
-    def __init__(self, x, rank: int, world: int, R: int, device):
+    def __init__(self, x, rank: int, world: int, R: int, device, fmt: str = "coo", block_bits: int = 7,
+                 hicoo=None):
         import torch
 
-        from . import pasta_coo_partition, pasta_coo_shard
-        self.rank, self.world, self.R = rank, world, R
+        from . import pasta_coo_partition, pasta_coo_shard, pasta_coo_to_hicoo, pasta_hicoo_shard
+        self.rank, self.world, self.R, self.fmt = rank, world, R, fmt
         self.order, self.dims, self.nnz = x.order, x.dims, x.nnz
         self.bounds = [pasta_coo_partition(x, n, world) for n in range(x.order)]
         self.shards = []
+        h = None
+        if fmt == "hicoo":
+            h = hicoo if hicoo is not None else pasta_coo_to_hicoo(x, block_bits)
         for n in range(x.order):
             lo, hi = int(self.bounds[n][rank]), int(self.bounds[n][rank + 1])
-            self.shards.append(pasta_coo_shard(x, n, lo, hi))
+            self.shards.append(pasta_hicoo_shard(h, n, lo, hi) if h is not None else pasta_coo_shard(x, n, lo, hi))
+        del h
         self.out = [torch.empty((d, R), dtype=torch.float32, device=device) for d in self.dims]
 
     def shard_nnz(self) -> List[int]:
@@ -111,10 +118,11 @@ class RowPartitionedMTTKRP:
     def step(self, factors, gather: bool = True, stream=None):
         """MTTKRP of every mode on this rank's shards (+ the all-gather of each output
         when world > 1).  The gather of mode n overlaps the compute of mode n + 1."""
-        from . import pasta_mttkrp_coo
+        from . import pasta_mttkrp_coo, pasta_mttkrp_hicoo
+        fn = pasta_mttkrp_hicoo if self.fmt == "hicoo" else pasta_mttkrp_coo
         works = []
         for n in range(self.order):
-            pasta_mttkrp_coo(self.shards[n], n, factors, out=self.out[n], stream=stream)
+            fn(self.shards[n], n, factors, out=self.out[n], stream=stream)
             if gather and self.world > 1:
                 works += gather_rows(self.out[n], self.bounds[n], async_op=True)
         for w in works:

@@ -25,14 +25,15 @@ def main():
     U = si.factors(dims, 16, seed=9)
     Ud = [torch.from_numpy(u).cuda() for u in U]
     x = pasta.pasta_coo_from_arrays(dims, inds, vals)
-    part = RowPartitionedMTTKRP(x, rank, world, 16, torch.device("cuda", 0))
-    outs = part.step(Ud, gather=True)
-    torch.cuda.synchronize()
     ok = True
-    for n in range(3):
-        ref, ab = oracle.mttkrp(dims, inds, vals, n, U)
-        g = outs[n].cpu().numpy().astype(np.float64)
-        ok &= bool(np.all(np.abs(g - ref) <= 1e-4 * ab + 1e-6))
+    for fmt in ("coo", "hicoo"):  # COO shards, and HiCOO shards (pasta_hicoo_shard)
+        part = RowPartitionedMTTKRP(x, rank, world, 16, torch.device("cuda", 0), fmt=fmt)
+        outs = part.step(Ud, gather=True)
+        torch.cuda.synchronize()
+        for n in range(3):
+            ref, ab = oracle.mttkrp(dims, inds, vals, n, U)
+            g = outs[n].cpu().numpy().astype(np.float64)
+            ok &= bool(np.all(np.abs(g - ref) <= 1e-4 * ab + 1e-6))
     flag = torch.tensor([1 if ok else 0])
     dist.all_reduce(flag, op=dist.ReduceOp.MIN)
     dist.destroy_process_group()

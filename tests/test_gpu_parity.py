@@ -219,6 +219,48 @@ def test_shards_cover_the_output(env):
             _check(out, ref, ab, f"shards mode {n} P={P}")
 
 
+@pytest.mark.parametrize("cmask", [0b111, 0b101])
+def test_hicoo_shards_bit_exact_and_cover_the_output(env, cmask):
+    """pasta_hicoo_shard: every shard equals the oracle's conversion of the
+    COO sub-tensor of its rows, bit for bit; the shards' MTTKRPs write disjoint row ranges
+    that together give the full result.  cmask 0b101: gHiCOO with mode 1 uncompressed."""
+    pasta, oracle, torch = env
+    dims = (2000, 300, 400)
+    inds, vals = si.hot_row_coo(dims, 20_000, 60_000, seed=9, mode=1, hot_row=17)
+    U = si.factors(dims, 16, seed=4)
+    Ud = _dev(torch, U)
+    x = pasta.pasta_coo_from_arrays(dims, inds, vals)
+    h = pasta.pasta_coo_to_hicoo(x, 7) if cmask == 0b111 else pasta.pasta_coo_to_ghicoo(x, 7, cmask)
+    for n in range(3):
+        ref, ab = oracle.mttkrp(dims, inds, vals, n, U)
+        bounds = pasta.pasta_coo_partition(x, n, 3)
+        out = torch.full((dims[n], 16), float("nan"), device="cuda")
+        total = 0
+        for p in range(3):
+            lo, hi = int(bounds[p]), int(bounds[p + 1])
+            sh = pasta.pasta_hicoo_shard(h, n, lo, hi)
+            total += sh.nnz
+            mine = (inds[n] >= lo) & (inds[n] < hi)
+            si_, sv_ = np.ascontiguousarray(inds[:, mine]), vals[mine]
+            if cmask == 0b111:
+                got, want = pasta.pasta_hicoo_export(sh), oracle.coo_to_hicoo(si_, sv_, 7)
+                keys = ("bptr", "binds", "einds")
+                for k in keys:
+                    assert np.array_equal(got[k], want[k]), (n, p, k)
+            else:
+                got, want = pasta.pasta_ghicoo_export(sh), oracle.coo_to_ghicoo(si_, sv_, 7, cmask)
+                assert np.array_equal(got["bptr"], want["bptr"]), (n, p)
+                for k in range(3):
+                    for key in ("binds", "einds", "uinds"):
+                        if want[key][k] is not None:
+                            assert np.array_equal(got[key][k], want[key][k]), (n, p, key, k)
+            assert got["nblocks"] == want["nblocks"]
+            assert np.array_equal(got["vals"].view(np.uint32), want["vals"].view(np.uint32))
+            pasta.pasta_mttkrp_hicoo(sh, n, Ud, out=out)  # writes only its rows
+        assert total == vals.shape[0]
+        _check(out, ref, ab, f"hicoo shards mode {n}")
+
+
 def test_allmodes_host_e2e_matches_device(env):
     pasta, oracle, torch = env
     dims = (500, 400, 300)

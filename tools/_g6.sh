@@ -6,3 +6,5 @@ ncu -i /tmp/split$SPLIT.ncu-rep --page raw --csv > $O/raw_split$SPLIT.csv 2>/dev
 done
 git checkout profiles/ncu_summary.json 2>/dev/null
 head -40 $O/ncu_full_coo_h_split1.md
+timeout 1200 python -m pytest tests/test_gpu_parity.py tests/test_gpu_cpals.py tests/test_gpu_multirank.py -q -x -k "shards or generator or tns or cpals or row_partitioned" > $O/pytest.log 2>&1; echo rc=$? >> $O/pytest.log
+tail -3 $O/pytest.log
