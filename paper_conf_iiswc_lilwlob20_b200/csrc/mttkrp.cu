@@ -89,7 +89,7 @@ struct KArgs {
 // Per-thread L2 cache policies (createpolicy, sm_80+): the nonzero stream is touched once
 // and must not displace the power-law-hot factor rows, which is what L2 is for here.
 struct Policies {
-  uint64_t stream, gather, out;
+  uint64_t stream, gather, cold, out;
   __device__ __forceinline__ explicit Policies(uint32_t mode) {
     uint64_t first, normal, last;
     asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(first));
@@ -97,6 +97,9 @@ struct Policies {
     asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(last));
     stream = (mode & 1) ? first : normal;
     gather = (mode & 2) ? last : normal;
+    // bit 3: gathers of COLD rows (not in a hot tier) evict_first, so that the rows that are
+    // used once or twice per launch do not push the hot tier out of L2
+    cold = (mode & 8) ? first : gather;
     out = (mode & 4) ? first : normal;
   }
 };
@@ -151,6 +154,24 @@ __device__ __forceinline__ Vec<4> ld_tiered(uint32_t saddr, const float *gp, uin
       "@pg ld.global.nc.L2::cache_hint.v4.f32 {%0, %1, %2, %3}, [%7], %8;\n\t}"
       : "=f"(r.v[0]), "=f"(r.v[1]), "=f"(r.v[2]), "=f"(r.v[3])
       : "r"(saddr), "r"(ps), "r"(pg), "l"(gp), "l"(pol));
+  return r;
+}
+
+// Three-way predicated 128-bit load: shared-memory tier (ps), L2-tier buffer (ph, policy ph_pol)
+// or a cold factor row (pc, policy pc_pol); gp is the global address of whichever of the two.
+__device__ __forceinline__ Vec<4> ld_tiered3(uint32_t saddr, const float *gp, uint64_t ph_pol, uint64_t pc_pol,
+                                             int ps, int ph, int pc) {
+  Vec<4> r;
+  asm volatile(
+      "{\n\t.reg .pred ps, ph, pc;\n\t"
+      "setp.ne.s32 ps, %5, 0;\n\t"
+      "setp.ne.s32 ph, %6, 0;\n\t"
+      "setp.ne.s32 pc, %7, 0;\n\t"
+      "@ps ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];\n\t"
+      "@ph ld.global.nc.L2::cache_hint.v4.f32 {%0, %1, %2, %3}, [%8], %9;\n\t"
+      "@pc ld.global.nc.L2::cache_hint.v4.f32 {%0, %1, %2, %3}, [%8], %10;\n\t}"
+      : "=f"(r.v[0]), "=f"(r.v[1]), "=f"(r.v[2]), "=f"(r.v[3])
+      : "r"(saddr), "r"(ps), "r"(ph), "r"(pc), "l"(gp), "l"(ph_pol), "l"(pc_pol));
   return r;
 }
 
@@ -928,8 +949,12 @@ __global__ void __launch_bounds__(HS ? WPC_ * 32 : kThreads, HS ? 1 : (WA == 6 ?
                   const bool in_h = (id >> 30) == 2u;
                   const uint64_t off = uint64_t(id & 0x3FFFFFFFu) * R + col;
                   const float *gptr = (in_h ? a.hot_buf : a.Uo[j]) + off;
-                  f[j][u] = ld_tiered(hs_saddr + uint32_t(off) * 4u, gptr, pol.gather, u < cnt && in_s,
-                                      u < cnt && !in_s);
+                  if constexpr (WA == 12)  // cold rows with their own L2 policy (Policies::cold)
+                    f[j][u] = ld_tiered3(hs_saddr + uint32_t(off) * 4u, gptr, pol.gather, pol.cold, u < cnt && in_s,
+                                         u < cnt && in_h, u < cnt && !in_s && !in_h);
+                  else
+                    f[j][u] = ld_tiered(hs_saddr + uint32_t(off) * 4u, gptr, pol.gather, u < cnt && in_s,
+                                        u < cnt && !in_s);
                 } else {
                   const uint32_t boff = ((id & 0x3FFFFFFFu) * R + col) * 4u;  // < 4 GB
                   const float *gptr = reinterpret_cast<const float *>(
@@ -1319,6 +1344,8 @@ void launch_coo_mttkrp(const pasta_coo *x, uint32_t mode, const float *const *fa
     using I16 = std::integral_constant<int, 16>;
     if (hs) {
       if (hs_cfg == 1) pick_hs(std::integral_constant<int, 24>(), I16());
+      else if (hs_cfg == 2 && no <= 2 && l2t && (a.cache_mode & 8u))  // cold gathers evict_first
+        with_no_lpn<2>(no, lpn, [&](auto NOt, auto Lt) { go(coo_staged_kernel<NOt.value, Lt.value, 12, true, 16, 32, 8>); });
       else if (hs_cfg == 2 && no <= 2)
         with_no_lpn<2>(no, lpn, [&](auto NOt, auto Lt) { go(coo_staged_kernel<NOt.value, Lt.value, 1, true, 16, 32, 8>); });
       else pick_hs(I16(), std::integral_constant<int, 32>());

@@ -22,7 +22,7 @@ def main():
     ap.add_argument("--runs", default="128")
     ap.add_argument("--formats", default="coo")
     ap.add_argument("--reps", type=int, default=10)
-    ap.add_argument("--caches", default="0")
+    ap.add_argument("--caches", default="", help="PASTA_MTTKRP_CACHE values (default: leave the env)")
     ap.add_argument("--cmask", type=int, default=0, help="gHiCOO mask (0 = auto)")
     ap.add_argument("--R", type=int, default=0, help="override the config's rank")
     args = ap.parse_args()
@@ -47,8 +47,9 @@ def main():
         which = 0 if fmt == "coo" else 1
         for n in range(len(dims)):
             fn(t, n, U, out=outs[n])  # prepare
+        caches = args.caches.split(",") if args.caches else [os.environ.get("PASTA_MTTKRP_CACHE", "0")]
         combos = [(r, v, c) for r in args.runs.split(",") for v in args.variants.split(",")
-                  for c in args.caches.split(",")]
+                  for c in caches]
         for run, var, cache in [(int(r), int(v), int(c)) for r, v, c in combos]:
             if True:
                 os.environ["PASTA_MTTKRP_CACHE"] = str(cache)
