@@ -344,7 +344,10 @@ static void hicoo_prepare_rowslice(pasta_hicoo *h, uint32_t mode, cudaStream_t s
   DevArray<uint32_t> starts;
   mc.nsb = select_flagged(flag.p, M, starts, s);
   mc.sbptr.alloc(mc.nsb + 1, s);
-  mc.sbrow.alloc(mc.nsb, s);
+  // slice rows / bases carry kSlicePad zero slots past nsb: the raw-staged decode copies 36
+  // aligned slots from any window's first slice without bounds checks
+  mc.sbrow.alloc(mc.nsb + kSlicePad, s);
+  PASTA_CUDA(cudaMemsetAsync(mc.sbrow.p + mc.nsb, 0, kSlicePad * 4, s));
   SliceOut o{};
   o.order = N;
   o.mode = mode;
@@ -353,7 +356,8 @@ static void hicoo_prepare_rowslice(pasta_hicoo *h, uint32_t mode, cudaStream_t s
   for (uint32_t k = 0; k < N; ++k) {
     o.binds[k] = h->binds[k].p;
     if (k != mode && comp(k)) {
-      mc.sbbase[k].alloc(mc.nsb, s);
+      mc.sbbase[k].alloc(mc.nsb + kSlicePad, s);
+      PASTA_CUDA(cudaMemsetAsync(mc.sbbase[k].p + mc.nsb, 0, kSlicePad * 4, s));
       o.base[k] = mc.sbbase[k].p;
     }
   }

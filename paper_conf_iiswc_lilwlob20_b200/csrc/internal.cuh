@@ -196,6 +196,7 @@ struct CooModeCopy {
 };
 
 constexpr int kCountBuckets = 256;  // 8 sub-buckets per octave of a row's nonzero count
+constexpr uint64_t kSlicePad = 40;  // padding slots after the row-slice arrays (raw decode)
 
 struct HicooModeCopy {
   bool ready = false;
@@ -224,6 +225,10 @@ struct HicooModeCopy {
   // staged decode (launch_hicoo_mttkrp): slice holding the first entry of every group run
   DevArray<uint64_t> run_sb;
   uint64_t run_sb_run = 0;
+  // raw-staged decode (WA 11): slice holding entry 32 w of every 32-entry window w, and the
+  // slice ends as u32 padded with nnz (kSlicePad slots)
+  DevArray<uint32_t> win_sb;
+  DevArray<uint32_t> sbend32;
   // Hot-BLOCK tiers (hicoo_mark_hot, R#34): the row-slice copy has no per-entry coordinate
   // to retag (entries carry 8-bit offsets from a per-slice block base), so the tiers of the
   // COO hot-row cache are built at block granularity: the most frequent block rows [b B,

@@ -84,6 +84,11 @@ struct KArgs {
   uint64_t split_x;
   unsigned long long *claim;
   const int8_t *die_of;
+  // HiCOO raw-staged decode (WA 11): win_sb[w] = slice holding entry 32 w; u32 slice ends;
+  // words per group window of the raw buffer (layout: see coo_staged_kernel)
+  const uint32_t *win_sb;
+  const uint32_t *sbend32;
+  uint32_t raw_words;
 };
 
 // Per-thread L2 cache policies (createpolicy, sm_80+): the nonzero stream is touched once
@@ -732,8 +737,12 @@ __global__ void __launch_bounds__(HS ? WPC_ * 32 : kThreads, HS ? 1 : (WA == 6 ?
   // no base-pointer select, 32-bit byte offsets.  9: HiCOO row slices decoded warp-wide into
   // the stage buffer (no hot tiers, 64-bit offsets).  10: the same decode with the hot-block
   // tiers (R#34): decoded coordinates carry the tier tags of their retagged slice bases
-  constexpr bool kHic = WA == 9 || WA == 10;
-  constexpr bool kL2T = WA != 7 && WA != 9;
+  // 11: HiCOO row slices whose raw arrays (values, 8-bit element indices, slice ends, rows,
+  // block bases) are copied into shared memory with cp.async one stage ahead and decoded from
+  // there -- the decode of WA 9 waits on dependent global loads every stage
+  constexpr bool kHicRaw = WA == 11;
+  constexpr bool kHic = WA == 9 || WA == 10 || kHicRaw;
+  constexpr bool kL2T = WA != 7 && WA != 9 && WA != 11;
   constexpr bool kGather = WA != 4 && WA != 5;
   constexpr bool kWrite = WA != 3 && WA != 5;
   constexpr int kBuf = (WA == 0 || WA == 2) ? WA : 1;  // 6: form 1 with 3 CTAs per SM
@@ -866,7 +875,139 @@ __global__ void __launch_bounds__(HS ? WPC_ * 32 : kThreads, HS ? 1 : (WA == 6 ?
       gsb[gi] = sb0 + uint64_t(clast) + (elast <= uint32_t(SG) ? 1u : 0u);
     }
   };
+  // ---- WA 11: raw windows.  Per group window (32 entries from p, slices from sb0), at word
+  // offsets: [0] sb0 & 3 | [4, 36) values | per other mode j: 8 words of 8-bit einds, or 32 of
+  // u32 coordinates (gHiCOO wide) | 36 slice ends (u32, slots (sb0 & ~3) + t) | 36 slice rows |
+  // per compressed mode j: 36 block bases.  The slice arrays are padded (ends with nnz) so the
+  // aligned 36-slot copies never leave them.
+  uint32_t *raw = reinterpret_cast<uint32_t *>(hs_tile + size_t(a.hs_lo[NO]) * R) + size_t(warp) * G * a.raw_words;
+  int off_e[NO > 0 ? NO : 1], off_b[NO > 0 ? NO : 1], off_end = 36, off_row = 72;
+  if constexpr (kHicRaw) {
+    int o = 36;
+#pragma unroll
+    for (int j = 0; j < NO; ++j) { off_e[j] = o; o += ((a.wide >> j) & 1u) ? 32 : 8; }
+    off_end = o;
+    off_row = o + 36;
+    o += 72;
+#pragma unroll
+    for (int j = 0; j < NO; ++j) { off_b[j] = o; o += ((a.wide >> j) & 1u) ? 0 : 36; }
+  }
+  const uint64_t nst_total = (uint64_t(a.chunk) / G) / SG;  // stages per chunk
+  // the position after (cc, s) in this warp's static schedule (cc = a.nnz: none)
+  auto next_pos = [&](uint64_t &cc, int &s) {
+    if (cc >= a.nnz) return;
+    if (uint64_t(s) + 1 < nst_total) { ++s; return; }
+    s = 0;
+    cc += wstep * a.chunk;
+    if (cc >= a.nnz) cc = a.nnz;
+  };
+  auto win_of = [&](uint64_t cc, int s) -> uint32_t {  // lane gi < G: win_sb of its group
+    const uint64_t p = cc + uint64_t(lane) * (a.chunk / G) + uint64_t(s) * SG;
+    return (lane < G && p < a.nnz) ? __ldg(a.win_sb + p / 32) : 0u;
+  };
+  auto raw_issue = [&](uint64_t cc, int s, uint32_t wsb) {
+    if (cc < a.nnz) {
+#pragma unroll 1
+      for (int gi = 0; gi < G; ++gi) {
+        const uint64_t p = cc + uint64_t(gi) * (a.chunk / G) + uint64_t(s) * SG;
+        if (p >= a.nnz) break;  // warp-uniform; later groups start later
+        const uint32_t sb0 = __shfl_sync(0xFFFFFFFFu, wsb, gi);
+        uint32_t *rw = raw + gi * a.raw_words;
+        if (lane == 0) rw[0] = sb0 & 3u;
+        const uint32_t sa = sb0 & ~3u;
+        auto cp16 = [&](uint32_t *dst, const void *src, int valid) {
+          asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(smem_addr(dst)), "l"(src),
+                       "r"(valid) : "memory");
+        };
+        const uint64_t left = a.nnz - p;  // entries of this window that exist (>= 1)
+        if (lane < 8) {  // values
+          const uint64_t q = uint64_t(lane) * 4;
+          cp16(rw + 4 + lane * 4, a.val + (q < left ? p + q : 0), q < left ? int(left - q >= 4 ? 16 : (left - q) * 4) : 0);
+        }
+#pragma unroll
+        for (int j = 0; j < NO; ++j) {
+          if ((a.wide >> j) & 1u) {
+            if (lane < 8) {
+              const uint64_t q = uint64_t(lane) * 4;
+              cp16(rw + off_e[j] + lane * 4, a.io[j] + (q < left ? p + q : 0),
+                   q < left ? int(left - q >= 4 ? 16 : (left - q) * 4) : 0);
+            }
+          } else if (lane < 2) {
+            const uint64_t q = uint64_t(lane) * 16;
+            cp16(rw + off_e[j] + lane * 4, a.eo[j] + (q < left ? p + q : 0),
+                 q < left ? int(left - q >= 16 ? 16 : left - q) : 0);
+          }
+        }
+        if (lane < 9) {  // 36 slots of ends, rows and bases from the aligned slot sa
+          cp16(rw + off_end + lane * 4, a.sbend32 + sa + lane * 4, 16);
+          cp16(rw + off_row + lane * 4, a.sbrow + sa + lane * 4, 16);
+#pragma unroll
+          for (int j = 0; j < NO; ++j)
+            if (!((a.wide >> j) & 1u)) cp16(rw + off_b[j] + lane * 4, a.sbbase[j] + sa + lane * 4, 16);
+        }
+      }
+    }
+    asm volatile("cp.async.commit_group;" ::: "memory");
+  };
+  // decode a landed raw stage into a stage buffer (same output as decode_to)
+  auto raw_decode = [&](uint64_t cc, int s, uint32_t *dst) {
+    if (cc >= a.nnz) return;
+#pragma unroll 1
+    for (int gi = 0; gi < G; ++gi) {
+      const uint64_t p = cc + uint64_t(gi) * (a.chunk / G) + uint64_t(s) * SG;
+      if (p >= a.nnz) break;
+      const uint32_t *rw = raw + gi * a.raw_words;
+      const uint32_t bi = rw[0] + uint32_t(lane);
+      const uint32_t p32 = uint32_t(p);
+      const uint32_t eabs = rw[off_end + bi];
+      const uint32_t erel = eabs - p32 > 64u ? 64u : eabs - p32;
+      const uint32_t srow = rw[off_row + bi];
+      const bool ok = p + lane < a.nnz;
+      const float v = ok ? __uint_as_float(rw[4 + lane]) : 0.f;
+      uint32_t sbase[NO > 0 ? NO : 1], e[NO > 0 ? NO : 1];
+#pragma unroll
+      for (int j = 0; j < NO; ++j) {
+        const bool wj = (a.wide >> j) & 1u;
+        sbase[j] = wj ? 0u : rw[off_b[j] + bi];
+        e[j] = !ok ? 0u : wj ? rw[off_e[j] + lane] : ((rw[off_e[j] + (lane >> 2)] >> (8 * (lane & 3))) & 0xFFu);
+      }
+      int c = 0;
+#pragma unroll
+      for (int k = 16; k >= 1; k >>= 1) {
+        const uint32_t et = __shfl_sync(0xFFFFFFFFu, erel, c + k - 1);
+        if (et <= uint32_t(lane)) c += k;
+      }
+      const uint32_t row = __shfl_sync(0xFFFFFFFFu, srow, c);
+      const int d = gi * SG + (((lane / 4) ^ (gi / GL)) & (CG - 1)) * 4 + (lane & 3);
+      dst[d] = row;
+#pragma unroll
+      for (int j = 0; j < NO; ++j) dst[(1 + j) * SW + d] = __shfl_sync(0xFFFFFFFFu, sbase[j], c) + e[j];
+      dst[(NA - 1) * SW + d] = __float_as_uint(v);
+    }
+  };
+  uint32_t wsb_next = 0;
+  bool raw_primed = false;
   auto issue = [&](uint64_t cc, int s, int b) {
+    if constexpr (kHicRaw) {
+      uint64_t c2 = cc;
+      int s2 = s;
+      next_pos(c2, s2);
+      if (!raw_primed) {  // first position of this warp: raw-issue it synchronously
+        raw_issue(cc, s, win_of(cc, s));
+        wsb_next = win_of(c2, s2);
+        raw_primed = true;
+      }
+      asm volatile("cp.async.wait_group 0;" ::: "memory");
+      __syncwarp();
+      raw_decode(cc, s, wbuf + b * NA * SW);
+      __syncwarp();  // every lane has read the raw buffer before it is refilled
+      raw_issue(c2, s2, wsb_next);
+      uint64_t c3 = c2;
+      int s3 = s2;
+      next_pos(c3, s3);
+      wsb_next = win_of(c3, s3);
+      return;
+    }
     if constexpr (kHic) {
       decode_to(cc, s, wbuf + b * NA * SW);
       return;
@@ -941,7 +1082,7 @@ __global__ void __launch_bounds__(HS ? WPC_ * 32 : kThreads, HS ? 1 : (WA == 6 ?
           for (int j = 0; j < NO; ++j) {
             if (kGather) {
               const uint32_t id = idx[j][u];
-              if constexpr (WA == 9) {  // decoded HiCOO coordinate: plain factor row
+              if constexpr (WA == 9 || WA == 11) {  // decoded HiCOO coordinate: plain factor row
                 if (u < cnt) f[j][u] = ldg_vec<4>(a.Uo[j] + uint64_t(id) * R + col, pol.gather);
               } else if constexpr (HS) {  // shared-memory tier, L2-tier buffer or plain factor row
                 const bool in_s = (id >> 30) == 3u;
@@ -1380,6 +1521,24 @@ void launch_heavy_lpn(const HArgs &h, int lpn, uint64_t n_pieces, size_t smem, c
 }
 
 namespace {
+// win_sb[w] = last slice s with sbptr[s] <= 32 w; end32[s] = sbptr[s + 1] (u32), nnz past nsb
+__global__ void win_slice_kernel(const uint64_t *__restrict__ sbptr, uint64_t nsb, uint64_t nwin,
+                                 uint32_t *__restrict__ win_sb) {
+  for (uint64_t w = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; w < nwin; w += uint64_t(gridDim.x) * blockDim.x) {
+    const uint64_t x = w * 32;
+    uint64_t lo = 0, hi = nsb;
+    while (hi - lo > 1) {
+      const uint64_t mid = (lo + hi) / 2;
+      if (sbptr[mid] <= x) lo = mid; else hi = mid;
+    }
+    win_sb[w] = uint32_t(lo);
+  }
+}
+__global__ void end32_kernel(const uint64_t *__restrict__ sbptr, uint64_t nsb, uint64_t nnz, uint64_t n,
+                             uint32_t *__restrict__ end32) {
+  for (uint64_t i = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; i < n; i += uint64_t(gridDim.x) * blockDim.x)
+    end32[i] = uint32_t(i < nsb ? sbptr[i + 1] : nnz);
+}
 // run_sb[r] = last slice s with sbptr[s] <= r * run (the slice holding entry r * run)
 __global__ void run_slice_kernel(const uint64_t *__restrict__ sbptr, uint64_t nsb, uint64_t run,
                                  uint64_t nruns, uint64_t *__restrict__ run_sb) {
@@ -1481,9 +1640,34 @@ void launch_hicoo_mttkrp(const pasta_hicoo *h, uint32_t mode, const float *const
       a.hs_lo[jj] = uint32_t(mc.hs_total);
       if (mc.hot_total) launch_hot_fill(mc, factors, h->order, mode, R, s);
     }
+    // raw-staged decode (WA 11): orders 2 and 3 (R >= 16: a warp's raw windows and stage
+    // buffers fit the 227 KB), no tiers; PASTA_HICOO_RAW=0 keeps the WA 9 decode
+    uint32_t raw_words = 36 + 72;
+    for (int j = 0; j < hno; ++j) raw_words += ((a.wide >> j) & 1u) ? 32 : 8 + 36;
+    const size_t raw_bytes = size_t(16) * G * raw_words * 4;
+    const bool use_raw = !tiers && hno <= 2 && env_int("PASTA_HICOO_RAW", 1) && stage + raw_bytes <= 227 * 1024 &&
+                         h->nnz < 0xFFFFFFFFull;
+    if (use_raw) {
+      const uint64_t nwin = (h->nnz + 31) / 32;
+      if (mcw.win_sb.n != nwin) {
+        mcw.win_sb.alloc(nwin, s);
+        uint64_t g = (nwin + 255) / 256;
+        if (g > 148 * 32) g = 148 * 32;
+        win_slice_kernel<<<unsigned(g), 256, 0, s>>>(mc.sbptr.p, mc.nsb, nwin, mcw.win_sb.p);
+        PASTA_LAUNCHED();
+        mcw.sbend32.alloc(mc.nsb + kSlicePad, s);
+        g = (mc.nsb + kSlicePad + 255) / 256;
+        if (g > 148 * 32) g = 148 * 32;
+        end32_kernel<<<unsigned(g), 256, 0, s>>>(mc.sbptr.p, mc.nsb, h->nnz, mc.nsb + kSlicePad, mcw.sbend32.p);
+        PASTA_LAUNCHED();
+      }
+      a.win_sb = mcw.win_sb.p;
+      a.sbend32 = mcw.sbend32.p;
+      a.raw_words = raw_words;
+    }
     ProfScope prof(kProfHicoo, s);
     const int cfg = env_int("PASTA_HS_CFG", 0);  // 2 (8-deep steps) spills here
-    const size_t smem = stage + (tiers ? size_t(mc.hs_total) * R * sizeof(float) : 0);
+    const size_t smem = stage + (tiers ? size_t(mc.hs_total) * R * sizeof(float) : 0) + (use_raw ? raw_bytes : 0);
     const uint64_t nwarps = (a.nnz + a.chunk - 1) / a.chunk;
     const uint64_t nblk = std::min<uint64_t>((nwarps + 15) / 16, uint64_t(sm_count()));
     auto go = [&](auto kern) {
@@ -1492,7 +1676,9 @@ void launch_hicoo_mttkrp(const pasta_hicoo *h, uint32_t mode, const float *const
       PASTA_LAUNCHED();
       mcw.fence.record(s);
     };
-    if (tiers)
+    if (use_raw)
+      with_no_lpn<2>(hno, lpn, [&](auto NOt, auto Lt) { go(coo_staged_kernel<NOt.value, Lt.value, 11, true, 16, 32, 4>); });
+    else if (tiers)
       with_no_lpn<3>(hno, lpn, [&](auto NOt, auto Lt) { go(coo_staged_kernel<NOt.value, Lt.value, 10, true, 16, 32, 4>); });
     else if (cfg == 2 && hno <= 2)
       with_no_lpn<2>(hno, lpn, [&](auto NOt, auto Lt) { go(coo_staged_kernel<NOt.value, Lt.value, 9, true, 16, 32, 8>); });
