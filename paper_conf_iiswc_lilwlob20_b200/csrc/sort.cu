@@ -343,11 +343,11 @@ void gather_any(const float *in, const uint32_t *perm, float *out, uint64_t n, c
 
 // die-split segment of each nonzero (R#35); n01 counts the die-0 segments (half of ia == 0)
 __global__ void split_seg_kernel(const uint32_t *__restrict__ ia, const uint32_t *__restrict__ ib, uint64_t M,
-                                 uint32_t ka, uint32_t kb, uint32_t ta, uint32_t tb, uint32_t *__restrict__ seg,
-                                 unsigned long long *__restrict__ n01) {
+                                 uint32_t ka, uint32_t kb, uint32_t ta, uint32_t tb, uint32_t sh,
+                                 uint32_t *__restrict__ seg, unsigned long long *__restrict__ n01) {
   unsigned long long c = 0;
   for (uint64_t x = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; x < M; x += uint64_t(gridDim.x) * blockDim.x) {
-    const uint32_t ha = die_half(ia[x], ka, ta), hb = die_half(ib[x], kb, tb);
+    const uint32_t ha = die_half(ia[x] >> sh, ka, ta), hb = die_half(ib[x] >> sh, kb, tb);
     seg[x] = ha ? (hb ? 2u : 3u) : (hb ? 1u : 0u);
     c += ha == 0;
   }
@@ -397,6 +397,10 @@ void coo_mark_hot(pasta_coo *x, uint32_t mode, uint32_t R, bool global_tier, uin
   // die-0 shares: the first gathered factor in proportion to the dies' SM counts, the second
   // half and half, so both phases of both dies get work in proportion to their SMs
   uint32_t tsplit[kMaxOrder] = {};
+  // the halves are made of 2-KB runs of factor rows (row >> split_sh): a die's L2 keeps whole
+  // lines its SMs read, so rows of the two halves must not share lines (nor 2-KB chunks)
+  uint32_t split_sh = 0;
+  while (split_sh < 16 && (uint64_t(R) * 4u << split_sh) < 2048u) ++split_sh;
   if (die_split) {
     int j = 0;
     for (uint32_t k = 0; k < N; ++k) {
@@ -467,8 +471,8 @@ void coo_mark_hot(pasta_coo *x, uint32_t mode, uint32_t R, bool global_tier, uin
         part.reserve(hl.size());
         PASTA_CUDA(cudaMemcpyAsync(hl.data(), lists[k].p, hl.size() * 4, cudaMemcpyDeviceToHost, s));
         PASTA_CUDA(cudaStreamSynchronize(s));
-        for (uint32_t r : hl) if (die_half(r, k, tsplit[k]) == 0) part.push_back(r);
-        for (uint32_t r : hl) if (die_half(r, k, tsplit[k]) == 1) part.push_back(r);
+        for (uint32_t r : hl) if (die_half(r >> split_sh, k, tsplit[k]) == 0) part.push_back(r);
+        for (uint32_t r : hl) if (die_half(r >> split_sh, k, tsplit[k]) == 1) part.push_back(r);
         PASTA_CUDA(cudaMemcpyAsync(lists[k].p, part.data(), part.size() * 4, cudaMemcpyHostToDevice, s));
         PASTA_CUDA(cudaStreamSynchronize(s));
       }
@@ -508,8 +512,8 @@ void coo_mark_hot(pasta_coo *x, uint32_t mode, uint32_t R, bool global_tier, uin
     DevArray<uint32_t> seg(M, s), perm(M, s);
     DevArray<unsigned long long> n01(1, s);
     PASTA_CUDA(cudaMemsetAsync(n01.p, 0, sizeof(unsigned long long), s));
-    split_seg_kernel<<<grid8(M), 256, 0, s>>>(mc.inds[ka], mc.inds[kb], M, ka, kb, tsplit[ka], tsplit[kb], seg.p,
-                                              n01.p);
+    split_seg_kernel<<<grid8(M), 256, 0, s>>>(mc.inds[ka], mc.inds[kb], M, ka, kb, tsplit[ka], tsplit[kb], split_sh,
+                                              seg.p, n01.p);
     PASTA_LAUNCHED();
     iota_u32(perm.p, M, s);
     const uint32_t *comps[1] = {seg.p};
