@@ -189,6 +189,42 @@ def cpu_oracle_child(args):
                       "modes": list(modes), "nnz": nnz, "cores": cores}), flush=True)
 
 
+def cpu_omp_child(args):
+    """Child process: the paper's CPU method (baselines/: COO-MTTKRP-OMP, fp32 + omp atomic,
+    all host threads) on the same host-drawn workload; prints one JSON line."""
+    import baselines
+    cfg = si.CONFIGS[args.config]
+    dims, R = cfg["dims"], cfg["R"]
+    nnz = min(args.cpu_sample or cfg["nnz"], cfg["nnz"])
+    inds, vals = host_workload(cfg, nnz)
+    U = si.factors(dims, R, seed=cfg["seed"])
+    baselines.build()
+    modes = range(len(dims)) if args.cpu_modes == "all" else [int(m) for m in args.cpu_modes.split(",")]
+    baselines.mttkrp(dims, inds[:, :1000], vals[:1000], 0, U)  # thread-pool warm-up
+    secs = []
+    for n in modes:
+        t0 = time.perf_counter()
+        baselines.mttkrp(dims, inds, vals, n, U)
+        secs.append(time.perf_counter() - t0)
+    flops = sum(model_flops(len(dims), nnz, R) for _ in modes)
+    print(json.dumps({"gflops": flops / sum(secs) / 1e9, "seconds_per_mode": [round(t, 3) for t in secs],
+                      "modes": list(modes), "nnz": nnz, "threads": baselines.threads()}), flush=True)
+
+
+def cpu_omp(args, cfg):
+    cmd = [sys.executable, os.path.abspath(__file__), "--cpu-omp-child", "--config", args.config,
+           "--cpu-modes", args.cpu_modes, "--cpu-sample", str(args.cpu_sample or 0)]
+    try:
+        r = subprocess.run(cmd, capture_output=True, text=True, timeout=900)
+        d = json.loads([l for l in r.stdout.splitlines() if l.startswith("{")][-1])
+    except Exception as e:
+        return {"unavailable": f"omp child failed: {str(e)[:160]}"}
+    return {"value": round(d["gflops"], 3), "unit": "GFLOP/s", "cores": d["threads"],
+            "kind": "paper CPU method (COO-MTTKRP-OMP, fp32, omp atomic; P:157, P:282), not the oracle",
+            "sample": f"the same {d['nnz']} host-drawn nonzeros as cpu_baseline, modes {d['modes']}",
+            "seconds_per_mode": d["seconds_per_mode"]}
+
+
 def cpu_baseline(args, cfg):
     """Run cpu_oracle_child pinned to core 0 (taskset when present) and report it."""
     cmd = [sys.executable, os.path.abspath(__file__), "--cpu-oracle-child", "--config", args.config,
@@ -365,6 +401,7 @@ def main():
     ap.add_argument("--ew-steps", type=int, default=20)
     ap.add_argument("--dram-probe", action="store_true", help=argparse.SUPPRESS)
     ap.add_argument("--cpu-oracle-child", action="store_true", help=argparse.SUPPRESS)
+    ap.add_argument("--cpu-omp-child", action="store_true", help=argparse.SUPPRESS)
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3  # timing rule: >= 3 warm-up steps
@@ -375,6 +412,8 @@ def main():
         return dram_probe_child(args)
     if args.cpu_oracle_child:
         return cpu_oracle_child(args)
+    if args.cpu_omp_child:
+        return cpu_omp_child(args)
     if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
         sys.exit(spawn_ranks(args))
     world, rank, local = dist_env()
@@ -817,9 +856,10 @@ def main():
         counters = dram_counters(args, cfg)
     traffic = counters.get("bytes_per_launch") if counters else None
 
-    cpu = None
+    cpu = comp_omp = None
     if not args.no_cpu_baseline and world == 1:
         cpu = cpu_baseline(args, cfg)
+        comp_omp = cpu_omp(args, cfg)
 
     line = {
         "metric": METRIC, "value": round(value, 3), "unit": "GFLOP/s", "n_gpus": world,
@@ -864,6 +904,7 @@ def main():
         "ttm": ttm,
         "gpu_launches": launches,
         "cpu_baseline": cpu,
+        "cpu_omp": comp_omp,
         "max_shard_nnz": max(shard_nnz),
         "shard_max_over_mean": balance,
     }

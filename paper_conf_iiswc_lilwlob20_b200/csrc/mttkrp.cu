@@ -1369,7 +1369,7 @@ void launch_coo_mttkrp(const pasta_coo *x, uint32_t mode, const float *const *fa
     if (const int cap = env_int("PASTA_HOT_SMEM_ROWS", 0)) hs_rows_budget = std::min(hs_rows_budget, uint32_t(cap));
     bool hs = env_int("PASTA_HOT_SMEM", 1) != 0 && hs_rows_budget >= 64;
     // die split (R#35): order 3 with DRAM-bound gathers (an L2 tier), persistent kernel only
-    const bool split_want = env_int("PASTA_DIE_SPLIT", 1) != 0 && no == 2 && want_hot;
+    const bool split_want = env_int("PASTA_DIE_SPLIT", 0) != 0 && no == 2 && want_hot;
     if (hs) {
       // the nonzero order changes with the die split: wait for launches still reading the copy
       const_cast<CooModeCopy &>(mc).fence.wait(s);
@@ -1645,7 +1645,7 @@ void launch_hicoo_mttkrp(const pasta_hicoo *h, uint32_t mode, const float *const
     uint32_t raw_words = 36 + 72;
     for (int j = 0; j < hno; ++j) raw_words += ((a.wide >> j) & 1u) ? 32 : 8 + 36;
     const size_t raw_bytes = size_t(16) * G * raw_words * 4;
-    const bool use_raw = !tiers && hno <= 2 && env_int("PASTA_HICOO_RAW", 1) && stage + raw_bytes <= 227 * 1024 &&
+    const bool use_raw = !tiers && hno <= 2 && env_int("PASTA_HICOO_RAW", 0) && stage + raw_bytes <= 227 * 1024 &&
                          h->nnz < 0xFFFFFFFFull;
     if (use_raw) {
       const uint64_t nwin = (h->nnz + 31) / 32;

@@ -386,8 +386,9 @@ void coo_mark_hot(pasta_coo *x, uint32_t mode, uint32_t R, bool global_tier, uin
       mc.split == die_split)
     return;
   // die split (R#35): two gathered factors, an L2 tier and a measured SM -> die map
-  const DieMap &dm = die_map();
-  die_split = die_split && global_tier && x->order == 3 && dm.ok;
+  die_split = die_split && global_tier && x->order == 3;
+  const DieMap *dmp = die_split ? &die_map() : nullptr;  // calibrates on first use only
+  die_split = die_split && dmp->ok;
   mc.split = false;
   const char *env = getenv("PASTA_HOT_MB");
   // the die split holds half of each factor's tier per die, so the tier can be larger
@@ -405,7 +406,7 @@ void coo_mark_hot(pasta_coo *x, uint32_t mode, uint32_t R, bool global_tier, uin
     int j = 0;
     for (uint32_t k = 0; k < N; ++k) {
       if (k == mode) continue;
-      tsplit[k] = j == 0 ? uint32_t(4294967296.0 * dm.n[0] / double(dm.n[0] + dm.n[1])) : 0x80000000u;
+      tsplit[k] = j == 0 ? uint32_t(4294967296.0 * dmp->n[0] / double(dmp->n[0] + dmp->n[1])) : 0x80000000u;
       ++j;
     }
   }

@@ -513,7 +513,7 @@ def test_coo_shared_memory_hot_tier(env, l2_tier, hs_cfg, monkeypatch):
         _check(pasta.pasta_mttkrp_coo(x, 1, Ud2), ref, ab, "smem tier refill")
 
 
-@pytest.mark.parametrize("staged", ["1", "0"])
+@pytest.mark.parametrize("staged", ["1", "0", "raw"])
 def test_hicoo_row_slices_staged_decode(env, staged, monkeypatch):
     """HiCOO / gHiCOO row-slice MTTKRP with the slices decoded warp-wide into the staged kernel
     (default) and with the per-group slice walk (PASTA_HICOO_STAGED=0): hypersparse blocks
@@ -521,7 +521,8 @@ def test_hicoo_row_slices_staged_decode(env, staged, monkeypatch):
     hot row (slices longer than any window), R = 16 / 32, orders 2-4, gHiCOO masks with
     uncompressed (32-bit) modes, and enough nonzeros for several chunks per persistent warp."""
     pasta, oracle, torch = env
-    monkeypatch.setenv("PASTA_HICOO_STAGED", staged)
+    monkeypatch.setenv("PASTA_HICOO_STAGED", "0" if staged == "0" else "1")
+    monkeypatch.setenv("PASTA_HICOO_RAW", "1" if staged == "raw" else "0")  # WA 11 raw-staged decode
     cases = [((1 << 20, 1 << 20, 1 << 20), 400_000, 16, "powerlaw", 7, None),
              ((300, 200, 500), 2_500_000, 16, "uniform", 7, None),
              ((600, 500, 400), 200_000, 32, "uniform", 5, None),
