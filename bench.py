@@ -487,8 +487,6 @@ def main():
             if not shared or turn == rank:
                 t0 = time.perf_counter()
                 x = pasta.pasta_gen_powerlaw(dims, M, cfg["seed"], kind=0 if cfg["kind"] == "uniform" else 1)
-                for n in range(N):
-                    pasta.pasta_coo_prepare(x, n)
                 torch.cuda.synchronize()
                 t_gen = time.perf_counter() - t0
                 if scaling == "strong" and rank == 0:
@@ -502,7 +500,8 @@ def main():
                     t1 = timed(step1, max(3, min(args.steps, 10)))
                     del full
                 t0 = time.perf_counter()
-                part = RowPartitionedMTTKRP(x, rank, world, R, dev)
+                # shards cut mode by mode, each full sorted copy released after its shard
+                part = RowPartitionedMTTKRP(x, rank, world, R, dev, release=True)
                 del x
                 torch.cuda.synchronize()
                 t_prep = time.perf_counter() - t0

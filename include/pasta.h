@@ -171,6 +171,10 @@ pasta_status pasta_ghicoo_auto_mask(const pasta_coo *x, uint32_t block_bits, uin
  * binds_mode with entries by einds_mode (dense blocks then run one per CTA with TMA-staged
  * factor tiles).  Optional: MTTKRP prepares on first use. */
 pasta_status pasta_coo_prepare(pasta_coo *x, uint32_t mode, void *stream);
+/* Free the mode-`mode` working copy of `x` and its caches (hot-row tiers, die split), after
+ * the launches that read them; the next use prepares it again.  Lets a caller keep only one
+ * sorted copy alive at a time (e.g. while cutting per-mode shards). */
+pasta_status pasta_coo_release_mode(pasta_coo *x, uint32_t mode);
 pasta_status pasta_hicoo_prepare(pasta_hicoo *h, uint32_t mode, void *stream);
 
 /* --------------------------------------------------------------- MTTKRP (a5-a8) ------ */

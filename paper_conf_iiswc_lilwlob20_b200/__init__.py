@@ -18,7 +18,7 @@ from ._native import MAX_ORDER, Allocator, ALLOC_FN, FREE_FN, GenParams, PastaEr
 __all__ = [
     "PastaError", "Coo", "Hicoo", "pasta_version", "pasta_set_allocator", "use_torch_allocator",
     "pasta_load_coo", "pasta_save_coo", "pasta_coo_from_arrays", "pasta_gen_powerlaw",
-    "pasta_coo_to_hicoo", "pasta_coo_prepare", "pasta_hicoo_prepare", "pasta_mttkrp_coo",
+    "pasta_coo_to_hicoo", "pasta_coo_prepare", "pasta_coo_release_mode", "pasta_hicoo_prepare", "pasta_mttkrp_coo",
     "pasta_mttkrp_hicoo", "pasta_mttkrp_coo_allmodes_host", "pasta_mttkrp_coo_allmodes_host_batch",
     "pasta_coo_row_counts",
     "pasta_row_partition", "pasta_coo_partition", "pasta_coo_shard", "pasta_hicoo_shard", "pasta_coo_info",
@@ -217,6 +217,11 @@ def pasta_ghicoo_auto_mask(x: Coo, block_bits: int = 7):
 
 def pasta_coo_prepare(x: Coo, mode: int, stream=None) -> None:
     check(lib().pasta_coo_prepare(x.ptr, mode, _stream_ptr(stream)))
+
+
+def pasta_coo_release_mode(x: Coo, mode: int) -> None:
+    """Free the mode-`mode` working copy and its caches (rebuilt on next use)."""
+    check(lib().pasta_coo_release_mode(x.ptr, mode))
 
 
 def pasta_hicoo_prepare(h: Hicoo, mode: int, stream=None) -> None:

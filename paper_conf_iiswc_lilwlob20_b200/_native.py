@@ -63,6 +63,7 @@ SIGNATURES = {
     "pasta_ghicoo_export": (_st, [_vp, _u64p, C.POINTER(_u32p), C.POINTER(_u8p), C.POINTER(_u32p), _f32p]),
     "pasta_coo_prepare": (_st, [_vp, C.c_uint32, _vp]),
     "pasta_hicoo_prepare": (_st, [_vp, C.c_uint32, _vp]),
+    "pasta_coo_release_mode": (_st, [_vp, C.c_uint32]),
     "pasta_mttkrp_coo": (_st, [_vp, C.c_uint32, C.POINTER(_vp), C.c_uint32, _vp, _vp]),
     "pasta_mttkrp_hicoo": (_st, [_vp, C.c_uint32, C.POINTER(_vp), C.c_uint32, _vp, _vp]),
     "pasta_mttkrp_coo_allmodes_host": (_st, [_vp, C.POINTER(_vp), C.c_uint32, C.POINTER(_vp), _vp]),

@@ -567,6 +567,34 @@ pasta_status pasta_coo_prepare(pasta_coo *x, uint32_t mode, void *stream) {
   API_END
 }
 
+pasta_status pasta_coo_release_mode(pasta_coo *x, uint32_t mode) {
+  API_BEGIN
+  require(x != nullptr, "x is NULL");
+  require(mode < x->order, "mode >= order");
+  check_device(x->device);
+  std::lock_guard<std::mutex> lk(x->mu);
+  CooModeCopy &mc = x->mc[mode];
+  if (mc.fence.e) PASTA_CUDA(cudaEventSynchronize(mc.fence.e));  // launches still reading it
+  for (uint32_t k = 0; k < kMaxOrder; ++k) {
+    mc.own_inds[k].reset();
+    mc.hot_inds[k].reset();
+    mc.inds[k] = nullptr;
+  }
+  mc.own_val.reset();
+  mc.val = nullptr;
+  mc.hot_rows.reset();
+  mc.hot_buf.reset();
+  mc.hs_rows.reset();
+  mc.split_irow.reset();
+  mc.split_val.reset();
+  mc.claim.reset();
+  mc.hot_R = 0;
+  mc.hot_total = mc.hs_total = 0;
+  mc.split = false;
+  mc.ready = false;
+  API_END
+}
+
 pasta_status pasta_hicoo_prepare(pasta_hicoo *h, uint32_t mode, void *stream) {
   API_BEGIN
   require(h != nullptr, "h is NULL");

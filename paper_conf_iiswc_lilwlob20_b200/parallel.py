@@ -92,13 +92,15 @@ def partition_bounds(counts_per_mode: Sequence[np.ndarray], world: int) -> List[
 class RowPartitionedMTTKRP:
     """Holds this rank's per-mode shards of a COO tensor and runs all-mode MTTKRP steps.
     fmt="hicoo": the shards are HiCOO (pasta_hicoo_shard of the tensor's HiCOO form with
-    block_bits, or of `hicoo` when given) and the step runs the HiCOO MTTKRP."""
+    block_bits, or of `hicoo` when given) and the step runs the HiCOO MTTKRP.  release=True
+    frees each mode's full sorted copy of `x` once its shard is cut."""
 
     def __init__(self, x, rank: int, world: int, R: int, device, fmt: str = "coo", block_bits: int = 7,
-                 hicoo=None):
+                 hicoo=None, release: bool = False):
         import torch
 
-        from . import pasta_coo_partition, pasta_coo_shard, pasta_coo_to_hicoo, pasta_hicoo_shard
+        from . import (pasta_coo_partition, pasta_coo_release_mode, pasta_coo_shard, pasta_coo_to_hicoo,
+                       pasta_hicoo_shard)
         self.rank, self.world, self.R, self.fmt = rank, world, R, fmt
         self.order, self.dims, self.nnz = x.order, x.dims, x.nnz
         self.bounds = [pasta_coo_partition(x, n, world) for n in range(x.order)]
@@ -109,6 +111,8 @@ class RowPartitionedMTTKRP:
         for n in range(x.order):
             lo, hi = int(self.bounds[n][rank]), int(self.bounds[n][rank + 1])
             self.shards.append(pasta_hicoo_shard(h, n, lo, hi) if h is not None else pasta_coo_shard(x, n, lo, hi))
+            if release:  # keep one full sorted copy alive at a time (bounded peak memory)
+                pasta_coo_release_mode(x, n)
         del h
         self.out = [torch.empty((d, R), dtype=torch.float32, device=device) for d in self.dims]
 

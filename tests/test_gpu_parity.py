@@ -217,6 +217,9 @@ def test_shards_cover_the_output(env):
                 pasta.pasta_mttkrp_coo(s, n, Ud, out=out)  # writes only its rows
             assert total == vals.shape[0]
             _check(out, ref, ab, f"shards mode {n} P={P}")
+        # the full sorted copy freed after sharding is rebuilt on the next use
+        pasta.pasta_coo_release_mode(x, n)
+        _check(pasta.pasta_mttkrp_coo(x, n, Ud), ref, ab, f"after release mode {n}")
 
 
 @pytest.mark.parametrize("cmask", [0b111, 0b101])
