@@ -5,8 +5,9 @@
   compute-sanitizer --tool memcheck|racecheck|synccheck --error-exitcode 9 \
       python tests/sanitize_cases.py
 
-COO MTTKRP (N = 3, 4; R = 8, 16, 32; default and forced hot-row cache), HiCOO and gHiCOO
-MTTKRP, mode sort, TTV / TTM, CP-ALS, TS / TEW, both generators."""
+COO MTTKRP (N = 3, 4; R = 8, 16, 32; default and forced hot-row cache, die split), HiCOO
+(staged decode, raw-staged decode, hot-block tiers, shards) and gHiCOO MTTKRP, mode sort,
+TTV / TTM, CP-ALS (incl. the fit kernel), TS / TEW, both generators (with relabelling)."""
 import os
 import sys
 
@@ -42,8 +43,23 @@ def main():
             for force in ("0", "1"):
                 os.environ["PASTA_HOT_FORCE"] = force
                 close(pasta.pasta_mttkrp_coo(x, n, Ud), ref, ab, (dims, R, n, "coo", force))
+            if len(dims) == 3:  # die-split COO (R#35), forced
+                os.environ["PASTA_HOT_FORCE"] = "1"
+                os.environ["PASTA_DIE_SPLIT"] = "1"
+                close(pasta.pasta_mttkrp_coo(x, n, Ud), ref, ab, (dims, R, n, "coo split"))
+                os.environ["PASTA_DIE_SPLIT"] = "0"
             os.environ["PASTA_HOT_FORCE"] = "0"
             close(pasta.pasta_mttkrp_hicoo(h, n, Ud), ref, ab, (dims, R, n, "hicoo"))
+            for env in ("PASTA_HICOO_RAW", "PASTA_HICOO_HOT"):  # WA 11 raw decode, WA 10 hot blocks
+                os.environ[env] = "1"
+                close(pasta.pasta_mttkrp_hicoo(h, n, Ud), ref, ab, (dims, R, n, "hicoo", env))
+                os.environ[env] = "0"
+            bounds = pasta.pasta_coo_partition(x, n, 2)
+            out = torch.zeros((dims[n], R), device="cuda")
+            for p in range(2):
+                pasta.pasta_mttkrp_hicoo(pasta.pasta_hicoo_shard(h, n, int(bounds[p]), int(bounds[p + 1])), n, Ud,
+                                         out=out)
+            close(out, ref, ab, (dims, R, n, "hicoo shards"))
             close(pasta.pasta_mttkrp_hicoo(g, n, Ud), ref, ab, (dims, R, n, "ghicoo"))
             si_, sv_ = pasta.pasta_coo_export_mode(x, n)
             oi, ov = oracle.mode_sort(inds, vals, n)
@@ -85,6 +101,10 @@ def main():
         gi, gv = pasta.pasta_coo_export(x)
         oi, ov = fn(dims, 5000, 3)
         assert np.array_equal(gi, oi) and np.array_equal(gv, ov), kind
+    x = pasta.pasta_gen_powerlaw((1000, 700, 33), 5000, 3, permute=1)  # relabelled (R#22)
+    gi, gv = pasta.pasta_coo_export(x)
+    oi, ov = oracle.gen_powerlaw((1000, 700, 33), 5000, 3, permute=True)
+    assert np.array_equal(gi, oi) and np.array_equal(gv, ov), "permute"
     print("ok generators", flush=True)
     torch.cuda.synchronize()
     print("sanitize cases done", flush=True)
