@@ -773,17 +773,18 @@ __global__ void __launch_bounds__(HS ? WPC_ * 32 : kThreads, HS ? 1 : (WA == 6 ?
     __syncthreads();
   }
   // the nonzero range this CTA works on: all of them, or its die's half (die split)
-  uint64_t xbeg = 0, xend = a.nnz;
-  int die = 0;
+  // die split (dyn): die 0's range is [0, split_x), die 1's [split_x, nnz); a CTA claims the
+  // chunks of its own die's range first, then (work stealing) the other die's, so every chunk is
+  // processed whatever the CTA placement (a CTA may not exist on some die at all)
   const bool dyn = HS && !kHic && a.split;
+  int die = 0;
   if (dyn) {
     uint32_t sm;
     asm volatile("mov.u32 %0, %%smid;" : "=r"(sm));
     die = a.die_of[sm];
-    xbeg = die ? a.split_x : 0;
-    xend = die ? a.nnz : a.split_x;
   }
-  const uint64_t nchunks = (xend - xbeg + a.chunk - 1) / a.chunk;
+  auto range_end = [&](uint64_t c) { return (dyn && c < a.split_x) ? a.split_x : a.nnz; };
+  const uint64_t nchunks = (a.nnz + a.chunk - 1) / a.chunk;  // static schedule
   const uint64_t wstep = HS ? uint64_t(gridDim.x) * WPC : nchunks;
   const uint64_t run = a.chunk / G;  // multiple of SG
   const int nstages = int(run / SG);
@@ -801,6 +802,7 @@ __global__ void __launch_bounds__(HS ? WPC_ * 32 : kThreads, HS ? 1 : (WA == 6 ?
   // issue the cp.async copies of stage s of the chunk starting at cc into dst (one commit
   // group; an empty group when cc is past the end, so that wait_group counts stay uniform)
   auto issue_to = [&](uint64_t cc, int s, uint32_t *dst) {
+    const uint64_t xend = range_end(cc);
     if (cc < xend) {
       for (int i = lane; i < SW / 4; i += 32) {  // 16-B chunks of one array
         const int gi = i / (SG / 4), k = i % (SG / 4);
@@ -1025,20 +1027,42 @@ __global__ void __launch_bounds__(HS ? WPC_ * 32 : kThreads, HS ? 1 : (WA == 6 ?
   // one atomic per chunk -- the CTA -> SM placement is not known in advance, so a static
   // split by die rank could skip or repeat chunks.  The claim of the chunk after next is
   // issued at the start of a chunk and consumed at its end (its latency hides behind it).
-  auto claim_issue = [&]() -> unsigned long long {
+  auto claim_issue = [&](int d) -> unsigned long long {
     unsigned long long v = 0;
-    if (lane == 0) v = atomicAdd(a.claim + die, 1ull);
+    if (lane == 0) v = atomicAdd(a.claim + d, 1ull);
     return v;
   };
   auto claim_get = [&](unsigned long long v) { return uint64_t(__shfl_sync(0xFFFFFFFFu, v, 0)); };
+  const uint64_t kDone = a.nnz;
+  int dcl = die;            // die range currently claimed from
+  bool stolen = false;      // switched to the other die's range
+  // chunk index v of range d -> first entry, or (range exhausted) steal once from the other
+  auto resolve = [&](uint64_t v, int d) -> uint64_t {
+    for (;;) {
+      const uint64_t base = d ? a.split_x : 0, end = d ? a.nnz : a.split_x;
+      if (v < (end - base + a.chunk - 1) / a.chunk) return base + v * a.chunk;
+      if (stolen) return kDone;
+      stolen = true;
+      dcl = d = 1 - d;
+      v = claim_get(claim_issue(d));
+    }
+  };
   int bsel = 0;
-  uint64_t w = dyn ? claim_get(claim_issue()) : uint64_t(blockIdx.x) * WPC + warp;
-  uint64_t wn = dyn ? (w < nchunks ? claim_get(claim_issue()) : nchunks) : w + wstep;
-  if (w < nchunks) issue(xbeg + w * a.chunk, 0, 0);
-  while (w < nchunks) {
-  const unsigned long long wnn_v = (dyn && wn < nchunks) ? claim_issue() : 0ull;
-  const uint64_t c0 = xbeg + w * a.chunk;
+  uint64_t c0, cn;  // first entry of the current / next chunk (kDone: none)
+  if (dyn) {
+    c0 = resolve(claim_get(claim_issue(dcl)), dcl);
+    cn = c0 < kDone ? resolve(claim_get(claim_issue(dcl)), dcl) : kDone;
+  } else {
+    const uint64_t w0 = uint64_t(blockIdx.x) * WPC + warp;
+    c0 = w0 < nchunks ? w0 * a.chunk : kDone;
+    cn = w0 + wstep < nchunks ? (w0 + wstep) * a.chunk : kDone;
+  }
+  if (c0 < kDone) issue(c0, 0, 0);
+  while (c0 < kDone) {
+  const int dpend = dcl;  // claim of the chunk after next, in flight during this chunk
+  const unsigned long long pend = (dyn && cn < kDone) ? claim_issue(dpend) : 0ull;
   const uint64_t x0 = c0 + uint64_t(g) * run;
+  const uint64_t xend = range_end(c0);
   const uint64_t x1 = (x0 + run < xend) ? x0 + run : xend;
   Vec<4> acc;
 #pragma unroll
@@ -1048,7 +1072,7 @@ __global__ void __launch_bounds__(HS ? WPC_ * 32 : kThreads, HS ? 1 : (WA == 6 ?
   const bool active = x0 < x1 && col < R;
   for (int s = 0; s < nstages; ++s) {
     if (s + 1 < nstages) issue(c0, s + 1, bsel ^ 1);
-    else issue(wn < nchunks ? xbeg + wn * a.chunk : xend, 0, bsel ^ 1);
+    else issue(cn, 0, bsel ^ 1);
     asm volatile("cp.async.wait_group 1;" ::: "memory");
     __syncwarp();
     const uint32_t *buf = wbuf + bsel * NA * SW + g * SG;
@@ -1153,8 +1177,10 @@ __global__ void __launch_bounds__(HS ? WPC_ * 32 : kThreads, HS ? 1 : (WA == 6 ?
   }
   if (active && cur != 0xFFFFFFFFu && (kWrite || acc.v[0] == 1.2345e-30f))
     red_vec<4>(a.out + uint64_t(cur) * R + col, acc, pol.out);
-  w = wn;
-  wn = dyn ? (w < nchunks ? claim_get(wnn_v) : nchunks) : w + wstep;
+  const uint64_t cprev = c0;
+  c0 = cn;
+  if (dyn) cn = c0 < kDone ? resolve(claim_get(pend), dpend) : kDone;
+  else cn = (c0 < kDone && cprev / a.chunk + 2 * wstep < nchunks) ? (cprev / a.chunk + 2 * wstep) * a.chunk : kDone;
   }  // chunk loop
 }
 
