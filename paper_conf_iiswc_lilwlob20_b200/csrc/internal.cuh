@@ -65,7 +65,9 @@ struct DevArray {
   void alloc(size_t count, cudaStream_t s = nullptr) {
     reset();
     n = count;
-    p = static_cast<T *>(dev_alloc((count ? count : 1) * sizeof(T), s));
+    // rounded up to 64 bytes: the kernels' 16-byte vector and cp.async reads of a ragged tail
+    // (with a partial src-size) stay inside the allocation
+    p = static_cast<T *>(dev_alloc(((count ? count : 1) * sizeof(T) + 63) & ~size_t(63), s));
   }
   void reset() {
     if (p) dev_free(p, nullptr);
