@@ -194,7 +194,9 @@ pasta_status pasta_hicoo_prepare(pasta_hicoo *h, uint32_t mode, void *stream);
  * L2-tier buffer is per handle and refilled from `factors` at every launch; the library
  * orders same-handle launches that use it (a launch on another stream waits for the previous
  * one through an event), so concurrent calls are safe but do not overlap.  Thread-safe: the
- * handle's caches are built and the launches enqueued under the handle's lock. */
+ * handle's caches are built and the launches enqueued under the handle's lock.  The cache tags
+ * use the top two bits of the indices, so it is off for tensors with a dimension >= 2^30 (the
+ * kernels then gather every row from the factors). */
 pasta_status pasta_mttkrp_coo(pasta_coo *x, uint32_t mode, const float *const *factors,
                               uint32_t R, float *out, void *stream);
 pasta_status pasta_mttkrp_hicoo(pasta_hicoo *h, uint32_t mode, const float *const *factors,
