@@ -833,48 +833,67 @@ __global__ void __launch_bounds__(HS ? WPC_ * 32 : kThreads, HS ? 1 : (WA == 6 ?
   // slot ends; row and block bases come from the owning lane by shuffle; i_k = base + e_k
   // (Alg. 3's rebased pointers).  gsb[g] = current slice of group g (warp-uniform).
   uint64_t gsb[G];
+  // The loads of GB groups' windows are issued together (branch-free, so the compiler can
+  // hoist them past the previous group's shuffles) before any is consumed: one memory latency
+  // per batch of groups instead of one per group.
   auto decode_to = [&](uint64_t cc, int s, uint32_t *dst) {
     if (cc >= a.nnz) return;
     const uint64_t r0 = cc / run;
+    if (s == 0) {
+      const uint64_t nruns = (a.nnz + run - 1) / run;
 #pragma unroll
-    for (int gi = 0; gi < G; ++gi) {
-      const uint64_t p = cc + uint64_t(gi) * run + uint64_t(s) * SG;
-      if (p >= a.nnz) continue;  // warp-uniform
-      if (s == 0) gsb[gi] = __ldg(a.run_sb + r0 + gi);
-      const uint64_t sb0 = gsb[gi];
-      const uint64_t st = sb0 + lane < a.nsb ? sb0 + lane : a.nsb - 1;
-      const uint64_t eabs = __ldg(a.sbptr + st + 1);
-      const uint32_t erel = eabs - p > 64 ? 64u : uint32_t(eabs - p);
-      const uint32_t srow = __ldg(a.sbrow + st);
-      uint32_t sbase[NO];
+      for (int gi = 0; gi < G; ++gi) gsb[gi] = __ldg(a.run_sb + (r0 + gi < nruns ? r0 + gi : nruns - 1));
+    }
+    constexpr int GB = G < 4 ? G : (NO >= 3 ? 2 : 4);
+    constexpr int NOA = NO > 0 ? NO : 1;
 #pragma unroll
-      for (int j = 0; j < NO; ++j) sbase[j] = ((a.wide >> j) & 1u) ? 0u : __ldg(a.sbbase[j] + st);
-      const uint64_t x = p + lane;
-      const bool ok = x < a.nnz;
-      const float v = ok ? __ldg(a.val + x) : 0.f;
-      uint32_t e[NO];
+    for (int gb = 0; gb < G; gb += GB) {
+      uint64_t eabs[GB];
+      uint32_t srow[GB], sbase[GB][NOA], e[GB][NOA];
+      float v[GB];
 #pragma unroll
-      for (int j = 0; j < NO; ++j)
-        e[j] = !ok ? 0u : ((a.wide >> j) & 1u) ? __ldg(a.io[j] + x) : uint32_t(__ldg(a.eo[j] + x));
-      int c = 0;  // <= 31: slot 0 holds entry p, so 32 entries span at most 32 slots
+      for (int q = 0; q < GB; ++q) {  // loads only
+        const uint64_t p = cc + uint64_t(gb + q) * run + uint64_t(s) * SG;
+        const uint64_t sb0 = gsb[gb + q];
+        const uint64_t st = sb0 + lane < a.nsb ? sb0 + lane : a.nsb - 1;
+        eabs[q] = __ldg(a.sbptr + st + 1);
+        srow[q] = __ldg(a.sbrow + st);
 #pragma unroll
-      for (int k = 16; k >= 1; k >>= 1) {
-        const uint32_t et = __shfl_sync(0xFFFFFFFFu, erel, c + k - 1);
-        if (et <= uint32_t(lane)) c += k;
+        for (int j = 0; j < NO; ++j) sbase[q][j] = ((a.wide >> j) & 1u) ? 0u : __ldg(a.sbbase[j] + st);
+        const uint64_t x = p + lane;
+        const bool ok = x < a.nnz;
+        v[q] = ok ? __ldg(a.val + x) : 0.f;
+#pragma unroll
+        for (int j = 0; j < NO; ++j)
+          e[q][j] = !ok ? 0u : ((a.wide >> j) & 1u) ? __ldg(a.io[j] + x) : uint32_t(__ldg(a.eo[j] + x));
       }
-      const uint32_t row = __shfl_sync(0xFFFFFFFFu, srow, c);
-      const int d = gi * SG + (((lane / 4) ^ (gi / GL)) & (CG - 1)) * 4 + (lane & 3);
-      dst[d] = row;
 #pragma unroll
-      for (int j = 0; j < NO; ++j) dst[(1 + j) * SW + d] = __shfl_sync(0xFFFFFFFFu, sbase[j], c) + e[j];
-      dst[(NA - 1) * SW + d] = __float_as_uint(v);
-      // the next window starts at the slice holding entry p + SG: the last entry's slice, or
-      // the one after it when that slice ends inside this window
-      const uint64_t nleft = a.nnz - p;
-      const int last = nleft >= uint64_t(SG) ? SG - 1 : int(nleft) - 1;
-      const int clast = __shfl_sync(0xFFFFFFFFu, c, last);
-      const uint32_t elast = __shfl_sync(0xFFFFFFFFu, erel, clast);
-      gsb[gi] = sb0 + uint64_t(clast) + (elast <= uint32_t(SG) ? 1u : 0u);
+      for (int q = 0; q < GB; ++q) {
+        const int gi = gb + q;
+        const uint64_t p = cc + uint64_t(gi) * run + uint64_t(s) * SG;
+        if (p >= a.nnz) continue;  // warp-uniform
+        const uint64_t sb0 = gsb[gi];
+        const uint32_t erel = eabs[q] - p > 64 ? 64u : uint32_t(eabs[q] - p);
+        int c = 0;  // <= 31: slot 0 holds entry p, so 32 entries span at most 32 slots
+#pragma unroll
+        for (int k = 16; k >= 1; k >>= 1) {
+          const uint32_t et = __shfl_sync(0xFFFFFFFFu, erel, c + k - 1);
+          if (et <= uint32_t(lane)) c += k;
+        }
+        const uint32_t row = __shfl_sync(0xFFFFFFFFu, srow[q], c);
+        const int d = gi * SG + (((lane / 4) ^ (gi / GL)) & (CG - 1)) * 4 + (lane & 3);
+        dst[d] = row;
+#pragma unroll
+        for (int j = 0; j < NO; ++j) dst[(1 + j) * SW + d] = __shfl_sync(0xFFFFFFFFu, sbase[q][j], c) + e[q][j];
+        dst[(NA - 1) * SW + d] = __float_as_uint(v[q]);
+        // the next window starts at the slice holding entry p + SG: the last entry's slice, or
+        // the one after it when that slice ends inside this window
+        const uint64_t nleft = a.nnz - p;
+        const int last = nleft >= uint64_t(SG) ? SG - 1 : int(nleft) - 1;
+        const int clast = __shfl_sync(0xFFFFFFFFu, c, last);
+        const uint32_t elast = __shfl_sync(0xFFFFFFFFu, erel, clast);
+        gsb[gi] = sb0 + uint64_t(clast) + (elast <= uint32_t(SG) ? 1u : 0u);
+      }
     }
   };
   // ---- WA 11: raw windows.  Per group window (32 entries from p, slices from sb0), at word
