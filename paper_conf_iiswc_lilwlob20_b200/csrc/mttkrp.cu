@@ -149,16 +149,28 @@ __device__ __forceinline__ Vec<VW> ldg_vec(const float *p, uint64_t pol) {
 
 // One predicated 128-bit load from either shared memory (ps) or global memory (pg), without a
 // branch: divergent per-group branches would serialise the batch of independent gathers.
+template <bool L1NA = false>
 __device__ __forceinline__ Vec<4> ld_tiered(uint32_t saddr, const float *gp, uint64_t pol, int ps, int pg) {
   Vec<4> r;
-  asm volatile(
-      "{\n\t.reg .pred ps, pg;\n\t"
-      "setp.ne.s32 ps, %5, 0;\n\t"
-      "setp.ne.s32 pg, %6, 0;\n\t"
-      "@ps ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];\n\t"
-      "@pg ld.global.nc.L2::cache_hint.v4.f32 {%0, %1, %2, %3}, [%7], %8;\n\t}"
-      : "=f"(r.v[0]), "=f"(r.v[1]), "=f"(r.v[2]), "=f"(r.v[3])
-      : "r"(saddr), "r"(ps), "r"(pg), "l"(gp), "l"(pol));
+  if constexpr (L1NA) {  // the global gather does not allocate in L1
+    asm volatile(
+        "{\n\t.reg .pred ps, pg;\n\t"
+        "setp.ne.s32 ps, %5, 0;\n\t"
+        "setp.ne.s32 pg, %6, 0;\n\t"
+        "@ps ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];\n\t"
+        "@pg ld.global.nc.L1::no_allocate.L2::cache_hint.v4.f32 {%0, %1, %2, %3}, [%7], %8;\n\t}"
+        : "=f"(r.v[0]), "=f"(r.v[1]), "=f"(r.v[2]), "=f"(r.v[3])
+        : "r"(saddr), "r"(ps), "r"(pg), "l"(gp), "l"(pol));
+  } else {
+    asm volatile(
+        "{\n\t.reg .pred ps, pg;\n\t"
+        "setp.ne.s32 ps, %5, 0;\n\t"
+        "setp.ne.s32 pg, %6, 0;\n\t"
+        "@ps ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];\n\t"
+        "@pg ld.global.nc.L2::cache_hint.v4.f32 {%0, %1, %2, %3}, [%7], %8;\n\t}"
+        : "=f"(r.v[0]), "=f"(r.v[1]), "=f"(r.v[2]), "=f"(r.v[3])
+        : "r"(saddr), "r"(ps), "r"(pg), "l"(gp), "l"(pol));
+  }
   return r;
 }
 
@@ -1137,8 +1149,8 @@ __global__ void __launch_bounds__(HS ? WPC_ * 32 : kThreads, HS ? 1 : (WA == 6 ?
                     f[j][u] = ld_tiered3(hs_saddr + uint32_t(off) * 4u, gptr, pol.gather, pol.cold, u < cnt && in_s,
                                          u < cnt && in_h, u < cnt && !in_s && !in_h);
                   else
-                    f[j][u] = ld_tiered(hs_saddr + uint32_t(off) * 4u, gptr, pol.gather, u < cnt && in_s,
-                                        u < cnt && !in_s);
+                    f[j][u] = ld_tiered<WA == 13>(hs_saddr + uint32_t(off) * 4u, gptr, pol.gather, u < cnt && in_s,
+                                                  u < cnt && !in_s);
                 } else {
                   const uint32_t boff = ((id & 0x3FFFFFFFu) * R + col) * 4u;  // < 4 GB
                   const float *gptr = reinterpret_cast<const float *>(
@@ -1532,6 +1544,8 @@ void launch_coo_mttkrp(const pasta_coo *x, uint32_t mode, const float *const *fa
       if (hs_cfg == 1) pick_hs(std::integral_constant<int, 24>(), I16());
       else if (hs_cfg == 2 && no <= 2 && l2t && (a.cache_mode & 8u))  // cold gathers evict_first
         with_no_lpn<2>(no, lpn, [&](auto NOt, auto Lt) { go(coo_staged_kernel<NOt.value, Lt.value, 12, true, 16, 32, 8>); });
+      else if (hs_cfg == 2 && no <= 2 && l2t && env_int("PASTA_GATHER_L1NA", 0))  // gathers skip L1
+        with_no_lpn<2>(no, lpn, [&](auto NOt, auto Lt) { go(coo_staged_kernel<NOt.value, Lt.value, 13, true, 16, 32, 8>); });
       else if (hs_cfg == 2 && no <= 2)
         with_no_lpn<2>(no, lpn, [&](auto NOt, auto Lt) { go(coo_staged_kernel<NOt.value, Lt.value, 1, true, 16, 32, 8>); });
       else pick_hs(I16(), std::integral_constant<int, 32>());
