@@ -856,11 +856,15 @@ __global__ void __launch_bounds__(HS ? WPC_ * 32 : kThreads, HS ? 1 : (WA == 6 ?
 #pragma unroll
       for (int gi = 0; gi < G; ++gi) gsb[gi] = __ldg(a.run_sb + (r0 + gi < nruns ? r0 + gi : nruns - 1));
     }
+#ifdef PASTA_DECODE_GB
+    constexpr int GB = G < PASTA_DECODE_GB ? G : PASTA_DECODE_GB;
+#else
     constexpr int GB = G < 4 ? G : (NO >= 3 ? 2 : 4);
+#endif
     constexpr int NOA = NO > 0 ? NO : 1;
 #pragma unroll
     for (int gb = 0; gb < G; gb += GB) {
-      uint64_t eabs[GB];
+      uint32_t eabs[GB];
       uint32_t srow[GB], sbase[GB][NOA], e[GB][NOA];
       float v[GB];
 #pragma unroll
@@ -868,7 +872,7 @@ __global__ void __launch_bounds__(HS ? WPC_ * 32 : kThreads, HS ? 1 : (WA == 6 ?
         const uint64_t p = cc + uint64_t(gb + q) * run + uint64_t(s) * SG;
         const uint64_t sb0 = gsb[gb + q];
         const uint64_t st = sb0 + lane < a.nsb ? sb0 + lane : a.nsb - 1;
-        eabs[q] = __ldg(a.sbptr + st + 1);
+        eabs[q] = __ldg(a.sbend32 + st);  // = sbptr[st + 1]
         srow[q] = __ldg(a.sbrow + st);
 #pragma unroll
         for (int j = 0; j < NO; ++j) sbase[q][j] = ((a.wide >> j) & 1u) ? 0u : __ldg(a.sbbase[j] + st);
@@ -885,7 +889,7 @@ __global__ void __launch_bounds__(HS ? WPC_ * 32 : kThreads, HS ? 1 : (WA == 6 ?
         const uint64_t p = cc + uint64_t(gi) * run + uint64_t(s) * SG;
         if (p >= a.nnz) continue;  // warp-uniform
         const uint64_t sb0 = gsb[gi];
-        const uint32_t erel = eabs[q] - p > 64 ? 64u : uint32_t(eabs[q] - p);
+        const uint32_t erel = eabs[q] - uint32_t(p) > 64u ? 64u : eabs[q] - uint32_t(p);
         int c = 0;  // <= 31: slot 0 holds entry p, so 32 entries span at most 32 slots
 #pragma unroll
         for (int k = 16; k >= 1; k >>= 1) {
@@ -1422,7 +1426,7 @@ void launch_coo_mttkrp(const pasta_coo *x, uint32_t mode, const float *const *fa
     const size_t smem_cap = 227 * 1024;
     uint32_t hs_rows_budget =
         stage_hs < smem_cap ? uint32_t((smem_cap - stage_hs) / (size_t(R) * sizeof(float))) : 0u;
-    if (want_hot) hs_rows_budget = std::min(hs_rows_budget, 512u);
+    if (want_hot) hs_rows_budget = std::min(hs_rows_budget, uint32_t(env_int("PASTA_HOT_SMEM_DRAM", 512)));
     if (const int cap = env_int("PASTA_HOT_SMEM_ROWS", 0)) hs_rows_budget = std::min(hs_rows_budget, uint32_t(cap));
     bool hs = env_int("PASTA_HOT_SMEM", 1) != 0 && hs_rows_budget >= 64;
     // die split (R#35): order 3 with DRAM-bound gathers (an L2 tier), persistent kernel only
@@ -1706,6 +1710,15 @@ void launch_hicoo_mttkrp(const pasta_hicoo *h, uint32_t mode, const float *const
     const size_t raw_bytes = size_t(16) * G * raw_words * 4;
     const bool use_raw = !tiers && hno <= 2 && env_int("PASTA_HICOO_RAW", 0) && stage + raw_bytes <= 227 * 1024 &&
                          h->nnz < 0xFFFFFFFFull;
+    // u32 slice ends (nnz < 2^32 by the API): half the bytes and registers of sbptr in the decode
+    if (mcw.sbend32.n != mc.nsb + kSlicePad) {
+      mcw.sbend32.alloc(mc.nsb + kSlicePad, s);
+      uint64_t g = (mc.nsb + kSlicePad + 255) / 256;
+      if (g > 148 * 32) g = 148 * 32;
+      end32_kernel<<<unsigned(g), 256, 0, s>>>(mc.sbptr.p, mc.nsb, h->nnz, mc.nsb + kSlicePad, mcw.sbend32.p);
+      PASTA_LAUNCHED();
+    }
+    a.sbend32 = mcw.sbend32.p;
     if (use_raw) {
       const uint64_t nwin = (h->nnz + 31) / 32;
       if (mcw.win_sb.n != nwin) {
@@ -1714,14 +1727,8 @@ void launch_hicoo_mttkrp(const pasta_hicoo *h, uint32_t mode, const float *const
         if (g > 148 * 32) g = 148 * 32;
         win_slice_kernel<<<unsigned(g), 256, 0, s>>>(mc.sbptr.p, mc.nsb, nwin, mcw.win_sb.p);
         PASTA_LAUNCHED();
-        mcw.sbend32.alloc(mc.nsb + kSlicePad, s);
-        g = (mc.nsb + kSlicePad + 255) / 256;
-        if (g > 148 * 32) g = 148 * 32;
-        end32_kernel<<<unsigned(g), 256, 0, s>>>(mc.sbptr.p, mc.nsb, h->nnz, mc.nsb + kSlicePad, mcw.sbend32.p);
-        PASTA_LAUNCHED();
       }
       a.win_sb = mcw.win_sb.p;
-      a.sbend32 = mcw.sbend32.p;
       a.raw_words = raw_words;
     }
     ProfScope prof(kProfHicoo, s);
