@@ -406,6 +406,8 @@ def main():
     if args.warmup < 3:
         args.warmup = 3  # timing rule: >= 3 warm-up steps
     cfg = si.CONFIGS[args.config]
+    if cfg["nnz"] >= 500_000_000:  # C5: the extra legs' copies would not fit next to the COO copies
+        args.hicoo_steps = args.cpals_iters = args.ew_steps = 0
     if args.cpu_sample == 0 and cfg["nnz"] > 200_000_000:
         args.cpu_sample = 100_000_000
     if args.dram_probe:

@@ -201,6 +201,18 @@ pasta_status pasta_mttkrp_coo(pasta_coo *x, uint32_t mode, const float *const *f
                               uint32_t R, float *out, void *stream);
 pasta_status pasta_mttkrp_hicoo(pasta_hicoo *h, uint32_t mode, const float *const *factors,
                                 uint32_t R, float *out, void *stream);
+/* Fused MTTKRP + all-gather over peer memory (a9; SURVEY 8(e) "fused variant"): as
+ * pasta_mttkrp_coo with out = outs[0], and every flush of a finished row segment is also stored
+ * (or atomically added) into outs[1 .. nout) -- the other ranks' replicas of the output,
+ * mapped with pasta_ipc_open -- so the rows this handle owns (all, or its shard's
+ * [row_lo, row_hi)) reach every replica while the kernel runs, tile by tile, over NVLink /
+ * NVSwitch P2P stores instead of a separate collective.  The owned rows are zeroed in every
+ * replica first.  nout in 1..8, all 16-byte aligned.  Ordering: the caller makes sure no rank
+ * still reads its replicas' rows before the call (a collective before it) and that peers read
+ * them only after it (a collective after it on the stream); the kernel ends with a
+ * system-scope fence. */
+pasta_status pasta_mttkrp_coo_bcast(pasta_coo *x, uint32_t mode, const float *const *factors,
+                                    uint32_t R, float *const *outs, uint32_t nout, void *stream);
 
 /* End-to-end variant over ALL modes with HOST buffers (the e2e path): copies the `order`
  * factor matrices host->device (pinned host memory gives full PCIe/C2C bandwidth), computes

@@ -19,7 +19,7 @@ __all__ = [
     "PastaError", "Coo", "Hicoo", "pasta_version", "pasta_set_allocator", "use_torch_allocator",
     "pasta_load_coo", "pasta_save_coo", "pasta_coo_from_arrays", "pasta_gen_powerlaw",
     "pasta_coo_to_hicoo", "pasta_coo_prepare", "pasta_coo_release_mode", "pasta_hicoo_prepare", "pasta_mttkrp_coo",
-    "pasta_mttkrp_hicoo", "pasta_mttkrp_coo_allmodes_host", "pasta_mttkrp_coo_allmodes_host_batch",
+    "pasta_mttkrp_hicoo", "pasta_mttkrp_coo_bcast", "pasta_mttkrp_coo_allmodes_host", "pasta_mttkrp_coo_allmodes_host_batch",
     "pasta_coo_row_counts",
     "pasta_row_partition", "pasta_coo_partition", "pasta_coo_shard", "pasta_hicoo_shard", "pasta_coo_info",
     "pasta_coo_export", "pasta_coo_export_mode", "pasta_hicoo_info", "pasta_hicoo_export",
@@ -284,6 +284,18 @@ def pasta_mttkrp_coo(x: Coo, mode: int, factors, out=None, stream=None, R=None):
     ptrs = _factor_ptrs(x.order, mode, factors, R, x.dims, out.device)
     check(lib().pasta_mttkrp_coo(x.ptr, mode, ptrs, R, C.c_void_p(out.data_ptr()),
                                  _stream_ptr(stream)))
+    return out
+
+
+def pasta_mttkrp_coo_bcast(x: Coo, mode: int, factors, out, dst_ptrs, stream=None, R=None):
+    """Fused MTTKRP + all-gather (include/pasta.h): `out` (local CUDA tensor) and every peer
+    replica in ``dst_ptrs`` (device addresses from pasta_ipc_open) receive the owned rows."""
+    R = _rank(factors, mode, R)
+    _check_out(out, x.dims[mode], R)
+    ptrs = _factor_ptrs(x.order, mode, factors, R, x.dims, out.device)
+    outs = [out.data_ptr()] + [int(p) for p in dst_ptrs]
+    op = (C.c_void_p * len(outs))(*outs)
+    check(lib().pasta_mttkrp_coo_bcast(x.ptr, mode, ptrs, R, op, len(outs), _stream_ptr(stream)))
     return out
 
 

@@ -66,6 +66,7 @@ SIGNATURES = {
     "pasta_coo_release_mode": (_st, [_vp, C.c_uint32]),
     "pasta_mttkrp_coo": (_st, [_vp, C.c_uint32, C.POINTER(_vp), C.c_uint32, _vp, _vp]),
     "pasta_mttkrp_hicoo": (_st, [_vp, C.c_uint32, C.POINTER(_vp), C.c_uint32, _vp, _vp]),
+    "pasta_mttkrp_coo_bcast": (_st, [_vp, C.c_uint32, C.POINTER(_vp), C.c_uint32, C.POINTER(_vp), C.c_uint32, _vp]),
     "pasta_mttkrp_coo_allmodes_host": (_st, [_vp, C.POINTER(_vp), C.c_uint32, C.POINTER(_vp), _vp]),
     "pasta_mttkrp_coo_allmodes_host_batch": (_st, [_vp, C.c_uint32, C.POINTER(_vp), C.c_uint32,
                                                    C.POINTER(_vp), _vp]),

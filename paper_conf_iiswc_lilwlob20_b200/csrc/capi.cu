@@ -634,6 +634,27 @@ pasta_status pasta_mttkrp_coo(pasta_coo *x, uint32_t mode, const float *const *f
   API_END
 }
 
+pasta_status pasta_mttkrp_coo_bcast(pasta_coo *x, uint32_t mode, const float *const *factors, uint32_t R,
+                                    float *const *outs, uint32_t nout, void *stream) {
+  API_BEGIN
+  require(x != nullptr && outs != nullptr, "x/outs is NULL");
+  require(nout >= 1 && nout <= kMaxOrder, "nout must be 1..8");
+  for (uint32_t d = 0; d < nout; ++d) {
+    require(outs[d] != nullptr, "outs[d] is NULL");
+    require((reinterpret_cast<uintptr_t>(outs[d]) & 15) == 0, "outs[d] must be 16-byte aligned");
+  }
+  validate_mttkrp(x->order, mode, factors, R, outs[0]);
+  check_device(x->device);
+  cudaStream_t s = as_stream(stream);
+  std::lock_guard<std::mutex> lk(x->mu);
+  if (!x->mc[mode].ready) coo_prepare_mode(x, mode, s);
+  uint64_t lo = 0, hi = x->dims[mode];
+  if (x->shard_mode == int(mode)) { lo = x->row_lo; hi = x->row_hi; }
+  for (uint32_t d = 0; d < nout; ++d) launch_zero_rows(outs[d], lo, hi, R, s);  // owned rows, every replica
+  launch_coo_mttkrp_bcast(x, mode, factors, R, outs, nout, s);
+  API_END
+}
+
 pasta_status pasta_mttkrp_hicoo(pasta_hicoo *h, uint32_t mode, const float *const *factors, uint32_t R,
                                 float *out, void *stream) {
   API_BEGIN

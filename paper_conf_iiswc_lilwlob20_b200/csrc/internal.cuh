@@ -358,6 +358,9 @@ uint64_t count_blocks_device(const pasta_coo *x, uint32_t block_bits, uint32_t c
 void launch_zero_rows(float *out, uint64_t row_lo, uint64_t row_hi, uint32_t R, cudaStream_t s);
 void launch_coo_mttkrp(const pasta_coo *x, uint32_t mode, const float *const *factors, uint32_t R,
                        float *out, cudaStream_t s);
+// fused MTTKRP + all-gather: outs[0] local output, outs[1..nout) peers' replicas (nout <= 8)
+void launch_coo_mttkrp_bcast(const pasta_coo *x, uint32_t mode, const float *const *factors, uint32_t R,
+                             float *const *outs, uint32_t nout, cudaStream_t s);
 void launch_hicoo_mttkrp(const pasta_hicoo *h, uint32_t mode, const float *const *factors,
                          uint32_t R, float *out, cudaStream_t s);
 void launch_gram(const float *U, uint64_t rows, uint32_t R, double *G, cudaStream_t s);

@@ -89,6 +89,10 @@ struct KArgs {
   const uint32_t *win_sb;
   const uint32_t *sbend32;
   uint32_t raw_words;
+  // fused MTTKRP + all-gather (WA 15): every flush also goes to the peers' replicas of the
+  // output (CUDA-IPC mapped, NVLink / NVSwitch P2P stores and atomics); outs[0] = out
+  float *outs[kMaxOrder];
+  uint32_t nout;
 };
 
 // Per-thread L2 cache policies (createpolicy, sm_80+): the nonzero stream is touched once
@@ -1193,7 +1197,12 @@ __global__ void __launch_bounds__(HS ? WPC_ * 32 : kThreads, HS ? 1 : (WA == 6 ?
             } else {
               if (cur != 0xFFFFFFFFu) {
                 float *dst = a.out + uint64_t(cur) * R + col;
-                if (kWrite) {
+                if constexpr (WA == 15) {  // the same flush into every replica
+                  for (uint32_t d = 0; d < a.nout; ++d) {
+                    float *dd = a.outs[d] + uint64_t(cur) * R + col;
+                    if (first) red_vec<4>(dd, acc, pol.out); else st_vec<4>(dd, acc, pol.out);
+                  }
+                } else if (kWrite) {
                   if (first || dyn) red_vec<4>(dst, acc, pol.out); else st_vec<4>(dst, acc, pol.out);
                 } else if (acc.v[0] == 1.2345e-30f) {
                   st_vec<4>(dst, acc, pol.out);  // keeps the arithmetic live in probes
@@ -1210,13 +1219,19 @@ __global__ void __launch_bounds__(HS ? WPC_ * 32 : kThreads, HS ? 1 : (WA == 6 ?
     __syncwarp();  // the buffer of this stage is refilled at the start of the next one
     bsel ^= 1;
   }
-  if (active && cur != 0xFFFFFFFFu && (kWrite || acc.v[0] == 1.2345e-30f))
-    red_vec<4>(a.out + uint64_t(cur) * R + col, acc, pol.out);
+  if (active && cur != 0xFFFFFFFFu && (kWrite || acc.v[0] == 1.2345e-30f)) {
+    if constexpr (WA == 15) {
+      for (uint32_t d = 0; d < a.nout; ++d) red_vec<4>(a.outs[d] + uint64_t(cur) * R + col, acc, pol.out);
+    } else {
+      red_vec<4>(a.out + uint64_t(cur) * R + col, acc, pol.out);
+    }
+  }
   const uint64_t cprev = c0;
   c0 = cn;
   if (dyn) cn = c0 < kDone ? resolve(claim_get(pend), dpend) : kDone;
   else cn = (c0 < kDone && cprev / a.chunk + 2 * wstep < nchunks) ? (cprev / a.chunk + 2 * wstep) * a.chunk : kDone;
   }  // chunk loop
+  if constexpr (WA == 15) __threadfence_system();  // the peer stores, before the kernel ends
 }
 
 template <int VW>
@@ -1364,6 +1379,26 @@ static bool vec4_ok(uint32_t order, uint32_t mode, const float *const *factors, 
 
 void launch_coo_mttkrp(const pasta_coo *x, uint32_t mode, const float *const *factors, uint32_t R,
                        float *out, cudaStream_t s) {
+  launch_coo_mttkrp_bcast(x, mode, factors, R, &out, 1, s);
+}
+
+// the rows this handle owns, copied from outs[0] into the peers' replicas outs[1..]
+static void bcast_owned_rows(const pasta_coo *x, uint32_t mode, uint32_t R, float *const *outs, uint32_t nout,
+                             cudaStream_t s) {
+  uint64_t lo = 0, hi = x->dims[mode];
+  if (x->shard_mode == int(mode)) { lo = x->row_lo; hi = x->row_hi; }
+  if (hi <= lo) return;
+  float *dsts[kMaxOrder];
+  for (uint32_t d = 1; d < nout; ++d) dsts[d - 1] = outs[d] + lo * R;
+  launch_bcast(outs[0] + lo * R, (hi - lo) * R, dsts, nout - 1, s);
+}
+
+// nout > 1: the fused MTTKRP + all-gather -- every flush is written into outs[0] (local) and
+// into the peers' replicas outs[1..]; the staged persistent kernel (WA 15) when it applies,
+// else the local kernel followed by a peer copy of the owned rows
+void launch_coo_mttkrp_bcast(const pasta_coo *x, uint32_t mode, const float *const *factors, uint32_t R,
+                             float *const *outs, uint32_t nout, cudaStream_t s) {
+  float *out = outs[0];
   const CooModeCopy &mc = x->mc[mode];
   KArgs a{};
   a.nnz = x->nnz;
@@ -1544,6 +1579,12 @@ void launch_coo_mttkrp(const pasta_coo *x, uint32_t mode, const float *const *fa
       });
     };
     using I16 = std::integral_constant<int, 16>;
+    a.nout = nout;
+    for (uint32_t d = 0; d < nout && d < uint32_t(kMaxOrder); ++d) a.outs[d] = outs[d];
+    if (hs && nout > 1) {  // fused MTTKRP + all-gather over peer memory
+      with_no_lpn<3>(no, lpn, [&](auto NOt, auto Lt) { go(coo_staged_kernel<NOt.value, Lt.value, 15, true, 16, 32, 4>); });
+      return;
+    }
     if (hs) {
       if (hs_cfg == 1) pick_hs(std::integral_constant<int, 24>(), I16());
       else if (hs_cfg == 2 && no <= 2 && l2t && (a.cache_mode & 8u))  // cold gathers evict_first
@@ -1560,9 +1601,11 @@ void launch_coo_mttkrp(const pasta_coo *x, uint32_t mode, const float *const *fa
     else if (wa == 5) pick(std::integral_constant<int, 5>());
     else if (wa == 6) pick(std::integral_constant<int, 6>());
     else pick(std::integral_constant<int, 0>());
+    if (nout > 1) bcast_owned_rows(x, mode, R, outs, nout, s);
     return;
   }
   dispatch<CooSrc>(a, vec4, s);
+  if (nout > 1) bcast_owned_rows(x, mode, R, outs, nout, s);
 }
 
 template <int NO>

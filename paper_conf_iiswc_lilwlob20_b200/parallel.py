@@ -119,6 +119,21 @@ class RowPartitionedMTTKRP:
     def shard_nnz(self) -> List[int]:
         return [s.nnz for s in self.shards]
 
+    def step_fused(self, factors, replicas, stream=None):
+        """MTTKRP of every mode with the all-gather fused into the kernel (COO shards):
+        ``replicas`` is a :class:`PeerReplicas` of the output shapes (dims, R); each rank's
+        kernel writes its owned rows into every rank's replica (pasta_mttkrp_coo_bcast, P2P
+        stores / atomics over NVLink).  A one-element all-reduce after the launches orders the
+        peers' reads; the caller orders the previous step's reads before it the same way."""
+        import torch
+
+        from . import pasta_mttkrp_coo_bcast
+        for n in range(self.order):
+            pasta_mttkrp_coo_bcast(self.shards[n], n, factors, replicas.tensors[n], replicas.dsts[n][1:],
+                                   stream=stream)
+        _all_reduce(torch.zeros(1, dtype=torch.float32, device=factors[0].device))
+        return replicas.tensors
+
     def step(self, factors, gather: bool = True, stream=None):
         """MTTKRP of every mode on this rank's shards (+ the all-gather of each output
         when world > 1).  The gather of mode n overlaps the compute of mode n + 1."""

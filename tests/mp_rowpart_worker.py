@@ -34,6 +34,22 @@ def main():
             ref, ab = oracle.mttkrp(dims, inds, vals, n, U)
             g = outs[n].cpu().numpy().astype(np.float64)
             ok &= bool(np.all(np.abs(g - ref) <= 1e-4 * ab + 1e-6))
+    # fused MTTKRP + all-gather over peer memory (CUDA IPC replicas; two ranks on one GPU here)
+    from paper_conf_iiswc_lilwlob20_b200.parallel import PeerReplicas
+    part = RowPartitionedMTTKRP(x, rank, world, 16, torch.device("cuda", 0))
+    reps = PeerReplicas(dims, 16)
+    for t in reps.tensors:
+        t.fill_(float("nan"))  # every row must be written by its owner
+    torch.cuda.synchronize()
+    dist.barrier()
+    outs = part.step_fused(Ud, reps)
+    torch.cuda.synchronize()
+    for n in range(3):
+        ref, ab = oracle.mttkrp(dims, inds, vals, n, U)
+        g = outs[n].cpu().numpy().astype(np.float64)
+        ok &= bool(np.all(np.abs(g - ref) <= 1e-4 * ab + 1e-6))
+    dist.barrier()
+    reps.close()
     flag = torch.tensor([1 if ok else 0])
     dist.all_reduce(flag, op=dist.ReduceOp.MIN)
     dist.destroy_process_group()
