@@ -647,6 +647,16 @@ def main():
                                 "gbs_per_rank": round(recv / (p_ms * 1e-3) / 1e9, 1),
                                 "how": "owned rows stored into every peer's replica by one kernel "
                                        "per mode (CUDA IPC P2P stores) + a 1-element all-reduce"}
+            # MTTKRP and all-gather fused in one kernel per mode (pasta_mttkrp_coo_bcast)
+            for _ in range(2):
+                part.step_fused(U, reps)
+            dist.barrier()
+            f_ms = max_over_ranks(timed(lambda: part.step_fused(U, reps), max(3, min(args.steps, 10))))
+            allgather["fused"] = {"ms_per_step": round(f_ms, 4),
+                                  "value": round(total_flops / (f_ms * 1e-3) / 1e9, 3),
+                                  "how": "MTTKRP step with the all-gather fused into the kernel: every "
+                                         "row flush also stored into the peers' replicas over P2P "
+                                         "(pasta_mttkrp_coo_bcast) + a 1-element all-reduce"}
             dist.barrier()
             reps.close()
         except Exception as e:  # e.g. no IPC between the ranks' GPUs

@@ -53,6 +53,7 @@ def test_bench_two_ranks_shared_gpu_weak():
     assert d["config"]["nnz"] == 2 * 54_000_000  # the tensor grows with the GPU count
     ag = d["allgather"]
     assert ag["ms_per_step"] > 0 and ag["bytes_received_per_rank"] > 0 and ag["broadcast"]["ms_per_step"] > 0
+    assert ag["p2p"]["ms_per_step"] > 0 and ag["fused"]["ms_per_step"] > 0  # CUDA IPC on one GPU
     assert d["e2e"]["value"] > 0 and d["gpu_launches"] > 0
     assert 0 < d["roofline"]["frac"] < 1.0  # compulsory bytes of this rank's launches
     bal = d["shard_max_over_mean"]  # nnz-balanced row ranges: max / mean nonzeros per rank
