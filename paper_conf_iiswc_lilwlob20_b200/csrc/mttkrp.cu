@@ -1200,7 +1200,7 @@ __global__ void __launch_bounds__(HS ? WPC_ * 32 : kThreads, HS ? 1 : (WA == 6 ?
                 if constexpr (WA == 15) {  // the same flush into every replica
                   for (uint32_t d = 0; d < a.nout; ++d) {
                     float *dd = a.outs[d] + uint64_t(cur) * R + col;
-                    if (first) red_vec<4>(dd, acc, pol.out); else st_vec<4>(dd, acc, pol.out);
+                    if (first || dyn) red_vec<4>(dd, acc, pol.out); else st_vec<4>(dd, acc, pol.out);
                   }
                 } else if (kWrite) {
                   if (first || dyn) red_vec<4>(dst, acc, pol.out); else st_vec<4>(dst, acc, pol.out);
@@ -1581,8 +1581,13 @@ void launch_coo_mttkrp_bcast(const pasta_coo *x, uint32_t mode, const float *con
     using I16 = std::integral_constant<int, 16>;
     a.nout = nout;
     for (uint32_t d = 0; d < nout && d < uint32_t(kMaxOrder); ++d) a.outs[d] = outs[d];
-    if (hs && nout > 1) {  // fused MTTKRP + all-gather over peer memory
-      with_no_lpn<3>(no, lpn, [&](auto NOt, auto Lt) { go(coo_staged_kernel<NOt.value, Lt.value, 15, true, 16, 32, 4>); });
+    if (hs && nout > 1) {  // fused MTTKRP + all-gather over peer memory, same shape as below
+      if (hs_cfg == 1)
+        with_no_lpn<3>(no, lpn, [&](auto NOt, auto Lt) { go(coo_staged_kernel<NOt.value, Lt.value, 15, true, 24, 16, 4>); });
+      else if (hs_cfg == 2 && no <= 2)
+        with_no_lpn<2>(no, lpn, [&](auto NOt, auto Lt) { go(coo_staged_kernel<NOt.value, Lt.value, 15, true, 16, 32, 8>); });
+      else
+        with_no_lpn<3>(no, lpn, [&](auto NOt, auto Lt) { go(coo_staged_kernel<NOt.value, Lt.value, 15, true, 16, 32, 4>); });
       return;
     }
     if (hs) {
