@@ -251,6 +251,13 @@ struct HicooModeCopy {
   DevArray<uint32_t> tier_block[kMaxOrder];
   bool tagged = false;
   LaunchFence fence;
+  // row-granular shared-memory tier of the staged decode (WA 16, hicoo_mark_rows): hot rows of
+  // each gathered mode (ascending) in rs_rows, per mode k a bitmap rs_bm[k] over its rows and
+  // the per-word prefix counts rs_pre[k]; cached for (rs_R, rs_budget)
+  uint32_t rs_R = 0, rs_budget = 0;
+  uint64_t rs_total = 0, rs_base[kMaxOrder] = {}, rs_words[kMaxOrder] = {};
+  DevArray<uint32_t> rs_rows;
+  DevArray<uint32_t> rs_bm[kMaxOrder], rs_pre[kMaxOrder];
 };
 
 }  // namespace pasta
@@ -395,6 +402,10 @@ void launch_hot_fill(const HicooModeCopy &mc, const float *const *factors, uint3
 // (R, global_tier, smem_rows) or when the copy is not the row-slice layout
 void hicoo_mark_hot(pasta_hicoo *h, uint32_t mode, uint32_t R, bool global_tier, uint32_t smem_rows,
                     cudaStream_t s);
+// row-granular shared-memory tier of the HiCOO staged decode (WA 16): the `smem_rows` most
+// frequent rows of the gathered modes, with per-mode bitmaps of at most max_words words
+void hicoo_mark_rows(pasta_hicoo *h, uint32_t mode, uint32_t R, uint32_t smem_rows, uint64_t max_words,
+                     cudaStream_t s);
 void row_counts_device(const uint32_t *rows, uint64_t nnz, uint32_t nrows, uint64_t *counts_host,
                        cudaStream_t s);
 // first position x in the sorted array a[0..M) with a[x] >= v (device binary search).

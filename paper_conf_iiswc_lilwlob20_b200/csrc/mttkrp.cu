@@ -93,6 +93,12 @@ struct KArgs {
   // output (CUDA-IPC mapped, NVLink / NVSwitch P2P stores and atomics); outs[0] = out
   float *outs[kMaxOrder];
   uint32_t nout;
+  // HiCOO row tier (WA 16): per other-mode slot j a bitmap of the factor rows held in the
+  // shared-memory tier (bit i of word w = row 32 w + i) and, per word, the number of tier rows
+  // before it; both copied into shared memory after the tier rows, rs_off[j] words apart
+  const uint32_t *rs_bm[kMaxOrder - 1];
+  const uint32_t *rs_pre[kMaxOrder - 1];
+  uint32_t rs_words[kMaxOrder - 1];
 };
 
 // Per-thread L2 cache policies (createpolicy, sm_80+): the nonzero stream is touched once
@@ -757,8 +763,12 @@ __global__ void __launch_bounds__(HS ? WPC_ * 32 : kThreads, HS ? 1 : (WA == 6 ?
   // block bases) are copied into shared memory with cp.async one stage ahead and decoded from
   // there -- the decode of WA 9 waits on dependent global loads every stage
   constexpr bool kHicRaw = WA == 11;
-  constexpr bool kHic = WA == 9 || WA == 10 || kHicRaw;
-  constexpr bool kL2T = WA != 7 && WA != 9 && WA != 11;
+  // 16: WA 9's decode with a ROW-granular shared-memory tier: the decoded coordinate of a hot
+  // row (bitmap + per-word prefix count, in shared memory) is retagged 0xC0000000 | smem slot,
+  // and the gathers use the WA 7 path (shared memory or a plain row, 32-bit byte offsets)
+  constexpr bool kHicRows = WA == 16;
+  constexpr bool kHic = WA == 9 || WA == 10 || kHicRaw || kHicRows;
+  constexpr bool kL2T = WA != 7 && WA != 9 && WA != 11 && WA != 16;
   constexpr bool kGather = WA != 4 && WA != 5;
   constexpr bool kWrite = WA != 3 && WA != 5;
   constexpr int kBuf = (WA == 0 || WA == 2) ? WA : 1;  // 6: form 1 with 3 CTAs per SM
@@ -785,6 +795,17 @@ __global__ void __launch_bounds__(HS ? WPC_ * 32 : kThreads, HS ? 1 : (WA == 6 ?
       for (int jj = 1; jj < NO; ++jj) j += slot >= a.hs_lo[jj];
       const float4 *Uj = reinterpret_cast<const float4 *>(a.Uo[j]);
       reinterpret_cast<float4 *>(hs_tile)[e] = __ldg(Uj + uint64_t(__ldg(a.hs_rows + slot)) * r4 + c);
+    }
+    if constexpr (kHicRows) {  // the tier's row bitmaps and per-word prefixes, after the rows
+      uint32_t *rs = reinterpret_cast<uint32_t *>(hs_tile + size_t(a.hs_lo[NO]) * R);
+#pragma unroll
+      for (int j = 0; j < NO; ++j) {
+        for (uint32_t w = threadIdx.x; w < a.rs_words[j]; w += blockDim.x) {
+          rs[w] = __ldg(a.rs_bm[j] + w);
+          rs[a.rs_words[j] + w] = __ldg(a.rs_pre[j] + w);
+        }
+        rs += 2 * a.rs_words[j];
+      }
     }
     __syncthreads();
   }
@@ -849,6 +870,20 @@ __global__ void __launch_bounds__(HS ? WPC_ * 32 : kThreads, HS ? 1 : (WA == 6 ?
   // slot ends; row and block bases come from the owning lane by shuffle; i_k = base + e_k
   // (Alg. 3's rebased pointers).  gsb[g] = current slice of group g (warp-uniform).
   uint64_t gsb[G];
+  uint32_t rs_j[NO > 0 ? NO : 1];  // WA 16: shared addresses of each mode's bitmap (prefixes follow)
+  if constexpr (kHicRows) {
+    uint32_t rs = hs_saddr + a.hs_lo[NO] * R * 4u;
+#pragma unroll
+    for (int j = 0; j < NO; ++j) {
+      rs_j[j] = rs;
+      rs += 8u * a.rs_words[j];
+    }
+  }
+  auto lds32 = [](uint32_t addr) {
+    uint32_t v;
+    asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(addr));
+    return v;
+  };
   // The loads of GB groups' windows are issued together (branch-free, so the compiler can
   // hoist them past the previous group's shuffles) before any is consumed: one memory latency
   // per batch of groups instead of one per group.
@@ -863,7 +898,7 @@ __global__ void __launch_bounds__(HS ? WPC_ * 32 : kThreads, HS ? 1 : (WA == 6 ?
 #ifdef PASTA_DECODE_GB
     constexpr int GB = G < PASTA_DECODE_GB ? G : PASTA_DECODE_GB;
 #else
-    constexpr int GB = G < 4 ? G : (NO >= 3 ? 2 : 4);
+    constexpr int GB = G < 4 ? G : ((NO >= 3 || kHicRows) ? 2 : 4);
 #endif
     constexpr int NOA = NO > 0 ? NO : 1;
 #pragma unroll
@@ -904,7 +939,17 @@ __global__ void __launch_bounds__(HS ? WPC_ * 32 : kThreads, HS ? 1 : (WA == 6 ?
         const int d = gi * SG + (((lane / 4) ^ (gi / GL)) & (CG - 1)) * 4 + (lane & 3);
         dst[d] = row;
 #pragma unroll
-        for (int j = 0; j < NO; ++j) dst[(1 + j) * SW + d] = __shfl_sync(0xFFFFFFFFu, sbase[q][j], c) + e[q][j];
+        for (int j = 0; j < NO; ++j) {
+          uint32_t id = __shfl_sync(0xFFFFFFFFu, sbase[q][j], c) + e[q][j];
+          if constexpr (kHicRows) {  // hot row -> its shared-memory slot
+            const uint32_t w = id >> 5;
+            const uint32_t bits = lds32(rs_j[j] + 4u * w);
+            if ((bits >> (id & 31)) & 1u)
+              id = 0xC0000000u | (a.hs_lo[j] + lds32(rs_j[j] + 4u * (a.rs_words[j] + w)) +
+                                  __popc(bits & ((1u << (id & 31)) - 1u)));
+          }
+          dst[(1 + j) * SW + d] = id;
+        }
         dst[(NA - 1) * SW + d] = __float_as_uint(v[q]);
         // the next window starts at the slice holding entry p + SG: the last entry's slice, or
         // the one after it when that slice ends inside this window
@@ -1779,9 +1824,48 @@ void launch_hicoo_mttkrp(const pasta_hicoo *h, uint32_t mode, const float *const
       a.win_sb = mcw.win_sb.p;
       a.raw_words = raw_words;
     }
+    // row-granular shared-memory tier (WA 16) when the factors are L2-resident and every
+    // gathered mode's row bitmap fits next to the stage buffers (C2- / C4-like tensors)
+    uint64_t max_factor16 = 0, words = 0;
+    uint64_t gathered16 = 0;
+    for (uint32_t k = 0; k < h->order; ++k)
+      if (k != mode) {
+        max_factor16 = std::max<uint64_t>(max_factor16, uint64_t(h->dims[k]) * R * sizeof(float));
+        gathered16 += uint64_t(h->dims[k]) * R * sizeof(float);
+        words += (uint64_t(h->dims[k]) + 31) / 32;
+      }
+    static int l2b = 0;
+    if (!l2b) {
+      int dev = 0;
+      cudaGetDevice(&dev);
+      cudaDeviceGetAttribute(&l2b, cudaDevAttrL2CacheSize, dev);
+      if (l2b <= 0) l2b = 126 << 20;
+    }
+    bool rowtier = false;
+    if (!tiers && !use_raw && env_int("PASTA_HICOO_ROWTIER", 0) && max_factor16 < (uint64_t(1) << 32) &&
+        gathered16 <= uint64_t(l2b) / 2 && stage + 8 * words + 64 * R * 4 <= 227 * 1024) {
+      uint32_t budget = uint32_t((227 * 1024 - stage - 8 * words) / (size_t(R) * 4));
+      if (const int cap = env_int("PASTA_HOT_SMEM_ROWS", 0)) budget = std::min(budget, uint32_t(cap));
+      hicoo_mark_rows(const_cast<pasta_hicoo *>(h), mode, R, budget, (227 * 1024 - stage) / 8, s);
+      rowtier = mc.rs_R == R && mc.rs_total > 0;
+    }
+    if (rowtier) {
+      a.hs_rows = mc.rs_rows.p;
+      int jj = 0;
+      for (uint32_t k = 0; k < h->order; ++k)
+        if (k != mode) {
+          a.hs_lo[jj] = uint32_t(mc.rs_base[k]);
+          a.rs_bm[jj] = mc.rs_bm[k].p;
+          a.rs_pre[jj] = mc.rs_pre[k].p;
+          a.rs_words[jj] = uint32_t(mc.rs_words[k]);
+          ++jj;
+        }
+      a.hs_lo[jj] = uint32_t(mc.rs_total);
+    }
     ProfScope prof(kProfHicoo, s);
     const int cfg = env_int("PASTA_HS_CFG", 0);  // 2 (8-deep steps) spills here
-    const size_t smem = stage + (tiers ? size_t(mc.hs_total) * R * sizeof(float) : 0) + (use_raw ? raw_bytes : 0);
+    const size_t smem = stage + (tiers ? size_t(mc.hs_total) * R * sizeof(float) : 0) + (use_raw ? raw_bytes : 0) +
+                        (rowtier ? size_t(mc.rs_total) * R * sizeof(float) + 8 * words : 0);
     const uint64_t nwarps = (a.nnz + a.chunk - 1) / a.chunk;
     const uint64_t nblk = std::min<uint64_t>((nwarps + 15) / 16, uint64_t(sm_count()));
     auto go = [&](auto kern) {
@@ -1790,7 +1874,9 @@ void launch_hicoo_mttkrp(const pasta_hicoo *h, uint32_t mode, const float *const
       PASTA_LAUNCHED();
       mcw.fence.record(s);
     };
-    if (use_raw)
+    if (rowtier)
+      with_no_lpn<3>(hno, lpn, [&](auto NOt, auto Lt) { go(coo_staged_kernel<NOt.value, Lt.value, 16, true, 16, 32, 4>); });
+    else if (use_raw)
       with_no_lpn<2>(hno, lpn, [&](auto NOt, auto Lt) { go(coo_staged_kernel<NOt.value, Lt.value, 11, true, 16, 32, 4>); });
     else if (tiers)
       with_no_lpn<3>(hno, lpn, [&](auto NOt, auto Lt) { go(coo_staged_kernel<NOt.value, Lt.value, 10, true, 16, 32, 4>); });

@@ -730,4 +730,89 @@ void hicoo_mark_hot(pasta_hicoo *h, uint32_t mode, uint32_t R, bool global_tier,
             (unsigned long long)mc.hs_total, (unsigned long long)mc.hot_total);
 }
 
+namespace {
+// cnt[i_k(x)] += 1 over the canonical HiCOO entries (i_k decoded from the block of entry x)
+__global__ void hicoo_row_count_kernel(const uint64_t *__restrict__ bptr, uint64_t nb, const uint32_t *__restrict__ binds,
+                                       const uint8_t *__restrict__ einds, const uint32_t *__restrict__ uinds,
+                                       uint32_t bb, uint64_t M, uint32_t *__restrict__ cnt) {
+  for (uint64_t x = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; x < M; x += uint64_t(gridDim.x) * blockDim.x) {
+    uint32_t row;
+    if (uinds) {
+      row = uinds[x];
+    } else {
+      uint64_t lo = 0, hi = nb;
+      while (hi - lo > 1) {
+        const uint64_t mid = (lo + hi) / 2;
+        if (bptr[mid] <= x) lo = mid; else hi = mid;
+      }
+      row = (binds[lo] << bb) | einds[x];
+    }
+    atomicAdd(&cnt[row], 1u);
+  }
+}
+}  // namespace
+
+void hicoo_mark_rows(pasta_hicoo *h, uint32_t mode, uint32_t R, uint32_t smem_rows, uint64_t max_words,
+                     cudaStream_t s) {
+  HicooModeCopy &mc = h->mc[mode];
+  if (mc.rs_R == R && mc.rs_budget == smem_rows) return;
+  const uint32_t N = h->order, bb = h->block_bits;
+  mc.rs_R = R;
+  mc.rs_budget = smem_rows;
+  mc.rs_total = 0;
+  uint64_t words = 0;
+  for (uint32_t k = 0; k < N; ++k)
+    if (k != mode) words += (uint64_t(h->dims[k]) + 31) / 32;
+  if (smem_rows == 0 || h->nnz == 0 || words > max_words) return;
+  struct Cand { uint32_t cnt, k, row; };
+  std::vector<Cand> cand;
+  std::vector<std::vector<uint32_t>> hc(N);
+  for (uint32_t k = 0; k < N; ++k) {
+    if (k == mode) continue;
+    DevArray<uint32_t> c(h->dims[k], s);
+    PASTA_CUDA(cudaMemsetAsync(c.p, 0, c.bytes(), s));
+    const bool comp = (h->cmask >> k) & 1u;
+    hicoo_row_count_kernel<<<grid8(h->nnz), 256, 0, s>>>(h->bptr.p, h->nblocks, comp ? h->binds[k].p : nullptr,
+                                                         comp ? h->einds[k].p : nullptr, comp ? nullptr : h->uinds[k].p,
+                                                         bb, h->nnz, c.p);
+    PASTA_LAUNCHED();
+    hc[k].resize(h->dims[k]);
+    PASTA_CUDA(cudaMemcpyAsync(hc[k].data(), c.p, c.bytes(), cudaMemcpyDeviceToHost, s));
+    PASTA_CUDA(cudaStreamSynchronize(s));
+    for (uint32_t r = 0; r < h->dims[k]; ++r)
+      if (hc[k][r]) cand.push_back({hc[k][r], k, r});
+  }
+  std::stable_sort(cand.begin(), cand.end(), [](const Cand &a, const Cand &b) { return a.cnt > b.cnt; });
+  if (cand.size() > smem_rows) cand.resize(smem_rows);
+  std::vector<std::vector<uint32_t>> rows(N);
+  for (const Cand &c : cand) rows[c.k].push_back(c.row);
+  std::vector<uint32_t> all;
+  for (uint32_t k = 0; k < N; ++k) {
+    mc.rs_base[k] = all.size();
+    mc.rs_words[k] = 0;
+    if (k == mode) continue;
+    std::sort(rows[k].begin(), rows[k].end());  // slot order = row order (prefix counts)
+    const uint64_t nw = (uint64_t(h->dims[k]) + 31) / 32;
+    std::vector<uint32_t> bm(nw, 0), pre(nw, 0);
+    for (uint32_t r : rows[k]) bm[r >> 5] |= 1u << (r & 31);
+    uint32_t run = 0;
+    for (uint64_t w = 0; w < nw; ++w) { pre[w] = run; run += uint32_t(__builtin_popcount(bm[w])); }
+    mc.rs_words[k] = nw;
+    mc.rs_bm[k].alloc(nw, s);
+    mc.rs_pre[k].alloc(nw, s);
+    PASTA_CUDA(cudaMemcpyAsync(mc.rs_bm[k].p, bm.data(), nw * 4, cudaMemcpyHostToDevice, s));
+    PASTA_CUDA(cudaMemcpyAsync(mc.rs_pre[k].p, pre.data(), nw * 4, cudaMemcpyHostToDevice, s));
+    all.insert(all.end(), rows[k].begin(), rows[k].end());
+    PASTA_CUDA(cudaStreamSynchronize(s));
+  }
+  mc.rs_total = all.size();
+  mc.rs_rows.alloc(std::max<size_t>(all.size(), 1), s);
+  if (!all.empty())
+    PASTA_CUDA(cudaMemcpyAsync(mc.rs_rows.p, all.data(), all.size() * 4, cudaMemcpyHostToDevice, s));
+  PASTA_CUDA(cudaStreamSynchronize(s));
+  if (getenv("PASTA_DEBUG"))
+    fprintf(stderr, "[pasta] hicoo row tier mode %u R %u: %llu smem rows, %llu bitmap words\n", mode, R,
+            (unsigned long long)mc.rs_total, (unsigned long long)words);
+}
+
 }  // namespace pasta
