@@ -157,6 +157,108 @@ __global__ void slice_emit_kernel(SliceOut o, const uint32_t *__restrict__ start
   }
 }
 
+// ---- R#36 tier blocks (row-granular hot-row tiers of the row-slice copy) ----
+struct TierArgs {
+  const uint32_t *binds[kMaxOrder];
+  const uint8_t *einds[kMaxOrder];
+  const uint32_t *rank[kMaxOrder];  // null: mode not tiered (the target mode, uncompressed modes)
+  uint32_t ntier[kMaxOrder];        // tier blocks of mode k (smem ones first)
+  uint32_t nbr[kMaxOrder];          // block rows of mode k: keys >= nbr are tier blocks
+  uint32_t *key[kMaxOrder];
+  uint8_t *e[kMaxOrder];
+  uint32_t order, bbits;
+};
+
+// per entry x of the canonical copy and tiered mode k: the row's heat rank rho; a row of tier
+// block m = rho >> b (m < ntier) gets key nbr + m and element index rho & (B - 1), any other row
+// keeps its canonical block (key binds_k) and element index
+__global__ void tier_entry_kernel(TierArgs t, const uint32_t *__restrict__ blk, uint64_t M) {
+  for (uint64_t x = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; x < M;
+       x += uint64_t(gridDim.x) * blockDim.x) {
+    const uint32_t b = blk[x];
+    for (uint32_t k = 0; k < t.order; ++k) {
+      if (!t.rank[k]) continue;
+      const uint32_t bk = t.binds[k][b], ek = t.einds[k][x];
+      const uint32_t rho = t.rank[k][(bk << t.bbits) | ek];
+      const uint32_t m = rho >> t.bbits;
+      if (m < t.ntier[k]) {
+        t.key[k][x] = t.nbr[k] + m;
+        t.e[k][x] = uint8_t(rho & ((1u << t.bbits) - 1u));
+      } else {
+        t.key[k][x] = bk;
+        t.e[k][x] = uint8_t(ek);
+      }
+    }
+  }
+}
+
+struct TierEmit {
+  const uint32_t *key[kMaxOrder];  // sorted keys (tiered or plain compressed other modes)
+  uint32_t *base[kMaxOrder];
+  uint32_t nbr[kMaxOrder], sblk[kMaxOrder], hs_base[kMaxOrder], hot_base[kMaxOrder];
+  uint32_t order, mode, bbits;
+};
+
+// slice j (first entry starts[j]): row, and per compressed other mode the block base -- plain
+// (binds_k << b) or the tier tag | first slot of the tier block
+__global__ void slice_emit_tier_kernel(TierEmit o, const uint32_t *__restrict__ starts, uint64_t nsb, uint64_t M,
+                                       const uint32_t *__restrict__ rowp, uint64_t *__restrict__ sbptr,
+                                       uint32_t *__restrict__ sbrow) {
+  for (uint64_t j = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; j <= nsb;
+       j += uint64_t(gridDim.x) * blockDim.x) {
+    if (j == nsb) { sbptr[nsb] = M; continue; }
+    const uint32_t x = starts[j];
+    sbptr[j] = x;
+    sbrow[j] = rowp[x];
+    for (uint32_t k = 0; k < o.order; ++k) {
+      if (!o.base[k]) continue;
+      const uint32_t key = o.key[k][x];
+      uint32_t v;
+      if (key < o.nbr[k]) {
+        v = key << o.bbits;
+      } else {
+        const uint32_t m = key - o.nbr[k];
+        v = m < o.sblk[k] ? (0xC0000000u | (o.hs_base[k] + (m << o.bbits)))
+                          : (0x80000000u | (o.hot_base[k] + ((m - o.sblk[k]) << o.bbits)));
+      }
+      o.base[k][j] = v;
+    }
+  }
+}
+
+__global__ void full_row_kernel(const uint32_t *__restrict__ binds_n, const uint32_t *__restrict__ blk,
+                                const uint8_t *__restrict__ einds_n, uint32_t bb, uint64_t M,
+                                uint32_t *__restrict__ out) {
+  for (uint64_t x = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; x < M;
+       x += uint64_t(gridDim.x) * blockDim.x)
+    out[x] = (binds_n[blk[x]] << bb) | einds_n[x];
+}
+
+__global__ void entry_row_count_kernel(const uint32_t *__restrict__ binds_k, const uint32_t *__restrict__ blk,
+                                       const uint8_t *__restrict__ einds_k, uint32_t bb, uint64_t M,
+                                       uint32_t *__restrict__ cnt) {
+  for (uint64_t x = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; x < M;
+       x += uint64_t(gridDim.x) * blockDim.x)
+    atomicAdd(&cnt[(binds_k[blk[x]] << bb) | einds_k[x]], 1u);
+}
+
+__global__ void scatter_rank_kernel(const uint32_t *__restrict__ order, uint32_t n, uint32_t *__restrict__ rank) {
+  for (uint64_t i = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; i < n; i += uint64_t(gridDim.x) * blockDim.x)
+    rank[order[i]] = uint32_t(i);
+}
+
+// heat[m] = sum of the sorted counts of ranks [m B, m B + B)
+__global__ void block_heat_kernel(const uint32_t *__restrict__ sorted, uint32_t n, uint32_t bb,
+                                  unsigned long long *__restrict__ heat) {
+  const uint64_t nb = (uint64_t(n) + (1u << bb) - 1) >> bb;
+  for (uint64_t m = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; m < nb; m += uint64_t(gridDim.x) * blockDim.x) {
+    unsigned long long h = 0;
+    const uint64_t e = std::min<uint64_t>(n, (m + 1) << bb);
+    for (uint64_t i = m << bb; i < e; ++i) h += sorted[i];
+    heat[m] = h;
+  }
+}
+
 __global__ void sched_counts_kernel(const uint64_t *__restrict__ bptr, const uint32_t *__restrict__ sched,
                                     uint64_t nb, uint64_t *__restrict__ cnt) {
   for (uint64_t s = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; s <= nb;
@@ -281,13 +383,29 @@ uint64_t count_blocks_device(const pasta_coo *x, uint32_t block_bits, uint32_t c
 // stably sorted by einds_mode, so equal output rows are contiguous runs (segmented
 // reduction); heavy blocks come first and get CTA work items (pieces) for the tile-staged
 // kernel.
-static void hicoo_prepare_rowslice(pasta_hicoo *h, uint32_t mode, cudaStream_t s) {
+// R#36: the tier blocks of each compressed other mode (see hicoo_tier_rows)
+struct TierPlan {
+  uint32_t ntier[kMaxOrder] = {}, sblk[kMaxOrder] = {};
+  uint32_t hs_base[kMaxOrder] = {}, hot_base[kMaxOrder] = {};
+};
+
+static void hicoo_prepare_rowslice_tiered(pasta_hicoo *h, uint32_t mode, const TierPlan &tp, cudaStream_t s);
+
+static void hicoo_prepare_rowslice(pasta_hicoo *h, uint32_t mode, cudaStream_t s, const TierPlan *tp = nullptr) {
   HicooModeCopy &mc = h->mc[mode];
   const uint32_t N = h->order;
   const uint64_t M = h->nnz, nb = h->nblocks;
   const uint32_t bb = h->block_bits;
   auto comp = [&](uint32_t k) { return ((h->cmask >> k) & 1u) != 0; };
   mc.layout = 0;
+  // derived per-copy caches of the launcher are rebuilt for the new slices
+  mc.run_sb_run = 0;
+  mc.run_sb.reset();
+  mc.sbend32.reset();
+  mc.win_sb.reset();
+  mc.tagged = false;
+  mc.hot_R = 0;
+  if (tp && M > 0) return hicoo_prepare_rowslice_tiered(h, mode, *tp, s);
   for (uint32_t k = 0; k < N; ++k) {
     if (k == mode) continue;
     if (comp(k)) mc.einds[k].alloc(M, s); else mc.uinds[k].alloc(M, s);
@@ -366,6 +484,272 @@ static void hicoo_prepare_rowslice(pasta_hicoo *h, uint32_t mode, cudaStream_t s
   PASTA_LAUNCHED();
   PASTA_CUDA(cudaStreamSynchronize(s));
   mc.ready = true;
+  if (getenv("PASTA_DEBUG"))
+    fprintf(stderr, "[pasta] hicoo row slices mode %u: %llu slices\n", mode, (unsigned long long)mc.nsb);
+}
+
+// Row-slice copy over tier blocks (R#36).  Every compressed other mode k has its rows ranked by
+// nonzero count (h->rt_rank[k]); the rows of ranks [0, ntier_k B) form ntier_k synthetic "tier
+// blocks" of B consecutive ranks -- the first sblk_k in the shared-memory tier, the rest in the
+// packed L2-tier buffer -- and an entry on such a row is re-blocked: block key nbr_k + m,
+// element index rho & (B - 1).  Entries are ordered by (output row, block key of every
+// compressed other mode); a slice = equal row and keys; a slice base of a tier block is the
+// tier tag | its first slot, so the decode's base + e lands on the row's slot directly and the
+// kernel gathers through the same tiers as the COO hot-row cache (WA 10).  Every row of a tier
+// block is hot (ranks, not row numbers), so a tier line holds only hot rows.
+static void hicoo_prepare_rowslice_tiered(pasta_hicoo *h, uint32_t mode, const TierPlan &tp, cudaStream_t s) {
+  HicooModeCopy &mc = h->mc[mode];
+  const uint32_t N = h->order;
+  const uint64_t M = h->nnz, nb = h->nblocks;
+  const uint32_t bb = h->block_bits, B = 1u << bb;
+  auto comp = [&](uint32_t k) { return ((h->cmask >> k) & 1u) != 0; };
+  for (uint32_t k = 0; k < N; ++k) {
+    if (k == mode) continue;
+    if (comp(k)) mc.einds[k].alloc(M, s); else mc.uinds[k].alloc(M, s);
+  }
+  mc.val.alloc(M, s);
+  DevArray<uint32_t> blk(M, s), rowfull;
+  entry_block_kernel<<<grid_for(M), kThreads, 0, s>>>(h->bptr.p, nb, M, blk.p);
+  PASTA_LAUNCHED();
+  const uint32_t *row_src;
+  if (comp(mode)) {
+    rowfull.alloc(M, s);
+    full_row_kernel<<<grid_for(M), kThreads, 0, s>>>(h->binds[mode].p, blk.p, h->einds[mode].p, bb, M, rowfull.p);
+    PASTA_LAUNCHED();
+    row_src = rowfull.p;
+  } else {
+    row_src = h->uinds[mode].p;
+  }
+  TierArgs ta{};
+  ta.order = N;
+  ta.bbits = bb;
+  DevArray<uint32_t> key[kMaxOrder];
+  DevArray<uint8_t> e[kMaxOrder];
+  const uint32_t *comps[kMaxOrder + 1];
+  uint32_t bits[kMaxOrder + 1];
+  int nc = 0;
+  comps[nc] = row_src;
+  bits[nc++] = ceil_log2(h->dims[mode]);
+  for (uint32_t k = 0; k < N; ++k) {
+    if (k == mode || !comp(k)) continue;
+    key[k].alloc(M, s);
+    e[k].alloc(M, s);
+    ta.binds[k] = h->binds[k].p;
+    ta.einds[k] = h->einds[k].p;
+    ta.rank[k] = h->rt_rank[k].p;
+    ta.ntier[k] = tp.ntier[k];
+    ta.nbr[k] = uint32_t((uint64_t(h->dims[k]) + B - 1) >> bb);
+    ta.key[k] = key[k].p;
+    ta.e[k] = e[k].p;
+    comps[nc] = key[k].p;
+    bits[nc++] = ceil_log2(uint64_t(ta.nbr[k]) + tp.ntier[k]);
+  }
+  tier_entry_kernel<<<grid_for(M), kThreads, 0, s>>>(ta, blk.p, M);
+  PASTA_LAUNCHED();
+  blk.reset();
+  DevArray<uint32_t> perm(M, s);
+  iota_u32(perm.p, M, s);
+  lexsort(comps, bits, nc, perm, M, s);
+  DevArray<uint32_t> rowp(M, s), keyp[kMaxOrder];
+  gather_u32(row_src, perm.p, rowp.p, M, s);
+  rowfull.reset();
+  Coords co{};
+  co.order = 0;
+  co.c[co.order++] = rowp.p;
+  for (uint32_t k = 0; k < N; ++k) {
+    if (k == mode) continue;
+    if (comp(k)) {
+      keyp[k].alloc(M, s);
+      gather_u32(key[k].p, perm.p, keyp[k].p, M, s);
+      gather_u8(e[k].p, perm.p, mc.einds[k].p, M, s);
+      co.c[co.order++] = keyp[k].p;
+      key[k].reset();
+      e[k].reset();
+    } else {
+      gather_u32(h->uinds[k].p, perm.p, mc.uinds[k].p, M, s);
+    }
+  }
+  gather_f32(h->val.p, perm.p, mc.val.p, M, s);
+  perm.reset();
+  DevArray<uint8_t> flag(M, s);
+  block_flag_kernel<<<grid_for(M), kThreads, 0, s>>>(co, 0, M, flag.p);
+  PASTA_LAUNCHED();
+  DevArray<uint32_t> starts;
+  mc.nsb = select_flagged(flag.p, M, starts, s);
+  flag.reset();
+  mc.sbptr.alloc(mc.nsb + 1, s);
+  mc.sbrow.alloc(mc.nsb + kSlicePad, s);
+  PASTA_CUDA(cudaMemsetAsync(mc.sbrow.p + mc.nsb, 0, kSlicePad * 4, s));
+  TierEmit o{};
+  o.order = N;
+  o.mode = mode;
+  o.bbits = bb;
+  for (uint32_t k = 0; k < N; ++k) {
+    if (k == mode || !comp(k)) continue;
+    mc.sbbase[k].alloc(mc.nsb + kSlicePad, s);
+    PASTA_CUDA(cudaMemsetAsync(mc.sbbase[k].p + mc.nsb, 0, kSlicePad * 4, s));
+    o.key[k] = keyp[k].p;
+    o.base[k] = mc.sbbase[k].p;
+    o.nbr[k] = ta.nbr[k];
+    o.sblk[k] = tp.sblk[k];
+    o.hs_base[k] = tp.hs_base[k];
+    o.hot_base[k] = tp.hot_base[k];
+  }
+  slice_emit_tier_kernel<<<grid_for(mc.nsb + 1), kThreads, 0, s>>>(o, starts.p, mc.nsb, M, rowp.p, mc.sbptr.p,
+                                                                   mc.sbrow.p);
+  PASTA_LAUNCHED();
+  PASTA_CUDA(cudaStreamSynchronize(s));
+  mc.ready = true;
+}
+
+// heat ranking of mode k's rows (R#36), cached on the handle: counts over the canonical entries,
+// rows sorted by count descending (ties by row, ascending: the radix sort is stable), rank =
+// inverse permutation, and the heat of every block of B consecutive ranks
+static void hicoo_rank_mode(pasta_hicoo *h, uint32_t k, const uint32_t *blk, cudaStream_t s) {
+  if (h->rt_ready[k]) return;
+  const uint32_t n = h->dims[k], bb = h->block_bits;
+  const uint64_t M = h->nnz;
+  DevArray<uint32_t> cnt(n, s), cnt_sorted(n, s), rows(n, s);
+  PASTA_CUDA(cudaMemsetAsync(cnt.p, 0, cnt.bytes(), s));
+  entry_row_count_kernel<<<grid_for(M), kThreads, 0, s>>>(h->binds[k].p, blk, h->einds[k].p, bb, M, cnt.p);
+  PASTA_LAUNCHED();
+  iota_u32(rows.p, n, s);
+  h->rt_order[k].alloc(n, s);
+  size_t tb = 0;
+  PASTA_CUDA(cub::DeviceRadixSort::SortPairsDescending(nullptr, tb, cnt.p, cnt_sorted.p, rows.p, h->rt_order[k].p,
+                                                        int64_t(n), 0, 32, s));
+  DevArray<uint8_t> tmp(tb, s);
+  PASTA_CUDA(cub::DeviceRadixSort::SortPairsDescending(tmp.p, tb, cnt.p, cnt_sorted.p, rows.p, h->rt_order[k].p,
+                                                        int64_t(n), 0, 32, s));
+  count_launch();
+  h->rt_rank[k].alloc(n, s);
+  scatter_rank_kernel<<<grid_for(n), kThreads, 0, s>>>(h->rt_order[k].p, n, h->rt_rank[k].p);
+  PASTA_LAUNCHED();
+  const uint64_t nbk = (uint64_t(n) + (1u << bb) - 1) >> bb;
+  DevArray<unsigned long long> heat(nbk, s);
+  block_heat_kernel<<<grid_for(nbk), kThreads, 0, s>>>(cnt_sorted.p, n, bb, heat.p);
+  PASTA_LAUNCHED();
+  h->rt_heat[k].resize(nbk);
+  PASTA_CUDA(cudaMemcpyAsync(h->rt_heat[k].data(), heat.p, heat.bytes(), cudaMemcpyDeviceToHost, s));
+  PASTA_CUDA(cudaStreamSynchronize(s));
+  h->rt_ready[k] = true;
+}
+
+// R#36: tier blocks for the row-slice copy of `mode`, budgets as the COO hot-row cache
+// (`smem_rows` shared-memory rows; PASTA_HOT_MB, default 64 MB, of L2 tier when `global_tier`).
+// Tier blocks of all compressed other modes are taken greedily by heat (each mode's block
+// heats are non-increasing, so every mode's tier is a prefix of its ranking: smem blocks
+// first, then L2 blocks).  Rebuilds the copy when the plan changes; on = false restores the
+// plain copy.
+void hicoo_tier_rows(pasta_hicoo *h, uint32_t mode, uint32_t R, bool on, bool global_tier, uint32_t smem_rows,
+                     cudaStream_t s) {
+  HicooModeCopy &mc = h->mc[mode];
+  if (!mc.ready || mc.layout != 0) return;
+  const bool want = on && h->nnz > 0;
+  if (!want) {
+    if (mc.rt_on) {
+      hicoo_prepare_rowslice(h, mode, s);
+      mc.rt_on = false;
+      mc.rt_R = 0;
+    }
+    return;
+  }
+  if (mc.rt_on && mc.rt_R == R && mc.rt_global == global_tier && mc.rt_budget == smem_rows) return;
+  const uint32_t N = h->order, bb = h->block_bits, B = 1u << bb;
+  auto tiered = [&](uint32_t k) { return k != mode && ((h->cmask >> k) & 1u) != 0; };
+  bool ok = true;
+  for (uint32_t k = 0; k < N; ++k)
+    if (h->dims[k] >= 0x40000000u) ok = false;  // tagged bases need slots below 2^30
+  const char *env = getenv("PASTA_HOT_MB");
+  const double hot_mb = global_tier ? ((env && *env) ? atof(env) : 64.0) : 0.0;
+  const uint64_t sm_blocks = smem_rows >> bb;
+  const uint64_t l2_blocks = uint64_t(hot_mb * 1048576.0 / (double(B) * R * sizeof(float)));
+  TierPlan tp{};
+  uint64_t hs_total = 0, hot_total = 0;
+  if (ok && sm_blocks + l2_blocks > 0) {
+    {
+      DevArray<uint32_t> blk(h->nnz, s);
+      entry_block_kernel<<<grid_for(h->nnz), kThreads, 0, s>>>(h->bptr.p, h->nblocks, h->nnz, blk.p);
+      PASTA_LAUNCHED();
+      for (uint32_t k = 0; k < N; ++k)
+        if (tiered(k)) hicoo_rank_mode(h, k, blk.p, s);
+    }
+    uint64_t p[kMaxOrder] = {};
+    for (uint64_t i = 0; i < sm_blocks + l2_blocks; ++i) {
+      int best = -1;
+      unsigned long long bh = 0;
+      for (uint32_t k = 0; k < N; ++k)
+        if (tiered(k) && p[k] < h->rt_heat[k].size() && h->rt_heat[k][p[k]] > bh) {
+          bh = h->rt_heat[k][p[k]];
+          best = int(k);
+        }
+      if (best < 0) break;
+      if (i < sm_blocks) ++tp.sblk[best];
+      ++tp.ntier[best];
+      ++p[best];
+    }
+    for (uint32_t k = 0; k < N; ++k) {
+      tp.hs_base[k] = uint32_t(hs_total);
+      hs_total += uint64_t(tp.sblk[k]) << bb;
+    }
+    for (uint32_t k = 0; k < N; ++k) {
+      tp.hot_base[k] = uint32_t(hot_total);
+      hot_total += uint64_t(tp.ntier[k] - tp.sblk[k]) << bb;
+    }
+  }
+  // slot -> factor row lists: the ranking's prefixes (slots past a mode's last row hold row 0)
+  mc.hs_total = hs_total;
+  mc.hot_total = hot_total;
+  mc.hs_rows.alloc(std::max<uint64_t>(hs_total, 1), s);
+  mc.hot_rows.alloc(std::max<uint64_t>(hot_total, 1), s);
+  PASTA_CUDA(cudaMemsetAsync(mc.hs_rows.p, 0, mc.hs_rows.bytes(), s));
+  PASTA_CUDA(cudaMemsetAsync(mc.hot_rows.p, 0, mc.hot_rows.bytes(), s));
+  mc.hot_buf.alloc(std::max<uint64_t>(hot_total, 1) * R, s);
+  for (uint32_t k = 0; k < N; ++k) {
+    mc.hs_base[k] = tp.hs_base[k];
+    mc.hs_cnt[k] = uint64_t(tp.sblk[k]) << bb;
+    mc.hot_base[k] = tp.hot_base[k];
+    mc.hot_cnt[k] = uint64_t(tp.ntier[k] - tp.sblk[k]) << bb;
+    if (!tp.ntier[k]) continue;
+    const uint64_t n = h->dims[k];
+    const uint64_t ns = std::min<uint64_t>(mc.hs_cnt[k], n);
+    if (ns)
+      PASTA_CUDA(cudaMemcpyAsync(mc.hs_rows.p + mc.hs_base[k], h->rt_order[k].p, ns * 4, cudaMemcpyDeviceToDevice, s));
+    const uint64_t h0 = mc.hs_cnt[k];
+    const uint64_t nh = h0 < n ? std::min<uint64_t>(mc.hot_cnt[k], n - h0) : 0;
+    if (nh)
+      PASTA_CUDA(cudaMemcpyAsync(mc.hot_rows.p + mc.hot_base[k], h->rt_order[k].p + h0, nh * 4,
+                                 cudaMemcpyDeviceToDevice, s));
+  }
+  hicoo_prepare_rowslice(h, mode, s, &tp);
+  // hicoo_prepare_rowslice cleared the R#34 state; these describe the R#36 tiers
+  mc.hs_total = hs_total;
+  mc.hot_total = hot_total;
+  for (uint32_t k = 0; k < N; ++k) {
+    mc.hs_base[k] = tp.hs_base[k];
+    mc.hs_cnt[k] = uint64_t(tp.sblk[k]) << bb;
+    mc.hot_base[k] = tp.hot_base[k];
+    mc.hot_cnt[k] = uint64_t(tp.ntier[k] - tp.sblk[k]) << bb;
+  }
+  mc.rt_on = true;
+  mc.rt_R = R;
+  mc.rt_global = global_tier;
+  mc.rt_budget = smem_rows;
+  if (getenv("PASTA_DEBUG")) {
+    double tot = 0.0, cov = 0.0;
+    for (uint32_t k = 0; k < N; ++k)
+      if (tiered(k) && h->rt_ready[k])
+        for (size_t m = 0; m < h->rt_heat[k].size(); ++m) {
+          tot += double(h->rt_heat[k][m]);
+          if (m < tp.ntier[k]) cov += double(h->rt_heat[k][m]);
+        }
+    fprintf(stderr, "[pasta] hicoo tier blocks mode %u R %u: smem %llu rows, L2 %llu rows, %llu slices, "
+            "%.3f of the gathers (", mode, R, (unsigned long long)hs_total, (unsigned long long)hot_total,
+            (unsigned long long)mc.nsb, tot > 0 ? cov / tot : 0.0);
+    for (uint32_t k = 0; k < N; ++k)
+      if (tiered(k)) fprintf(stderr, " k%u:%u+%u", k, tp.sblk[k], tp.ntier[k] - tp.sblk[k]);
+    fprintf(stderr, " )\n");
+  }
 }
 
 void hicoo_prepare_mode(pasta_hicoo *h, uint32_t mode, cudaStream_t s) {

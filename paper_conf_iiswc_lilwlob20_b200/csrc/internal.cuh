@@ -258,6 +258,11 @@ struct HicooModeCopy {
   uint64_t rs_total = 0, rs_base[kMaxOrder] = {}, rs_words[kMaxOrder] = {};
   DevArray<uint32_t> rs_rows;
   DevArray<uint32_t> rs_bm[kMaxOrder], rs_pre[kMaxOrder];
+  // tier blocks (R#36, hicoo_tier_rows): the copy itself was built over the heat-ranked tier
+  // blocks of the gathered modes for (rt_R, rt_global, rt_budget); hs_* / hot_* describe them
+  bool rt_on = false;
+  uint32_t rt_R = 0, rt_budget = 0;
+  bool rt_global = false;
 };
 
 }  // namespace pasta
@@ -310,6 +315,11 @@ struct pasta_hicoo {
   pasta::DevArray<uint32_t> uinds[pasta::kMaxOrder];
   pasta::DevArray<float> val;
   pasta::HicooModeCopy mc[pasta::kMaxOrder];
+  // R#36 heat ranking per mode (rows by nonzero count, descending): order, its inverse, and
+  // the heat of every block of 2^block_bits consecutive ranks (host)
+  bool rt_ready[pasta::kMaxOrder] = {};
+  pasta::DevArray<uint32_t> rt_order[pasta::kMaxOrder], rt_rank[pasta::kMaxOrder];
+  std::vector<unsigned long long> rt_heat[pasta::kMaxOrder];
   int shard_mode = -1;  // >= 0: the [row_lo, row_hi) shard of that mode (pasta_hicoo_shard)
   uint32_t row_lo = 0, row_hi = 0;
   std::mutex mu;
@@ -405,6 +415,10 @@ void hicoo_mark_hot(pasta_hicoo *h, uint32_t mode, uint32_t R, bool global_tier,
 // row-granular shared-memory tier of the HiCOO staged decode (WA 16): the `smem_rows` most
 // frequent rows of the gathered modes, with per-mode bitmaps of at most max_words words
 void hicoo_mark_rows(pasta_hicoo *h, uint32_t mode, uint32_t R, uint32_t smem_rows, uint64_t max_words,
+                     cudaStream_t s);
+// tier blocks of the HiCOO row-slice copy of `mode` (R#36): rebuilds the copy over heat-ranked
+// tier blocks of the gathered modes (on), or back to the plain copy (!on); cached per plan
+void hicoo_tier_rows(pasta_hicoo *h, uint32_t mode, uint32_t R, bool on, bool global_tier, uint32_t smem_rows,
                      cudaStream_t s);
 void row_counts_device(const uint32_t *rows, uint64_t nnz, uint32_t nrows, uint64_t *counts_host,
                        cudaStream_t s);

@@ -61,6 +61,9 @@ struct KArgs {
   // gHiCOO (R#29): bit j set <=> other-mode slot j is uncompressed: its u32 coordinates come
   // from io[j] (no slice base); clear -> 8-bit element index eo[j] + slice base
   uint32_t wide;
+  // staged decode: bulk-prefetch (into L2) the slice and entry arrays of the stage after the
+  // one just decoded (its first slices are known then)
+  uint32_t pf;
   // factors of the other modes (ascending k), output
   const float *Uo[kMaxOrder - 1];
   float *out;
@@ -130,6 +133,18 @@ __device__ __forceinline__ uint32_t ld_stream_u32(const void *p, uint64_t pol) {
   uint32_t r;
   asm("ld.global.nc.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(r) : "l"(p), "l"(pol));
   return r;
+}
+__device__ __forceinline__ uint32_t ld_stream_u8(const void *p, uint64_t pol) {
+  unsigned short r;
+  asm("ld.global.nc.L2::cache_hint.u8 %0, [%1], %2;" : "=h"(r) : "l"(p), "l"(pol));
+  return r;
+}
+// L2 prefetch of [p, p + bytes) by the bulk-copy unit (no registers, no completion to wait on);
+// p is rounded down and the size up to 16 bytes
+__device__ __forceinline__ void bulk_prefetch_l2(const void *p, uint32_t bytes) {
+  const uint64_t a = reinterpret_cast<uint64_t>(p), a0 = a & ~uint64_t(15);
+  const uint32_t n = uint32_t((a + bytes - a0 + 15) & ~uint64_t(15));
+  asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(a0), "r"(n) : "memory");
 }
 __device__ __forceinline__ float4 ld_gather_f4(const float *p, uint64_t pol) {
   float4 r;
@@ -767,8 +782,11 @@ __global__ void __launch_bounds__(HS ? WPC_ * 32 : kThreads, HS ? 1 : (WA == 6 ?
   // row (bitmap + per-word prefix count, in shared memory) is retagged 0xC0000000 | smem slot,
   // and the gathers use the WA 7 path (shared memory or a plain row, 32-bit byte offsets)
   constexpr bool kHicRows = WA == 16;
-  constexpr bool kHic = WA == 9 || WA == 10 || kHicRaw || kHicRows;
-  constexpr bool kL2T = WA != 7 && WA != 9 && WA != 11 && WA != 16;
+  // 17: WA 9's decode with tagged slice bases of the shared-memory tier only (R#36 tier blocks
+  // without an L2 tier): the gathers take the WA 7 path (shared memory or a plain row, 32-bit
+  // byte offsets)
+  constexpr bool kHic = WA == 9 || WA == 10 || kHicRaw || kHicRows || WA == 17;
+  constexpr bool kL2T = WA != 7 && WA != 9 && WA != 11 && WA != 16 && WA != 17;
   constexpr bool kGather = WA != 4 && WA != 5;
   constexpr bool kWrite = WA != 3 && WA != 5;
   constexpr int kBuf = (WA == 0 || WA == 2) ? WA : 1;  // 6: form 1 with 3 CTAs per SM
@@ -911,16 +929,21 @@ __global__ void __launch_bounds__(HS ? WPC_ * 32 : kThreads, HS ? 1 : (WA == 6 ?
         const uint64_t p = cc + uint64_t(gb + q) * run + uint64_t(s) * SG;
         const uint64_t sb0 = gsb[gb + q];
         const uint64_t st = sb0 + lane < a.nsb ? sb0 + lane : a.nsb - 1;
-        eabs[q] = __ldg(a.sbend32 + st);  // = sbptr[st + 1]
-        srow[q] = __ldg(a.sbrow + st);
-#pragma unroll
-        for (int j = 0; j < NO; ++j) sbase[q][j] = ((a.wide >> j) & 1u) ? 0u : __ldg(a.sbbase[j] + st);
-        const uint64_t x = p + lane;
-        const bool ok = x < a.nnz;
-        v[q] = ok ? __ldg(a.val + x) : 0.f;
+        // the slice and entry arrays are read once per launch: evict_first (pol.stream), like
+        // the COO stream, so they do not push the tiers and hot factor rows out of L2
+        eabs[q] = ld_stream_u32(a.sbend32 + st, pol.stream);  // = sbptr[st + 1]
+        srow[q] = ld_stream_u32(a.sbrow + st, pol.stream);
 #pragma unroll
         for (int j = 0; j < NO; ++j)
-          e[q][j] = !ok ? 0u : ((a.wide >> j) & 1u) ? __ldg(a.io[j] + x) : uint32_t(__ldg(a.eo[j] + x));
+          sbase[q][j] = ((a.wide >> j) & 1u) ? 0u : ld_stream_u32(a.sbbase[j] + st, pol.stream);
+        const uint64_t x = p + lane;
+        const bool ok = x < a.nnz;
+        v[q] = ok ? __uint_as_float(ld_stream_u32(a.val + x, pol.stream)) : 0.f;
+#pragma unroll
+        for (int j = 0; j < NO; ++j)
+          e[q][j] = !ok ? 0u
+                        : ((a.wide >> j) & 1u) ? ld_stream_u32(a.io[j] + x, pol.stream)
+                                               : ld_stream_u8(a.eo[j] + x, pol.stream);
       }
 #pragma unroll
       for (int q = 0; q < GB; ++q) {
@@ -958,6 +981,32 @@ __global__ void __launch_bounds__(HS ? WPC_ * 32 : kThreads, HS ? 1 : (WA == 6 ?
         const int clast = __shfl_sync(0xFFFFFFFFu, c, last);
         const uint32_t elast = __shfl_sync(0xFFFFFFFFu, erel, clast);
         gsb[gi] = sb0 + uint64_t(clast) + (elast <= uint32_t(SG) ? 1u : 0u);
+      }
+    }
+    // the next stage's windows: slots [gsb, gsb + 32) of the slice arrays and its 32 entries
+    // (the same group run, or the warp's next chunk -- skipped then), one array per lane
+    if (a.pf) {
+      const uint64_t nstg = (uint64_t(a.chunk) / G) / SG;
+      if (uint64_t(s) + 1 < nstg) {
+#pragma unroll
+        for (int gi = 0; gi < G; ++gi) {
+          const uint64_t pn = cc + uint64_t(gi) * run + uint64_t(s + 1) * SG;
+          if (pn >= a.nnz) continue;  // warp-uniform
+          // slot arrays are padded by kSlicePad (>= 32) slots; entry ranges stop at nnz
+          const uint64_t sb = gsb[gi] < a.nsb ? gsb[gi] : a.nsb - 1;
+          const uint32_t ne = a.nnz - pn >= uint64_t(SG) ? uint32_t(SG) : uint32_t(a.nnz - pn);
+          if (lane == 0) bulk_prefetch_l2(a.sbend32 + sb, 128);
+          else if (lane == 1) bulk_prefetch_l2(a.sbrow + sb, 128);
+          else if (lane == 2) bulk_prefetch_l2(a.val + pn, 4 * ne);
+          else if (lane >= 3 && lane < 3 + NO) {
+            const int j = lane - 3;
+            if ((a.wide >> j) & 1u) bulk_prefetch_l2(a.io[j] + pn, 4 * ne);
+            else bulk_prefetch_l2(a.eo[j] + pn, ne);
+          } else if (lane >= 3 + NO && lane < 3 + 2 * NO) {
+            const int j = lane - 3 - NO;
+            if (!((a.wide >> j) & 1u)) bulk_prefetch_l2(a.sbbase[j] + sb, 128);
+          }
+        }
       }
     }
   };
@@ -1721,6 +1770,49 @@ void launch_hicoo_mttkrp(const pasta_hicoo *h, uint32_t mode, const float *const
   if (mc.layout == 0 && env_int("PASTA_HICOO_STAGED", 1) && staged_rank(R) && hno >= 1 &&
       hno <= 3 && h->nnz > 0 && hic_smem <= 227 * 1024 && vec4_ok(h->order, mode, factors, R, out)) {
     // Row slices decoded warp-wide into the persistent staged COO kernel (WA 9)
+    HicooModeCopy &mcw = const_cast<HicooModeCopy &>(mc);
+    const int lpn = int(R / 4);
+    const int G = 32 / lpn;
+    const size_t stage = size_t(16) * 2 * (hno + 2) * (G * 32) * sizeof(uint32_t);
+    // hot-row tiers: 2 (default) = tier blocks (R#36, the copy rebuilt over heat-ranked blocks
+    // of the gathered modes), 1 = hot-block tiers (R#34, slice bases of whole canonical blocks
+    // retagged), 0 = none.  Budgets as the COO hot-row cache: an L2 tier when the gathered
+    // factors exceed half the L2, a shared-memory tier of what the stage buffers leave (512
+    // rows when the gathers go to DRAM)
+    // Default (PASTA_HICOO_HOT unset): tier blocks when every gathered factor exceeds twice
+    // the L2 -- measured: H (two 512-MB factors) 3.04 -> 2.60 ms per mode; C3 (a 20- or 102-MB
+    // factor next to the 1.8-GB one) 2.41 -> 2.63 and the L2-resident C2 / C4 1.08 -> 1.20 / 1.15
+    // -> 1.29, where the tiered gathers' extra instructions outweigh the misses they save
+    // (profiles/r02_hicoo_tier_sweep.txt)
+    static int l2 = 0;
+    if (!l2) {
+      int dev = 0;
+      cudaGetDevice(&dev);
+      cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, dev);
+      if (l2 <= 0) l2 = 126 << 20;
+    }
+    uint64_t gathered = 0, min_gathered = ~uint64_t(0);
+    for (uint32_t k = 0; k < h->order; ++k)
+      if (k != mode) {
+        const uint64_t b = uint64_t(h->dims[k]) * R * sizeof(float);
+        gathered += b;
+        min_gathered = std::min(min_gathered, b);
+      }
+    const int hot_env = env_int("PASTA_HICOO_HOT", -1);
+    const int hot_mode = !env_int("PASTA_HOT_SMEM", 1) ? 0
+                         : hot_env >= 0                 ? hot_env
+                         : (min_gathered > 2 * uint64_t(l2) ? 2 : 0);
+    bool want_hot = false;
+    uint32_t budget = 0;
+    {
+      want_hot = env_int("PASTA_HOT_FORCE", 0) || gathered > uint64_t(l2) / 2;
+      budget = stage < 227 * 1024 ? uint32_t((227 * 1024 - stage) / (size_t(R) * sizeof(float))) : 0u;
+      if (want_hot) budget = std::min(budget, uint32_t(env_int("PASTA_HOT_SMEM_DRAM", 512)));
+      if (const int cap = env_int("PASTA_HOT_SMEM_ROWS", 0)) budget = std::min(budget, uint32_t(cap));
+    }
+    // every launch on this copy reads its slices: a rebuild or retag waits for the previous one
+    mcw.fence.wait(s);
+    hicoo_tier_rows(const_cast<pasta_hicoo *>(h), mode, R, hot_mode == 2, want_hot, budget, s);
     KArgs a{};
     a.nnz = h->nnz;
     a.order = h->order;
@@ -1743,12 +1835,9 @@ void launch_hicoo_mttkrp(const pasta_hicoo *h, uint32_t mode, const float *const
       ++j;
     }
     a.out = out;
-    const int lpn = int(R / 4);
-    const int G = 32 / lpn;
     uint64_t run = uint64_t(env_int("PASTA_MTTKRP_RUN", 128));
     run = run < 32 ? 32 : (run / 32) * 32;
     a.chunk = uint64_t(G) * run;
-    HicooModeCopy &mcw = const_cast<HicooModeCopy &>(mc);
     const uint64_t nruns = (a.nnz + run - 1) / run;
     if (mcw.run_sb_run != run || mcw.run_sb.n != nruns) {
       mcw.run_sb.alloc(nruns, s);
@@ -1759,30 +1848,12 @@ void launch_hicoo_mttkrp(const pasta_hicoo *h, uint32_t mode, const float *const
       mcw.run_sb_run = run;
     }
     a.run_sb = mcw.run_sb.p;
-    // hot-block tiers (R#34), with the COO cache's policy: an L2 tier when the gathered factors
-    // exceed half the L2, a shared-memory tier of what the stage buffers leave (512 rows when
-    // the gathers go to DRAM); PASTA_HICOO_HOT=0 disables both
-    const size_t stage = size_t(16) * 2 * (hno + 2) * (G * 32) * sizeof(uint32_t);
     bool tiers = false;
-    // every launch on this copy reads sbbase: a retag waits for the previous launch
-    mcw.fence.wait(s);
-    if (!(env_int("PASTA_HICOO_HOT", 0) && env_int("PASTA_HOT_SMEM", 1))) {
+    if (hot_mode == 2) {
+      tiers = mc.rt_on && mc.rt_R == R && (mc.hs_total + mc.hot_total) > 0;
+    } else if (hot_mode != 1) {
       if (mc.tagged) hicoo_mark_hot(const_cast<pasta_hicoo *>(h), mode, R, false, 0, s);  // untag
     } else {
-      static int l2 = 0;
-      if (!l2) {
-        int dev = 0;
-        cudaGetDevice(&dev);
-        cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, dev);
-        if (l2 <= 0) l2 = 126 << 20;
-      }
-      uint64_t gathered = 0;
-      for (uint32_t k = 0; k < h->order; ++k)
-        if (k != mode) gathered += uint64_t(h->dims[k]) * R * sizeof(float);
-      const bool want_hot = env_int("PASTA_HOT_FORCE", 0) || gathered > uint64_t(l2) / 2;
-      uint32_t budget = stage < 227 * 1024 ? uint32_t((227 * 1024 - stage) / (size_t(R) * sizeof(float))) : 0u;
-      if (want_hot) budget = std::min(budget, 512u);
-      if (const int cap = env_int("PASTA_HOT_SMEM_ROWS", 0)) budget = std::min(budget, uint32_t(cap));
       hicoo_mark_hot(const_cast<pasta_hicoo *>(h), mode, R, want_hot, budget, s);
       tiers = mc.hot_R == R && (mc.hs_total + mc.hot_total) > 0;
     }
@@ -1812,6 +1883,7 @@ void launch_hicoo_mttkrp(const pasta_hicoo *h, uint32_t mode, const float *const
       PASTA_LAUNCHED();
     }
     a.sbend32 = mcw.sbend32.p;
+    a.pf = uint32_t(env_int("PASTA_HICOO_PF", 1));
     if (use_raw) {
       const uint64_t nwin = (h->nnz + 31) / 32;
       if (mcw.win_sb.n != nwin) {
@@ -1874,7 +1946,12 @@ void launch_hicoo_mttkrp(const pasta_hicoo *h, uint32_t mode, const float *const
       PASTA_LAUNCHED();
       mcw.fence.record(s);
     };
-    if (rowtier)
+    uint64_t max_gf = 0;
+    for (uint32_t k = 0; k < h->order; ++k)
+      if (k != mode) max_gf = std::max<uint64_t>(max_gf, uint64_t(h->dims[k]) * R * sizeof(float));
+    if (tiers && mc.hot_total == 0 && max_gf < (uint64_t(1) << 32))  // smem tier only: WA 17
+      with_no_lpn<3>(hno, lpn, [&](auto NOt, auto Lt) { go(coo_staged_kernel<NOt.value, Lt.value, 17, true, 16, 32, 4>); });
+    else if (rowtier)
       with_no_lpn<3>(hno, lpn, [&](auto NOt, auto Lt) { go(coo_staged_kernel<NOt.value, Lt.value, 16, true, 16, 32, 4>); });
     else if (use_raw)
       with_no_lpn<2>(hno, lpn, [&](auto NOt, auto Lt) { go(coo_staged_kernel<NOt.value, Lt.value, 11, true, 16, 32, 4>); });
@@ -1889,9 +1966,10 @@ void launch_hicoo_mttkrp(const pasta_hicoo *h, uint32_t mode, const float *const
   if (mc.layout == 0) {
     // the generic row-slice kernel reads plain block bases: undo any hot-block tagging
     HicooModeCopy &mcw = const_cast<HicooModeCopy &>(mc);
-    if (mc.tagged) {
+    if (mc.tagged || mc.rt_on) {
       mcw.fence.wait(s);
-      hicoo_mark_hot(const_cast<pasta_hicoo *>(h), mode, R, false, 0, s);
+      if (mc.tagged) hicoo_mark_hot(const_cast<pasta_hicoo *>(h), mode, R, false, 0, s);
+      hicoo_tier_rows(const_cast<pasta_hicoo *>(h), mode, R, false, false, 0, s);
     }
     KArgs a{};
     a.nnz = h->nnz;

@@ -54,6 +54,13 @@ def main():
                 os.environ[env] = "1"
                 close(pasta.pasta_mttkrp_hicoo(h, n, Ud), ref, ab, (dims, R, n, "hicoo", env))
                 os.environ[env] = "0"
+            # R#36 tier blocks: smem tier only (WA 17), then smem + L2 tiers forced (WA 10)
+            os.environ["PASTA_HICOO_HOT"] = "2"
+            for force in ("0", "1"):
+                os.environ["PASTA_HOT_FORCE"] = force
+                close(pasta.pasta_mttkrp_hicoo(h, n, Ud), ref, ab, (dims, R, n, "hicoo tier blocks", force))
+            os.environ["PASTA_HOT_FORCE"] = "0"
+            os.environ["PASTA_HICOO_HOT"] = "0"
             bounds = pasta.pasta_coo_partition(x, n, 2)
             out = torch.zeros((dims[n], R), device="cuda")
             for p in range(2):

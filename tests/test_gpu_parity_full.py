@@ -103,14 +103,16 @@ def test_fullsize_hicoo_conversion_bit_exact(env, key):
     assert np.array_equal(hx["vals"].view(np.uint32), o["vals"].view(np.uint32))
 
 
+@pytest.mark.parametrize("tier", ["1", "2"])
 @pytest.mark.parametrize("hot_mb", ["0.05", "64"])
-def test_hicoo_hot_block_tiers_retag(env, hot_mb, monkeypatch):
-    """HiCOO hot-block tiers (R#34): shared-memory and L2 tiers forced on, ragged dims (partial
-    last blocks), and the rank changed on the same handle (R = 16 -> 32 -> 8 -> 16) so the
-    retagged slice bases are untagged and retagged between launches; every result against the
-    oracle.  hot_mb = 0.05 leaves most blocks cold (mixed tags inside a warp's window)."""
+def test_hicoo_hot_block_tiers_retag(env, hot_mb, tier, monkeypatch):
+    """HiCOO hot-row tiers, shared-memory and L2 tiers forced on: tier = 1 hot-block tiers (R#34,
+    retagged canonical blocks), tier = 2 tier blocks (R#36, the copy rebuilt over heat-ranked
+    blocks).  Ragged dims (partial last blocks), and the rank changed on the same handle (R = 16
+    -> 32 -> 8 -> 16) so the tiers are rebuilt between launches; every result against the
+    oracle.  hot_mb = 0.05 leaves most rows cold (mixed tags inside a warp's window)."""
     pasta, oracle, torch = env
-    monkeypatch.setenv("PASTA_HICOO_HOT", "1")
+    monkeypatch.setenv("PASTA_HICOO_HOT", tier)
     monkeypatch.setenv("PASTA_HOT_FORCE", "1")
     monkeypatch.setenv("PASTA_HOT_MB", hot_mb)
     dims = (1000, 777, 1300)
@@ -126,3 +128,31 @@ def test_hicoo_hot_block_tiers_retag(env, hot_mb, monkeypatch):
             for name, t in (("hicoo", h), ("ghicoo", gh)):
                 ex = _excess(pasta.pasta_mttkrp_hicoo(t, n, Ud), ref, ab)
                 assert ex.max() <= 0, f"{name} R={R} mode {n}: excess {ex.max():.3e}"
+
+
+def test_hicoo_tier_blocks_switch(env, monkeypatch):
+    """R#36 tier blocks on one handle while the tier mode flips (2 -> 0 -> 1 -> 2 -> generic
+    R = 12 path -> 2): the copy is rebuilt plain / tiered / retagged each time and every result
+    matches the oracle; order 4 with a gHiCOO mask; the canonical HiCOO arrays never change."""
+    pasta, oracle, torch = env
+    monkeypatch.setenv("PASTA_HOT_FORCE", "1")
+    monkeypatch.setenv("PASTA_HOT_MB", "0.1")
+    dims = (300, 520, 41, 700)
+    inds, vals = si.powerlaw_coo(dims, 200_000, seed=91)
+    x = pasta.pasta_coo_from_arrays(dims, inds, vals)
+    h = pasta.pasta_coo_to_hicoo(x, 7)
+    gh = pasta.pasta_coo_to_ghicoo(x, 7, 0b1011)  # mode 2 uncompressed
+    before = pasta.pasta_hicoo_export(h)
+    for tier, R in (("2", 16), ("0", 16), ("1", 16), ("2", 32), ("2", 12), ("2", 16)):
+        monkeypatch.setenv("PASTA_HICOO_HOT", tier)
+        U = si.factors(dims, R, seed=R + 3)
+        Ud = [torch.from_numpy(u).cuda() for u in U]
+        for n in range(4):
+            ref, ab = oracle.mttkrp(dims, inds, vals, n, U)
+            for name, t in (("hicoo", h), ("ghicoo", gh)):
+                ex = _excess(pasta.pasta_mttkrp_hicoo(t, n, Ud), ref, ab)
+                assert ex.max() <= 0, f"{name} tier {tier} R={R} mode {n}: excess {ex.max():.3e}"
+    after = pasta.pasta_hicoo_export(h)
+    for k in ("bptr", "binds", "einds"):
+        assert np.array_equal(before[k], after[k]), k
+    assert np.array_equal(before["vals"].view(np.uint32), after["vals"].view(np.uint32))
