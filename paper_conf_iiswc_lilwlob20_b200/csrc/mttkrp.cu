@@ -61,9 +61,6 @@ struct KArgs {
   // gHiCOO (R#29): bit j set <=> other-mode slot j is uncompressed: its u32 coordinates come
   // from io[j] (no slice base); clear -> 8-bit element index eo[j] + slice base
   uint32_t wide;
-  // staged decode: bulk-prefetch (into L2) the slice and entry arrays of the stage after the
-  // one just decoded (its first slices are known then)
-  uint32_t pf;
   // factors of the other modes (ascending k), output
   const float *Uo[kMaxOrder - 1];
   float *out;
@@ -138,13 +135,6 @@ __device__ __forceinline__ uint32_t ld_stream_u8(const void *p, uint64_t pol) {
   unsigned short r;
   asm("ld.global.nc.L2::cache_hint.u8 %0, [%1], %2;" : "=h"(r) : "l"(p), "l"(pol));
   return r;
-}
-// L2 prefetch of [p, p + bytes) by the bulk-copy unit (no registers, no completion to wait on);
-// p is rounded down and the size up to 16 bytes
-__device__ __forceinline__ void bulk_prefetch_l2(const void *p, uint32_t bytes) {
-  const uint64_t a = reinterpret_cast<uint64_t>(p), a0 = a & ~uint64_t(15);
-  const uint32_t n = uint32_t((a + bytes - a0 + 15) & ~uint64_t(15));
-  asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(a0), "r"(n) : "memory");
 }
 __device__ __forceinline__ float4 ld_gather_f4(const float *p, uint64_t pol) {
   float4 r;
@@ -981,32 +971,6 @@ __global__ void __launch_bounds__(HS ? WPC_ * 32 : kThreads, HS ? 1 : (WA == 6 ?
         const int clast = __shfl_sync(0xFFFFFFFFu, c, last);
         const uint32_t elast = __shfl_sync(0xFFFFFFFFu, erel, clast);
         gsb[gi] = sb0 + uint64_t(clast) + (elast <= uint32_t(SG) ? 1u : 0u);
-      }
-    }
-    // the next stage's windows: slots [gsb, gsb + 32) of the slice arrays and its 32 entries
-    // (the same group run, or the warp's next chunk -- skipped then), one array per lane
-    if (a.pf) {
-      const uint64_t nstg = (uint64_t(a.chunk) / G) / SG;
-      if (uint64_t(s) + 1 < nstg) {
-#pragma unroll
-        for (int gi = 0; gi < G; ++gi) {
-          const uint64_t pn = cc + uint64_t(gi) * run + uint64_t(s + 1) * SG;
-          if (pn >= a.nnz) continue;  // warp-uniform
-          // slot arrays are padded by kSlicePad (>= 32) slots; entry ranges stop at nnz
-          const uint64_t sb = gsb[gi] < a.nsb ? gsb[gi] : a.nsb - 1;
-          const uint32_t ne = a.nnz - pn >= uint64_t(SG) ? uint32_t(SG) : uint32_t(a.nnz - pn);
-          if (lane == 0) bulk_prefetch_l2(a.sbend32 + sb, 128);
-          else if (lane == 1) bulk_prefetch_l2(a.sbrow + sb, 128);
-          else if (lane == 2) bulk_prefetch_l2(a.val + pn, 4 * ne);
-          else if (lane >= 3 && lane < 3 + NO) {
-            const int j = lane - 3;
-            if ((a.wide >> j) & 1u) bulk_prefetch_l2(a.io[j] + pn, 4 * ne);
-            else bulk_prefetch_l2(a.eo[j] + pn, ne);
-          } else if (lane >= 3 + NO && lane < 3 + 2 * NO) {
-            const int j = lane - 3 - NO;
-            if (!((a.wide >> j) & 1u)) bulk_prefetch_l2(a.sbbase[j] + sb, 128);
-          }
-        }
       }
     }
   };
@@ -1883,7 +1847,6 @@ void launch_hicoo_mttkrp(const pasta_hicoo *h, uint32_t mode, const float *const
       PASTA_LAUNCHED();
     }
     a.sbend32 = mcw.sbend32.p;
-    a.pf = uint32_t(env_int("PASTA_HICOO_PF", 1));
     if (use_raw) {
       const uint64_t nwin = (h->nnz + 31) / 32;
       if (mcw.win_sb.n != nwin) {
