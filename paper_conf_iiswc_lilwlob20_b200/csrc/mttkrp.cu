@@ -1898,14 +1898,18 @@ void launch_hicoo_mttkrp(const pasta_hicoo *h, uint32_t mode, const float *const
       a.hs_lo[jj] = uint32_t(mc.rs_total);
     }
     ProfScope prof(kProfHicoo, s);
-    const int cfg = env_int("PASTA_HS_CFG", 0);  // 2 (8-deep steps) spills here
+    // shape: 0 = 16 warps x 4-nonzero steps; 2 = 16 x 8 (spills here: H 3.59 ms); 3 = 12 warps x
+    // 8-nonzero steps (168 registers), the default with an L2 tier at order 3 (H 2.61 -> 2.53 ms,
+    // profiles/r02_hicoo_tier_sweep.txt)
+    const int cfg = env_int("PASTA_HS_CFG", (tiers && mc.hot_total > 0 && hno <= 2) ? 3 : 0);
     const size_t smem = stage + (tiers ? size_t(mc.hs_total) * R * sizeof(float) : 0) + (use_raw ? raw_bytes : 0) +
                         (rowtier ? size_t(mc.rs_total) * R * sizeof(float) + 8 * words : 0);
     const uint64_t nwarps = (a.nnz + a.chunk - 1) / a.chunk;
-    const uint64_t nblk = std::min<uint64_t>((nwarps + 15) / 16, uint64_t(sm_count()));
+    const int wpc = (cfg == 3 && tiers && hno <= 2) ? 12 : 16;  // warps per CTA
+    const uint64_t nblk = std::min<uint64_t>((nwarps + wpc - 1) / wpc, uint64_t(sm_count()));
     auto go = [&](auto kern) {
       PASTA_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem)));
-      kern<<<unsigned(nblk), 512, smem, s>>>(a);
+      kern<<<unsigned(nblk), wpc * 32, smem, s>>>(a);
       PASTA_LAUNCHED();
       mcw.fence.record(s);
     };
@@ -1919,7 +1923,12 @@ void launch_hicoo_mttkrp(const pasta_hicoo *h, uint32_t mode, const float *const
     else if (use_raw)
       with_no_lpn<2>(hno, lpn, [&](auto NOt, auto Lt) { go(coo_staged_kernel<NOt.value, Lt.value, 11, true, 16, 32, 4>); });
     else if (tiers)
-      with_no_lpn<3>(hno, lpn, [&](auto NOt, auto Lt) { go(coo_staged_kernel<NOt.value, Lt.value, 10, true, 16, 32, 4>); });
+      if (cfg == 2 && hno <= 2)  // 8-nonzero steps (the COO shape on DRAM-bound gathers)
+        with_no_lpn<2>(hno, lpn, [&](auto NOt, auto Lt) { go(coo_staged_kernel<NOt.value, Lt.value, 10, true, 16, 32, 8>); });
+      else if (cfg == 3 && hno <= 2)  // 12 warps x 8-nonzero steps: 168 registers, no spills
+        with_no_lpn<2>(hno, lpn, [&](auto NOt, auto Lt) { go(coo_staged_kernel<NOt.value, Lt.value, 10, true, 12, 32, 8>); });
+      else
+        with_no_lpn<3>(hno, lpn, [&](auto NOt, auto Lt) { go(coo_staged_kernel<NOt.value, Lt.value, 10, true, 16, 32, 4>); });
     else if (cfg == 2 && hno <= 2)
       with_no_lpn<2>(hno, lpn, [&](auto NOt, auto Lt) { go(coo_staged_kernel<NOt.value, Lt.value, 9, true, 16, 32, 8>); });
     else
