@@ -877,7 +877,7 @@ __global__ void __launch_bounds__(HS ? WPC_ * 32 : kThreads, HS ? 1 : (WA == 6 ?
   // an entry's slot = #{slots whose end <= entry} by a 5-step shuffle search over the sorted
   // slot ends; row and block bases come from the owning lane by shuffle; i_k = base + e_k
   // (Alg. 3's rebased pointers).  gsb[g] = current slice of group g (warp-uniform).
-  uint64_t gsb[G];
+  uint32_t gsb[G];  // slice indices < nnz < 2^32 (API)
   uint32_t rs_j[NO > 0 ? NO : 1];  // WA 16: shared addresses of each mode's bitmap (prefixes follow)
   if constexpr (kHicRows) {
     uint32_t rs = hs_saddr + a.hs_lo[NO] * R * 4u;
@@ -901,7 +901,7 @@ __global__ void __launch_bounds__(HS ? WPC_ * 32 : kThreads, HS ? 1 : (WA == 6 ?
     if (s == 0) {
       const uint64_t nruns = (a.nnz + run - 1) / run;
 #pragma unroll
-      for (int gi = 0; gi < G; ++gi) gsb[gi] = __ldg(a.run_sb + (r0 + gi < nruns ? r0 + gi : nruns - 1));
+      for (int gi = 0; gi < G; ++gi) gsb[gi] = uint32_t(__ldg(a.run_sb + (r0 + gi < nruns ? r0 + gi : nruns - 1)));
     }
 #ifdef PASTA_DECODE_GB
     constexpr int GB = G < PASTA_DECODE_GB ? G : PASTA_DECODE_GB;
@@ -970,7 +970,7 @@ __global__ void __launch_bounds__(HS ? WPC_ * 32 : kThreads, HS ? 1 : (WA == 6 ?
         const int last = nleft >= uint64_t(SG) ? SG - 1 : int(nleft) - 1;
         const int clast = __shfl_sync(0xFFFFFFFFu, c, last);
         const uint32_t elast = __shfl_sync(0xFFFFFFFFu, erel, clast);
-        gsb[gi] = sb0 + uint64_t(clast) + (elast <= uint32_t(SG) ? 1u : 0u);
+        gsb[gi] = uint32_t(sb0) + uint32_t(clast) + (elast <= uint32_t(SG) ? 1u : 0u);
       }
     }
   };
@@ -1902,10 +1902,17 @@ void launch_hicoo_mttkrp(const pasta_hicoo *h, uint32_t mode, const float *const
     // 8-nonzero steps (168 registers), the default with an L2 tier at order 3 (H 2.61 -> 2.53 ms,
     // profiles/r02_hicoo_tier_sweep.txt)
     const int cfg = env_int("PASTA_HS_CFG", (tiers && mc.hot_total > 0 && hno <= 2) ? 3 : 0);
-    const size_t smem = stage + (tiers ? size_t(mc.hs_total) * R * sizeof(float) : 0) + (use_raw ? raw_bytes : 0) +
+    uint64_t max_gf = 0;
+    for (uint32_t k = 0; k < h->order; ++k)
+      if (k != mode) max_gf = std::max<uint64_t>(max_gf, uint64_t(h->dims[k]) * R * sizeof(float));
+    // kernel choice (below) and its warps per CTA
+    const bool wa17 = tiers && mc.hot_total == 0 && max_gf < (uint64_t(1) << 32);
+    const int wpc = wa17 || rowtier || use_raw ? 16
+                    : tiers                    ? ((cfg == 3 && hno <= 2) ? 12 : 16)
+                                               : 16;
+    const size_t smem = stage * wpc / 16 + (tiers ? size_t(mc.hs_total) * R * sizeof(float) : 0) + (use_raw ? raw_bytes : 0) +
                         (rowtier ? size_t(mc.rs_total) * R * sizeof(float) + 8 * words : 0);
     const uint64_t nwarps = (a.nnz + a.chunk - 1) / a.chunk;
-    const int wpc = (cfg == 3 && tiers && hno <= 2) ? 12 : 16;  // warps per CTA
     const uint64_t nblk = std::min<uint64_t>((nwarps + wpc - 1) / wpc, uint64_t(sm_count()));
     auto go = [&](auto kern) {
       PASTA_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem)));
@@ -1913,23 +1920,20 @@ void launch_hicoo_mttkrp(const pasta_hicoo *h, uint32_t mode, const float *const
       PASTA_LAUNCHED();
       mcw.fence.record(s);
     };
-    uint64_t max_gf = 0;
-    for (uint32_t k = 0; k < h->order; ++k)
-      if (k != mode) max_gf = std::max<uint64_t>(max_gf, uint64_t(h->dims[k]) * R * sizeof(float));
-    if (tiers && mc.hot_total == 0 && max_gf < (uint64_t(1) << 32))  // smem tier only: WA 17
+    if (wa17)  // smem tier only: WA 17
       with_no_lpn<3>(hno, lpn, [&](auto NOt, auto Lt) { go(coo_staged_kernel<NOt.value, Lt.value, 17, true, 16, 32, 4>); });
     else if (rowtier)
       with_no_lpn<3>(hno, lpn, [&](auto NOt, auto Lt) { go(coo_staged_kernel<NOt.value, Lt.value, 16, true, 16, 32, 4>); });
     else if (use_raw)
       with_no_lpn<2>(hno, lpn, [&](auto NOt, auto Lt) { go(coo_staged_kernel<NOt.value, Lt.value, 11, true, 16, 32, 4>); });
-    else if (tiers)
+    else if (tiers) {
       if (cfg == 2 && hno <= 2)  // 8-nonzero steps (the COO shape on DRAM-bound gathers)
         with_no_lpn<2>(hno, lpn, [&](auto NOt, auto Lt) { go(coo_staged_kernel<NOt.value, Lt.value, 10, true, 16, 32, 8>); });
       else if (cfg == 3 && hno <= 2)  // 12 warps x 8-nonzero steps: 168 registers, no spills
         with_no_lpn<2>(hno, lpn, [&](auto NOt, auto Lt) { go(coo_staged_kernel<NOt.value, Lt.value, 10, true, 12, 32, 8>); });
       else
         with_no_lpn<3>(hno, lpn, [&](auto NOt, auto Lt) { go(coo_staged_kernel<NOt.value, Lt.value, 10, true, 16, 32, 4>); });
-    else if (cfg == 2 && hno <= 2)
+    } else if (cfg == 2 && hno <= 2)
       with_no_lpn<2>(hno, lpn, [&](auto NOt, auto Lt) { go(coo_staged_kernel<NOt.value, Lt.value, 9, true, 16, 32, 8>); });
     else
       with_no_lpn<3>(hno, lpn, [&](auto NOt, auto Lt) { go(coo_staged_kernel<NOt.value, Lt.value, 9, true, 16, 32, 4>); });
