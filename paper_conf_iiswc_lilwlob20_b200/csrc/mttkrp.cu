@@ -131,11 +131,6 @@ __device__ __forceinline__ uint32_t ld_stream_u32(const void *p, uint64_t pol) {
   asm("ld.global.nc.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(r) : "l"(p), "l"(pol));
   return r;
 }
-__device__ __forceinline__ uint32_t ld_stream_u8(const void *p, uint64_t pol) {
-  unsigned short r;
-  asm("ld.global.nc.L2::cache_hint.u8 %0, [%1], %2;" : "=h"(r) : "l"(p), "l"(pol));
-  return r;
-}
 __device__ __forceinline__ float4 ld_gather_f4(const float *p, uint64_t pol) {
   float4 r;
   asm("ld.global.nc.L2::cache_hint.v4.f32 {%0, %1, %2, %3}, [%4], %5;"
@@ -919,21 +914,20 @@ __global__ void __launch_bounds__(HS ? WPC_ * 32 : kThreads, HS ? 1 : (WA == 6 ?
         const uint64_t p = cc + uint64_t(gb + q) * run + uint64_t(s) * SG;
         const uint64_t sb0 = gsb[gb + q];
         const uint64_t st = sb0 + lane < a.nsb ? sb0 + lane : a.nsb - 1;
-        // the slice and entry arrays are read once per launch: evict_first (pol.stream), like
-        // the COO stream, so they do not push the tiers and hot factor rows out of L2
-        eabs[q] = ld_stream_u32(a.sbend32 + st, pol.stream);  // = sbptr[st + 1]
-        srow[q] = ld_stream_u32(a.sbrow + st, pol.stream);
+        // the slice and entry arrays are read once per launch: cache-streaming loads (ld.cs,
+        // evict-first in L2), like the COO stream, so they do not push the tiers and hot factor
+        // rows out of L2.  (The same loads with an L2::cache_hint policy operand faulted for
+        // order-2 instantiations at R >= 32 under ptxas 12.9.)
+        eabs[q] = __ldcs(a.sbend32 + st);  // = sbptr[st + 1]
+        srow[q] = __ldcs(a.sbrow + st);
 #pragma unroll
-        for (int j = 0; j < NO; ++j)
-          sbase[q][j] = ((a.wide >> j) & 1u) ? 0u : ld_stream_u32(a.sbbase[j] + st, pol.stream);
+        for (int j = 0; j < NO; ++j) sbase[q][j] = ((a.wide >> j) & 1u) ? 0u : __ldcs(a.sbbase[j] + st);
         const uint64_t x = p + lane;
         const bool ok = x < a.nnz;
-        v[q] = ok ? __uint_as_float(ld_stream_u32(a.val + x, pol.stream)) : 0.f;
+        v[q] = ok ? __ldcs(a.val + x) : 0.f;
 #pragma unroll
         for (int j = 0; j < NO; ++j)
-          e[q][j] = !ok ? 0u
-                        : ((a.wide >> j) & 1u) ? ld_stream_u32(a.io[j] + x, pol.stream)
-                                               : ld_stream_u8(a.eo[j] + x, pol.stream);
+          e[q][j] = !ok ? 0u : ((a.wide >> j) & 1u) ? __ldcs(a.io[j] + x) : uint32_t(__ldcs(a.eo[j] + x));
       }
 #pragma unroll
       for (int q = 0; q < GB; ++q) {

@@ -143,7 +143,7 @@ def test_hicoo_tier_blocks_switch(env, monkeypatch):
     h = pasta.pasta_coo_to_hicoo(x, 7)
     gh = pasta.pasta_coo_to_ghicoo(x, 7, 0b1011)  # mode 2 uncompressed
     before = pasta.pasta_hicoo_export(h)
-    for tier, R in (("2", 16), ("0", 16), ("1", 16), ("2", 32), ("2", 12), ("2", 16)):
+    for tier, R in (("2", 16), ("0", 16), ("1", 16), ("2", 32), ("2", 64), ("2", 12), ("2", 16)):
         monkeypatch.setenv("PASTA_HICOO_HOT", tier)
         U = si.factors(dims, R, seed=R + 3)
         Ud = [torch.from_numpy(u).cuda() for u in U]
@@ -156,3 +156,49 @@ def test_hicoo_tier_blocks_switch(env, monkeypatch):
     for k in ("bptr", "binds", "einds"):
         assert np.array_equal(before[k], after[k]), k
     assert np.array_equal(before["vals"].view(np.uint32), after["vals"].view(np.uint32))
+
+
+@pytest.mark.parametrize("hot,cfg", [("0", "0"), ("2", "0"), ("2", "2"), ("2", "3")])
+def test_hicoo_staged_orders_ranks(env, hot, cfg, monkeypatch):
+    """The staged HiCOO kernels (plain decode WA 9, tier blocks WA 10 / 17) in every shape
+    (PASTA_HS_CFG 0 = 16 warps x 4-nonzero steps, 2 = 16 x 8, 3 = 12 x 8) at orders 2, 3, 4 and
+    R = 16, 32, 64, tiers forced on (order 2 at R >= 32 once faulted with cache-hinted decode
+    loads; the decode now uses ld.cs)."""
+    pasta, oracle, torch = env
+    monkeypatch.setenv("PASTA_HICOO_HOT", hot)
+    monkeypatch.setenv("PASTA_HS_CFG", cfg)
+    monkeypatch.setenv("PASTA_HOT_FORCE", "1")
+    monkeypatch.setenv("PASTA_HOT_MB", "0.2")
+    for dims in ((5000, 3000), (900, 1300, 700), (300, 520, 41, 700)):
+        inds, vals = si.powerlaw_coo(dims, 120_000, seed=5)
+        x = pasta.pasta_coo_from_arrays(dims, inds, vals)
+        h = pasta.pasta_coo_to_hicoo(x, 7)
+        for R in (16, 32, 64):
+            U = si.factors(dims, R, seed=R + 11)
+            Ud = [torch.from_numpy(u).cuda() for u in U]
+            for n in range(len(dims)):
+                ref, ab = oracle.mttkrp(dims, inds, vals, n, U)
+                ex = _excess(pasta.pasta_mttkrp_hicoo(h, n, Ud), ref, ab)
+                assert ex.max() <= 0, f"hot {hot} cfg {cfg} dims {dims} R={R} mode {n}: excess {ex.max():.3e}"
+
+
+@pytest.mark.parametrize("shape", ["12x8", "16x4"])
+def test_hicoo_tier_blocks_orders_2_3(env, shape, monkeypatch):
+    """R#36 tier blocks with both tiers forced on, at orders 2 (SpMM-like) and 3, in the default
+    12-warp x 8-nonzero-step shape and the 16 x 4 shape, R = 16 and 32."""
+    pasta, oracle, torch = env
+    monkeypatch.setenv("PASTA_HICOO_HOT", "2")
+    monkeypatch.setenv("PASTA_HOT_FORCE", "1")
+    monkeypatch.setenv("PASTA_HOT_MB", "0.2")
+    monkeypatch.setenv("PASTA_HS_CFG", "3" if shape == "12x8" else "0")
+    for dims, nnz, seed in (((5000, 3000), 120_000, 5), ((900, 1300, 700), 250_000, 6)):
+        inds, vals = si.powerlaw_coo(dims, nnz, seed=seed)
+        x = pasta.pasta_coo_from_arrays(dims, inds, vals)
+        h = pasta.pasta_coo_to_hicoo(x, 7)
+        for R in (16, 32):
+            U = si.factors(dims, R, seed=R + 11)
+            Ud = [torch.from_numpy(u).cuda() for u in U]
+            for n in range(len(dims)):
+                ref, ab = oracle.mttkrp(dims, inds, vals, n, U)
+                ex = _excess(pasta.pasta_mttkrp_hicoo(h, n, Ud), ref, ab)
+                assert ex.max() <= 0, f"{shape} dims {dims} R={R} mode {n}: excess {ex.max():.3e}"
