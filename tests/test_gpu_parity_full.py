@@ -180,6 +180,13 @@ def test_hicoo_staged_orders_ranks(env, hot, cfg, monkeypatch):
                 ref, ab = oracle.mttkrp(dims, inds, vals, n, U)
                 ex = _excess(pasta.pasta_mttkrp_hicoo(h, n, Ud), ref, ab)
                 assert ex.max() <= 0, f"hot {hot} cfg {cfg} dims {dims} R={R} mode {n}: excess {ex.max():.3e}"
+                if R == 32:  # two row shards (pasta_hicoo_shard) into one output, tiers rebuilt per shard
+                    b = pasta.pasta_coo_partition(x, n, 2)
+                    out = torch.zeros((dims[n], R), device="cuda")
+                    for q in range(2):
+                        pasta.pasta_mttkrp_hicoo(pasta.pasta_hicoo_shard(h, n, int(b[q]), int(b[q + 1])), n, Ud, out=out)
+                    ex = _excess(out, ref, ab)
+                    assert ex.max() <= 0, f"shards hot {hot} cfg {cfg} dims {dims} mode {n}: excess {ex.max():.3e}"
 
 
 @pytest.mark.parametrize("shape", ["12x8", "16x4"])
