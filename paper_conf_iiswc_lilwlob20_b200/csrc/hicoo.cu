@@ -161,7 +161,7 @@ __global__ void slice_emit_kernel(SliceOut o, const uint32_t *__restrict__ start
 struct TierArgs {
   const uint32_t *binds[kMaxOrder];
   const uint8_t *einds[kMaxOrder];
-  const uint32_t *rank[kMaxOrder];  // null: mode not tiered (the target mode, uncompressed modes)
+  const uint32_t *rank[kMaxOrder];  // null: not ranked (no tiers)
   uint32_t ntier[kMaxOrder];        // tier blocks of mode k (smem ones first)
   uint32_t nbr[kMaxOrder];          // block rows of mode k: keys >= nbr are tier blocks
   uint32_t *key[kMaxOrder];
@@ -177,17 +177,19 @@ __global__ void tier_entry_kernel(TierArgs t, const uint32_t *__restrict__ blk, 
        x += uint64_t(gridDim.x) * blockDim.x) {
     const uint32_t b = blk[x];
     for (uint32_t k = 0; k < t.order; ++k) {
-      if (!t.rank[k]) continue;
+      if (!t.key[k]) continue;  // the target mode, uncompressed modes
       const uint32_t bk = t.binds[k][b], ek = t.einds[k][x];
-      const uint32_t rho = t.rank[k][(bk << t.bbits) | ek];
-      const uint32_t m = rho >> t.bbits;
-      if (m < t.ntier[k]) {
-        t.key[k][x] = t.nbr[k] + m;
-        t.e[k][x] = uint8_t(rho & ((1u << t.bbits) - 1u));
-      } else {
-        t.key[k][x] = bk;
-        t.e[k][x] = uint8_t(ek);
+      if (t.rank[k] && t.ntier[k]) {
+        const uint32_t rho = t.rank[k][(bk << t.bbits) | ek];
+        const uint32_t m = rho >> t.bbits;
+        if (m < t.ntier[k]) {
+          t.key[k][x] = t.nbr[k] + m;
+          t.e[k][x] = uint8_t(rho & ((1u << t.bbits) - 1u));
+          continue;
+        }
       }
+      t.key[k][x] = bk;
+      t.e[k][x] = uint8_t(ek);
     }
   }
 }
@@ -240,6 +242,25 @@ __global__ void entry_row_count_kernel(const uint32_t *__restrict__ binds_k, con
   for (uint64_t x = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; x < M;
        x += uint64_t(gridDim.x) * blockDim.x)
     atomicAdd(&cnt[(binds_k[blk[x]] << bb) | einds_k[x]], 1u);
+}
+
+__global__ void coord_count_kernel(const uint32_t *__restrict__ c, uint64_t M, uint32_t *__restrict__ cnt) {
+  for (uint64_t x = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; x < M;
+       x += uint64_t(gridDim.x) * blockDim.x)
+    atomicAdd(&cnt[c[x]], 1u);
+}
+
+// gHiCOO uncompressed mode (R#36): the entry's full coordinate, or the tag | slot of its tier row
+__global__ void tier_coord_kernel(const uint32_t *__restrict__ c, const uint32_t *__restrict__ perm, uint64_t M,
+                                  const uint32_t *__restrict__ rank, uint32_t nrank_tier, uint32_t nrank_smem,
+                                  uint32_t hs_base, uint32_t hot_base, uint32_t *__restrict__ out) {
+  for (uint64_t x = blockIdx.x * uint64_t(blockDim.x) + threadIdx.x; x < M;
+       x += uint64_t(gridDim.x) * blockDim.x) {
+    const uint32_t v = c[perm[x]], rho = rank[v];
+    out[x] = rho >= nrank_tier ? v
+             : rho < nrank_smem ? (0xC0000000u | (hs_base + rho))
+                                : (0x80000000u | (hot_base + rho - nrank_smem));
+  }
 }
 
 __global__ void scatter_rank_kernel(const uint32_t *__restrict__ order, uint32_t n, uint32_t *__restrict__ rank) {
@@ -565,6 +586,11 @@ static void hicoo_prepare_rowslice_tiered(pasta_hicoo *h, uint32_t mode, const T
       co.c[co.order++] = keyp[k].p;
       key[k].reset();
       e[k].reset();
+    } else if (tp.ntier[k]) {
+      tier_coord_kernel<<<grid_for(M), kThreads, 0, s>>>(h->uinds[k].p, perm.p, M, h->rt_rank[k].p, tp.ntier[k] << bb,
+                                                         tp.sblk[k] << bb, tp.hs_base[k], tp.hot_base[k],
+                                                         mc.uinds[k].p);
+      PASTA_LAUNCHED();
     } else {
       gather_u32(h->uinds[k].p, perm.p, mc.uinds[k].p, M, s);
     }
@@ -611,7 +637,10 @@ static void hicoo_rank_mode(pasta_hicoo *h, uint32_t k, const uint32_t *blk, cud
   const uint64_t M = h->nnz;
   DevArray<uint32_t> cnt(n, s), cnt_sorted(n, s), rows(n, s);
   PASTA_CUDA(cudaMemsetAsync(cnt.p, 0, cnt.bytes(), s));
-  entry_row_count_kernel<<<grid_for(M), kThreads, 0, s>>>(h->binds[k].p, blk, h->einds[k].p, bb, M, cnt.p);
+  if ((h->cmask >> k) & 1u)
+    entry_row_count_kernel<<<grid_for(M), kThreads, 0, s>>>(h->binds[k].p, blk, h->einds[k].p, bb, M, cnt.p);
+  else  // gHiCOO uncompressed mode: full coordinates
+    coord_count_kernel<<<grid_for(M), kThreads, 0, s>>>(h->uinds[k].p, M, cnt.p);
   PASTA_LAUNCHED();
   iota_u32(rows.p, n, s);
   h->rt_order[k].alloc(n, s);
@@ -656,7 +685,9 @@ void hicoo_tier_rows(pasta_hicoo *h, uint32_t mode, uint32_t R, bool on, bool gl
   }
   if (mc.rt_on && mc.rt_R == R && mc.rt_global == global_tier && mc.rt_budget == smem_rows) return;
   const uint32_t N = h->order, bb = h->block_bits, B = 1u << bb;
-  auto tiered = [&](uint32_t k) { return k != mode && ((h->cmask >> k) & 1u) != 0; };
+  // every gathered mode: compressed ones through re-blocked slices, uncompressed (gHiCOO) ones
+  // through tagged per-entry coordinates
+  auto tiered = [&](uint32_t k) { return k != mode; };
   bool ok = true;
   for (uint32_t k = 0; k < N; ++k)
     if (h->dims[k] >= 0x40000000u) ok = false;  // tagged bases need slots below 2^30
