@@ -371,11 +371,12 @@ unsigned grid8(uint64_t n) {
 //    the kernel is bound by L2->SM bandwidth, and power-law-hot rows carry most gathers);
 //  * L2 tier (`global_tier`, when the gathered factors exceed L2): the next rows, as many as fit
 //    PASTA_HOT_MB (default 64 MB) at R*4 bytes per row, get contiguous slots of one buffer
-//    refilled from the factors before every launch.  Packed hot rows fill whole L2 lines and
-//    stay resident, where scattered ones share lines with cold neighbours and are evicted by
-//    the cold-row and stream traffic: L2 turns from LRU over scattered rows into a
-//    frequency-based cache for the power-law gathers (cache reuse is why MTTKRP beats its
-//    DRAM roofline).
+//    refilled from the factors before every launch.  Packed hot rows fill whole L2 lines, and
+//    their misses land on a 64-MB region instead of the whole factor: on H the DRAM bytes stay
+//    about the same (8.10 vs 8.32 GB per launch) but the kernel runs 2.4x faster, because
+//    scattered misses are bound by the rate of DRAM row activations (~37 G/s) and packed ones
+//    are not (profiles/r02_coo_l2_tier_effect.txt; cache reuse is why MTTKRP beats its DRAM
+//    roofline).
 // The per-mode index copies hot_inds[k] encode 0xC0000000 | smem slot (slot numbered over all
 // gathered factors, factor k at [hs_base[k], +hs_cnt[k])), 0x80000000 | L2-tier slot, or the
 // plain row.  Needs dims < 2^30.
