@@ -199,6 +199,12 @@ pasta_status pasta_hicoo_prepare(pasta_hicoo *h, uint32_t mode, void *stream);
  * kernels then gather every row from the factors). */
 pasta_status pasta_mttkrp_coo(pasta_coo *x, uint32_t mode, const float *const *factors,
                               uint32_t R, float *out, void *stream);
+/* As pasta_mttkrp_coo over the HiCOO handle's per-mode working copy (Alg. 3; R#27).
+ * When every gathered factor exceeds twice the L2 (or PASTA_HICOO_HOT=2), the first call per
+ * (mode, R) rebuilds that copy over heat-ranked "tier blocks" of the gathered modes (R#36:
+ * hot rows served from the shared-memory / L2-tier buffers, synchronising once); the canonical
+ * HiCOO arrays (pasta_hicoo_export) never change.  Same concurrency and thread-safety as
+ * pasta_mttkrp_coo. */
 pasta_status pasta_mttkrp_hicoo(pasta_hicoo *h, uint32_t mode, const float *const *factors,
                                 uint32_t R, float *out, void *stream);
 /* Fused MTTKRP + all-gather over peer memory (a9; SURVEY 8(e) "fused variant"): as
