@@ -195,6 +195,7 @@ struct CooModeCopy {
   DevArray<uint32_t> split_irow;
   DevArray<float> split_val;
   DevArray<unsigned long long> claim;   // per-die chunk counters, zeroed before each launch
+  bool smem_fill = false;               // PASTA_HOT_SMEM_FILL: smem tier filled from the next bucket
 };
 
 constexpr int kCountBuckets = 256;  // 8 sub-buckets per octave of a row's nonzero count

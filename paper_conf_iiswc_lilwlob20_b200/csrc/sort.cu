@@ -364,6 +364,11 @@ unsigned grid8(uint64_t n) {
 
 }  // namespace
 
+static bool env_flag(const char *name) {
+  const char *v = getenv(name);
+  return v && *v && atoi(v) != 0;
+}
+
 // Hot-row cache for the COO factor gathers, two tiers.  The most frequent rows of the gathered
 // factors (row nonzero counts, bucketed 8 per octave) are ranked jointly over the factors:
 //  * shared-memory tier: as many as fit `smem_rows` rows (the kernel copies them into every
@@ -383,9 +388,16 @@ unsigned grid8(uint64_t n) {
 void coo_mark_hot(pasta_coo *x, uint32_t mode, uint32_t R, bool global_tier, uint32_t smem_rows,
                   cudaStream_t s, bool die_split) {
   CooModeCopy &mc = x->mc[mode];
+  // the shared-memory tier filled to its budget from the next count bucket down: on
+  // L2-resident factors (no L2 tier) every row it serves is an L1TEX wavefront saved (C2 0.757
+  // -> 0.729 ms per mode); with DRAM-bound gathers it takes L1 from the in-flight misses (H 1.56
+  // -> 1.71), so off there (profiles/r02_smem_fill_sweep.txt).  PASTA_HOT_SMEM_FILL overrides.
+  const char *fenv = getenv("PASTA_HOT_SMEM_FILL");
+  const bool smem_fill = (fenv && *fenv) ? atoi(fenv) != 0 : !global_tier;
   if (mc.hot_R == R && mc.hot_global == global_tier && mc.hot_smem_budget == smem_rows &&
-      mc.split == die_split)
+      mc.split == die_split && mc.smem_fill == smem_fill)
     return;
+  mc.smem_fill = smem_fill;
   // die split (R#35): two gathered factors, an L2 tier and a measured SM -> die map
   die_split = die_split && global_tier && x->order == 3;
   const DieMap *dmp = die_split ? &die_map() : nullptr;  // calibrates on first use only
@@ -446,6 +458,19 @@ void coo_mark_hot(pasta_coo *x, uint32_t mode, uint32_t R, bool global_tier, uin
   const uint32_t hsb = threshold(double(smem_rows));  // smem tier: bucket >= hsb
   const uint32_t hb =                                  // L2 tier: hb <= bucket < hsb
       hot_mb > 0 ? threshold(double(smem_rows) + hot_mb * 1048576.0 / (double(R) * 4.0)) : hsb;
+  uint64_t smem_fill_extra[kMaxOrder] = {};
+  if (smem_fill && hsb > 1 && hsb <= kCountBuckets && smem_rows > 0) {
+    double in_tier = 0.0, next = 0.0;
+    for (uint32_t k = 0; k < N; ++k) {
+      if (k == mode) continue;
+      for (uint32_t b = hsb; b < kCountBuckets; ++b) in_tier += double(x->count_hist[k][b]);
+      next += double(x->count_hist[k][hsb - 1]);
+    }
+    const double left = double(smem_rows) - in_tier;
+    if (left > 0 && next > 0)
+      for (uint32_t k = 0; k < N; ++k)
+        if (k != mode) smem_fill_extra[k] = uint64_t(double(x->count_hist[k][hsb - 1]) * std::min(1.0, left / next));
+  }
   // both tiers -> contiguous slots (per tier, factor after factor, rows ascending)
   uint64_t total = 0, stotal = 0;
   std::vector<DevArray<uint32_t>> lists(N), slists(N);
@@ -462,6 +487,22 @@ void coo_mark_hot(pasta_coo *x, uint32_t mode, uint32_t R, bool global_tier, uin
       PASTA_LAUNCHED();
       mc.hs_cnt[k] = select_flagged(flag.p, x->dims[k], slists[k], s);
       stotal += mc.hs_cnt[k];
+    }
+    // smem fill: the budget the whole buckets leave is filled with rows of the next bucket
+    // down (each factor in proportion to its rows there; with an L2 tier they keep that slot too)
+    if (hsb > 1 && hsb <= kCountBuckets && smem_fill_extra[k] > 0) {
+      hot_flag_kernel<<<grid8(x->dims[k]), 256, 0, s>>>(x->row_count[k].p, x->dims[k], hsb - 1, hsb, flag.p);
+      PASTA_LAUNCHED();
+      DevArray<uint32_t> more;
+      const uint64_t nm = std::min<uint64_t>(select_flagged(flag.p, x->dims[k], more, s), smem_fill_extra[k]);
+      DevArray<uint32_t> cat(mc.hs_cnt[k] + nm, s);
+      if (mc.hs_cnt[k])
+        PASTA_CUDA(cudaMemcpyAsync(cat.p, slists[k].p, mc.hs_cnt[k] * 4, cudaMemcpyDeviceToDevice, s));
+      PASTA_CUDA(cudaMemcpyAsync(cat.p + mc.hs_cnt[k], more.p, nm * 4, cudaMemcpyDeviceToDevice, s));
+      PASTA_CUDA(cudaStreamSynchronize(s));
+      slists[k] = std::move(cat);
+      mc.hs_cnt[k] += nm;
+      stotal += nm;
     }
     if (hb < hsb) {
       hot_flag_kernel<<<grid8(x->dims[k]), 256, 0, s>>>(x->row_count[k].p, x->dims[k], hb, hsb, flag.p);
