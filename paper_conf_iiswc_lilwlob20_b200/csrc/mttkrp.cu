@@ -1506,9 +1506,12 @@ void launch_coo_mttkrp_bcast(const pasta_coo *x, uint32_t mode, const float *con
     // registers) and 12 warps x 8-deep steps are slower everywhere (H 1.80 / 1.73 ms).
     // (R = 8 with DRAM-bound gathers: the 32-deep shape does not fit -> non-persistent kernel,
     // which measured faster there than forcing the 16-deep shape: H 1.80 vs 2.01 ms)
-    const int hs_cfg = env_int("PASTA_HS_CFG", no <= 2 ? (want_hot ? 2 : 1) : 0);
-    const int hs_wpc = hs_cfg == 1 ? 24 : 16;
-    const int hs_sg = hs_cfg == 1 ? 16 : 32;
+    // L2-resident factors: 20 warps x 16-deep (order <= 3) / 16 x 16-deep (order 4) -- the
+    // shallower stage leaves the shared-memory tier 256-640 more rows (C2 0.728 -> 0.699, C4
+    // 0.687 -> 0.676 ms per mode, profiles/r02_smem_fill_sweep.txt)
+    const int hs_cfg = env_int("PASTA_HS_CFG", no <= 2 ? (want_hot ? 2 : 6) : (want_hot ? 0 : 5));
+    const int hs_wpc = hs_cfg == 1 ? 24 : hs_cfg == 6 ? 20 : 16;
+    const int hs_sg = (hs_cfg == 1 || hs_cfg == 5 || hs_cfg == 6) ? 16 : 32;  // 5: 16 x 16 x 4, 6: 20 x 16 x 4
     const size_t stage_hs = size_t(hs_wpc) * 2 * (no + 2) * (G * hs_sg) * sizeof(uint32_t);
     const size_t smem_cap = 227 * 1024;
     uint32_t hs_rows_budget =
@@ -1636,6 +1639,10 @@ void launch_coo_mttkrp_bcast(const pasta_coo *x, uint32_t mode, const float *con
     if (hs && nout > 1) {  // fused MTTKRP + all-gather over peer memory, same shape as below
       if (hs_cfg == 1)
         with_no_lpn<3>(no, lpn, [&](auto NOt, auto Lt) { go(coo_staged_kernel<NOt.value, Lt.value, 15, true, 24, 16, 4>); });
+      else if (hs_cfg == 5)
+        with_no_lpn<3>(no, lpn, [&](auto NOt, auto Lt) { go(coo_staged_kernel<NOt.value, Lt.value, 15, true, 16, 16, 4>); });
+      else if (hs_cfg == 6)
+        with_no_lpn<3>(no, lpn, [&](auto NOt, auto Lt) { go(coo_staged_kernel<NOt.value, Lt.value, 15, true, 20, 16, 4>); });
       else if (hs_cfg == 2 && no <= 2)
         with_no_lpn<2>(no, lpn, [&](auto NOt, auto Lt) { go(coo_staged_kernel<NOt.value, Lt.value, 15, true, 16, 32, 8>); });
       else
@@ -1644,6 +1651,8 @@ void launch_coo_mttkrp_bcast(const pasta_coo *x, uint32_t mode, const float *con
     }
     if (hs) {
       if (hs_cfg == 1) pick_hs(std::integral_constant<int, 24>(), I16());
+      else if (hs_cfg == 5) pick_hs(I16(), I16());
+      else if (hs_cfg == 6) pick_hs(std::integral_constant<int, 20>(), I16());
       else if (hs_cfg == 2 && no <= 2 && l2t && (a.cache_mode & 8u))  // cold gathers evict_first
         with_no_lpn<2>(no, lpn, [&](auto NOt, auto Lt) { go(coo_staged_kernel<NOt.value, Lt.value, 12, true, 16, 32, 8>); });
       else if (hs_cfg == 2 && no <= 2 && l2t && env_int("PASTA_GATHER_L1NA", 0))  // gathers skip L1
